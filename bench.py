@@ -1,0 +1,312 @@
+#!/usr/bin/env python
+"""bench.py — AIG node-pattern evals/s of the exhaustive-simulation hot path on B200.
+
+One "step" = one full cec_plan_run of the workload: every window's whole 2^k pattern space
+simulated and every candidate pair compared, plus the NCCL min
+all-reduce when N > 1. Default workload = C5 (BASELINE.json configs[4], the config the metric is
+quoted on at 1/2/4/8 GPUs): 256 disjoint copies, ~2.1M ANDs, 6320 PO pairs, k = 24 per copy.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config c5|c2|c2bug|c1] [--impl ours|reference]
+
+value      = W (node-patterns of one step, all ranks) / device time per step (CUDA events on the
+             launch stream, max over ranks), schedules resident in HBM, L2 flushed between steps
+e2e        = same metric through the public blocking C call cec_sim_exhaustive with host arrays
+             (planning + H2D of schedules + kernels + all-reduce + D2H of results per step)
+roofline   = ALU (LOP3) bound: 1 LOP3 per node per 32 patterns (u32 word) is the algorithmic work;
+             peak = 148 SMs x 64 LOP3/clk/SM x SM clock
+cpu_baseline / --impl reference = the oracle (oracle/, plain single-threaded C) timed on a bounded
+             sample of the same workload on this host.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "AIG node-pattern evals/s"
+UNIT = "node-patterns/s"
+LOP3_PER_CLK_PER_SM = 64  # alu pipe: rt = 2 cycles per warp-instr per SMSP, 4 SMSPs (B300_MICROARCH.md)
+
+
+def make_workload(name: str):
+    from workloads import c1_add8, c2_mul12, c2_mul12_bug, c5_big
+
+    if name == "c5":
+        m = c5_big()
+        desc = ("c5_big2m: 256 disjoint copies (176 random-block sin_10xd-shaped miters of 3 types + 80 "
+                "mul12 array-vs-Wallace miters), 8 seeded single-gate bug copies, 24 PIs per copy")
+        return m, desc, 0  # copy index 0 for the oracle sample
+    if name == "c2":
+        return c2_mul12(), "c2_mul12: 12x12 array vs Wallace multiplier miter", None
+    if name == "c2bug":
+        return c2_mul12_bug(seed=1), "c2_mul12_bug1: C2 with one flipped complement in B's tree", None
+    if name == "c1":
+        return c1_add8(), "c1_add8: 8-bit ripple-carry vs Kogge-Stone adder miter", None
+    raise SystemExit(f"unknown config {name}")
+
+
+def sample_pairs(m, copy_idx):
+    """Pairs of one copy (C5) or all pairs."""
+    import numpy as np
+
+    if copy_idx is None or "pairs_per_copy" not in m.meta:
+        return m.lit_a, m.lit_b, "all pairs"
+    off = int(np.sum(m.meta["pairs_per_copy"][:copy_idx]))
+    n = m.meta["pairs_per_copy"][copy_idx]
+    return m.lit_a[off:off + n], m.lit_b[off:off + n], f"the {n} PO pairs of copy {copy_idx}"
+
+
+def oracle_sample(m, copy_idx, log2_patterns):
+    """Time the oracle (as it stands) on patterns [0, 2^log2_patterns) of one copy's pair group."""
+    import oracle
+
+    la, lb, what = sample_pairs(m, copy_idx)
+    orc = oracle.Oracle.from_aig(m.aig)
+    t = time.perf_counter()
+    _, _, _, evals = orc.check_pairs(la, lb, k_max=32, lo=0, hi=1 << log2_patterns)
+    dt = time.perf_counter() - t
+    return evals, dt, f"{what}, patterns [0, 2^{log2_patterns}) of its 2^24-pattern window, single thread"
+
+
+class ClockSampler:
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu: int):
+        self.gpu = gpu
+        self.proc = None
+        self.path = None
+
+    def __enter__(self):
+        fd, self.path = tempfile.mkstemp(suffix=".csv")
+        os.close(fd)
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.FIELDS}",
+                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                         stdout=open(self.path, "w"), stderr=subprocess.DEVNULL)
+        except OSError:
+            self.proc = None
+        return self
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except subprocess.TimeoutExpired:
+                self.proc.kill()
+
+    def summary(self):
+        if not self.path or not os.path.exists(self.path):
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        rows = []
+        for line in open(self.path):
+            f = [x.strip() for x in line.split(",")]
+            if len(f) >= 9 and f[1].replace(".", "").isdigit():
+                rows.append(f)
+        os.unlink(self.path)
+        if not rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["no samples"]}
+        sm = [float(r[1]) for r in rows]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in rows for i in range(4) if r[5 + i].lower() == "active"})
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": float(rows[0][2]), "reasons": reasons,
+                "samples": len(rows), "power_w_max": max(float(r[3]) for r in rows if r[3].replace(".", "").isdigit())}
+
+
+def run_reference(args):
+    """--impl reference: the oracle as it stands, on rank 0's host cores, bounded sample per step."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    import oracle
+
+    oracle.build()
+    m, desc, copy_idx = make_workload(args.config)
+    log2p = args.ref_log2_patterns
+    for _ in range(args.warmup):
+        oracle_sample(m, copy_idx, log2p)
+    evals = 0
+    secs = 0.0
+    for _ in range(args.steps):
+        e, dt, what = oracle_sample(m, copy_idx, log2p)
+        evals += e
+        secs += dt
+    v = evals / secs
+    line = {
+        "impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * secs / args.steps,
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u8",
+        "data": "synthetic",
+        "config": {"workload": args.config, "description": desc, "sample": what},
+        "cpu_baseline": {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": what},
+        "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="c5")
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--engine", type=int, default=0)
+    ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--cpu-log2-patterns", type=int, default=19)
+    ap.add_argument("--ref-log2-patterns", type=int, default=17)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3
+    if args.impl == "reference":
+        return run_reference(args)
+
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_dac_liuy25_b200 import capi
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    stream = torch.cuda.current_stream()
+
+    m, desc, copy_idx = make_workload(args.config)
+    uid = None
+    if world > 1:
+        obj = [capi.cec_nccl_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0)
+        uid = obj[0]
+    t_load = time.perf_counter()
+    ctx = capi.Context.from_aig(m.aig, device=local, rank=rank, world=world, stream=stream.cuda_stream,
+                                engine=args.engine, nccl_unique_id=uid)
+    load_ms = 1e3 * (time.perf_counter() - t_load)
+    plan = capi.cec_plan_exhaustive(ctx.handle, m.lit_a, m.lit_b)
+    info = capi.cec_plan_info(plan)
+    st0 = ctx.stats()
+
+    for _ in range(args.warmup):
+        capi.cec_plan_run(ctx.handle, plan)
+    torch.cuda.synchronize()
+    v, cex, k = capi.cec_plan_results(ctx.handle, plan, m.num_pairs)
+    verdicts = {"EQ": int((v == capi.CEC_EQUIVALENT).sum()), "NEQ": int((v == capi.CEC_NOT_EQUIVALENT).sum()),
+                "UND": int((v == capi.CEC_UNDECIDED).sum())}
+    stats = ctx.stats()
+    W_rank, W_all = stats["node_patterns"], stats["node_patterns_all"]
+    launches_per_step = stats["num_launches"]
+
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
+    starts = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    ends = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    with ClockSampler(local) as clk:
+        t0 = time.perf_counter()
+        for i in range(args.steps):
+            flush.zero_()  # L2 flush between timed steps (outside the events)
+            starts[i].record(stream)
+            capi.cec_plan_run(ctx.handle, plan)
+            ends[i].record(stream)
+        torch.cuda.synchronize()
+        wall = time.perf_counter() - t0
+    if world > 1:
+        dist.barrier()
+    step_ms = [s.elapsed_time(e) for s, e in zip(starts, ends)]
+    ms = sum(step_ms) / len(step_ms)
+    if world > 1:
+        t = torch.tensor([ms], device="cuda", dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+    value = W_all / (ms / 1e3)
+
+    # e2e: the public blocking call with host arrays (plan + H2D + kernels + reduce + D2H)
+    e2e_ms = []
+    la_h, lb_h = np.ascontiguousarray(m.lit_a), np.ascontiguousarray(m.lit_b)
+    for _ in range(max(1, args.e2e_steps)):
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        t = time.perf_counter()
+        ve, ce, ke = ctx.sim_exhaustive(la_h, lb_h)
+        e2e_ms.append(1e3 * (time.perf_counter() - t))
+        assert np.array_equal(ve, v) and np.array_equal(ce, cex)
+    st_e2e = ctx.stats()
+    e2e = statistics.median(e2e_ms)
+    if world > 1:
+        t = torch.tensor([e2e], device="cuda", dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        e2e = float(t.item())
+
+    clocks = clk.summary()
+    sm_clock = clocks.get("sm_max_mhz") or 1965.0
+    props = torch.cuda.get_device_properties(local)
+    peak = props.multi_processor_count * LOP3_PER_CLK_PER_SM * sm_clock * 1e6 / 1e12  # TLOP3/s
+    achieved = (W_rank / 32.0) / (ms / 1e3) / 1e12
+    traffic = None
+    prof = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    if os.path.exists(prof):
+        try:
+            traffic = json.load(open(prof)).get(args.config, {}).get("dram_bytes_per_launch")
+        except Exception:
+            traffic = None
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        import oracle
+
+        oracle.build()
+        evals, dt, what = oracle_sample(m, copy_idx, args.cpu_log2_patterns)
+        cpu = {"value": evals / dt, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": what,
+               "seconds": round(dt, 2)}
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+            "config": {"workload": args.config, "description": desc, "ands": int(m.aig.num_ands),
+                       "pairs": int(m.num_pairs), "windows": info["num_windows"], "max_k": info["max_k"],
+                       "max_slots": info["max_slots"], "node_patterns_per_step": W_all,
+                       "parallelism": f"pattern-space shards x{world}" + (" + NCCL min all-reduce" if world > 1 else ""),
+                       "l2": "flushed between timed steps (256 MiB write, outside the events)",
+                       "engine": "interp", "verdicts": verdicts},
+            "clocks": clocks,
+            "gpu_launches": int(launches_per_step * args.steps),
+            "e2e": {"value": W_all / (e2e / 1e3), "unit": UNIT, "ms_per_miter": e2e,
+                    "h2d_bytes_per_step": int(st_e2e["h2d_bytes"]), "d2h_bytes_per_step": int(st_e2e["d2h_bytes"]),
+                    "host_prep_ms": st_e2e["host_prep_ms"], "aig_load_ms": load_ms},
+            "roofline": {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "TLOP3/s",
+                         "frac": achieved / peak, "traffic": traffic,
+                         "peak_basis": f"{props.multi_processor_count} SMs x {LOP3_PER_CLK_PER_SM} LOP3/clk x {sm_clock:.0f} MHz (guide unit counts, max SM clock)"},
+            "step_ms": step_ms, "wall_s": wall,
+        }
+        if cpu:
+            line["cpu_baseline"] = cpu
+        print(json.dumps(line), flush=True)
+    capi.cec_plan_free(plan)
+    ctx.close()
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

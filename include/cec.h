@@ -1,0 +1,192 @@
+/*
+ * cec.h — C ABI of the B200 exhaustive-simulation CEC hot path (libcec.so).
+ *
+ * The boundary follows the paper's problem statement: given a combinational And-Inverter Graph
+ * holding two circuits with shared PIs (a miter, §II-B) and candidate node pairs,
+ * decide for each pair equivalent / not equivalent with a counter-example (§III-A,
+ * footnote 1 at :69) / undecided (§III-D); and, for pairs whose support is too large,
+ * check their local functions on a common cut (§III-C1).
+ *
+ * Conventions used by every call
+ *  - Node ids: 0 = constant 0; 1..num_pis = PIs in input order; num_pis+1 .. num_pis+num_ands =
+ *    AND nodes. Every AND's fanin ids are smaller than its own id (AIGER-binary order), so the id
+ *    order is a topological order.
+ *  - A literal is 2*id + complement ("signals can be optionally inverted").
+ *  - Pattern index / truth-table convention (§II-A): for a window with inputs
+ *    S[0] < S[1] < ... < S[k-1] (increasing node id), pattern i assigns input S[j]
+ *    the value of bit j of i. CEX indices are given in the PAIR'S OWN support order with every
+ *    non-support PI = 0, and are the MINIMUM mismatching index (canonical CEX).
+ *  - Ownership: the caller owns every array passed in and every output array; the library copies
+ *    what it keeps. A context owns its device buffers and plans. A context is not thread-safe.
+ *  - Errors: every call returns cec_status; no C++ exception crosses the ABI. On error,
+ *    cec_last_error(ctx) returns a NUL-terminated message (valid until the next call on ctx).
+ *  - No CPU fallback: simulation entry points need a CUDA device and return CEC_E_CUDA without
+ *    one. A context created with opts.device = -1 is "host only": it can load, validate and plan
+ *    (cec_pair_support, cec_plan_*_info) but every simulation call returns CEC_E_CUDA.
+ */
+#ifndef CEC_H
+#define CEC_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define CEC_ABI_VERSION 1
+#define CEC_NO_CEX UINT64_MAX
+
+typedef struct cec_ctx cec_ctx;
+typedef struct cec_plan cec_plan;
+
+typedef enum {
+    CEC_OK = 0,
+    CEC_E_ARG = 1,    /* bad argument (NULL pointer, literal out of range, k_max > 63, ...) */
+    CEC_E_AIG = 2,    /* malformed AIG: fanin id >= own id, literal out of range */
+    CEC_E_CUT = 3,    /* a local-check leaf set is not a cut of its roots */
+    CEC_E_NOMEM = 4,  /* host or device allocation failed, or a window exceeds on-chip capacity */
+    CEC_E_CUDA = 5,   /* CUDA error, or no CUDA device (host-only context) */
+    CEC_E_NCCL = 6,   /* NCCL error in the cross-GPU reduction */
+    CEC_E_NOCEX = 7,  /* cec_get_cex on a pair that was not NOT_EQUIVALENT */
+    CEC_E_STATE = 8   /* call order violated (e.g. cec_get_cex before any cec_sim_exhaustive) */
+} cec_status;
+
+typedef enum {
+    CEC_BAD_CUT = -1,          /* local check only: the leaves are not a cut of the pair */
+    CEC_UNDECIDED = 0,         /* support above k_max (global) or local functions differ (local) */
+    CEC_EQUIVALENT = 1,
+    CEC_NOT_EQUIVALENT = 2     /* global check only: a counter-example exists */
+} cec_verdict;
+
+typedef enum {
+    CEC_MERGE_OFF = 0,
+    CEC_MERGE_PAPER = 1, /* lexicographic sort + greedy consecutive merge, union <= k_s */
+    CEC_MERGE_COST = 2   /* same sort and greedy pass, but a merge is taken only if it does not
+                            increase the estimated work (nodes x 2^k); results are identical (Q8) */
+} cec_merge_policy;
+
+typedef enum {
+    CEC_ENGINE_AUTO = 0,
+    CEC_ENGINE_INTERP = 1, /* schedule interpreter: values in shared memory slots */
+    CEC_ENGINE_JIT = 2     /* per-window-structure register-resident kernel compiled with NVRTC */
+} cec_engine;
+
+typedef struct {
+    uint32_t num_pis;
+    uint32_t num_ands;
+    uint32_t num_pos;
+    const uint32_t *fanin_lits; /* [2*num_ands]: AND i (id num_pis+1+i) = (lit[2i], lit[2i+1]) */
+    const uint32_t *po_lits;    /* [num_pos] (informational; pairs are passed explicitly) */
+} cec_aig;
+
+typedef struct {
+    int32_t device;            /* CUDA device ordinal; -1 = host-only context (no simulation) */
+    int32_t rank, world;       /* world > 1: SPMD over `world` GPUs; every rank passes the same
+                                  AIG, pairs and options; results are identical on every rank */
+    const void *nccl_unique_id;/* 128-byte ncclUniqueId (required when world > 1); the caller
+                                  bootstraps it, e.g. through torch.distributed */
+    void *stream;              /* cudaStream_t to launch on, or NULL for the library's own stream */
+    uint32_t k_max;            /* exhaustive support limit, <= 63. Default 32 (= k_P) */
+    uint32_t k_s;              /* window-merge threshold; 0 = k_max */
+    int32_t merge;             /* cec_merge_policy; default CEC_MERGE_PAPER */
+    int32_t engine;            /* cec_engine; default CEC_ENGINE_AUTO */
+    uint64_t reserved[6];      /* must be zero */
+} cec_opts;
+
+typedef struct {
+    uint64_t node_patterns;    /* W: sum over simulated windows of (#AND nodes) x (#patterns
+                                  simulated by this rank), after merging */
+    uint64_t node_patterns_all;/* same, all ranks together */
+    uint32_t num_windows;      /* windows after merging */
+    uint32_t max_k;            /* largest window input count */
+    uint32_t max_slots;        /* largest on-chip live set (interpreter slots) */
+    uint32_t num_launches;     /* kernel launches of the last run */
+    float kernel_ms;           /* device time of the last run (first launch .. reduction done) */
+    float host_prep_ms;        /* host planning time of the last plan */
+    uint64_t h2d_bytes;        /* bytes copied host->device by the last plan (schedules, items) */
+    uint64_t d2h_bytes;        /* bytes copied device->host by the last results read-back */
+} cec_stats;
+
+/* Fill *opts with the defaults above. */
+void cec_default_opts(cec_opts *opts);
+
+/* Create a context: copy and validate the AIG (CEC_E_AIG if any fanin id >= own id or a literal
+ * is out of range), select the device, and when opts->world > 1 create the NCCL communicator
+ * (collective: every rank must call it). *ctx is set only on CEC_OK. */
+cec_status cec_load_aig(cec_ctx **ctx, const cec_aig *aig, const cec_opts *opts);
+
+/* Global exhaustive check of num_pairs literal pairs (Alg. 1 :89-108).
+ * For a pair with k = |supp(a) U supp(b)| <= k_max the verdict is exact: EQUIVALENT, or
+ * NOT_EQUIVALENT with cex_index_out = the minimum mismatching pattern in the pair's own support
+ * order. k > k_max gives UNDECIDED and CEC_NO_CEX (the caller may fall back to local cuts).
+ * lit_a == lit_b -> EQUIVALENT; lit_a == lit_b ^ 1 -> NOT_EQUIVALENT at index 0.
+ * verdict_out / cex_index_out / k_out are caller-owned host arrays of num_pairs (cex_index_out and
+ * k_out may be NULL). Blocking: returns after the kernels, the cross-GPU reduction and the copy
+ * back. Windows are merged per opts->merge. */
+cec_status cec_sim_exhaustive(cec_ctx *ctx, uint32_t num_pairs, const uint32_t *lit_a, const uint32_t *lit_b,
+                              int32_t *verdict_out, uint64_t *cex_index_out, uint32_t *k_out);
+
+/* Local function checks (§III-C1). Check q compares lit_a[q] and lit_b[q] as
+ * functions of the leaves cut_leaves[cut_off[q] .. cut_off[q+1]) (node ids, any order, taken in
+ * increasing id; at most k_max and at most 24 leaves). verdict_out[q] = EQUIVALENT if the two local
+ * functions are identical; UNDECIDED if they differ (the difference may be an SDC, so
+ * no CEX is produced); CEC_BAD_CUT if the backward traversal from a root reaches a PI that is not a
+ * leaf, in which case the call returns CEC_E_CUT after filling every other verdict. */
+cec_status cec_check_local_cuts(cec_ctx *ctx, uint32_t num_checks, const uint32_t *lit_a, const uint32_t *lit_b,
+                                const uint32_t *cut_off, const uint32_t *cut_leaves, int32_t *verdict_out);
+
+/* Counter-example of pair `pair_idx` of the most recent cec_sim_exhaustive / cec_plan_results:
+ * pi_values_out[i] = value of PI id i+1 (0/1): PI S[j] = bit j of the CEX index, every other PI 0.
+ * CEC_E_NOCEX unless that pair was NOT_EQUIVALENT; CEC_E_STATE before any global check. */
+cec_status cec_get_cex(cec_ctx *ctx, uint32_t pair_idx, uint8_t *pi_values_out);
+
+/* Structural support of {var(lit_a), var(lit_b)}: writes min(k, cap) PI ids in
+ * increasing order to support_out (may be NULL when cap = 0) and returns k via *k_out. */
+cec_status cec_pair_support(cec_ctx *ctx, uint32_t lit_a, uint32_t lit_b, uint32_t *support_out, uint32_t cap,
+                            uint32_t *k_out);
+
+/* ---- Plans: split cec_sim_exhaustive into host planning, device run and result read-back, so a
+ * caller can time the device part with the inputs already resident in HBM. ------------------------ */
+
+/* Host planning for a global check: supports, windows, merging, schedules; uploads the schedules.
+ * A host-only context plans without uploading. */
+cec_status cec_plan_exhaustive(cec_ctx *ctx, uint32_t num_pairs, const uint32_t *lit_a, const uint32_t *lit_b,
+                               cec_plan **plan);
+/* Launch the plan's kernels (and the cross-GPU reduction) on the context stream; asynchronous. */
+cec_status cec_plan_run(cec_ctx *ctx, cec_plan *plan);
+/* Wait for the plan, copy the results back and decode them exactly as cec_sim_exhaustive does. */
+cec_status cec_plan_results(cec_ctx *ctx, cec_plan *plan, int32_t *verdict_out, uint64_t *cex_index_out,
+                            uint32_t *k_out);
+/* Plan shape: windows after merging, W for one full run, largest k and live set. */
+cec_status cec_plan_info(const cec_plan *plan, uint32_t *num_windows, uint64_t *node_patterns, uint32_t *max_k,
+                         uint32_t *max_slots);
+/* Per-window description, for tests of the host logic: window w's inputs (node ids, increasing),
+ * its AND-node count and its pair indices. Arrays may be NULL to query sizes only. */
+cec_status cec_plan_window(const cec_plan *plan, uint32_t w, uint32_t *inputs, uint32_t *k, uint32_t *num_nodes,
+                           uint32_t *pairs, uint32_t *num_pairs);
+void cec_plan_free(cec_plan *plan);
+
+/* The CUDA stream the context launches on (cudaStream_t). */
+void *cec_stream(cec_ctx *ctx);
+/* Statistics of the last run on this context. */
+cec_status cec_get_stats(cec_ctx *ctx, cec_stats *stats);
+
+/* Create a 128-byte ncclUniqueId (rank 0 calls it and shares the bytes with the other ranks, e.g.
+ * through torch.distributed) using the NCCL library libcec loads on demand. CEC_E_NCCL if NCCL is
+ * unavailable. */
+cec_status cec_nccl_unique_id(void *out128);
+
+/* Host utility exported for tests: the contiguous slice range [*begin, *end) of `n` slices that
+ * rank `rank` of `world` simulates (pattern-space sharding). */
+void cec_shard_range(uint64_t n, int32_t rank, int32_t world, uint64_t *begin, uint64_t *end);
+/* Host utility exported for tests: parallel bit extract (idx_own = pext(idx_merged, ownmask)). */
+uint64_t cec_pext64(uint64_t value, uint64_t mask);
+
+void cec_free(cec_ctx *ctx);
+const char *cec_last_error(const cec_ctx *ctx);
+int cec_abi_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* CEC_H */

@@ -1,0 +1,296 @@
+"""Thin ctypes binding of include/cec.h (argument marshalling only; every step of the hot path runs
+in libcec.so's sm_100a kernels and its C++ host driver). Function names match the C ABI.
+
+There is no fallback: if libcec.so is missing this module raises ImportError, and on a machine
+without a CUDA device every simulation call raises CecError(CEC_E_CUDA).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from typing import Optional, Sequence, Tuple
+
+import numpy as np
+
+HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(HERE, "libcec.so")
+
+CEC_OK, CEC_E_ARG, CEC_E_AIG, CEC_E_CUT, CEC_E_NOMEM, CEC_E_CUDA, CEC_E_NCCL, CEC_E_NOCEX, CEC_E_STATE = range(9)
+CEC_BAD_CUT, CEC_UNDECIDED, CEC_EQUIVALENT, CEC_NOT_EQUIVALENT = -1, 0, 1, 2
+CEC_MERGE_OFF, CEC_MERGE_PAPER, CEC_MERGE_COST = 0, 1, 2
+CEC_ENGINE_AUTO, CEC_ENGINE_INTERP, CEC_ENGINE_JIT = 0, 1, 2
+CEC_NO_CEX = (1 << 64) - 1
+STATUS_NAMES = ["CEC_OK", "CEC_E_ARG", "CEC_E_AIG", "CEC_E_CUT", "CEC_E_NOMEM", "CEC_E_CUDA", "CEC_E_NCCL",
+                "CEC_E_NOCEX", "CEC_E_STATE"]
+
+# every symbol include/cec.h declares (tests check the library exports all of them)
+EXPORTS = ["cec_default_opts", "cec_load_aig", "cec_sim_exhaustive", "cec_check_local_cuts", "cec_get_cex",
+           "cec_pair_support", "cec_plan_exhaustive", "cec_plan_run", "cec_plan_results", "cec_plan_info",
+           "cec_plan_window", "cec_plan_free", "cec_stream", "cec_get_stats", "cec_shard_range", "cec_pext64",
+           "cec_free", "cec_last_error", "cec_abi_version", "cec_nccl_unique_id"]
+
+
+class CecOpts(ctypes.Structure):
+    _fields_ = [("device", ctypes.c_int32), ("rank", ctypes.c_int32), ("world", ctypes.c_int32),
+                ("nccl_unique_id", ctypes.c_void_p), ("stream", ctypes.c_void_p), ("k_max", ctypes.c_uint32),
+                ("k_s", ctypes.c_uint32), ("merge", ctypes.c_int32), ("engine", ctypes.c_int32),
+                ("reserved", ctypes.c_uint64 * 6)]
+
+
+class CecAig(ctypes.Structure):
+    _fields_ = [("num_pis", ctypes.c_uint32), ("num_ands", ctypes.c_uint32), ("num_pos", ctypes.c_uint32),
+                ("fanin_lits", ctypes.c_void_p), ("po_lits", ctypes.c_void_p)]
+
+
+class CecStats(ctypes.Structure):
+    _fields_ = [("node_patterns", ctypes.c_uint64), ("node_patterns_all", ctypes.c_uint64),
+                ("num_windows", ctypes.c_uint32), ("max_k", ctypes.c_uint32), ("max_slots", ctypes.c_uint32),
+                ("num_launches", ctypes.c_uint32), ("kernel_ms", ctypes.c_float), ("host_prep_ms", ctypes.c_float),
+                ("h2d_bytes", ctypes.c_uint64), ("d2h_bytes", ctypes.c_uint64)]
+
+    def as_dict(self):
+        return {f: getattr(self, f) for f, _ in self._fields_}
+
+
+class CecError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        self.status = status
+        super().__init__(f"{STATUS_NAMES[status] if 0 <= status < len(STATUS_NAMES) else status}: {msg}")
+
+
+def _load() -> ctypes.CDLL:
+    if not os.path.exists(LIB_PATH):
+        raise ImportError(f"{LIB_PATH} is missing: run `python -c 'import __graft_entry__ as g; g.build()'` "
+                          "(there is no CPU fallback)")
+    L = ctypes.CDLL(LIB_PATH)
+    P, u32, u64, i32 = ctypes.c_void_p, ctypes.c_uint32, ctypes.c_uint64, ctypes.c_int32
+    sig = {
+        "cec_default_opts": (None, [P]),
+        "cec_load_aig": (ctypes.c_int, [P, P, P]),
+        "cec_sim_exhaustive": (ctypes.c_int, [P, u32, P, P, P, P, P]),
+        "cec_check_local_cuts": (ctypes.c_int, [P, u32, P, P, P, P, P]),
+        "cec_get_cex": (ctypes.c_int, [P, u32, P]),
+        "cec_pair_support": (ctypes.c_int, [P, u32, u32, P, u32, P]),
+        "cec_plan_exhaustive": (ctypes.c_int, [P, u32, P, P, P]),
+        "cec_plan_run": (ctypes.c_int, [P, P]),
+        "cec_plan_results": (ctypes.c_int, [P, P, P, P, P]),
+        "cec_plan_info": (ctypes.c_int, [P, P, P, P, P]),
+        "cec_plan_window": (ctypes.c_int, [P, u32, P, P, P, P, P]),
+        "cec_plan_free": (None, [P]),
+        "cec_stream": (P, [P]),
+        "cec_get_stats": (ctypes.c_int, [P, P]),
+        "cec_shard_range": (None, [u64, i32, i32, P, P]),
+        "cec_pext64": (u64, [u64, u64]),
+        "cec_free": (None, [P]),
+        "cec_last_error": (ctypes.c_char_p, [P]),
+        "cec_abi_version": (ctypes.c_int, []),
+        "cec_nccl_unique_id": (ctypes.c_int, [P]),
+    }
+    for name, (res, args) in sig.items():
+        fn = getattr(L, name)
+        fn.restype = res
+        fn.argtypes = args
+    return L
+
+
+lib = _load()
+
+
+def _p(a: Optional[np.ndarray]):
+    return None if a is None else a.ctypes.data_as(ctypes.c_void_p)
+
+
+def _u32(x) -> np.ndarray:
+    return np.ascontiguousarray(np.asarray(x, dtype=np.uint32).reshape(-1))
+
+
+def cec_default_opts(**kw) -> CecOpts:
+    o = CecOpts()
+    lib.cec_default_opts(ctypes.byref(o))
+    for k, v in kw.items():
+        setattr(o, k, v)
+    return o
+
+
+def cec_last_error(ctx) -> str:
+    s = lib.cec_last_error(ctx)
+    return s.decode() if s else ""
+
+
+def _check(st: int, ctx=None):
+    if st != CEC_OK:
+        raise CecError(st, cec_last_error(ctx))
+
+
+def cec_load_aig(num_pis: int, fanins: np.ndarray, pos: np.ndarray, opts: Optional[CecOpts] = None,
+                 nccl_unique_id: Optional[bytes] = None):
+    fan = _u32(fanins)
+    po = _u32(pos)
+    aig = CecAig(num_pis, fan.size // 2, po.size, fan.ctypes.data if fan.size else None,
+                 po.ctypes.data if po.size else None)
+    opts = opts if opts is not None else cec_default_opts()
+    keep = None
+    if nccl_unique_id is not None:
+        keep = ctypes.create_string_buffer(bytes(nccl_unique_id), 128)
+        opts.nccl_unique_id = ctypes.cast(keep, ctypes.c_void_p)
+    ctx = ctypes.c_void_p()
+    st = lib.cec_load_aig(ctypes.byref(ctx), ctypes.byref(aig), ctypes.byref(opts))
+    _check(st, None)
+    return ctx
+
+
+def cec_free(ctx) -> None:
+    lib.cec_free(ctx)
+
+
+def cec_sim_exhaustive(ctx, lit_a, lit_b) -> Tuple[np.ndarray, np.ndarray, np.ndarray]:
+    la, lb = _u32(lit_a), _u32(lit_b)
+    n = la.size
+    v = np.zeros(max(n, 1), np.int32)
+    cex = np.zeros(max(n, 1), np.uint64)
+    k = np.zeros(max(n, 1), np.uint32)
+    _check(lib.cec_sim_exhaustive(ctx, n, _p(la), _p(lb), _p(v), _p(cex), _p(k)), ctx)
+    return v[:n], cex[:n], k[:n]
+
+
+def cec_check_local_cuts(ctx, lit_a, lit_b, cut_off, cut_leaves, raise_on_bad_cut: bool = False) -> np.ndarray:
+    la, lb, off = _u32(lit_a), _u32(lit_b), _u32(cut_off)
+    lv = _u32(cut_leaves) if len(cut_leaves) else np.zeros(1, np.uint32)
+    n = la.size
+    v = np.zeros(max(n, 1), np.int32)
+    st = lib.cec_check_local_cuts(ctx, n, _p(la), _p(lb), _p(off), _p(lv), _p(v))
+    if st == CEC_E_CUT and not raise_on_bad_cut:
+        return v[:n]
+    _check(st, ctx)
+    return v[:n]
+
+
+def cec_get_cex(ctx, pair_idx: int, num_pis: int) -> np.ndarray:
+    out = np.zeros(max(num_pis, 1), np.uint8)
+    _check(lib.cec_get_cex(ctx, pair_idx, _p(out)), ctx)
+    return out[:num_pis]
+
+
+def cec_pair_support(ctx, lit_a: int, lit_b: int) -> list:
+    """Full structural support (sorted PI ids) of {var(lit_a), var(lit_b)}."""
+    k = cec_pair_k(ctx, lit_a, lit_b)
+    buf = np.zeros(max(k, 1), np.uint32)
+    kk = ctypes.c_uint32()
+    _check(lib.cec_pair_support(ctx, lit_a, lit_b, _p(buf), k, ctypes.byref(kk)), ctx)
+    return [int(x) for x in buf[:k]]
+
+
+def cec_pair_k(ctx, lit_a: int, lit_b: int) -> int:
+    k = ctypes.c_uint32()
+    _check(lib.cec_pair_support(ctx, lit_a, lit_b, None, 0, ctypes.byref(k)), ctx)
+    return int(k.value)
+
+
+def cec_plan_exhaustive(ctx, lit_a, lit_b):
+    la, lb = _u32(lit_a), _u32(lit_b)
+    plan = ctypes.c_void_p()
+    _check(lib.cec_plan_exhaustive(ctx, la.size, _p(la), _p(lb), ctypes.byref(plan)), ctx)
+    return plan
+
+
+def cec_plan_run(ctx, plan) -> None:
+    _check(lib.cec_plan_run(ctx, plan), ctx)
+
+
+def cec_plan_results(ctx, plan, num_pairs: int):
+    v = np.zeros(max(num_pairs, 1), np.int32)
+    cex = np.zeros(max(num_pairs, 1), np.uint64)
+    k = np.zeros(max(num_pairs, 1), np.uint32)
+    _check(lib.cec_plan_results(ctx, plan, _p(v), _p(cex), _p(k)), ctx)
+    return v[:num_pairs], cex[:num_pairs], k[:num_pairs]
+
+
+def cec_plan_info(plan) -> dict:
+    nw, W, mk, ms = ctypes.c_uint32(), ctypes.c_uint64(), ctypes.c_uint32(), ctypes.c_uint32()
+    _check(lib.cec_plan_info(plan, ctypes.byref(nw), ctypes.byref(W), ctypes.byref(mk), ctypes.byref(ms)))
+    return {"num_windows": nw.value, "node_patterns": W.value, "max_k": mk.value, "max_slots": ms.value}
+
+
+def cec_plan_window(plan, w: int) -> dict:
+    k, nn, np_ = ctypes.c_uint32(), ctypes.c_uint32(), ctypes.c_uint32()
+    _check(lib.cec_plan_window(plan, w, None, ctypes.byref(k), ctypes.byref(nn), None, ctypes.byref(np_)))
+    ins = np.zeros(max(k.value, 1), np.uint32)
+    pairs = np.zeros(max(np_.value, 1), np.uint32)
+    _check(lib.cec_plan_window(plan, w, _p(ins), None, None, _p(pairs), None))
+    return {"inputs": [int(x) for x in ins[:k.value]], "num_nodes": nn.value,
+            "pairs": [int(x) for x in pairs[:np_.value]]}
+
+
+def cec_plan_free(plan) -> None:
+    lib.cec_plan_free(plan)
+
+
+def cec_stream(ctx) -> int:
+    return lib.cec_stream(ctx) or 0
+
+
+def cec_get_stats(ctx) -> dict:
+    s = CecStats()
+    _check(lib.cec_get_stats(ctx, ctypes.byref(s)), ctx)
+    return s.as_dict()
+
+
+def cec_shard_range(n: int, rank: int, world: int) -> Tuple[int, int]:
+    b, e = ctypes.c_uint64(), ctypes.c_uint64()
+    lib.cec_shard_range(n, rank, world, ctypes.byref(b), ctypes.byref(e))
+    return b.value, e.value
+
+
+def cec_pext64(value: int, mask: int) -> int:
+    return int(lib.cec_pext64(value, mask))
+
+
+def cec_nccl_unique_id() -> bytes:
+    buf = ctypes.create_string_buffer(128)
+    _check(lib.cec_nccl_unique_id(buf), None)
+    return buf.raw
+
+
+def cec_abi_version() -> int:
+    return int(lib.cec_abi_version())
+
+
+class Context:
+    """RAII wrapper around a cec_ctx for one AIG."""
+
+    def __init__(self, num_pis: int, fanins: np.ndarray, pos: np.ndarray, **opt):
+        uid = opt.pop("nccl_unique_id", None)
+        self.opts = cec_default_opts(**opt)
+        self.num_pis = num_pis
+        self._ctx = cec_load_aig(num_pis, fanins, pos, self.opts, nccl_unique_id=uid)
+
+    @classmethod
+    def from_aig(cls, aig, **opt) -> "Context":
+        return cls(aig.num_pis, aig.fanins, aig.pos, **opt)
+
+    @property
+    def handle(self):
+        return self._ctx
+
+    def sim_exhaustive(self, lit_a, lit_b):
+        return cec_sim_exhaustive(self._ctx, lit_a, lit_b)
+
+    def check_local_cuts(self, lit_a, lit_b, cut_off, leaves):
+        return cec_check_local_cuts(self._ctx, lit_a, lit_b, cut_off, leaves)
+
+    def get_cex(self, pair_idx: int) -> np.ndarray:
+        return cec_get_cex(self._ctx, pair_idx, self.num_pis)
+
+    def pair_k(self, lit_a: int, lit_b: int) -> int:
+        return cec_pair_k(self._ctx, lit_a, lit_b)
+
+    def stats(self) -> dict:
+        return cec_get_stats(self._ctx)
+
+    def close(self):
+        if getattr(self, "_ctx", None):
+            cec_free(self._ctx)
+            self._ctx = None
+
+    def __del__(self):
+        self.close()

@@ -1,0 +1,71 @@
+// cec_internal.hpp — structures shared by the host driver (cec_host.cpp) and the sm_100a kernels
+// (sim_interp.cu). Not part of the ABI; include/cec.h is the boundary.
+#pragma once
+#include <cstdint>
+#include <string>
+#include <vector>
+
+namespace cec {
+
+// ---- Interpreter program encoding (one uint2 per op) ------------------------------------------
+// AND op  (TT(n)[w] = (TT(f0)[w] ^ m0) & (TT(f1)[w] ^ m1), Alg. 1 l.10-11):
+//   x = (slot0 << 1 | c0) | (slot1 << 1 | c1) << 16 ;  y = out_slot
+// CMP op  (XOR-compare of a pair's root words, Alg. 1 l.12-14):
+//   x = (slotA << 1 | cA) | (slotB << 1 | cB) << 16 ;  y = OP_CMP | cmp_index
+// A slot holds one u32 truth-table word per lane of a warp (32 consecutive words per warp pass).
+constexpr uint32_t OP_CMP = 0x80000000u;
+constexpr uint32_t MAX_SLOTS = 32767;   // 15-bit slot field
+constexpr uint32_t MAX_CMPS = 0x7FFFFFFFu;
+
+struct DevWin {            // one simulation window (§III-B1) after merging
+    uint32_t prog_off;     // first op in the program array
+    uint32_t prog_len;     // number of ops (ANDs + CMPs)
+    uint32_t k;            // number of inputs; input j lives in slot j at the start of a pass
+    uint32_t const_slot;   // slot holding constant 0, or 0xFFFFFFFF if unused
+    uint32_t cmp_off;      // this window's compare indices are [cmp_off, cmp_off + ncmp)
+    uint32_t ncmp;
+    uint32_t tt_words_lo;  // truth-table length in u32 words = max(1, 2^(k-5))
+    uint32_t tt_words_hi;
+};
+
+struct Item {              // a contiguous range of 32-word slices of one window
+    uint32_t win;
+    uint32_t s_begin;
+    uint32_t s_end;
+    uint32_t pad;
+};
+
+struct LaunchGroup {       // windows sharing one kernel launch (same shared-memory slot budget)
+    uint32_t nslots;       // slots per warp in this launch
+    uint32_t item_off, nitems;
+};
+
+// Device buffers of one plan.
+struct DevPlan {
+    DevWin *wins = nullptr;
+    uint2 *prog = nullptr;
+    Item *items = nullptr;
+    unsigned long long *first = nullptr;  // [ncmp] minimum mismatching merged pattern index
+    unsigned long long *bound = nullptr;  // [nwin] early-exit bound (all pairs NEQ below it)
+    uint32_t *neq_cnt = nullptr;          // [nwin]
+    uint32_t *item_ctr = nullptr;         // [ngroups]
+};
+
+// sim_interp.cu
+const char *launch_interp(const DevPlan &d, const std::vector<LaunchGroup> &groups, uint32_t nwin, uint32_t ncmp,
+                          void *stream, int num_sms, uint32_t *launches);
+const char *dev_alloc(void **p, size_t bytes);
+const char *dev_free(void *p);
+const char *h2d(void *dst, const void *src, size_t bytes, void *stream);
+const char *d2h(void *dst, const void *src, size_t bytes, void *stream);
+const char *dev_memset(void *dst, int v, size_t bytes, void *stream);
+const char *stream_sync(void *stream);
+const char *dev_init(int device, void **own_stream, int *num_sms);
+const char *stream_destroy(void *stream);
+const char *event_create(void **ev);
+const char *event_record(void *ev, void *stream);
+const char *event_elapsed(float *ms, void *a, void *b);
+void event_destroy(void *ev);
+uint32_t interp_max_slots_per_warp();
+
+}  // namespace cec

@@ -1,0 +1,205 @@
+// sim_interp.cu — sm_100a schedule-interpreter kernel for exhaustive bit-parallel simulation.
+//
+// What it computes (§III-B, Alg. 1 reconstructed in SURVEY.md App. A): for every
+// window, every u32 word w of the 2^k-pattern truth table of every window node, with the input
+// (projection) words generated arithmetically, AND nodes evaluated in topological
+// order, and every candidate pair XOR-compared; the minimum mismatching pattern index per pair is
+// recorded with atomicMin (canonical CEX).
+//
+// B200 design (differs from the paper's Alg. 1):
+//  * no simulation table in HBM: each warp owns a 32-word slice of the pattern space and carries it
+//    through the whole window; node words live in shared-memory slots [slot][lane] allocated by
+//    liveness on the host, so a window's working set is (live nodes) x 128 B per warp;
+//  * levels are program order inside a warp (no grid-wide level barrier, no per-level launch);
+//  * windows and slices are work items pulled by warps from a global counter (dims 2 and 3 of
+//    PAPER.md:114-116 folded into one dynamic queue, largest windows first);
+//  * compare ops are interleaved right after the later root is computed; __ballot_sync finds the
+//    lowest mismatching lane (= lowest word), __ffs the lowest bit; a window whose pairs are all
+//    refuted publishes a bound and later slices above it are skipped (bounded early exit, Q9).
+#include <cuda_runtime.h>
+
+#include <cstdint>
+#include <vector>
+
+#include "cec_internal.hpp"
+
+namespace cec {
+
+namespace {
+
+constexpr uint32_t FULL = 0xFFFFFFFFu;
+constexpr int MAX_WPB = 4;  // warps per block
+constexpr size_t SMEM_PER_SM = 227 * 1024;
+
+__device__ __forceinline__ uint32_t proj_word(uint32_t j, uint64_t w) {
+    // projection truth table of input j at word w: bit b of word w is pattern
+    // i = 32 w + b, and input j takes bit j of i.
+    switch (j) {
+        case 0: return 0xAAAAAAAAu;
+        case 1: return 0xCCCCCCCCu;
+        case 2: return 0xF0F0F0F0u;
+        case 3: return 0xFF00FF00u;
+        case 4: return 0xFFFF0000u;
+        default: return 0u - (uint32_t)((w >> (j - 5)) & 1u);
+    }
+}
+
+__device__ __noinline__ void record_mismatch(uint32_t c, uint64_t idx, uint32_t win, const DevWin &W,
+                                             unsigned long long *first, unsigned long long *bound,
+                                             uint32_t *neq_cnt) {
+    unsigned long long old = atomicMin(&first[c], (unsigned long long)idx);
+    if (old == ~0ull) {
+        __threadfence();
+        uint32_t n = atomicAdd(&neq_cnt[win], 1u) + 1u;
+        if (n == W.ncmp) {  // every pair of the window is refuted: publish an early-exit bound
+            __threadfence();
+            unsigned long long mx = 0;
+            for (uint32_t t = 0; t < W.ncmp; ++t) {
+                unsigned long long v = atomicAdd(&first[W.cmp_off + t], 0ull);
+                mx = v > mx ? v : mx;
+            }
+            atomicMin(&bound[win], mx);
+        }
+    }
+}
+
+__global__ void __launch_bounds__(MAX_WPB * 32)
+interp_kernel(const Item *__restrict__ items, uint32_t nitems, uint32_t *__restrict__ item_ctr,
+              const DevWin *__restrict__ wins, const uint2 *__restrict__ prog, unsigned long long *first,
+              unsigned long long *bound, uint32_t *neq_cnt, uint32_t nslots) {
+    extern __shared__ uint32_t smem[];
+    const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31u;
+    uint32_t *vals = smem + (size_t)warp * (nslots * 32u + 64u);
+    uint2 *ibuf = reinterpret_cast<uint2 *>(vals + nslots * 32u);
+    uint32_t *my = vals + lane;  // this lane's column: slot s at my[s * 32]
+
+    for (;;) {
+        uint32_t it = 0;
+        if (lane == 0) it = atomicAdd(item_ctr, 1u);
+        it = __shfl_sync(FULL, it, 0);
+        if (it >= nitems) break;
+        const Item item = items[it];
+        const DevWin W = wins[item.win];
+        const uint64_t tt_words = ((uint64_t)W.tt_words_hi << 32) | W.tt_words_lo;
+        for (uint32_t s = item.s_begin; s < item.s_end; ++s) {
+            const uint64_t base_idx = (uint64_t)s << 10;  // first pattern of this 32-word slice
+            if (base_idx >= *((volatile unsigned long long *)&bound[item.win])) break;
+            const uint64_t word = ((uint64_t)s << 5) + lane;
+            const bool active = word < tt_words;
+            for (uint32_t j = 0; j < W.k; ++j) my[j * 32u] = proj_word(j, word);
+            if (W.const_slot != 0xFFFFFFFFu) my[W.const_slot * 32u] = 0u;
+            for (uint32_t p = 0; p < W.prog_len; p += 32u) {
+                const uint32_t n = min(32u, W.prog_len - p);
+                __syncwarp();
+                if (lane < n) ibuf[lane] = prog[W.prog_off + p + lane];
+                __syncwarp();
+                for (uint32_t j = 0; j < n; ++j) {
+                    const uint2 ins = ibuf[j];
+                    const uint32_t a = my[(ins.x & 0xFFFEu) << 4] ^ (0u - (ins.x & 1u));
+                    const uint32_t b = my[((ins.x >> 16) & 0xFFFEu) << 4] ^ (0u - ((ins.x >> 16) & 1u));
+                    if (!(ins.y & OP_CMP)) {
+                        my[ins.y << 5] = a & b;
+                    } else {
+                        const uint32_t d = active ? (a ^ b) : 0u;
+                        const uint32_t bal = __ballot_sync(FULL, d != 0u);
+                        if (bal) {
+                            const uint32_t l = (uint32_t)__ffs(bal) - 1u;
+                            const uint32_t dl = __shfl_sync(FULL, d, l);
+                            if (lane == 0) {
+                                const uint64_t idx = ((((uint64_t)s << 5) + l) << 5) + (uint32_t)(__ffs(dl) - 1);
+                                record_mismatch(ins.y & ~OP_CMP, idx, item.win, W, first, bound, neq_cnt);
+                            }
+                        }
+                    }
+                }
+            }
+        }
+    }
+}
+
+inline const char *ck(cudaError_t e) { return e == cudaSuccess ? nullptr : cudaGetErrorString(e); }
+
+}  // namespace
+
+uint32_t interp_max_slots_per_warp() {
+    // one warp per block, whole shared memory: (nslots*32 + 64) * 4 <= 227 KB
+    return (uint32_t)((SMEM_PER_SM / 4 - 64) / 32);
+}
+
+const char *launch_interp(const DevPlan &d, const std::vector<LaunchGroup> &groups, uint32_t nwin, uint32_t ncmp,
+                          void *stream, int num_sms, uint32_t *launches) {
+    cudaStream_t st = (cudaStream_t)stream;
+    const char *e;
+    if ((e = ck(cudaMemsetAsync(d.first, 0xFF, sizeof(unsigned long long) * (ncmp ? ncmp : 1), st)))) return e;
+    if ((e = ck(cudaMemsetAsync(d.bound, 0xFF, sizeof(unsigned long long) * (nwin ? nwin : 1), st)))) return e;
+    if ((e = ck(cudaMemsetAsync(d.neq_cnt, 0, sizeof(uint32_t) * (nwin ? nwin : 1), st)))) return e;
+    if ((e = ck(cudaMemsetAsync(d.item_ctr, 0, sizeof(uint32_t) * (groups.size() ? groups.size() : 1), st)))) return e;
+    uint32_t nl = 0;
+    for (size_t g = 0; g < groups.size(); ++g) {
+        const LaunchGroup &G = groups[g];
+        if (G.nitems == 0) continue;
+        const size_t per_warp = ((size_t)G.nslots * 32 + 64) * 4;
+        int wpb = MAX_WPB;
+        while (wpb > 1 && per_warp * wpb > SMEM_PER_SM) wpb >>= 1;
+        const size_t smem = per_warp * wpb;
+        if (smem > SMEM_PER_SM) return "window live set exceeds shared memory";
+        if ((e = ck(cudaFuncSetAttribute(interp_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem))))
+            return e;
+        int per_sm = 0;
+        if ((e = ck(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, interp_kernel, wpb * 32, smem)))) return e;
+        if (per_sm < 1) per_sm = 1;
+        uint64_t grid = (uint64_t)num_sms * per_sm;
+        const uint64_t need = (G.nitems + wpb - 1) / wpb;
+        if (grid > need) grid = need;
+        interp_kernel<<<(unsigned)grid, wpb * 32, smem, st>>>(d.items + G.item_off, G.nitems, d.item_ctr + g, d.wins,
+                                                              d.prog, d.first, d.bound, d.neq_cnt, G.nslots);
+        if ((e = ck(cudaGetLastError()))) return e;
+        ++nl;
+    }
+    if (launches) *launches = nl;
+    return nullptr;
+}
+
+const char *dev_alloc(void **p, size_t bytes) { return ck(cudaMalloc(p, bytes ? bytes : 16)); }
+const char *dev_free(void *p) { return p ? ck(cudaFree(p)) : nullptr; }
+const char *h2d(void *dst, const void *src, size_t bytes, void *stream) {
+    return bytes ? ck(cudaMemcpyAsync(dst, src, bytes, cudaMemcpyHostToDevice, (cudaStream_t)stream)) : nullptr;
+}
+const char *d2h(void *dst, const void *src, size_t bytes, void *stream) {
+    return bytes ? ck(cudaMemcpyAsync(dst, src, bytes, cudaMemcpyDeviceToHost, (cudaStream_t)stream)) : nullptr;
+}
+const char *dev_memset(void *dst, int v, size_t bytes, void *stream) {
+    return bytes ? ck(cudaMemsetAsync(dst, v, bytes, (cudaStream_t)stream)) : nullptr;
+}
+const char *stream_sync(void *stream) { return ck(cudaStreamSynchronize((cudaStream_t)stream)); }
+const char *dev_init(int device, void **own_stream, int *num_sms) {
+    int n = 0;
+    const char *e;
+    if ((e = ck(cudaGetDeviceCount(&n)))) return e;
+    if (device < 0 || device >= n) return "no such CUDA device";
+    if ((e = ck(cudaSetDevice(device)))) return e;
+    cudaDeviceProp prop;
+    if ((e = ck(cudaGetDeviceProperties(&prop, device)))) return e;
+    if (prop.major != 10) return "libcec is built for sm_100a (B200); this device is not compute capability 10.x";
+    *num_sms = prop.multiProcessorCount;
+    cudaStream_t s;
+    if ((e = ck(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking)))) return e;
+    *own_stream = s;
+    return nullptr;
+}
+const char *stream_destroy(void *stream) { return stream ? ck(cudaStreamDestroy((cudaStream_t)stream)) : nullptr; }
+const char *event_create(void **ev) {
+    cudaEvent_t e;
+    const char *r = ck(cudaEventCreate(&e));
+    *ev = r ? nullptr : e;
+    return r;
+}
+const char *event_record(void *ev, void *stream) { return ck(cudaEventRecord((cudaEvent_t)ev, (cudaStream_t)stream)); }
+const char *event_elapsed(float *ms, void *a, void *b) {
+    return ck(cudaEventElapsedTime(ms, (cudaEvent_t)a, (cudaEvent_t)b));
+}
+void event_destroy(void *ev) {
+    if (ev) cudaEventDestroy((cudaEvent_t)ev);
+}
+
+}  // namespace cec

@@ -1,0 +1,210 @@
+"""GPU parity: the CUDA path (through the C-ABI) against the CPU oracle, element by element on the
+same seeded inputs. Integer/bitwise path => bit-exact: verdicts, k, canonical CEX indices and CEX
+vectors (zero tolerance)."""
+import json
+import os
+
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+import oracle  # noqa: E402
+from oracle import Oracle  # noqa: E402
+from paper_conf_dac_liuy25_b200 import capi  # noqa: E402
+from workloads import Builder, c1_add8, c2_mul12, c2_mul12_bug, c5_big, circuits, tiny_random  # noqa: E402
+
+GOLD = os.path.join(os.path.dirname(__file__), "golden")
+NO = oracle.NO_CEX
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _need_gpu():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+
+
+def gpu_ctx(aig, **kw):
+    return capi.Context.from_aig(aig, **kw)
+
+
+def assert_same(gv, gc, gk, ov, oc, ok, tag=""):
+    assert list(map(int, gk)) == list(map(int, ok)), f"{tag} k differs"
+    assert list(map(int, gv)) == list(map(int, ov)), f"{tag} verdicts differ"
+    gc = [int(c) if int(v) == oracle.NOT_EQUIVALENT else NO for v, c in zip(gv, gc)]
+    oc = [int(c) if int(v) == oracle.NOT_EQUIVALENT else NO for v, c in zip(ov, oc)]
+    assert gc == oc, f"{tag} CEX indices differ"
+
+
+def check_vs_oracle(m, k_max=32, **kw):
+    ctx = gpu_ctx(m.aig, k_max=k_max, **kw)
+    gv, gc, gk = ctx.sim_exhaustive(m.lit_a, m.lit_b)
+    orc = Oracle.from_aig(m.aig)
+    ov, oc, ok, _ = orc.check_pairs(m.lit_a, m.lit_b, k_max=k_max)
+    assert_same(gv, gc, gk, ov, oc, ok, m.name)
+    for p in np.nonzero(gv == capi.CEC_NOT_EQUIVALENT)[0][:64]:
+        vec = ctx.get_cex(int(p))
+        assert np.array_equal(vec, orc.cex_vector(int(m.lit_a[p]), int(m.lit_b[p]), int(oc[p])))
+        assert orc.eval_lit(int(m.lit_a[p]), vec) != orc.eval_lit(int(m.lit_b[p]), vec)
+    return ctx, gv, gc, gk
+
+
+def test_paper_examples_on_gpu():
+    bd = Builder(3, strash=False)
+    x, y, z = bd.pi(0), bd.pi(1), bd.pi(2)
+    n4 = bd.raw_and(x, y ^ 1)
+    n5 = bd.raw_and(n4, z)
+    f = bd.raw_and(n4 ^ 1, n5 ^ 1) ^ 1
+    s4 = bd.raw_and(x ^ 1, y ^ 1)  # SDC example: n1 = !s4
+    s5 = bd.raw_and(y, z)
+    s6 = bd.raw_and(s4 ^ 1, s5)
+    aig = bd.finish([f])
+    ctx = gpu_ctx(aig)
+    v, c, k = ctx.sim_exhaustive([f, f, 0, s6, f], [n4, x, 1, s5, f ^ 1])
+    assert list(v) == [capi.CEC_EQUIVALENT, capi.CEC_NOT_EQUIVALENT, capi.CEC_NOT_EQUIVALENT,
+                       capi.CEC_EQUIVALENT, capi.CEC_NOT_EQUIVALENT]
+    assert int(c[1]) == 3 and int(c[2]) == 0 and list(k[:3]) == [3, 3, 0]
+    lv = ctx.check_local_cuts([s6, s6], [s5, s5], [0, 2, 5], [s4 >> 1, s5 >> 1, 1, 2, 3])
+    assert list(lv) == [capi.CEC_UNDECIDED, capi.CEC_EQUIVALENT]  # PAPER.md:35/:130 SDC; cut = support
+
+
+@pytest.mark.parametrize("seed", range(60))
+def test_fuzz_tiny_random(seed):
+    rng = np.random.default_rng(seed)
+    I = int(rng.integers(1, 13))
+    m = tiny_random(I, int(rng.integers(1, 120)), 24, 7000 + seed)
+    kmax = int(rng.integers(0, 13))
+    merge = int(rng.integers(0, 3))
+    check_vs_oracle(m, k_max=kmax, merge=merge)
+
+
+def test_c1_add8():
+    check_vs_oracle(c1_add8())
+
+
+@pytest.mark.parametrize("n", [6, 8, 10])
+def test_small_multipliers_and_bugs(n):
+    check_vs_oracle(circuits.c2_mul12(n))
+    check_vs_oracle(circuits.c2_mul12_bug(seed=1, n=n))
+    check_vs_oracle(circuits.c2_mul12_bug(seed=3, n=n), merge=capi.CEC_MERGE_OFF)
+
+
+def test_invariance_merge_and_kmax():
+    m = c5_big(copies=6, n_random=4, n_bugs=3, rand_pis=14, rand_ands=700, mul_n=7)
+    ref = None
+    for merge in (capi.CEC_MERGE_OFF, capi.CEC_MERGE_PAPER, capi.CEC_MERGE_COST):
+        for k_max in (32, 40):
+            ctx = gpu_ctx(m.aig, merge=merge, k_max=k_max, k_s=28 if merge else 0)
+            got = ctx.sim_exhaustive(m.lit_a, m.lit_b)
+            if ref is None:
+                ref = got
+                orc = Oracle.from_aig(m.aig)
+                ov, oc, ok, _ = orc.check_pairs(m.lit_a, m.lit_b, k_max=32)
+                assert_same(*got, ov, oc, ok, "c5-mini")
+            else:
+                for a, b in zip(ref, got):
+                    assert np.array_equal(a, b)
+
+
+def test_c5_reduced_vs_oracle():
+    m = c5_big(copies=16, n_random=10, n_bugs=4, rand_pis=16, rand_ands=1500, mul_n=8)
+    check_vs_oracle(m)
+
+
+def _golden(name):
+    path = os.path.join(GOLD, name + ".json")
+    if not os.path.exists(path):
+        pytest.skip(f"{path} missing (run scripts/make_golden.py)")
+    return json.load(open(path))
+
+
+@pytest.mark.parametrize("name,fn", [("c2_mul12", lambda: c2_mul12()), ("c2_mul12_bug1", lambda: c2_mul12_bug(seed=1))])
+def test_c2_full_vs_stored_oracle(name, fn):
+    g = _golden(name)
+    m = fn()
+    assert [int(x) for x in m.lit_a] == g["lit_a"] and [int(x) for x in m.lit_b] == g["lit_b"]
+    assert int(m.aig.num_ands) == g["num_ands"]
+    ctx = gpu_ctx(m.aig)
+    gv, gc, gk = ctx.sim_exhaustive(m.lit_a, m.lit_b)
+    assert_same(gv, gc, gk, g["verdict"], g["cex"], g["k"], name)
+    orc = Oracle.from_aig(m.aig)
+    for p in np.nonzero(gv == capi.CEC_NOT_EQUIVALENT)[0]:
+        vec = ctx.get_cex(int(p))
+        n = 12
+        a = sum(int(vec[i]) << i for i in range(n))
+        b = sum(int(vec[n + i]) << i for i in range(n))
+        assert orc.eval_lit(int(m.lit_a[p]), vec) == ((a * b) >> int(p)) & 1  # closed form side
+        assert orc.eval_lit(int(m.lit_b[p]), vec) != ((a * b) >> int(p)) & 1
+
+
+def test_c5_full_size_sampled():
+    """Full BASELINE C5 size in the bench's launch configuration: copy invariance for every copy and
+    oracle confirmation of sampled outputs (every NEQ CEX re-derived as the first mismatch by the
+    oracle scanning [0, cex]; EQ pairs of bug copies checked on a sampled pattern range)."""
+    m = c5_big()
+    ctx = gpu_ctx(m.aig)
+    gv, gc, gk = ctx.sim_exhaustive(m.lit_a, m.lit_b)
+    types = m.meta["types"]
+    ppc = m.meta["pairs_per_copy"]
+    off = np.concatenate([[0], np.cumsum(ppc)])
+    by_type = {}
+    for c, t in enumerate(types):
+        sl = slice(off[c], off[c + 1])
+        sig = (tuple(gv[sl]), tuple(gc[sl]), tuple(gk[sl]))
+        by_type.setdefault(t, sig)
+        assert by_type[t] == sig, f"copy {c} differs from its type {t}"
+    assert all(int(x) == 24 or int(x) <= 24 for x in gk)
+    orc = Oracle.from_aig(m.aig)
+    rng = np.random.default_rng(0)
+    for c in m.meta["bug_copies"]:
+        sl = range(off[c], off[c + 1])
+        la, lb = m.lit_a[off[c]:off[c + 1]], m.lit_b[off[c]:off[c + 1]]
+        neq = [p for p in sl if gv[p] == capi.CEC_NOT_EQUIVALENT]
+        for p in neq:
+            hi = int(gc[p]) + 1
+            if hi > (1 << 22):
+                continue
+            ov, oc, ok, _ = orc.check_pairs([m.lit_a[p]], [m.lit_b[p]], lo=0, hi=hi)
+            assert int(ov[0]) == oracle.NOT_EQUIVALENT and int(oc[0]) == int(gc[p])
+        eqs = [p for p in sl if gv[p] == capi.CEC_EQUIVALENT]
+        if eqs:
+            lo = int(rng.integers(0, (1 << 24) - 4096))
+            ov, oc, ok, _ = orc.check_pairs(m.lit_a[eqs], m.lit_b[eqs], lo=lo, hi=lo + 4096)
+            assert all(int(v) == oracle.EQUIVALENT for v in ov)
+    assert any(gv == capi.CEC_NOT_EQUIVALENT)
+
+
+@pytest.mark.parametrize("seed", range(20))
+def test_local_checks_vs_oracle(seed):
+    rng = np.random.default_rng(500 + seed)
+    I = int(rng.integers(3, 12))
+    m = tiny_random(I, int(rng.integers(5, 80)), 16, 500 + seed)
+    N = m.aig.num_nodes
+    la, lb, off, lv = [], [], [0], []
+    for q in range(m.num_pairs):
+        cand = rng.choice(np.arange(1, N), size=int(rng.integers(1, min(N - 1, 10) + 1)), replace=False)
+        if rng.random() < 0.6:
+            cand = np.unique(np.concatenate([cand, rng.choice(np.arange(1, I + 1), size=I, replace=False)]))
+        cand = cand[:16]
+        la.append(int(m.lit_a[q])); lb.append(int(m.lit_b[q]))
+        lv += [int(x) for x in cand]
+        off.append(len(lv))
+    ctx = gpu_ctx(m.aig)
+    got = ctx.check_local_cuts(la, lb, off, lv)
+    want = Oracle.from_aig(m.aig).check_local(la, lb, off, lv)
+    assert list(map(int, got)) == list(map(int, want))
+
+
+def test_plan_rerun_is_deterministic():
+    m = c2_mul12_bug(seed=1, n=10)
+    ctx = gpu_ctx(m.aig)
+    plan = capi.cec_plan_exhaustive(ctx.handle, m.lit_a, m.lit_b)
+    outs = []
+    for _ in range(3):
+        capi.cec_plan_run(ctx.handle, plan)
+        outs.append(capi.cec_plan_results(ctx.handle, plan, m.num_pairs))
+    for o in outs[1:]:
+        for a, b in zip(outs[0], o):
+            assert np.array_equal(a, b)
+    capi.cec_plan_free(plan)

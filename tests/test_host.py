@@ -1,0 +1,167 @@
+"""CPU tests of the C-ABI library: it loads, exports every symbol include/cec.h declares, and its
+host logic (validation, supports, routing, windows, merging, sharding, pext) behaves as the paper
+and SURVEY.md §8 say. No compute call runs here (no GPU); simulation calls must refuse loudly."""
+import ctypes
+import os
+import re
+
+import numpy as np
+import pytest
+
+import paper_conf_dac_liuy25_b200 as pkg
+from paper_conf_dac_liuy25_b200 import capi
+from workloads import Builder, c1_add8, c2_mul12, c5_big
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def host_ctx(aig, **kw):
+    kw.setdefault("device", -1)
+    return capi.Context.from_aig(aig, **kw)
+
+
+def test_exports_match_header():
+    hdr = open(os.path.join(ROOT, "include", "cec.h")).read()
+    declared = set(re.findall(r"\b(cec_[a-z0-9_]+)\s*\(", hdr))
+    assert declared == set(capi.EXPORTS), declared ^ set(capi.EXPORTS)
+    for name in declared:
+        assert hasattr(capi.lib, name)  # dlsym succeeds
+    assert capi.cec_abi_version() == 1
+
+
+def test_opts_layout_and_defaults():
+    o = capi.cec_default_opts()
+    assert (o.device, o.rank, o.world, o.k_max, o.k_s, o.merge, o.engine) == (0, 0, 1, 32, 0, 1, 0)
+    assert ctypes.sizeof(capi.CecOpts) == 4 * 3 + 4 + 8 + 8 + 4 * 4 + 8 * 6
+
+
+def test_validation_rejects_non_topological():
+    fan = np.array([[2, 8]], dtype=np.uint32)  # AND id 3 (I=2) reading id 4
+    with pytest.raises(capi.CecError) as e:
+        capi.cec_load_aig(2, fan, np.array([6], np.uint32), capi.cec_default_opts(device=-1))
+    assert e.value.status == capi.CEC_E_AIG
+    with pytest.raises(capi.CecError) as e:
+        capi.cec_load_aig(2, fan, np.array([6], np.uint32), capi.cec_default_opts(device=-1, k_max=64))
+    assert e.value.status == capi.CEC_E_ARG
+
+
+def test_no_cpu_fallback():
+    m = c1_add8()
+    ctx = host_ctx(m.aig)
+    with pytest.raises(capi.CecError) as e:
+        ctx.sim_exhaustive(m.lit_a, m.lit_b)
+    assert e.value.status == capi.CEC_E_CUDA
+    with pytest.raises(capi.CecError) as e:
+        ctx.check_local_cuts(m.lit_a[:1], m.lit_b[:1], [0, 2], [1, 9])
+    assert e.value.status == capi.CEC_E_CUDA
+
+
+def test_supports_C1():
+    m = c1_add8()
+    ctx = host_ctx(m.aig)
+    for j in range(8):
+        S = capi.cec_pair_support(ctx.handle, int(m.lit_a[j]), int(m.lit_b[j]))
+        assert S == list(range(1, j + 2)) + list(range(9, 9 + j + 1))  # {a_0..a_j, b_0..b_j}
+    assert ctx.pair_k(int(m.lit_a[8]), int(m.lit_b[8])) == 16
+
+
+def test_plan_C1_single_window():
+    m = c1_add8()
+    ctx = host_ctx(m.aig)
+    plan = capi.cec_plan_exhaustive(ctx.handle, m.lit_a, m.lit_b)
+    info = capi.cec_plan_info(plan)
+    w = capi.cec_plan_window(plan, 0)
+    assert info["num_windows"] == 1 and info["max_k"] == 16
+    assert w["inputs"] == list(range(1, 17)) and sorted(w["pairs"]) == list(range(9))
+    assert info["node_patterns"] == w["num_nodes"] * (1 << 16)
+    # the window is exactly the ANDs in the TFI of the PO pairs (KS leaves unused prefix P terms)
+    I, fan = m.aig.num_pis, m.aig.fanins
+    seen, todo = set(), [int(x) >> 1 for x in list(m.lit_a) + list(m.lit_b)]
+    while todo:
+        v = todo.pop()
+        if v in seen or v <= I:
+            continue
+        seen.add(v)
+        todo += [int(fan[v - I - 1, 0]) >> 1, int(fan[v - I - 1, 1]) >> 1]
+    assert w["num_nodes"] == len(seen)
+    capi.cec_plan_free(plan)
+
+
+def merge_example_aig():
+    """windows with inputs {a,b}, {a,b,c}, {a,c}, {a,e}, {a,f}; ids a..f = 1..6.
+    (The printed list has four windows for "five"; {a,c} is the reading-Q10 fifth window.)"""
+    bd = Builder(6, strash=False)
+    a, b, c, d, e, f = (bd.pi(i) for i in range(6))
+    ab = bd.raw_and(a, b)
+    abc = bd.raw_and(ab, c)
+    ac = bd.raw_and(a, c)
+    ae = bd.raw_and(a, e)
+    af = bd.raw_and(a, f)
+    aig = bd.finish([ab, abc, ac, ae, af])
+    # pairs (node, a): support = the node's support
+    la = [ab, abc, ac, ae, af]
+    lb = [a] * 5
+    return aig, la, lb
+
+
+def test_window_merging_paper_example():
+    aig, la, lb = merge_example_aig()
+    ctx = host_ctx(aig, k_s=3)
+    plan = capi.cec_plan_exhaustive(ctx.handle, la, lb)
+    groups = sorted(capi.cec_plan_window(plan, w)["inputs"] for w in range(capi.cec_plan_info(plan)["num_windows"]))
+    assert groups == [[1, 2, 3], [1, 5, 6]]  # "the first three and the last two are merged"
+    capi.cec_plan_free(plan)
+    ctx2 = host_ctx(aig, k_s=3, merge=capi.CEC_MERGE_OFF)
+    plan = capi.cec_plan_exhaustive(ctx2.handle, la, lb)
+    assert capi.cec_plan_info(plan)["num_windows"] == 5
+    capi.cec_plan_free(plan)
+
+
+def test_routing_k_max_and_trivial_pairs():
+    m = c1_add8()
+    ctx = host_ctx(m.aig, k_max=10)
+    plan = capi.cec_plan_exhaustive(ctx.handle, m.lit_a, m.lit_b)
+    info = capi.cec_plan_info(plan)
+    assert info["max_k"] <= 10
+    ks = [ctx.pair_k(int(a), int(b)) for a, b in zip(m.lit_a, m.lit_b)]
+    simulated = sum(len(capi.cec_plan_window(plan, w)["pairs"]) for w in range(info["num_windows"]))
+    assert simulated == sum(1 for k in ks if k <= 10)
+    capi.cec_plan_free(plan)
+
+
+def test_c5_plan_one_window_per_copy():
+    m = c5_big(copies=8, n_random=6, n_bugs=2)
+    ctx = host_ctx(m.aig)
+    plan = capi.cec_plan_exhaustive(ctx.handle, m.lit_a, m.lit_b)
+    info = capi.cec_plan_info(plan)
+    assert info["num_windows"] == 8 and info["max_k"] == 24
+    W = 0
+    for w in range(8):
+        win = capi.cec_plan_window(plan, w)
+        c = (win["inputs"][0] - 1) // 24
+        assert win["inputs"] == list(range(24 * c + 1, 24 * c + 25))
+        W += win["num_nodes"] << 24
+    assert W == info["node_patterns"]
+    capi.cec_plan_free(plan)
+
+
+def test_shard_range_partition():
+    for n in [0, 1, 7, 2048, 16384, 10**9 + 7]:
+        for G in [1, 2, 3, 4, 8]:
+            rs = [capi.cec_shard_range(n, g, G) for g in range(G)]
+            assert rs[0][0] == 0 and rs[-1][1] == n
+            assert all(rs[g][1] == rs[g + 1][0] for g in range(G - 1))
+            assert max(e - b for b, e in rs) - min(e - b for b, e in rs) <= 1
+
+
+def test_pext():
+    assert capi.cec_pext64(6, 0b110) == 3  # survey vector V3
+    rng = np.random.default_rng(0)
+    for _ in range(200):
+        v, m = int(rng.integers(0, 2**63)), int(rng.integers(0, 2**63))
+        want, j = 0, 0
+        for b in range(64):
+            if (m >> b) & 1:
+                want |= ((v >> b) & 1) << j
+                j += 1
+        assert capi.cec_pext64(v, m) == want
