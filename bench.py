@@ -163,7 +163,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--config", default="c5")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--engine", type=int, default=0)
+    ap.add_argument("--engine", type=int, default=0, help="0 auto, 1 interpreter, 2 JIT")
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--cpu-log2-patterns", type=int, default=19)
     ap.add_argument("--ref-log2-patterns", type=int, default=17)
@@ -186,7 +186,8 @@ def main():
     torch.cuda.set_device(local)
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    stream = torch.cuda.current_stream()
+    stream = torch.cuda.Stream()  # the library launches on this stream; events are recorded on it
+    torch.cuda.set_stream(stream)
 
     m, desc, copy_idx = make_workload(args.config)
     uid = None
@@ -201,6 +202,8 @@ def main():
     plan = capi.cec_plan_exhaustive(ctx.handle, m.lit_a, m.lit_b)
     info = capi.cec_plan_info(plan)
     st0 = ctx.stats()
+    engine_name = ("jit" if st0["jit_windows"] == info["num_windows"] else
+                   "interp" if st0["jit_windows"] == 0 else f"jit({st0['jit_windows']} windows)+interp")
 
     for _ in range(args.warmup):
         capi.cec_plan_run(ctx.handle, plan)
@@ -287,7 +290,8 @@ def main():
                        "max_slots": info["max_slots"], "node_patterns_per_step": W_all,
                        "parallelism": f"pattern-space shards x{world}" + (" + NCCL min all-reduce" if world > 1 else ""),
                        "l2": "flushed between timed steps (256 MiB write, outside the events)",
-                       "engine": "interp", "verdicts": verdicts},
+                       "engine": engine_name, "jit_kernels": st0["jit_kernels"], "jit_compile_ms": st0["jit_ms"],
+                       "verdicts": verdicts},
             "clocks": clocks,
             "gpu_launches": int(launches_per_step * args.steps),
             "e2e": {"value": W_all / (e2e / 1e3), "unit": UNIT, "ms_per_miter": e2e,

@@ -105,6 +105,9 @@ typedef struct {
     float host_prep_ms;        /* host planning time of the last plan */
     uint64_t h2d_bytes;        /* bytes copied host->device by the last plan (schedules, items) */
     uint64_t d2h_bytes;        /* bytes copied device->host by the last results read-back */
+    float jit_ms;              /* NVRTC compile + load time spent by the last plan (0 if cached) */
+    uint32_t jit_kernels;      /* distinct window structures compiled for the last plan */
+    uint32_t jit_windows;      /* windows of the last plan run by JIT kernels (rest: interpreter) */
 } cec_stats;
 
 /* Fill *opts with the defaults above. */

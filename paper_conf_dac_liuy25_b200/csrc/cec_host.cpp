@@ -12,6 +12,7 @@
 #include <nccl.h>
 
 #include <algorithm>
+#include <atomic>
 #include <chrono>
 #include <cstdarg>
 #include <cstdio>
@@ -20,6 +21,7 @@
 #include <memory>
 #include <new>
 #include <string>
+#include <thread>
 #include <unordered_map>
 #include <vector>
 
@@ -122,7 +124,10 @@ struct cec_plan {
     std::vector<DevWin> dwin;
     std::vector<uint2> prog;
     std::vector<Item> items;
+    std::vector<JItem> jitems;
     std::vector<LaunchGroup> groups;
+    uint32_t jit_windows = 0, jit_kernels = 0;
+    float jit_ms = 0.f;
     uint64_t W_rank = 0, W_all = 0;
     uint32_t max_k = 0, max_slots = 0;
     float host_ms = 0.f;
@@ -393,8 +398,7 @@ cec_status cec_load_aig(cec_ctx **out, const cec_aig *aig, const cec_opts *opts)
     if (!c) return CEC_E_NOMEM;
     cec_default_opts(&c->opts);
     if (opts) c->opts = *opts;
-    if (c->opts.k_max == 0) c->opts.k_max = 32;
-    if (c->opts.k_max > 63) return CEC_E_ARG;
+    if (c->opts.k_max > 63) return fail(nullptr, CEC_E_ARG, "k_max > 63");
     if (c->opts.k_s == 0) c->opts.k_s = c->opts.k_max;
     if (c->opts.world < 1) c->opts.world = 1;
     if (c->opts.rank < 0 || c->opts.rank >= c->opts.world) return CEC_E_ARG;
@@ -480,6 +484,7 @@ cec_status cec_pair_support(cec_ctx *ctx, uint32_t la, uint32_t lb, uint32_t *su
 namespace {
 
 constexpr int32_t DECIDED_BY_SIM = -100;
+constexpr int JIT_MIN_BLOCKS = 4;  // 128-thread blocks -> <= 128 registers per thread
 
 uint64_t tt_words_of(uint32_t k) { return k <= 5 ? 1ull : (1ull << (k - 5)); }
 
@@ -490,6 +495,7 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
     P->dwin.clear();
     P->prog.clear();
     P->items.clear();
+    P->jitems.clear();
     P->groups.clear();
     P->win_inputs.clear();
     P->win_nodes.clear();
@@ -502,6 +508,9 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
     uint32_t max_slot_cap = interp_max_slots_per_warp();
     std::vector<uint32_t> nslots_of;
     std::vector<uint64_t> cost_of;
+    std::vector<int32_t> win_jit;                    // JIT structure index per window, -1 = interpreter
+    std::vector<JitProgram> jit_progs;
+    std::unordered_map<std::string, uint32_t> jit_index;
     for (size_t w = 0; w < wins.size(); ++w) {
         WinHost &W = wins[w];
         DevWin dw{};
@@ -562,6 +571,41 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         P->win_nodes.push_back((uint32_t)nodes.size());
         P->win_cmps.push_back(wc);
         nslots_of.push_back(sc.nslots);
+        // engine choice: straight-line register kernel for big windows (k >= 10 so a 32-word warp
+        // pass is never partial); the interpreter for small ones (JIT compile would dominate)
+        const uint64_t node_words = (uint64_t)nodes.size() * ttw;
+        bool jit = false;
+        if (dw.k >= 10 && !nodes.empty()) {
+            if (c->opts.engine == CEC_ENGINE_JIT) jit = true;
+            else if (c->opts.engine == CEC_ENGINE_AUTO) jit = node_words >= (1ull << 26);
+        }
+        if (jit) {
+            JitProgram jp;
+            jp.k = dw.k;
+            std::unordered_map<uint32_t, uint32_t> ref;
+            ref.reserve(2 * (nodes.size() + W.inputs.size()) + 4);
+            ref[0] = 0;
+            for (uint32_t j = 0; j < dw.k; ++j) ref[W.inputs[j]] = j + 1;
+            for (uint32_t t = 0; t < nodes.size(); ++t) ref[nodes[t]] = dw.k + 1 + t;
+            jp.nodes.reserve(2 * nodes.size());
+            for (uint32_t id : nodes) {
+                jp.nodes.push_back(ref.at(c->f0[id] >> 1) << 1 | (c->f0[id] & 1u));
+                jp.nodes.push_back(ref.at(c->f1[id] >> 1) << 1 | (c->f1[id] & 1u));
+            }
+            for (uint32_t ci : wc) {
+                jp.cmps.push_back(ref.at(cmps2[ci].la >> 1) << 1 | (cmps2[ci].la & 1u));
+                jp.cmps.push_back(ref.at(cmps2[ci].lb >> 1) << 1 | (cmps2[ci].lb & 1u));
+            }
+            std::string key = jit_key(jp);
+            auto it = jit_index.find(key);
+            if (it == jit_index.end()) {
+                it = jit_index.emplace(key, (uint32_t)jit_progs.size()).first;
+                jit_progs.push_back(std::move(jp));
+            }
+            win_jit.push_back((int32_t)it->second);
+        } else {
+            win_jit.push_back(-1);
+        }
         P->max_k = std::max(P->max_k, dw.k);
         P->max_slots = std::max(P->max_slots, sc.nslots);
         // W accounting: nodes x patterns, per rank and all ranks
@@ -578,14 +622,37 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
     P->cmps.swap(cmps2);
     for (auto &pc : P->pair_cmp)
         if (pc >= 0) pc = remap[pc];
-    // launch groups by slot budget (power-of-two buckets), items per group, largest windows first
-    std::map<uint32_t, std::vector<uint32_t>> buckets;
-    for (uint32_t w = 0; w < P->dwin.size(); ++w) {
-        uint32_t b = 32;
-        while (b < nslots_of[w]) b <<= 1;
-        b = std::min(b, max_slot_cap);
-        buckets[b].push_back(w);
+    // compile the distinct JIT structures (in parallel; cached process-wide by structure)
+    std::vector<JitKernel *> kernels(jit_progs.size(), nullptr);
+    P->jit_ms = 0.f;
+    if (!jit_progs.empty()) {
+        auto t0 = std::chrono::steady_clock::now();
+        std::vector<const char *> errs(jit_progs.size(), nullptr);
+        const bool load = !c->host_only;
+        // compile (CPU-heavy, thread-safe) in parallel without loading, then load serially
+        const unsigned hw = std::max(1u, std::min(16u, std::thread::hardware_concurrency()));
+        std::vector<std::thread> pool;
+        std::atomic<size_t> next{0};
+        for (unsigned t = 0; t < std::min<size_t>(hw, jit_progs.size()); ++t)
+            pool.emplace_back([&]() {
+                for (size_t i; (i = next.fetch_add(1)) < jit_progs.size();)
+                    errs[i] = jit_get_kernel(jit_progs[i], JIT_MIN_BLOCKS, false, &kernels[i]);
+            });
+        for (auto &th : pool) th.join();
+        for (size_t i = 0; i < jit_progs.size(); ++i) {
+            if (errs[i]) return fail(c, CEC_E_CUDA, "JIT: %s", errs[i]);
+            if (load) {
+                const char *e = jit_get_kernel(jit_progs[i], JIT_MIN_BLOCKS, true, &kernels[i]);
+                if (e) return fail(c, CEC_E_CUDA, "JIT load: %s", e);
+            }
+        }
+        P->jit_ms = std::chrono::duration<float, std::milli>(std::chrono::steady_clock::now() - t0).count();
     }
+    P->jit_kernels = (uint32_t)jit_progs.size();
+    P->jit_windows = 0;
+    for (int32_t j : win_jit) P->jit_windows += j >= 0;
+    // work items: slices of each window split into chunks; interpreter windows grouped by slot
+    // budget, JIT windows by structure; largest windows first inside a group
     uint64_t total_slices = 0;
     for (uint32_t w = 0; w < P->dwin.size(); ++w) {
         uint64_t ttw = tt_words_of(P->dwin[w].k), sb, se;
@@ -595,27 +662,50 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
     const uint64_t target_items = std::max<uint64_t>(1, (uint64_t)std::max(c->num_sms, 148) * 64);
     uint64_t item_slices = std::max<uint64_t>(1, total_slices / target_items);
     item_slices = std::min<uint64_t>(item_slices, 4096);
-    for (auto &kv : buckets) {
-        LaunchGroup g{};
-        g.nslots = kv.first;
-        g.item_off = (uint32_t)P->items.size();
-        std::vector<uint32_t> ws = kv.second;
+    std::map<uint32_t, std::vector<uint32_t>> buckets;   // interpreter: slot budget -> windows
+    std::map<int32_t, std::vector<uint32_t>> jgroups;    // JIT: structure -> windows
+    for (uint32_t w = 0; w < P->dwin.size(); ++w) {
+        if (win_jit[w] >= 0) {
+            jgroups[win_jit[w]].push_back(w);
+            continue;
+        }
+        uint32_t b = (nslots_of[w] + 31) / 32 * 32;
+        b = std::min(b, max_slot_cap);
+        buckets[b].push_back(w);
+    }
+    auto add_items = [&](std::vector<uint32_t> ws, bool jit) {
         std::stable_sort(ws.begin(), ws.end(), [&](uint32_t a, uint32_t b) { return cost_of[a] > cost_of[b]; });
-        // interleave: items of big windows first, each window's slices ascending
         for (uint32_t w : ws) {
             uint64_t ttw = tt_words_of(P->dwin[w].k), sb, se;
             cec_shard_range((ttw + 31) / 32, rank, world, &sb, &se);
             for (uint64_t s = sb; s < se; s += item_slices) {
-                Item it{};
-                it.win = w;
-                it.s_begin = (uint32_t)s;
-                it.s_end = (uint32_t)std::min<uint64_t>(se, s + item_slices);
-                P->items.push_back(it);
+                const uint32_t e = (uint32_t)std::min<uint64_t>(se, s + item_slices);
+                if (jit)
+                    P->jitems.push_back(JItem{w, (uint32_t)s, e, P->dwin[w].cmp_off});
+                else
+                    P->items.push_back(Item{w, (uint32_t)s, e, 0});
             }
         }
+    };
+    for (auto &kv : jgroups) {
+        LaunchGroup g{};
+        g.jit = kernels[kv.first];
+        g.item_off = (uint32_t)P->jitems.size();
+        add_items(kv.second, true);
+        g.nitems = (uint32_t)(P->jitems.size() - g.item_off);
+        P->groups.push_back(g);
+    }
+    for (auto &kv : buckets) {
+        LaunchGroup g{};
+        g.nslots = kv.first;
+        g.item_off = (uint32_t)P->items.size();
+        add_items(kv.second, false);
         g.nitems = (uint32_t)(P->items.size() - g.item_off);
         P->groups.push_back(g);
     }
+    // biggest groups first so the small launches fill in behind them
+    std::stable_sort(P->groups.begin(), P->groups.end(),
+                     [](const LaunchGroup &a, const LaunchGroup &b) { return a.nitems > b.nitems; });
     (void)stop;
     (void)local;
     return CEC_OK;
@@ -632,12 +722,15 @@ cec_status upload(cec_ctx *c, cec_plan *P) {
     CUDA_TRY(c, dev_alloc((void **)&d.bound, sizeof(unsigned long long) * nwin));
     CUDA_TRY(c, dev_alloc((void **)&d.neq_cnt, sizeof(uint32_t) * nwin));
     CUDA_TRY(c, dev_alloc((void **)&d.item_ctr, sizeof(uint32_t) * std::max<size_t>(1, P->groups.size())));
+    CUDA_TRY(c, dev_alloc((void **)&d.jitems, sizeof(JItem) * std::max<size_t>(1, P->jitems.size())));
+    CUDA_TRY(c, h2d(d.jitems, P->jitems.data(), sizeof(JItem) * P->jitems.size(), c->stream));
     CUDA_TRY(c, h2d(d.wins, P->dwin.data(), sizeof(DevWin) * P->dwin.size(), c->stream));
     CUDA_TRY(c, h2d(d.prog, P->prog.data(), sizeof(uint2) * P->prog.size(), c->stream));
     CUDA_TRY(c, h2d(d.items, P->items.data(), sizeof(Item) * P->items.size(), c->stream));
     CUDA_TRY(c, event_create(&P->ev0));
     CUDA_TRY(c, event_create(&P->ev1));
-    c->stats.h2d_bytes = sizeof(DevWin) * P->dwin.size() + sizeof(uint2) * P->prog.size() + sizeof(Item) * P->items.size();
+    c->stats.h2d_bytes = sizeof(DevWin) * P->dwin.size() + sizeof(uint2) * P->prog.size() +
+                         sizeof(Item) * P->items.size() + sizeof(JItem) * P->jitems.size();
     P->uploaded = true;
     return CEC_OK;
 }
@@ -651,6 +744,7 @@ void free_dev(cec_plan *P) {
     dev_free(d.bound);
     dev_free(d.neq_cnt);
     dev_free(d.item_ctr);
+    dev_free(d.jitems);
     d = DevPlan{};
     event_destroy(P->ev0);
     event_destroy(P->ev1);
@@ -771,6 +865,9 @@ cec_status cec_plan_exhaustive(cec_ctx *c, uint32_t n, const uint32_t *la, const
     auto t1 = std::chrono::steady_clock::now();
     P->host_ms = std::chrono::duration<float, std::milli>(t1 - t0).count();
     c->stats.host_prep_ms = P->host_ms;
+    c->stats.jit_ms = P->jit_ms;
+    c->stats.jit_kernels = P->jit_kernels;
+    c->stats.jit_windows = P->jit_windows;
     st = upload(c, P.get());
     if (st != CEC_OK) {
         free_dev(P.get());
@@ -786,9 +883,9 @@ cec_status cec_plan_run(cec_ctx *c, cec_plan *P) {
     if (!P->uploaded) return fail(c, CEC_E_STATE, "plan not uploaded");
     CUDA_TRY(c, event_record(P->ev0, c->stream));
     uint32_t nl = 0;
-    const char *e = launch_interp(P->d, P->groups, (uint32_t)P->dwin.size(), (uint32_t)P->cmps.size(), c->stream,
+    const char *e = launch_run(P->d, P->groups, (uint32_t)P->dwin.size(), (uint32_t)P->cmps.size(), c->stream,
                                   c->num_sms, &nl);
-    if (e) return fail(c, CEC_E_CUDA, "CUDA: %s (interpreter launch)", e);
+    if (e) return fail(c, CEC_E_CUDA, "CUDA: %s (kernel launch)", e);
     if (c->opts.world > 1 && !P->cmps.empty()) {  // a10: one NCCL min all-reduce of first_idx
         ncclResult_t r = g_nccl.all_reduce(P->d.first, P->d.first, P->cmps.size(), ncclUint64, ncclMin, c->comm,
                                            (cudaStream_t)c->stream);

@@ -35,9 +35,25 @@ struct Item {              // a contiguous range of 32-word slices of one window
     uint32_t pad;
 };
 
-struct LaunchGroup {       // windows sharing one kernel launch (same shared-memory slot budget)
-    uint32_t nslots;       // slots per warp in this launch
+// ---- JIT engine (jit.cpp) -----------------------------------------------------------------------
+// A window as a straight-line SSA program. Operand refs: 0 = constant 0, 1..k = input j-1,
+// k+1+t = node t. nodes[2t], nodes[2t+1] = (ref << 1 | complement) of node t's fanins;
+// cmps[2c], cmps[2c+1] = the two roots of the window's c-th compare.
+struct JitProgram {
+    uint32_t k = 0;
+    std::vector<uint32_t> nodes;
+    std::vector<uint32_t> cmps;
+};
+struct JItem {             // a slice range of one JIT window instance
+    uint32_t win;          // window index (bound / neq_cnt)
+    uint32_t s_begin, s_end;
+    uint32_t cmp_off;      // first[] index of the window's compare 0
+};
+struct JitKernel;
+struct LaunchGroup {       // windows sharing one kernel launch
+    uint32_t nslots;       // interpreter: slots per warp in this launch
     uint32_t item_off, nitems;
+    JitKernel *jit = nullptr;  // non-null: a JIT structure group (items index DevPlan::jitems)
 };
 
 // Device buffers of one plan.
@@ -49,11 +65,21 @@ struct DevPlan {
     unsigned long long *bound = nullptr;  // [nwin] early-exit bound (all pairs NEQ below it)
     uint32_t *neq_cnt = nullptr;          // [nwin]
     uint32_t *item_ctr = nullptr;         // [ngroups]
+    JItem *jitems = nullptr;
 };
 
+// jit.cpp
+std::string jit_key(const JitProgram &p);
+std::string jit_source(const JitProgram &p, int min_blocks);
+const char *jit_compile_cubin(const std::string &src, std::vector<char> &cubin, std::string &log);
+const char *jit_get_kernel(const JitProgram &p, int min_blocks, bool load, JitKernel **out);
+double jit_compile_ms(const JitKernel *k);
+const char *jit_launch(JitKernel *K, const JItem *items, uint32_t nitems, uint32_t *ctr, unsigned long long *first,
+                       unsigned long long *bound, uint32_t *neq_cnt, void *stream, int num_sms);
+
 // sim_interp.cu
-const char *launch_interp(const DevPlan &d, const std::vector<LaunchGroup> &groups, uint32_t nwin, uint32_t ncmp,
-                          void *stream, int num_sms, uint32_t *launches);
+const char *launch_run(const DevPlan &d, const std::vector<LaunchGroup> &groups, uint32_t nwin, uint32_t ncmp,
+                       void *stream, int num_sms, uint32_t *launches);
 const char *dev_alloc(void **p, size_t bytes);
 const char *dev_free(void *p);
 const char *h2d(void *dst, const void *src, size_t bytes, void *stream);

@@ -1,0 +1,269 @@
+// jit.cpp — register-resident window kernels generated per window STRUCTURE and compiled at plan
+// time with NVRTC for sm_100a (CEC_ENGINE_JIT / AUTO).
+//
+// Why: the interpreter keeps node words in shared-memory slots, so every AND costs two loads and a
+// store of shared memory (~12 B per node-word) — it is bound by the shared-memory pipe, far below
+// the ALU (LOP3) pipe. A window's structure is fixed for the whole 2^k-pattern sweep, so we emit it
+// as straight-line code: every node word lives in a register and every AND is exactly ONE
+// `lop3.b32` whose 8-bit LUT folds both edge complements (0xC0 = a&b, 0x0C = !a&b, 0x30 = a&!b,
+// 0x03 = !a&!b). The LOP3s are emitted as inline PTX so the compiler cannot re-associate or
+// simplify the Boolean logic (that would silently skip node evaluations and falsify the
+// node-pattern count W; ptxas still allocates registers and schedules). Input (projection) words
+// are generated arithmetically from the word index; compares are warp-aggregated
+// (__any_sync, __ballot_sync) exactly like the interpreter, so the canonical minimum CEX index is
+// the same.
+//
+// Windows with identical structure (same k, same node list up to renaming, same compares) share
+// one compiled kernel; all their instances run in one launch (e.g. the disjoint copies of C5).
+#include <cuda_runtime.h>
+#include <dlfcn.h>
+
+#include <algorithm>
+#include <chrono>
+#include <cstdio>
+#include <cstring>
+#include <map>
+#include <memory>
+#include <mutex>
+#include <string>
+#include <vector>
+
+#include "cec_internal.hpp"
+
+namespace cec {
+
+namespace {
+
+// ---- NVRTC, loaded on demand --------------------------------------------------------------------
+typedef int nvrtcResult_t;
+typedef struct _nvrtcProgram *nvrtcProgram_t;
+struct Nvrtc {
+    void *h = nullptr;
+    nvrtcResult_t (*create)(nvrtcProgram_t *, const char *, const char *, int, const char *const *,
+                            const char *const *) = nullptr;
+    nvrtcResult_t (*compile)(nvrtcProgram_t, int, const char *const *) = nullptr;
+    nvrtcResult_t (*log_size)(nvrtcProgram_t, size_t *) = nullptr;
+    nvrtcResult_t (*log)(nvrtcProgram_t, char *) = nullptr;
+    nvrtcResult_t (*cubin_size)(nvrtcProgram_t, size_t *) = nullptr;
+    nvrtcResult_t (*cubin)(nvrtcProgram_t, char *) = nullptr;
+    nvrtcResult_t (*destroy)(nvrtcProgram_t *) = nullptr;
+    std::string why;
+    bool load() {
+        if (h) return true;
+        const char *cands[] = {"libnvrtc.so.12", "/usr/local/cuda/lib64/libnvrtc.so.12", "libnvrtc.so"};
+        for (const char *c : cands) {
+            h = dlopen(c, RTLD_NOW | RTLD_LOCAL);
+            if (h) break;
+        }
+        if (!h) {
+            why = "libnvrtc.so.12 not found";
+            return false;
+        }
+        create = (decltype(create))dlsym(h, "nvrtcCreateProgram");
+        compile = (decltype(compile))dlsym(h, "nvrtcCompileProgram");
+        log_size = (decltype(log_size))dlsym(h, "nvrtcGetProgramLogSize");
+        log = (decltype(log))dlsym(h, "nvrtcGetProgramLog");
+        cubin_size = (decltype(cubin_size))dlsym(h, "nvrtcGetCUBINSize");
+        cubin = (decltype(cubin))dlsym(h, "nvrtcGetCUBIN");
+        destroy = (decltype(destroy))dlsym(h, "nvrtcDestroyProgram");
+        if (!(create && compile && log_size && log && cubin_size && cubin && destroy)) {
+            why = "libnvrtc is missing symbols";
+            return false;
+        }
+        return true;
+    }
+};
+Nvrtc g_nvrtc;
+std::mutex g_mu;
+
+const char *kMask[5] = {"0xAAAAAAAAu", "0xCCCCCCCCu", "0xF0F0F0F0u", "0xFF00FF00u", "0xFFFF0000u"};
+
+std::string ref_name(const JitProgram &p, uint32_t ref) {
+    if (ref == 0) return "0u";
+    if (ref <= p.k) return "x" + std::to_string(ref - 1);
+    return "n" + std::to_string(ref - p.k - 1);
+}
+
+}  // namespace
+
+struct JitKernel {
+    cudaLibrary_t lib = nullptr;
+    cudaKernel_t kern = nullptr;
+    int block = 128;
+    int blocks_per_sm = 0;
+    double compile_ms = 0;
+    size_t src_bytes = 0, cubin_bytes = 0;
+};
+
+std::string jit_key(const JitProgram &p) {
+    std::string key;
+    key.reserve(16 + 8 * (p.nodes.size() + p.cmps.size()));
+    auto put = [&](uint32_t v) { key.append(reinterpret_cast<const char *>(&v), 4); };
+    put(p.k);
+    put((uint32_t)p.nodes.size());
+    put((uint32_t)p.cmps.size());
+    for (uint32_t v : p.nodes) put(v);
+    for (uint32_t v : p.cmps) put(v);
+    return key;
+}
+
+std::string jit_source(const JitProgram &p, int min_blocks) {
+    const uint32_t n = (uint32_t)(p.nodes.size() / 2), ncmp = (uint32_t)(p.cmps.size() / 2);
+    std::string s;
+    s.reserve(96 * (size_t)n + 160 * (size_t)ncmp + 4096);
+    char buf[256];
+    s += "typedef unsigned int u32; typedef unsigned long long u64;\n"
+         "struct JItem { u32 win, s_begin, s_end, cmp_off; };\n"
+         "__device__ __noinline__ void rep(u32 d, u32 c, u32 win, u32 s, u32 lane, u32 ncmp, u32 cmp_off,\n"
+         "    u64 *first, u64 *bound, u32 *neq_cnt) {\n"
+         "  const u32 bal = __ballot_sync(0xFFFFFFFFu, d != 0u);\n"
+         "  const u32 l = (u32)__ffs(bal) - 1u;\n"
+         "  const u32 dl = __shfl_sync(0xFFFFFFFFu, d, l);\n"
+         "  if (lane != 0u) return;\n"
+         "  const u64 idx = ((((u64)s << 5) + l) << 5) + (u32)(__ffs(dl) - 1);\n"
+         "  const u64 old = atomicMin(&first[cmp_off + c], idx);\n"
+         "  if (old != ~0ull) return;\n"
+         "  __threadfence();\n"
+         "  if (atomicAdd(&neq_cnt[win], 1u) + 1u != ncmp) return;\n"
+         "  __threadfence();\n"
+         "  u64 mx = 0;\n"
+         "  for (u32 t = 0; t < ncmp; ++t) { u64 v = atomicAdd(&first[cmp_off + t], 0ull); mx = v > mx ? v : mx; }\n"
+         "  atomicMin(&bound[win], mx);\n"
+         "}\n";
+    snprintf(buf, sizeof buf,
+             "extern \"C\" __global__ void __launch_bounds__(128, %d) cecjit(const JItem *__restrict__ items, u32 nitems,\n"
+             "    u32 *ctr, u64 *first, u64 *bound, u32 *neq_cnt) {\n",
+             min_blocks);
+    s += buf;
+    s += "  const u32 lane = threadIdx.x & 31u;\n"
+         "  for (;;) {\n"
+         "    u32 it = 0;\n"
+         "    if (lane == 0u) it = atomicAdd(ctr, 1u);\n"
+         "    it = __shfl_sync(0xFFFFFFFFu, it, 0);\n"
+         "    if (it >= nitems) return;\n"
+         "    const JItem I = items[it];\n"
+         "    for (u32 s = I.s_begin; s < I.s_end; ++s) {\n"
+         "      if (((u64)s << 10) >= *((volatile u64 *)&bound[I.win])) break;\n"
+         "      const u64 word = ((u64)s << 5) + lane;\n";
+    for (uint32_t j = 0; j < p.k; ++j) {
+        if (j < 5)
+            snprintf(buf, sizeof buf, "      const u32 x%u = %s;\n", j, kMask[j]);
+        else
+            snprintf(buf, sizeof buf, "      const u32 x%u = 0u - (u32)((word >> %u) & 1ull);\n", j, j - 5);
+        s += buf;
+    }
+    // compares are placed right after their later root so roots die early (fewer live registers)
+    std::vector<std::vector<uint32_t>> after(n + 1);
+    for (uint32_t c = 0; c < ncmp; ++c) {
+        const uint32_t ra = p.cmps[2 * c] >> 1, rb = p.cmps[2 * c + 1] >> 1;
+        const uint32_t m = std::max(ra, rb);
+        after[m > p.k ? m - p.k : 0].push_back(c);
+    }
+    auto emit_cmp = [&](uint32_t c) {
+        const uint32_t a = p.cmps[2 * c], b = p.cmps[2 * c + 1];
+        const bool inv = ((a ^ b) & 1u) != 0;
+        snprintf(buf, sizeof buf,
+                 "      { const u32 d = %s%s ^ %s%s; if (__any_sync(0xFFFFFFFFu, d != 0u)) rep(d, %uu, I.win, s, lane, %uu, I.cmp_off, first, bound, neq_cnt); }\n",
+                 inv ? "~(" : "", ref_name(p, a >> 1).c_str(), ref_name(p, b >> 1).c_str(), inv ? ")" : "", c, ncmp);
+        s += buf;
+    };
+    static const unsigned lut[4] = {0xC0, 0x0C, 0x30, 0x03};  // index = ca | cb << 1; a = 0xF0, b = 0xCC
+    for (uint32_t c : after[0]) emit_cmp(c);
+    for (uint32_t t = 0; t < n; ++t) {
+        const uint32_t a = p.nodes[2 * t], b = p.nodes[2 * t + 1];
+        const unsigned L = lut[(a & 1u) | ((b & 1u) << 1)];
+        snprintf(buf, sizeof buf, "      u32 n%u; asm(\"lop3.b32 %%0, %%1, %%2, 0, 0x%02X;\" : \"=r\"(n%u) : \"r\"(%s), \"r\"(%s));\n",
+                 t, L, t, ref_name(p, a >> 1).c_str(), ref_name(p, b >> 1).c_str());
+        s += buf;
+        for (uint32_t c : after[t + 1]) emit_cmp(c);
+    }
+    s += "    }\n  }\n}\n";
+    return s;
+}
+
+const char *jit_compile_cubin(const std::string &src, std::vector<char> &cubin, std::string &log) {
+    {
+        std::lock_guard<std::mutex> g(g_mu);
+        if (!g_nvrtc.load()) return g_nvrtc.why.c_str();
+    }
+    nvrtcProgram_t prog = nullptr;
+    if (g_nvrtc.create(&prog, src.c_str(), "cecjit.cu", 0, nullptr, nullptr) != 0) return "nvrtcCreateProgram failed";
+    const char *opts[] = {"--gpu-architecture=sm_100a", "--std=c++17", "-default-device", "-lineinfo"};
+    const int rc = g_nvrtc.compile(prog, 4, opts);
+    size_t ls = 0;
+    g_nvrtc.log_size(prog, &ls);
+    log.assign(ls, '\0');
+    if (ls) g_nvrtc.log(prog, &log[0]);
+    if (rc != 0) {
+        g_nvrtc.destroy(&prog);
+        return "NVRTC compilation failed";
+    }
+    size_t cs = 0;
+    g_nvrtc.cubin_size(prog, &cs);
+    cubin.resize(cs);
+    g_nvrtc.cubin(prog, cubin.data());
+    g_nvrtc.destroy(&prog);
+    return nullptr;
+}
+
+namespace {
+std::map<std::string, std::unique_ptr<JitKernel>> g_cache;  // process-wide, keyed by structure
+}
+
+const char *jit_get_kernel(const JitProgram &p, int min_blocks, bool load, JitKernel **out) {
+    const std::string key = jit_key(p) + std::string(1, (char)min_blocks);
+    {
+        std::lock_guard<std::mutex> g(g_mu);
+        auto it = g_cache.find(key);
+        if (it != g_cache.end() && (!load || it->second->kern)) {
+            *out = it->second.get();
+            return nullptr;
+        }
+    }
+    auto t0 = std::chrono::steady_clock::now();
+    const std::string src = jit_source(p, min_blocks);
+    std::vector<char> cubin;
+    std::string log;
+    const char *e = jit_compile_cubin(src, cubin, log);
+    if (e) {
+        static thread_local std::string msg;
+        msg = std::string(e) + ": " + log.substr(0, 400);
+        return msg.c_str();
+    }
+    std::unique_ptr<JitKernel> K(new JitKernel());
+    K->src_bytes = src.size();
+    K->cubin_bytes = cubin.size();
+    if (load) {
+        cudaError_t ce = cudaLibraryLoadData(&K->lib, cubin.data(), nullptr, nullptr, 0, nullptr, nullptr, 0);
+        if (ce != cudaSuccess) return cudaGetErrorString(ce);
+        ce = cudaLibraryGetKernel(&K->kern, K->lib, "cecjit");
+        if (ce != cudaSuccess) return cudaGetErrorString(ce);
+        int per_sm = 0;
+        ce = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, (const void *)K->kern, K->block, 0);
+        if (ce != cudaSuccess) return cudaGetErrorString(ce);
+        K->blocks_per_sm = per_sm > 0 ? per_sm : 1;
+    }
+    K->compile_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+    std::lock_guard<std::mutex> g(g_mu);
+    auto &slot = g_cache[key];
+    slot = std::move(K);
+    *out = slot.get();
+    return nullptr;
+}
+
+double jit_compile_ms(const JitKernel *k) { return k ? k->compile_ms : 0.0; }
+
+const char *jit_launch(JitKernel *K, const JItem *items, uint32_t nitems, uint32_t *ctr, unsigned long long *first,
+                       unsigned long long *bound, uint32_t *neq_cnt, void *stream, int num_sms) {
+    if (!K || !K->kern) return "JIT kernel not loaded";
+    if (nitems == 0) return nullptr;
+    uint64_t grid = (uint64_t)num_sms * K->blocks_per_sm;
+    const uint64_t need = (nitems + (K->block / 32) - 1) / (K->block / 32);
+    if (grid > need) grid = need;
+    void *args[] = {(void *)&items, (void *)&nitems, (void *)&ctr, (void *)&first, (void *)&bound, (void *)&neq_cnt};
+    cudaError_t e = cudaLaunchKernel((const void *)K->kern, dim3((unsigned)grid), dim3(K->block), args, 0,
+                                     (cudaStream_t)stream);
+    return e == cudaSuccess ? nullptr : cudaGetErrorString(e);
+}
+
+}  // namespace cec

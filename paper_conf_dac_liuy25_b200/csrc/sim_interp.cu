@@ -18,6 +18,7 @@
 //    refuted publishes a bound and later slices above it are skipped (bounded early exit, Q9).
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <cstdint>
 #include <vector>
 
@@ -126,8 +127,8 @@ uint32_t interp_max_slots_per_warp() {
     return (uint32_t)((SMEM_PER_SM / 4 - 64) / 32);
 }
 
-const char *launch_interp(const DevPlan &d, const std::vector<LaunchGroup> &groups, uint32_t nwin, uint32_t ncmp,
-                          void *stream, int num_sms, uint32_t *launches) {
+const char *launch_run(const DevPlan &d, const std::vector<LaunchGroup> &groups, uint32_t nwin, uint32_t ncmp,
+                       void *stream, int num_sms, uint32_t *launches) {
     cudaStream_t st = (cudaStream_t)stream;
     const char *e;
     if ((e = ck(cudaMemsetAsync(d.first, 0xFF, sizeof(unsigned long long) * (ncmp ? ncmp : 1), st)))) return e;
@@ -138,9 +139,25 @@ const char *launch_interp(const DevPlan &d, const std::vector<LaunchGroup> &grou
     for (size_t g = 0; g < groups.size(); ++g) {
         const LaunchGroup &G = groups[g];
         if (G.nitems == 0) continue;
+        if (G.jit) {
+            if ((e = jit_launch(G.jit, d.jitems + G.item_off, G.nitems, d.item_ctr + g, d.first, d.bound, d.neq_cnt,
+                                stream, num_sms)))
+                return e;
+            ++nl;
+            continue;
+        }
         const size_t per_warp = ((size_t)G.nslots * 32 + 64) * 4;
-        int wpb = MAX_WPB;
-        while (wpb > 1 && per_warp * wpb > SMEM_PER_SM) wpb >>= 1;
+        // warps per block: the choice that keeps the most warps resident per SM (smem-limited)
+        int wpb = 1;
+        size_t best = 0;
+        for (int w = MAX_WPB; w >= 1; w >>= 1) {
+            const size_t per_block = per_warp * w + 1024;  // + per-block reservation
+            const size_t resident = (size_t)w * std::min<size_t>(32 / w, (SMEM_PER_SM + 1024) / per_block);
+            if (resident > best) {
+                best = resident;
+                wpb = w;
+            }
+        }
         const size_t smem = per_warp * wpb;
         if (smem > SMEM_PER_SM) return "window live set exceeds shared memory";
         if ((e = ck(cudaFuncSetAttribute(interp_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem))))

@@ -69,6 +69,9 @@ def test_paper_examples_on_gpu():
     assert list(lv) == [capi.CEC_UNDECIDED, capi.CEC_EQUIVALENT]  # PAPER.md:35/:130 SDC; cut = support
 
 
+ENGINES = [capi.CEC_ENGINE_INTERP, capi.CEC_ENGINE_JIT]
+
+
 @pytest.mark.parametrize("seed", range(60))
 def test_fuzz_tiny_random(seed):
     rng = np.random.default_rng(seed)
@@ -76,26 +79,29 @@ def test_fuzz_tiny_random(seed):
     m = tiny_random(I, int(rng.integers(1, 120)), 24, 7000 + seed)
     kmax = int(rng.integers(0, 13))
     merge = int(rng.integers(0, 3))
-    check_vs_oracle(m, k_max=kmax, merge=merge)
+    check_vs_oracle(m, k_max=kmax, merge=merge, engine=ENGINES[seed % 2])
 
 
-def test_c1_add8():
-    check_vs_oracle(c1_add8())
+@pytest.mark.parametrize("engine", ENGINES)
+def test_c1_add8(engine):
+    check_vs_oracle(c1_add8(), engine=engine)
 
 
+@pytest.mark.parametrize("engine", ENGINES)
 @pytest.mark.parametrize("n", [6, 8, 10])
-def test_small_multipliers_and_bugs(n):
-    check_vs_oracle(circuits.c2_mul12(n))
-    check_vs_oracle(circuits.c2_mul12_bug(seed=1, n=n))
-    check_vs_oracle(circuits.c2_mul12_bug(seed=3, n=n), merge=capi.CEC_MERGE_OFF)
+def test_small_multipliers_and_bugs(n, engine):
+    check_vs_oracle(circuits.c2_mul12(n), engine=engine)
+    check_vs_oracle(circuits.c2_mul12_bug(seed=1, n=n), engine=engine)
+    check_vs_oracle(circuits.c2_mul12_bug(seed=3, n=n), merge=capi.CEC_MERGE_OFF, engine=engine)
 
 
-def test_invariance_merge_and_kmax():
+def test_invariance_merge_kmax_engine():
     m = c5_big(copies=6, n_random=4, n_bugs=3, rand_pis=14, rand_ands=700, mul_n=7)
     ref = None
-    for merge in (capi.CEC_MERGE_OFF, capi.CEC_MERGE_PAPER, capi.CEC_MERGE_COST):
-        for k_max in (32, 40):
-            ctx = gpu_ctx(m.aig, merge=merge, k_max=k_max, k_s=28 if merge else 0)
+    for merge, k_max, engine in [(m_, k_, e_) for m_ in (capi.CEC_MERGE_OFF, capi.CEC_MERGE_PAPER, capi.CEC_MERGE_COST)
+                                 for k_ in (32, 40) for e_ in ENGINES]:
+        if True:
+            ctx = gpu_ctx(m.aig, merge=merge, k_max=k_max, k_s=28 if merge else 0, engine=engine)
             got = ctx.sim_exhaustive(m.lit_a, m.lit_b)
             if ref is None:
                 ref = got
@@ -107,9 +113,10 @@ def test_invariance_merge_and_kmax():
                     assert np.array_equal(a, b)
 
 
-def test_c5_reduced_vs_oracle():
+@pytest.mark.parametrize("engine", ENGINES)
+def test_c5_reduced_vs_oracle(engine):
     m = c5_big(copies=16, n_random=10, n_bugs=4, rand_pis=16, rand_ands=1500, mul_n=8)
-    check_vs_oracle(m)
+    check_vs_oracle(m, engine=engine)
 
 
 def _golden(name):
@@ -119,13 +126,14 @@ def _golden(name):
     return json.load(open(path))
 
 
+@pytest.mark.parametrize("engine", ENGINES)
 @pytest.mark.parametrize("name,fn", [("c2_mul12", lambda: c2_mul12()), ("c2_mul12_bug1", lambda: c2_mul12_bug(seed=1))])
-def test_c2_full_vs_stored_oracle(name, fn):
+def test_c2_full_vs_stored_oracle(name, fn, engine):
     g = _golden(name)
     m = fn()
     assert [int(x) for x in m.lit_a] == g["lit_a"] and [int(x) for x in m.lit_b] == g["lit_b"]
     assert int(m.aig.num_ands) == g["num_ands"]
-    ctx = gpu_ctx(m.aig)
+    ctx = gpu_ctx(m.aig, engine=engine)
     gv, gc, gk = ctx.sim_exhaustive(m.lit_a, m.lit_b)
     assert_same(gv, gc, gk, g["verdict"], g["cex"], g["k"], name)
     orc = Oracle.from_aig(m.aig)

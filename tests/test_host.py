@@ -165,3 +165,21 @@ def test_pext():
                 want |= ((v >> b) & 1) << j
                 j += 1
         assert capi.cec_pext64(v, m) == want
+
+
+def test_jit_codegen_compiles_for_sm100a_host_only():
+    """The JIT engine's NVRTC path runs on the host (no GPU needed): one kernel per distinct window
+    structure; C5's 256 copies share 3 random + 1 mul12 + bug-variant structures."""
+    from workloads import circuits
+    m = c5_big(copies=12, n_random=8, n_bugs=2, rand_pis=12, rand_ands=300, mul_n=6)
+    ctx = host_ctx(m.aig, engine=capi.CEC_ENGINE_JIT)
+    plan = capi.cec_plan_exhaustive(ctx.handle, m.lit_a, m.lit_b)
+    st = ctx.stats()
+    n_struct = len(set(m.meta["types"]))
+    assert st["jit_windows"] == 12 and st["jit_kernels"] == n_struct
+    capi.cec_plan_free(plan)
+    # interpreter only: no JIT
+    ctx2 = host_ctx(m.aig, engine=capi.CEC_ENGINE_INTERP)
+    plan = capi.cec_plan_exhaustive(ctx2.handle, m.lit_a, m.lit_b)
+    assert ctx2.stats()["jit_windows"] == 0
+    capi.cec_plan_free(plan)

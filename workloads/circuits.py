@@ -46,17 +46,28 @@ def _remap_lits(lits: np.ndarray, num_pis: int, pi_base: int, and_base: int) -> 
 
 
 def concat_miter(a: Aig, b: Aig, name: str = "") -> Miter:
-    """Put A's ANDs then B's ANDs over the shared PIs. Pairs = (PO_A[i], PO_B[i])."""
+    """Miter of A and B over the shared PIs, structurally hashed like an ABC miter: A's ANDs first,
+    then B's ANDs re-created through the same hashing builder, so a B node identical to an A node
+    (same fanin literals) is not duplicated. Pairs = (PO_A[i], PO_B[i]).
+    meta: a_ands = #ANDs of A; b_ands = #ANDs created for B only (ids after A's)."""
     if a.num_pis != b.num_pis or a.pos.size != b.pos.size:
         raise ValueError("A and B must have the same PIs and PO count")
     I = a.num_pis
-    fa = a.fanins
-    fb = _remap_lits(b.fanins, I, 0, 1 + I + a.num_ands)
-    pb = _remap_lits(b.pos, I, 0, 1 + I + a.num_ands)
-    aig = Aig(I, np.concatenate([fa, fb]).astype(np.uint32).reshape(-1, 2),
-              np.concatenate([a.pos, pb]).astype(np.uint32))
-    aig.validate()
-    return Miter(aig, a.pos.copy(), pb.copy(), name=name, meta={"a_ands": a.num_ands, "b_ands": b.num_ands})
+    bd = Builder(I, strash=True)
+    for l0, l1 in a.fanins:
+        bd.raw_and(int(l0), int(l1))
+        bd._table[(min(int(l0), int(l1)), max(int(l0), int(l1)))] = 2 * (bd.next_id() - 1)
+    a_ands = len(bd.ands)
+    lit_map = np.zeros(1 + I + b.num_ands, dtype=np.int64)
+    lit_map[1:1 + I] = 2 * np.arange(1, I + 1)
+    for j, (l0, l1) in enumerate(b.fanins):
+        x = int(lit_map[int(l0) >> 1]) ^ (int(l0) & 1)
+        y = int(lit_map[int(l1) >> 1]) ^ (int(l1) & 1)
+        lit_map[1 + I + j] = bd.AND(x, y)
+    pb = np.array([int(lit_map[int(l) >> 1]) ^ (int(l) & 1) for l in b.pos], dtype=np.uint32)
+    aig = bd.finish(list(a.pos) + list(pb))
+    return Miter(aig, a.pos.astype(np.uint32).copy(), pb, name=name,
+                 meta={"a_ands": a_ands, "b_ands": len(bd.ands) - a_ands})
 
 
 def b_image(miter_a_ands: int, num_pis: int, lit_in_b: int) -> int:
@@ -476,10 +487,12 @@ def c5_big(copies: int = 256, n_random: int = 176, seed: int = 5, n_bugs: int = 
     all_bases = list(bases)
     for c in bug_copies:
         bm = bases[types[c]]
-        p = int(rng.integers(0, bm.num_pairs))
-        drv = int(bm.lit_b[p]) >> 1
-        if drv <= bm.aig.num_pis:
+        lo, hi = b_side_ids(bm)
+        cand = [p for p in range(bm.num_pairs) if lo <= (int(bm.lit_b[p]) >> 1) < hi]
+        if not cand:
             continue
+        p = cand[int(rng.integers(0, len(cand)))]
+        drv = int(bm.lit_b[p]) >> 1
         bugged = flip_fanin(bm, drv, int(rng.integers(0, 2)))
         all_bases.append(bugged)
         types[c] = len(all_bases) - 1
