@@ -72,11 +72,12 @@ def test_plan_C1_single_window():
     info = capi.cec_plan_info(plan)
     w = capi.cec_plan_window(plan, 0)
     assert info["num_windows"] == 1 and info["max_k"] == 16
-    assert w["inputs"] == list(range(1, 17)) and sorted(w["pairs"]) == list(range(9))
+    nontrivial = [p for p in range(9) if m.lit_a[p] != m.lit_b[p]]  # strashed-identical pairs need no sim
+    assert w["inputs"] == list(range(1, 17)) and sorted(w["pairs"]) == nontrivial
     assert info["node_patterns"] == w["num_nodes"] * (1 << 16)
     # the window is exactly the ANDs in the TFI of the PO pairs (KS leaves unused prefix P terms)
     I, fan = m.aig.num_pis, m.aig.fanins
-    seen, todo = set(), [int(x) >> 1 for x in list(m.lit_a) + list(m.lit_b)]
+    seen, todo = set(), [int(x) >> 1 for p in nontrivial for x in (m.lit_a[p], m.lit_b[p])]
     while todo:
         v = todo.pop()
         if v in seen or v <= I:
@@ -125,7 +126,7 @@ def test_routing_k_max_and_trivial_pairs():
     assert info["max_k"] <= 10
     ks = [ctx.pair_k(int(a), int(b)) for a, b in zip(m.lit_a, m.lit_b)]
     simulated = sum(len(capi.cec_plan_window(plan, w)["pairs"]) for w in range(info["num_windows"]))
-    assert simulated == sum(1 for k in ks if k <= 10)
+    assert simulated == sum(1 for k, a, b in zip(ks, m.lit_a, m.lit_b) if k <= 10 and a != b)
     capi.cec_plan_free(plan)
 
 
@@ -172,7 +173,7 @@ def test_jit_codegen_compiles_for_sm100a_host_only():
     structure; C5's 256 copies share 3 random + 1 mul12 + bug-variant structures."""
     from workloads import circuits
     m = c5_big(copies=12, n_random=8, n_bugs=2, rand_pis=12, rand_ands=300, mul_n=6)
-    ctx = host_ctx(m.aig, engine=capi.CEC_ENGINE_JIT)
+    ctx = host_ctx(m.aig, engine=capi.CEC_ENGINE_JIT, k_s=12)  # merge inside a copy, never across
     plan = capi.cec_plan_exhaustive(ctx.handle, m.lit_a, m.lit_b)
     st = ctx.stats()
     n_struct = len(set(m.meta["types"]))
