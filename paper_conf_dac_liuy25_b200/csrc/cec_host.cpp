@@ -80,6 +80,9 @@ struct cec_ctx {
     std::vector<int32_t> last_verdict;
     std::vector<uint64_t> last_cex;
     std::vector<std::vector<uint32_t>> last_support;
+    // scratch for the schedule builder
+    std::vector<uint32_t> sc_stamp, sc_pos, sc_last, sc_slot;
+    uint32_t sc_epoch = 0;
     // scratch for traversals
     std::vector<uint32_t> stamp;
     uint32_t epoch = 0;
@@ -228,95 +231,107 @@ bool build_schedule(cec_ctx *c, const std::vector<uint32_t> &inputs, const std::
                     std::string &why) {
     const uint32_t k = (uint32_t)inputs.size();
     const uint32_t n = (uint32_t)nodes.size();
-    // position of each value: inputs -> k slots fixed at pass start; AND node t -> op order
-    std::unordered_map<uint32_t, uint32_t> node_pos;  // id -> index in `nodes`
-    node_pos.reserve(n * 2 + 16);
-    std::unordered_map<uint32_t, uint32_t> input_idx;
-    input_idx.reserve(k * 2 + 4);
-    for (uint32_t j = 0; j < k; ++j) input_idx[inputs[j]] = j;
-    for (uint32_t t = 0; t < n; ++t) node_pos[nodes[t]] = t;
-    auto def_pos = [&](uint32_t id) -> int64_t {  // -1 for inputs / const
-        auto it = node_pos.find(id);
-        if (it != node_pos.end() && !input_idx.count(id)) return (int64_t)it->second;
-        return -1;
-    };
-    // compare placement
-    std::vector<std::vector<uint32_t>> cmp_after(n + 1);  // index 0 = before any node
-    for (uint32_t ci : win_cmps) {
-        const Cmp &cm = cmps[ci];
-        int64_t p = std::max(def_pos(cm.la >> 1), def_pos(cm.lb >> 1));
-        cmp_after[(size_t)(p + 1)].push_back(ci);
+    // per-node scratch, valid where sc_stamp == ep (flat arrays: no hashing on the hot host path)
+    if (c->sc_stamp.size() != c->N()) {
+        c->sc_stamp.assign(c->N(), 0);
+        c->sc_pos.assign(c->N(), 0);
+        c->sc_last.assign(c->N(), 0);
+        c->sc_slot.assign(c->N(), 0);
     }
-    // op list: (is_cmp, index)
-    struct Op { bool cmp; uint32_t i; };
+    if (++c->sc_epoch == 0) {
+        std::fill(c->sc_stamp.begin(), c->sc_stamp.end(), 0u);
+        c->sc_epoch = 1;
+    }
+    const uint32_t ep = c->sc_epoch;
+    auto &stamp = c->sc_stamp;
+    auto &pos = c->sc_pos;    // 0 = input/const, t+1 = AND node t
+    auto &last = c->sc_last;  // last reading op + 1 (0 = never read)
+    auto &slot = c->sc_slot;
+    auto touch = [&](uint32_t id) {
+        if (stamp[id] != ep) {
+            stamp[id] = ep;
+            pos[id] = 0;
+            last[id] = 0;
+            slot[id] = 0xFFFFFFFFu;
+        }
+    };
+    touch(0);
+    for (uint32_t j = 0; j < k; ++j) touch(inputs[j]);
+    for (uint32_t t = 0; t < n; ++t) {
+        touch(nodes[t]);
+        pos[nodes[t]] = t + 1;
+    }
+    // compare placement: right after the later root (PAPER.md:118 compares per round; here per pass)
+    std::vector<uint32_t> cnt(n + 2, 0);
+    std::vector<uint32_t> cmp_at(win_cmps.size());
+    for (size_t i = 0; i < win_cmps.size(); ++i) {
+        const Cmp &cm = cmps[win_cmps[i]];
+        touch(cm.la >> 1);
+        touch(cm.lb >> 1);
+        cmp_at[i] = std::max(pos[cm.la >> 1], pos[cm.lb >> 1]);  // 0 = before any node
+        ++cnt[cmp_at[i] + 1];
+    }
+    for (uint32_t t = 1; t < n + 2; ++t) cnt[t] += cnt[t - 1];
+    std::vector<uint32_t> cmp_sorted(win_cmps.size());
+    {
+        std::vector<uint32_t> fill(cnt.begin(), cnt.end());
+        for (size_t i = 0; i < win_cmps.size(); ++i) cmp_sorted[fill[cmp_at[i]]++] = win_cmps[i];
+    }
+    // op order: cmps at 0, then node t followed by cmps at t+1
+    struct Op { uint32_t la, lb, id; bool cmp; };
     std::vector<Op> order;
     order.reserve(n + win_cmps.size());
-    for (uint32_t ci : cmp_after[0]) order.push_back({true, ci});
+    auto push_cmps = [&](uint32_t at) {
+        for (uint32_t i = cnt[at]; i < cnt[at + 1]; ++i) {
+            const Cmp &cm = cmps[cmp_sorted[i]];
+            order.push_back(Op{cm.la, cm.lb, cmp_sorted[i], true});
+        }
+    };
+    push_cmps(0);
     for (uint32_t t = 0; t < n; ++t) {
-        order.push_back({false, t});
-        for (uint32_t ci : cmp_after[t + 1]) order.push_back({true, ci});
+        const uint32_t id = nodes[t];
+        order.push_back(Op{c->f0[id], c->f1[id], id, false});
+        push_cmps(t + 1);
     }
-    // value key: id. last use (op index) of each value
-    std::unordered_map<uint32_t, uint32_t> last;
-    last.reserve((n + k) * 2 + 4);
     bool uses_const = false;
     for (uint32_t o = 0; o < order.size(); ++o) {
-        uint32_t a, b;
-        if (order[o].cmp) {
-            a = cmps[order[o].i].la >> 1;
-            b = cmps[order[o].i].lb >> 1;
-        } else {
-            uint32_t id = nodes[order[o].i];
-            a = c->f0[id] >> 1;
-            b = c->f1[id] >> 1;
+        const uint32_t a = order[o].la >> 1, b = order[o].lb >> 1;
+        if (stamp[a] != ep || stamp[b] != ep) {
+            why = "schedule: operand outside the window";
+            return false;
         }
-        last[a] = o;
-        last[b] = o;
+        last[a] = o + 1;
+        last[b] = o + 1;
         uses_const |= (a == 0 || b == 0);
     }
-    std::unordered_map<uint32_t, uint32_t> slot;
-    slot.reserve((n + k) * 2 + 4);
     std::vector<uint32_t> free_list;
     uint32_t next = k;
     for (uint32_t j = 0; j < k; ++j) slot[inputs[j]] = j;
-    if (uses_const && !input_idx.count(0)) {
+    bool const_is_input = false;
+    for (uint32_t j = 0; j < k; ++j) const_is_input |= inputs[j] == 0;
+    if (uses_const && !const_is_input) {
         out.const_slot = next++;
         slot[0] = out.const_slot;
     }
-    // inputs never read are free from the start (they are still written at pass start)
-    for (uint32_t j = 0; j < k; ++j)
-        if (!last.count(inputs[j])) free_list.push_back(j);
-    std::reverse(free_list.begin(), free_list.end());
+    for (uint32_t j = k; j-- > 0;)  // inputs never read are free from the start
+        if (!last[inputs[j]]) free_list.push_back(j);
     out.ops.clear();
     out.ops.reserve(order.size());
-    auto enc = [&](uint32_t lit) -> uint32_t {
-        auto it = slot.find(lit >> 1);
-        return (it->second << 1) | (lit & 1u);
-    };
     for (uint32_t o = 0; o < order.size(); ++o) {
-        uint32_t la, lb;
-        if (order[o].cmp) {
-            la = cmps[order[o].i].la;
-            lb = cmps[order[o].i].lb;
-        } else {
-            uint32_t id = nodes[order[o].i];
-            la = c->f0[id];
-            lb = c->f1[id];
-        }
-        if (!slot.count(la >> 1) || !slot.count(lb >> 1)) {
+        const Op &op = order[o];
+        const uint32_t va = op.la >> 1, vb = op.lb >> 1;
+        if (slot[va] == 0xFFFFFFFFu || slot[vb] == 0xFFFFFFFFu) {
             why = "schedule: operand not defined before use";
             return false;
         }
-        uint2 op;
-        op.x = enc(la) | (enc(lb) << 16);
-        // free operands whose last reader is this op (read-before-write inside the kernel)
-        uint32_t va = la >> 1, vb = lb >> 1;
-        if (last[va] == o) free_list.push_back(slot[va]);
-        if (vb != va && last[vb] == o) free_list.push_back(slot[vb]);
-        if (order[o].cmp) {
-            op.y = OP_CMP | order[o].i;
+        uint2 e;
+        e.x = (slot[va] << 1 | (op.la & 1u)) | ((slot[vb] << 1 | (op.lb & 1u)) << 16);
+        // free operands whose last reader is this op (the kernel reads before it writes)
+        if (last[va] == o + 1) free_list.push_back(slot[va]);
+        if (vb != va && last[vb] == o + 1) free_list.push_back(slot[vb]);
+        if (op.cmp) {
+            e.y = OP_CMP | op.id;
         } else {
-            uint32_t id = nodes[order[o].i];
             uint32_t s;
             if (!free_list.empty()) {
                 s = free_list.back();
@@ -328,11 +343,11 @@ bool build_schedule(cec_ctx *c, const std::vector<uint32_t> &inputs, const std::
                 why = "schedule: live set exceeds the slot field";
                 return false;
             }
-            slot[id] = s;
-            op.y = s;
-            if (!last.count(id)) free_list.push_back(s);  // value never read (not in a valid window)
+            slot[op.id] = s;
+            e.y = s;
+            if (!last[op.id]) free_list.push_back(s);  // never read (cannot happen in a window)
         }
-        out.ops.push_back(op);
+        out.ops.push_back(e);
     }
     out.nslots = std::max<uint32_t>(next, 1);
     return true;
@@ -653,15 +668,6 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
     for (int32_t j : win_jit) P->jit_windows += j >= 0;
     // work items: slices of each window split into chunks; interpreter windows grouped by slot
     // budget, JIT windows by structure; largest windows first inside a group
-    uint64_t total_slices = 0;
-    for (uint32_t w = 0; w < P->dwin.size(); ++w) {
-        uint64_t ttw = tt_words_of(P->dwin[w].k), sb, se;
-        cec_shard_range((ttw + 31) / 32, rank, world, &sb, &se);
-        total_slices += se - sb;
-    }
-    const uint64_t target_items = std::max<uint64_t>(1, (uint64_t)std::max(c->num_sms, 148) * 64);
-    uint64_t item_slices = std::max<uint64_t>(1, total_slices / target_items);
-    item_slices = std::min<uint64_t>(item_slices, 4096);
     std::map<uint32_t, std::vector<uint32_t>> buckets;   // interpreter: slot budget -> windows
     std::map<int32_t, std::vector<uint32_t>> jgroups;    // JIT: structure -> windows
     for (uint32_t w = 0; w < P->dwin.size(); ++w) {
@@ -673,8 +679,18 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         b = std::min(b, max_slot_cap);
         buckets[b].push_back(w);
     }
+    // Each launch is a persistent grid pulling items; size items per GROUP so even a one-window
+    // group (e.g. a bug-variant structure) splits into enough items to fill every SM.
     auto add_items = [&](std::vector<uint32_t> ws, bool jit) {
         std::stable_sort(ws.begin(), ws.end(), [&](uint32_t a, uint32_t b) { return cost_of[a] > cost_of[b]; });
+        uint64_t group_slices = 0;
+        for (uint32_t w : ws) {
+            uint64_t ttw = tt_words_of(P->dwin[w].k), sb, se;
+            cec_shard_range((ttw + 31) / 32, rank, world, &sb, &se);
+            group_slices += se - sb;
+        }
+        const uint64_t target = (uint64_t)std::max(c->num_sms, 148) * 16 /*resident warps*/ * 8;
+        const uint64_t item_slices = std::min<uint64_t>(4096, std::max<uint64_t>(1, group_slices / target));
         for (uint32_t w : ws) {
             uint64_t ttw = tt_words_of(P->dwin[w].k), sb, se;
             cec_shard_range((ttw + 31) / 32, rank, world, &sb, &se);
@@ -786,11 +802,59 @@ cec_status cec_plan_exhaustive(cec_ctx *c, uint32_t n, const uint32_t *la, const
     std::map<std::pair<uint32_t, uint32_t>, uint32_t> seen;
     std::map<std::vector<uint32_t>, uint32_t> by_support;  // identical supports share a window
     std::vector<WinHost> wins0;
-    std::vector<uint32_t> S;
-    for (uint32_t p = 0; p < n; ++p) {
+    for (uint32_t p = 0; p < n; ++p)
         if ((la[p] >> 1) >= c->N() || (lb[p] >> 1) >= c->N())
             return fail(c, CEC_E_ARG, "pair %u: literal out of range", p);
-        uint64_t cone = support_of(c, la[p], lb[p], S);
+    // a2: structural supports of all pairs, in parallel (independent TFI walks, own scratch each)
+    std::vector<std::vector<uint32_t>> supp(n);
+    std::vector<uint64_t> cones(n, 0);
+    {
+        const unsigned hw = std::max(1u, std::min(16u, std::thread::hardware_concurrency()));
+        const unsigned nt = (unsigned)std::min<uint64_t>(hw, (n + 63) / 64);
+        std::atomic<uint32_t> next{0};
+        auto work = [&]() {
+            std::vector<uint32_t> stamp(c->N(), 0), st;
+            uint32_t ep = 0;
+            for (uint32_t p; (p = next.fetch_add(1)) < n;) {
+                ++ep;
+                auto &S = supp[p];
+                uint64_t nodes = 0;
+                st.clear();
+                for (uint32_t r : {la[p] >> 1, lb[p] >> 1})
+                    if (stamp[r] != ep) {
+                        stamp[r] = ep;
+                        st.push_back(r);
+                    }
+                while (!st.empty()) {
+                    const uint32_t v = st.back();
+                    st.pop_back();
+                    if (v >= 1 && v <= c->I) {
+                        S.push_back(v);
+                        continue;
+                    }
+                    if (v == 0) continue;
+                    ++nodes;
+                    for (uint32_t f : {c->f0[v] >> 1, c->f1[v] >> 1})
+                        if (stamp[f] != ep) {
+                            stamp[f] = ep;
+                            st.push_back(f);
+                        }
+                }
+                std::sort(S.begin(), S.end());
+                cones[p] = nodes;
+            }
+        };
+        if (nt <= 1) {
+            work();
+        } else {
+            std::vector<std::thread> pool;
+            for (unsigned t = 0; t < nt; ++t) pool.emplace_back(work);
+            for (auto &th : pool) th.join();
+        }
+    }
+    for (uint32_t p = 0; p < n; ++p) {
+        const std::vector<uint32_t> &S = supp[p];
+        const uint64_t cone = cones[p];
         P->k[p] = (uint32_t)S.size();
         if (la[p] == lb[p]) {
             P->pre_verdict[p] = CEC_EQUIVALENT;

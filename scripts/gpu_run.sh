@@ -1,0 +1,14 @@
+# usage: bash scripts/gpu_run.sh  (runs on the GPU box from the repo root; outputs under gpurun_out/)
+set -x
+mkdir -p gpurun_out
+nvidia-smi > gpurun_out/smi.txt 2>&1
+python -c "import __graft_entry__ as g; g.build(); g.smoke()" > gpurun_out/smoke.log 2>&1
+timeout 1500 python -m pytest tests -m gpu -q -rf -x > gpurun_out/pytest_gpu.log 2>&1
+timeout 600 python bench.py --steps 5 --warmup 3 > gpurun_out/bench.log 2>&1
+timeout 600 python bench.py --steps 3 --warmup 3 --engine 1 --no-cpu-baseline > gpurun_out/bench_interp.log 2>&1
+timeout 300 python bench.py --config c2 --steps 5 --warmup 3 --no-cpu-baseline > gpurun_out/bench_c2.log 2>&1
+timeout 300 python bench.py --config c2 --steps 5 --warmup 3 --engine 1 --no-cpu-baseline > gpurun_out/bench_c2_interp.log 2>&1
+timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches.csv python bench.py --steps 2 --warmup 3 --no-cpu-baseline --e2e-steps 1 > gpurun_out/b_ncu.log 2>&1
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:cecjit -s 3 -c 1 -o gpurun_out/prof_jit_c2 python bench.py --config c2 --steps 1 --warmup 3 --no-cpu-baseline --e2e-steps 1 > gpurun_out/ncu_full_c2.log 2>&1
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:interp -s 3 -c 1 -o gpurun_out/prof_interp_c2 python bench.py --config c2 --engine 1 --steps 1 --warmup 3 --no-cpu-baseline --e2e-steps 1 > gpurun_out/ncu_full_c2i.log 2>&1
+echo done
