@@ -82,9 +82,15 @@ typedef struct {
 typedef struct {
     int32_t device;            /* CUDA device ordinal; -1 = host-only context (no simulation) */
     int32_t rank, world;       /* world > 1: SPMD over `world` GPUs; every rank passes the same
-                                  AIG, pairs and options; results are identical on every rank */
-    const void *nccl_unique_id;/* 128-byte ncclUniqueId (required when world > 1); the caller
-                                  bootstraps it, e.g. through torch.distributed */
+                                  AIG, pairs and options; rank r simulates its contiguous share of
+                                  every window's pattern slices */
+    const void *nccl_unique_id;/* 128-byte ncclUniqueId for world > 1 (the caller bootstraps it,
+                                  e.g. through torch.distributed): one ncclAllReduce(min) of the
+                                  per-pair first-mismatch indices makes the results identical on
+                                  every rank. NULL with world > 1 = shard-only mode: no collective;
+                                  results cover this rank's slices only (NOT_EQUIVALENT iff a CEX
+                                  lies in them, with the minimum such index) and the caller combines
+                                  ranks by taking the per-pair minimum index */
     void *stream;              /* cudaStream_t to launch on, or NULL for the library's own stream */
     uint32_t k_max;            /* exhaustive support limit, <= 63. Default 32 (= k_P) */
     uint32_t k_s;              /* window-merge threshold; 0 = k_max */
@@ -137,6 +143,14 @@ cec_status cec_sim_exhaustive(cec_ctx *ctx, uint32_t num_pairs, const uint32_t *
  * leaf, in which case the call returns CEC_E_CUT after filling every other verdict. */
 cec_status cec_check_local_cuts(cec_ctx *ctx, uint32_t num_checks, const uint32_t *lit_a, const uint32_t *lit_b,
                                 const uint32_t *cut_off, const uint32_t *cut_leaves, int32_t *verdict_out);
+
+/* Partial random simulation (PAPER.md:41 §II-B, :61, :183): simulate every node on num_words*32
+ * random patterns (PI id i, word w gets the low 32 bits of splitmix64(seed ^ (i << 32) ^ w)) on the
+ * GPU and write one 64-bit signature per node id to sig_out[1+num_pis+num_ands], canonical under
+ * complement: phase_out[id] = 1 if the node evaluates to 1 on pattern 0 and was complemented
+ * before hashing. Nodes with equal signatures are candidate-equivalent (equivalence classes,
+ * representative = minimum id); a signature is a filter, never a proof. */
+cec_status cec_sim_random(cec_ctx *ctx, uint32_t num_words, uint64_t seed, uint64_t *sig_out, uint8_t *phase_out);
 
 /* Counter-example of pair `pair_idx` of the most recent cec_sim_exhaustive / cec_plan_results:
  * pi_values_out[i] = value of PI id i+1 (0/1): PI S[j] = bit j of the CEX index, every other PI 0.

@@ -27,7 +27,7 @@ STATUS_NAMES = ["CEC_OK", "CEC_E_ARG", "CEC_E_AIG", "CEC_E_CUT", "CEC_E_NOMEM", 
 EXPORTS = ["cec_default_opts", "cec_load_aig", "cec_sim_exhaustive", "cec_check_local_cuts", "cec_get_cex",
            "cec_pair_support", "cec_plan_exhaustive", "cec_plan_run", "cec_plan_results", "cec_plan_info",
            "cec_plan_window", "cec_plan_free", "cec_stream", "cec_get_stats", "cec_shard_range", "cec_pext64",
-           "cec_free", "cec_last_error", "cec_abi_version", "cec_nccl_unique_id"]
+           "cec_free", "cec_last_error", "cec_abi_version", "cec_nccl_unique_id", "cec_sim_random"]
 
 
 class CecOpts(ctypes.Structure):
@@ -86,6 +86,7 @@ def _load() -> ctypes.CDLL:
         "cec_last_error": (ctypes.c_char_p, [P]),
         "cec_abi_version": (ctypes.c_int, []),
         "cec_nccl_unique_id": (ctypes.c_int, [P]),
+        "cec_sim_random": (ctypes.c_int, [P, u32, u64, P, P]),
     }
     for name, (res, args) in sig.items():
         fn = getattr(L, name)
@@ -164,6 +165,14 @@ def cec_check_local_cuts(ctx, lit_a, lit_b, cut_off, cut_leaves, raise_on_bad_cu
         return v[:n]
     _check(st, ctx)
     return v[:n]
+
+
+def cec_sim_random(ctx, num_nodes: int, num_words: int = 64, seed: int = 1):
+    """Per-node complement-canonical random-simulation signatures (uint64[N]) and phases (uint8[N])."""
+    sig = np.zeros(max(num_nodes, 1), np.uint64)
+    ph = np.zeros(max(num_nodes, 1), np.uint8)
+    _check(lib.cec_sim_random(ctx, num_words, seed, _p(sig), _p(ph)), ctx)
+    return sig[:num_nodes], ph[:num_nodes]
 
 
 def cec_get_cex(ctx, pair_idx: int, num_pis: int) -> np.ndarray:

@@ -15,6 +15,7 @@
 #include <atomic>
 #include <chrono>
 #include <cstdarg>
+#include <cstdlib>
 #include <cstdio>
 #include <cstring>
 #include <map>
@@ -80,6 +81,9 @@ struct cec_ctx {
     std::vector<int32_t> last_verdict;
     std::vector<uint64_t> last_cex;
     std::vector<std::vector<uint32_t>> last_support;
+    // device copy of the AIG for random simulation (lazy)
+    uint32_t *d_f0 = nullptr, *d_f1 = nullptr, *d_level_ids = nullptr;
+    std::vector<uint32_t> level_off;
     // scratch for the schedule builder
     std::vector<uint32_t> sc_stamp, sc_pos, sc_last, sc_slot;
     uint32_t sc_epoch = 0;
@@ -453,9 +457,8 @@ cec_status cec_load_aig(cec_ctx **out, const cec_aig *aig, const cec_opts *opts)
             return CEC_E_CUDA;
         }
         c->stream = c->opts.stream ? c->opts.stream : c->own_stream;
-        if (c->opts.world > 1) {
-            if (!c->opts.nccl_unique_id) return CEC_E_ARG;
-            if (!g_nccl.load()) return CEC_E_NCCL;
+        if (c->opts.world > 1 && c->opts.nccl_unique_id) {  // NULL id: shard-only mode, no collective
+            if (!g_nccl.load()) return fail(nullptr, CEC_E_NCCL, "NCCL library not found");
             ncclUniqueId uid;
             std::memcpy(&uid, c->opts.nccl_unique_id, sizeof uid);
             ncclResult_t r = g_nccl.init_rank(&c->comm, c->opts.world, uid, c->opts.rank);
@@ -468,6 +471,9 @@ cec_status cec_load_aig(cec_ctx **out, const cec_aig *aig, const cec_opts *opts)
 
 void cec_free(cec_ctx *ctx) {
     if (!ctx) return;
+    dev_free(ctx->d_f0);
+    dev_free(ctx->d_f1);
+    dev_free(ctx->d_level_ids);
     if (ctx->comm && g_nccl.destroy) g_nccl.destroy(ctx->comm);
     if (ctx->own_stream) stream_destroy(ctx->own_stream);
     delete ctx;
@@ -499,7 +505,13 @@ cec_status cec_pair_support(cec_ctx *ctx, uint32_t la, uint32_t lb, uint32_t *su
 namespace {
 
 constexpr int32_t DECIDED_BY_SIM = -100;
-constexpr int JIT_MIN_BLOCKS = 4;  // 128-thread blocks -> <= 128 registers per thread
+JitConfig jit_config() {  // overridable for tuning: CEC_JIT_THREADS / CEC_JIT_MINB / CEC_JIT_SYNC
+    JitConfig cfg;
+    if (const char *e = getenv("CEC_JIT_THREADS")) cfg.threads = atoi(e);
+    if (const char *e = getenv("CEC_JIT_MINB")) cfg.min_blocks = atoi(e);
+    if (const char *e = getenv("CEC_JIT_SYNC")) cfg.sync_every = atoi(e);
+    return cfg;
+}
 
 uint64_t tt_words_of(uint32_t k) { return k <= 5 ? 1ull : (1ull << (k - 5)); }
 
@@ -548,12 +560,37 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         if (stop_mark.size() != c->N()) stop_mark.assign(c->N(), 0);
         const uint32_t sep = (uint32_t)w + 1;
         for (uint32_t x : W.inputs) stop_mark[x] = sep;
+        // Node order = a topological order chosen to keep the live set small (it sets the
+        // interpreter's shared-memory slots and the JIT kernel's register pressure): depth-first
+        // post-order from the roots, compare by compare, deeper fanin first (Sethi-Ullman style).
         std::vector<uint32_t> nodes;
-        walk_tfi(c, roots.data(), (int)roots.size(), &stop_mark, sep, [&](uint32_t v) {
-            if (c->is_and(v) && stop_mark[v] != sep) nodes.push_back(v);
-        });
+        {
+            const uint32_t ep = c->next_epoch();
+            std::vector<std::pair<uint32_t, uint8_t>> st;
+            for (uint32_t r : roots) {
+                if (c->stamp[r] == ep || !c->is_and(r) || stop_mark[r] == sep) continue;
+                st.push_back({r, 0});
+                c->stamp[r] = ep;
+                while (!st.empty()) {
+                    auto &top = st.back();
+                    const uint32_t v = top.first;
+                    if (top.second < 2) {
+                        uint32_t a = c->f0[v] >> 1, b = c->f1[v] >> 1;
+                        if (c->level[b] > c->level[a]) std::swap(a, b);  // deeper first
+                        const uint32_t nxt = top.second == 0 ? a : b;
+                        ++top.second;
+                        if (c->stamp[nxt] != ep && c->is_and(nxt) && stop_mark[nxt] != sep) {
+                            c->stamp[nxt] = ep;
+                            st.push_back({nxt, 0});
+                        }
+                    } else {
+                        nodes.push_back(v);
+                        st.pop_back();
+                    }
+                }
+            }
+        }
         for (uint32_t x : W.inputs) stop_mark[x] = 0;
-        std::sort(nodes.begin(), nodes.end());
         // own-support masks (a11 pext)
         for (uint32_t ci : wc) {
             Cmp &cm = cmps2[ci];
@@ -570,6 +607,16 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         Sched sc;
         std::string why;
         if (!build_schedule(c, W.inputs, nodes, cmps2, wc, sc, why)) return fail(c, CEC_E_NOMEM, "%s", why.c_str());
+        {  // the id order (the netlist's own construction order) is often the better one: keep the
+           // order with the smaller live set
+            std::vector<uint32_t> by_id(nodes);
+            std::sort(by_id.begin(), by_id.end());
+            Sched sc2;
+            if (build_schedule(c, W.inputs, by_id, cmps2, wc, sc2, why) && sc2.nslots < sc.nslots) {
+                sc = std::move(sc2);
+                nodes.swap(by_id);
+            }
+        }
         if (sc.nslots > max_slot_cap)
             return fail(c, CEC_E_NOMEM, "window %zu needs %u live slots > %u (on-chip capacity)", w, sc.nslots,
                         max_slot_cap);
@@ -639,6 +686,8 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         if (pc >= 0) pc = remap[pc];
     // compile the distinct JIT structures (in parallel; cached process-wide by structure)
     std::vector<JitKernel *> kernels(jit_progs.size(), nullptr);
+    const JitConfig jcfg = jit_config();
+    const uint64_t jit_pass = jcfg.sync_every > 0 ? (uint64_t)jcfg.threads / 32 : 1;
     P->jit_ms = 0.f;
     if (!jit_progs.empty()) {
         auto t0 = std::chrono::steady_clock::now();
@@ -651,13 +700,13 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         for (unsigned t = 0; t < std::min<size_t>(hw, jit_progs.size()); ++t)
             pool.emplace_back([&]() {
                 for (size_t i; (i = next.fetch_add(1)) < jit_progs.size();)
-                    errs[i] = jit_get_kernel(jit_progs[i], JIT_MIN_BLOCKS, false, &kernels[i]);
+                    errs[i] = jit_get_kernel(jit_progs[i], jcfg, false, &kernels[i]);
             });
         for (auto &th : pool) th.join();
         for (size_t i = 0; i < jit_progs.size(); ++i) {
             if (errs[i]) return fail(c, CEC_E_CUDA, "JIT: %s", errs[i]);
             if (load) {
-                const char *e = jit_get_kernel(jit_progs[i], JIT_MIN_BLOCKS, true, &kernels[i]);
+                const char *e = jit_get_kernel(jit_progs[i], jcfg, true, &kernels[i]);
                 if (e) return fail(c, CEC_E_CUDA, "JIT load: %s", e);
             }
         }
@@ -690,7 +739,9 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
             group_slices += se - sb;
         }
         const uint64_t target = (uint64_t)std::max(c->num_sms, 148) * 16 /*resident warps*/ * 8;
-        const uint64_t item_slices = std::min<uint64_t>(4096, std::max<uint64_t>(1, group_slices / target));
+        uint64_t item_slices = std::min<uint64_t>(4096, std::max<uint64_t>(1, group_slices / target));
+        if (jit && jit_pass > 1)  // block-synchronous JIT: whole passes of one slice per warp
+            item_slices = std::max<uint64_t>(jit_pass, (item_slices * 16 + jit_pass - 1) / jit_pass * jit_pass);
         for (uint32_t w : ws) {
             uint64_t ttw = tt_words_of(P->dwin[w].k), sb, se;
             cec_shard_range((ttw + 31) / 32, rank, world, &sb, &se);
@@ -929,6 +980,9 @@ cec_status cec_plan_exhaustive(cec_ctx *c, uint32_t n, const uint32_t *la, const
     auto t1 = std::chrono::steady_clock::now();
     P->host_ms = std::chrono::duration<float, std::milli>(t1 - t0).count();
     c->stats.host_prep_ms = P->host_ms;
+    c->stats.node_patterns = P->W_rank;
+    c->stats.node_patterns_all = P->W_all;
+    c->stats.num_windows = (uint32_t)P->dwin.size();
     c->stats.jit_ms = P->jit_ms;
     c->stats.jit_kernels = P->jit_kernels;
     c->stats.jit_windows = P->jit_windows;
@@ -950,7 +1004,7 @@ cec_status cec_plan_run(cec_ctx *c, cec_plan *P) {
     const char *e = launch_run(P->d, P->groups, (uint32_t)P->dwin.size(), (uint32_t)P->cmps.size(), c->stream,
                                   c->num_sms, &nl);
     if (e) return fail(c, CEC_E_CUDA, "CUDA: %s (kernel launch)", e);
-    if (c->opts.world > 1 && !P->cmps.empty()) {  // a10: one NCCL min all-reduce of first_idx
+    if (c->comm && !P->cmps.empty()) {  // a10: one NCCL min all-reduce of first_idx
         ncclResult_t r = g_nccl.all_reduce(P->d.first, P->d.first, P->cmps.size(), ncclUint64, ncclMin, c->comm,
                                            (cudaStream_t)c->stream);
         if (r != ncclSuccess) return fail(c, CEC_E_NCCL, "NCCL: %s", g_nccl.err(r));
@@ -1062,6 +1116,50 @@ cec_status cec_sim_exhaustive(cec_ctx *c, uint32_t n, const uint32_t *la, const 
     if (st == CEC_OK) st = cec_plan_results(c, P, verdict, cex, k_out);
     cec_plan_free(P);
     return st;
+}
+
+cec_status cec_sim_random(cec_ctx *c, uint32_t W, uint64_t seed, uint64_t *sig_out, uint8_t *phase_out) {
+    if (!c || !sig_out || W == 0) return fail(c, CEC_E_ARG, "null argument or num_words == 0");
+    if (c->host_only) return fail(c, CEC_E_CUDA, "host-only context: no CUDA device (no CPU fallback)");
+    const uint32_t N = c->N();
+    if (!c->d_f0) {  // AIG and level CSR on the device (a1)
+        uint32_t maxl = 0;
+        for (uint32_t id = 0; id < N; ++id) maxl = std::max(maxl, c->level[id]);
+        c->level_off.assign(maxl + 2, 0);
+        for (uint32_t id = 1 + c->I; id < N; ++id) ++c->level_off[c->level[id] + 1];
+        for (size_t l = 1; l < c->level_off.size(); ++l) c->level_off[l] += c->level_off[l - 1];
+        std::vector<uint32_t> ids(std::max<uint32_t>(1, c->A)), fill(c->level_off.begin(), c->level_off.end());
+        for (uint32_t id = 1 + c->I; id < N; ++id) ids[fill[c->level[id]]++] = id;
+        CUDA_TRY(c, dev_alloc((void **)&c->d_f0, sizeof(uint32_t) * N));
+        CUDA_TRY(c, dev_alloc((void **)&c->d_f1, sizeof(uint32_t) * N));
+        CUDA_TRY(c, dev_alloc((void **)&c->d_level_ids, sizeof(uint32_t) * ids.size()));
+        CUDA_TRY(c, h2d(c->d_f0, c->f0.data(), sizeof(uint32_t) * N, c->stream));
+        CUDA_TRY(c, h2d(c->d_f1, c->f1.data(), sizeof(uint32_t) * N, c->stream));
+        CUDA_TRY(c, h2d(c->d_level_ids, ids.data(), sizeof(uint32_t) * ids.size(), c->stream));
+        CUDA_TRY(c, stream_sync(c->stream));
+    }
+    uint32_t *tt = nullptr;
+    unsigned long long *sig = nullptr;
+    uint8_t *ph = nullptr;
+    struct Guard {
+        void **p[3];
+        ~Guard() {
+            for (auto q : p) dev_free(*q);
+        }
+    } guard{{(void **)&tt, (void **)&sig, (void **)&ph}};
+    CUDA_TRY(c, dev_alloc((void **)&tt, sizeof(uint32_t) * (size_t)N * W));
+    CUDA_TRY(c, dev_alloc((void **)&sig, sizeof(unsigned long long) * N));
+    CUDA_TRY(c, dev_alloc((void **)&ph, N));
+    uint32_t nl = 0;
+    const char *e = random_sim(c->d_f0, c->d_f1, c->d_level_ids, c->level_off, c->I, N, W, seed, tt, sig, ph, c->stream,
+                               c->num_sms, &nl);
+    if (e) return fail(c, CEC_E_CUDA, "CUDA: %s (random simulation)", e);
+    CUDA_TRY(c, d2h(sig_out, sig, sizeof(unsigned long long) * N, c->stream));
+    std::vector<uint8_t> phase(N);
+    CUDA_TRY(c, d2h(phase.data(), ph, N, c->stream));
+    CUDA_TRY(c, stream_sync(c->stream));
+    if (phase_out) std::memcpy(phase_out, phase.data(), N);
+    return CEC_OK;
 }
 
 cec_status cec_get_cex(cec_ctx *c, uint32_t p, uint8_t *pis) {

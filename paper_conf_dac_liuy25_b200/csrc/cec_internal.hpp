@@ -50,6 +50,11 @@ struct JItem {             // a slice range of one JIT window instance
     uint32_t cmp_off;      // first[] index of the window's compare 0
 };
 struct JitKernel;
+struct JitConfig {
+    int threads = 512;      // threads per block
+    int min_blocks = 1;     // __launch_bounds__ min blocks per SM (registers <= 64K / (threads*min_blocks))
+    int sync_every = 256;   // block-synchronous: __syncthreads() every this many nodes; 0 = warp-independent
+};
 struct LaunchGroup {       // windows sharing one kernel launch
     uint32_t nslots;       // interpreter: slots per warp in this launch
     uint32_t item_off, nitems;
@@ -70,12 +75,19 @@ struct DevPlan {
 
 // jit.cpp
 std::string jit_key(const JitProgram &p);
-std::string jit_source(const JitProgram &p, int min_blocks);
+std::string jit_source(const JitProgram &p, const JitConfig &cfg);
 const char *jit_compile_cubin(const std::string &src, std::vector<char> &cubin, std::string &log);
-const char *jit_get_kernel(const JitProgram &p, int min_blocks, bool load, JitKernel **out);
+const char *jit_get_kernel(const JitProgram &p, const JitConfig &cfg, bool load, JitKernel **out);
 double jit_compile_ms(const JitKernel *k);
+int jit_slices_per_pass(const JitKernel *k);
 const char *jit_launch(JitKernel *K, const JItem *items, uint32_t nitems, uint32_t *ctr, unsigned long long *first,
                        unsigned long long *bound, uint32_t *neq_cnt, void *stream, int num_sms);
+
+// sim_random.cu
+const char *random_sim(const uint32_t *d_f0, const uint32_t *d_f1, const uint32_t *d_level_ids,
+                       const std::vector<uint32_t> &level_off, uint32_t I, uint32_t N, uint32_t W, uint64_t seed,
+                       uint32_t *d_tt, unsigned long long *d_sig, uint8_t *d_phase, void *stream, int num_sms,
+                       uint32_t *launches);
 
 // sim_interp.cu
 const char *launch_run(const DevPlan &d, const std::vector<LaunchGroup> &groups, uint32_t nwin, uint32_t ncmp,

@@ -21,7 +21,9 @@
 #include <algorithm>
 #include <chrono>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
+#include <functional>
 #include <map>
 #include <memory>
 #include <mutex>
@@ -91,6 +93,7 @@ struct JitKernel {
     cudaKernel_t kern = nullptr;
     int block = 128;
     int blocks_per_sm = 0;
+    int slices_per_pass = 1;  // block-synchronous kernels: warps per block
     double compile_ms = 0;
     size_t src_bytes = 0, cubin_bytes = 0;
 };
@@ -107,11 +110,13 @@ std::string jit_key(const JitProgram &p) {
     return key;
 }
 
-std::string jit_source(const JitProgram &p, int min_blocks) {
+std::string jit_source(const JitProgram &p, const JitConfig &cfg) {
     const uint32_t n = (uint32_t)(p.nodes.size() / 2), ncmp = (uint32_t)(p.cmps.size() / 2);
+    const bool block_sync = cfg.sync_every > 0;
+    const int nw = cfg.threads / 32;
     std::string s;
     s.reserve(96 * (size_t)n + 160 * (size_t)ncmp + 4096);
-    char buf[256];
+    char buf[1024];
     s += "typedef unsigned int u32; typedef unsigned long long u64;\n"
          "struct JItem { u32 win, s_begin, s_end, cmp_off; };\n"
          "__device__ __noinline__ void rep(u32 d, u32 c, u32 win, u32 s, u32 lane, u32 ncmp, u32 cmp_off,\n"
@@ -131,20 +136,43 @@ std::string jit_source(const JitProgram &p, int min_blocks) {
          "  atomicMin(&bound[win], mx);\n"
          "}\n";
     snprintf(buf, sizeof buf,
-             "extern \"C\" __global__ void __launch_bounds__(128, %d) cecjit(const JItem *__restrict__ items, u32 nitems,\n"
-             "    u32 *ctr, u64 *first, u64 *bound, u32 *neq_cnt) {\n",
-             min_blocks);
+             "extern \"C\" __global__ void __launch_bounds__(%d, %d) cecjit(const JItem *__restrict__ items, u32 nitems,\n"
+             "    u32 *ctr, u64 *first, u64 *bound, u32 *neq_cnt) {\n"
+             "  const u32 lane = threadIdx.x & 31u;\n",
+             cfg.threads, cfg.min_blocks);
     s += buf;
-    s += "  const u32 lane = threadIdx.x & 31u;\n"
-         "  for (;;) {\n"
-         "    u32 it = 0;\n"
-         "    if (lane == 0u) it = atomicAdd(ctr, 1u);\n"
-         "    it = __shfl_sync(0xFFFFFFFFu, it, 0);\n"
-         "    if (it >= nitems) return;\n"
-         "    const JItem I = items[it];\n"
-         "    for (u32 s = I.s_begin; s < I.s_end; ++s) {\n"
-         "      if (((u64)s << 10) >= *((volatile u64 *)&bound[I.win])) break;\n"
-         "      const u64 word = ((u64)s << 5) + lane;\n";
+    if (!block_sync) {
+        // every warp independent: pulls items itself, one 32-word slice per pass
+        s += "  for (;;) {\n"
+             "    u32 it = 0;\n"
+             "    if (lane == 0u) it = atomicAdd(ctr, 1u);\n"
+             "    it = __shfl_sync(0xFFFFFFFFu, it, 0);\n"
+             "    if (it >= nitems) return;\n"
+             "    const JItem I = items[it];\n"
+             "    for (u32 s = I.s_begin; s < I.s_end; ++s) {\n"
+             "      if (((u64)s << 10) >= *((volatile u64 *)&bound[I.win])) break;\n"
+             "      const bool live = true;\n";
+    } else {
+        // block-synchronous: the block pulls an item and its warps take consecutive slices; a
+        // __syncthreads() every few hundred nodes keeps all warps of the SM inside the same stretch
+        // of the (large, straight-line) program so instruction-cache lines are shared, not thrashed
+        snprintf(buf, sizeof buf,
+                 "  const u32 warp = threadIdx.x >> 5;\n"
+                 "  __shared__ u32 s_it; __shared__ JItem s_item;\n"
+                 "  for (;;) {\n"
+                 "    if (threadIdx.x == 0u) { const u32 t = atomicAdd(ctr, 1u); s_it = t; if (t < nitems) s_item = items[t]; }\n"
+                 "    __syncthreads();\n"
+                 "    const u32 it = s_it;\n"
+                 "    if (it >= nitems) return;\n"
+                 "    const JItem I = s_item;\n"
+                 "    for (u32 s0 = I.s_begin; s0 < I.s_end; s0 += %du) {\n"
+                 "      const u32 s = s0 + warp;\n"
+                 "      const bool live = s < I.s_end && ((u64)s << 10) < *((volatile u64 *)&bound[I.win]);\n"
+                 "      if (!__syncthreads_or(live)) break;\n",
+                 nw);
+        s += buf;
+    }
+    s += "      const u64 word = ((u64)s << 5) + lane;\n";
     for (uint32_t j = 0; j < p.k; ++j) {
         if (j < 5)
             snprintf(buf, sizeof buf, "      const u32 x%u = %s;\n", j, kMask[j]);
@@ -163,7 +191,7 @@ std::string jit_source(const JitProgram &p, int min_blocks) {
         const uint32_t a = p.cmps[2 * c], b = p.cmps[2 * c + 1];
         const bool inv = ((a ^ b) & 1u) != 0;
         snprintf(buf, sizeof buf,
-                 "      { const u32 d = %s%s ^ %s%s; if (__any_sync(0xFFFFFFFFu, d != 0u)) rep(d, %uu, I.win, s, lane, %uu, I.cmp_off, first, bound, neq_cnt); }\n",
+                 "      { const u32 d = live ? (%s%s ^ %s%s) : 0u; if (__any_sync(0xFFFFFFFFu, d != 0u)) rep(d, %uu, I.win, s, lane, %uu, I.cmp_off, first, bound, neq_cnt); }\n",
                  inv ? "~(" : "", ref_name(p, a >> 1).c_str(), ref_name(p, b >> 1).c_str(), inv ? ")" : "", c, ncmp);
         s += buf;
     };
@@ -176,8 +204,9 @@ std::string jit_source(const JitProgram &p, int min_blocks) {
                  t, L, t, ref_name(p, a >> 1).c_str(), ref_name(p, b >> 1).c_str());
         s += buf;
         for (uint32_t c : after[t + 1]) emit_cmp(c);
+        if (block_sync && (t + 1) % (uint32_t)cfg.sync_every == 0 && t + 1 < n) s += "      __syncthreads();\n";
     }
-    s += "    }\n  }\n}\n";
+    s += block_sync ? "    }\n    __syncthreads();\n  }\n}\n" : "    }\n  }\n}\n";
     return s;
 }
 
@@ -210,8 +239,10 @@ namespace {
 std::map<std::string, std::unique_ptr<JitKernel>> g_cache;  // process-wide, keyed by structure
 }
 
-const char *jit_get_kernel(const JitProgram &p, int min_blocks, bool load, JitKernel **out) {
-    const std::string key = jit_key(p) + std::string(1, (char)min_blocks);
+const char *jit_get_kernel(const JitProgram &p, const JitConfig &cfg, bool load, JitKernel **out) {
+    char ck[64];
+    snprintf(ck, sizeof ck, "|%d,%d,%d", cfg.threads, cfg.min_blocks, cfg.sync_every);
+    const std::string key = jit_key(p) + ck;
     {
         std::lock_guard<std::mutex> g(g_mu);
         auto it = g_cache.find(key);
@@ -221,7 +252,7 @@ const char *jit_get_kernel(const JitProgram &p, int min_blocks, bool load, JitKe
         }
     }
     auto t0 = std::chrono::steady_clock::now();
-    const std::string src = jit_source(p, min_blocks);
+    const std::string src = jit_source(p, cfg);
     std::vector<char> cubin;
     std::string log;
     const char *e = jit_compile_cubin(src, cubin, log);
@@ -230,7 +261,23 @@ const char *jit_get_kernel(const JitProgram &p, int min_blocks, bool load, JitKe
         msg = std::string(e) + ": " + log.substr(0, 400);
         return msg.c_str();
     }
+    if (const char *dir = getenv("CEC_JIT_DUMP")) {  // inspection: cuobjdump -sass <dir>/cecjit_*.cubin
+        const size_t h = std::hash<std::string>()(key);
+        char path[512];
+        snprintf(path, sizeof path, "%s/cecjit_%016zx.cu", dir, h);
+        if (FILE *f = fopen(path, "w")) {
+            fwrite(src.data(), 1, src.size(), f);
+            fclose(f);
+        }
+        snprintf(path, sizeof path, "%s/cecjit_%016zx.cubin", dir, h);
+        if (FILE *f = fopen(path, "wb")) {
+            fwrite(cubin.data(), 1, cubin.size(), f);
+            fclose(f);
+        }
+    }
     std::unique_ptr<JitKernel> K(new JitKernel());
+    K->block = cfg.threads;
+    K->slices_per_pass = cfg.sync_every > 0 ? cfg.threads / 32 : 1;
     K->src_bytes = src.size();
     K->cubin_bytes = cubin.size();
     if (load) {
@@ -252,13 +299,14 @@ const char *jit_get_kernel(const JitProgram &p, int min_blocks, bool load, JitKe
 }
 
 double jit_compile_ms(const JitKernel *k) { return k ? k->compile_ms : 0.0; }
+int jit_slices_per_pass(const JitKernel *k) { return k ? k->slices_per_pass : 1; }
 
 const char *jit_launch(JitKernel *K, const JItem *items, uint32_t nitems, uint32_t *ctr, unsigned long long *first,
                        unsigned long long *bound, uint32_t *neq_cnt, void *stream, int num_sms) {
     if (!K || !K->kern) return "JIT kernel not loaded";
     if (nitems == 0) return nullptr;
     uint64_t grid = (uint64_t)num_sms * K->blocks_per_sm;
-    const uint64_t need = (nitems + (K->block / 32) - 1) / (K->block / 32);
+    const uint64_t need = K->slices_per_pass > 1 ? nitems : (nitems + (K->block / 32) - 1) / (K->block / 32);
     if (grid > need) grid = need;
     void *args[] = {(void *)&items, (void *)&nitems, (void *)&ctr, (void *)&first, (void *)&bound, (void *)&neq_cnt};
     cudaError_t e = cudaLaunchKernel((const void *)K->kern, dim3((unsigned)grid), dim3(K->block), args, 0,
