@@ -53,7 +53,7 @@ struct JitKernel;
 struct JitConfig {
     int threads = 512;      // threads per block
     int min_blocks = 1;     // __launch_bounds__ min blocks per SM (registers <= 64K / (threads*min_blocks))
-    int sync_every = 256;   // block-synchronous: __syncthreads() every this many nodes; 0 = warp-independent
+    int sync_every = 512;   // block-synchronous: __syncthreads() every this many nodes; 0 = warp-independent
 };
 struct LaunchGroup {       // windows sharing one kernel launch
     uint32_t nslots;       // interpreter: slots per warp in this launch

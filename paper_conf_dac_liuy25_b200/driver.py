@@ -1,0 +1,297 @@
+"""Host driver above the C ABI: the simulation-based CEC flow of PAPER.md §III-D (Fig. 5, :179-187).
+
+  P phase  PO pairs with support <= k_P (all) or <= k_p (subset) -> cec_sim_exhaustive
+  ECs partial random simulation on the GPU (cec_sim_random) -> classes,
+            representative = minimum id, pairs (repr, member)
+  G phase  candidate pairs with support <= k_g -> cec_sim_exhaustive
+  L phases  (§III-C) 3 passes of cut enumeration (Eq. 1, Table I orders) and local
+            checks (cec_check_local_cuts); reduce the miter after each phase; repeat until no progress
+  reduction proved pairs are merged (member -> representative) and the miter is
+            rebuilt with structural hashing
+
+Every simulation runs in libcec.so's CUDA kernels. The host part here is graph bookkeeping: cut
+enumeration (a host-minimal stand-in for the GPU cut generator), class
+formation from GPU signatures, and miter rebuilding. Undecided pairs remain undecided (the paper
+then hands the reduced miter to ABC, which is out of scope).
+"""
+from __future__ import annotations
+
+import dataclasses
+import time
+from typing import Dict, List, Optional, Tuple
+
+import numpy as np
+
+from . import capi
+from workloads.aig import Aig, Builder  # structural builder (strash) used for miter reduction
+
+
+@dataclasses.dataclass
+class CecParams:
+    k_P: int = 32
+    k_p: int = 16
+    k_g: int = 16
+    k_l: int = 8
+    C: int = 8
+    sim_words: int = 64    # random patterns = 32 * sim_words
+    seed: int = 1
+    max_phases: int = 64
+    max_cuts_per_pair: int = 8
+    device: int = 0
+    engine: int = capi.CEC_ENGINE_AUTO
+
+
+@dataclasses.dataclass
+class CecResult:
+    verdict: int                      # CEC_EQUIVALENT / CEC_NOT_EQUIVALENT / CEC_UNDECIDED
+    po_verdicts: np.ndarray
+    cex: Optional[np.ndarray] = None  # PI values (PI id i+1 = cex[i]) of the lowest NEQ PO pair
+    cex_pair: int = -1
+    log: List[dict] = dataclasses.field(default_factory=list)
+    checks: List[dict] = dataclasses.field(default_factory=list)  # replay log of every local check
+    versions: List[Aig] = dataclasses.field(default_factory=list)  # miter versions the checks refer to
+    final_ands: int = 0
+
+
+# ---------------------------------------------------------------------------------------------
+# miter bookkeeping
+# ---------------------------------------------------------------------------------------------
+
+class Miter:
+    """Current (reduced) miter: an AIG plus the PO pair literals expressed in it."""
+
+    def __init__(self, aig: Aig, lit_a, lit_b):
+        self.aig = aig
+        self.lit_a = np.asarray(lit_a, dtype=np.uint32).copy()
+        self.lit_b = np.asarray(lit_b, dtype=np.uint32).copy()
+
+    def reduce(self, subst: Dict[int, int]) -> "Miter":
+        """Merge proved pairs: node id -> literal of its (lower-id) representative,
+        then rebuild with structural hashing so merged fanouts collapse."""
+        I, A = self.aig.num_pis, self.aig.num_ands
+        fan = self.aig.fanins.astype(np.int64)
+        new = np.zeros(1 + I + A, dtype=np.int64)
+        new[1:1 + I] = 2 * np.arange(1, I + 1)
+        bd = Builder(I, strash=True)
+
+        def m(lit):
+            return int(new[lit >> 1]) ^ (lit & 1)
+
+        for j in range(A):
+            nid = 1 + I + j
+            if nid in subst:
+                new[nid] = m(subst[nid])
+            else:
+                new[nid] = bd.AND(m(int(fan[j, 0])), m(int(fan[j, 1])))
+        la = np.array([m(int(x)) for x in self.lit_a], dtype=np.uint32)
+        lb = np.array([m(int(x)) for x in self.lit_b], dtype=np.uint32)
+        return Miter(bd.finish(list(la) + list(lb)), la, lb), new
+
+
+def _ctx(aig: Aig, p: CecParams, k_max: int, k_s: Optional[int] = None) -> capi.Context:
+    return capi.Context.from_aig(aig, device=p.device, k_max=k_max, k_s=k_s or k_max, engine=p.engine)
+
+
+# ---------------------------------------------------------------------------------------------
+# cut enumeration (Eq. 1) with Table I selection — host-minimal
+# ---------------------------------------------------------------------------------------------
+
+def _bits(mask: int) -> List[int]:
+    out = []
+    while mask:
+        low = mask & -mask
+        out.append(low.bit_length() - 1)
+        mask ^= low
+    return out
+
+
+def enumerate_cuts(aig: Aig, k_l: int, C: int, pass_id: int) -> List[List[int]]:
+    """P(n) for every node id as bitmasks over node ids. E(n) = {u | v : u in P(n0) + {{n0}},
+    v in P(n1) + {{n1}}, |u | v| <= k_l} (Eq. 1); P(n) = the C best of E(n) under the
+    Table I order of this pass: pass 1 fanout > size > small level; pass 2 small
+    level > size > fanout; pass 3 large level > size > fanout. PIs: P = {{pi}} (Alg. 2 l.4-5)."""
+    I, A = aig.num_pis, aig.num_ands
+    N = 1 + I + A
+    fan = aig.fanins.astype(np.int64)
+    level = np.zeros(N, dtype=np.int64)
+    fanout = np.zeros(N, dtype=np.int64)
+    for j in range(A):
+        a, b = int(fan[j, 0]) >> 1, int(fan[j, 1]) >> 1
+        level[1 + I + j] = 1 + max(level[a], level[b])
+        fanout[a] += 1
+        fanout[b] += 1
+    P: List[List[int]] = [[] for _ in range(N)]
+    for i in range(1, I + 1):
+        P[i] = [1 << i]
+    P[0] = [1]  # constant: treat as its own leaf
+
+    def key(mask: int):
+        ids = _bits(mask)
+        sz = len(ids)
+        avg_f = sum(int(fanout[x]) for x in ids) / sz
+        avg_l = sum(int(level[x]) for x in ids) / sz
+        if pass_id == 0:
+            return (-avg_f, sz, avg_l)
+        if pass_id == 1:
+            return (avg_l, sz, -avg_f)
+        return (-avg_l, sz, -avg_f)
+
+    for j in range(A):
+        n = 1 + I + j
+        a, b = int(fan[j, 0]) >> 1, int(fan[j, 1]) >> 1
+        ua = P[a] + [1 << a]
+        vb = P[b] + [1 << b]
+        E = set()
+        for u in ua:
+            for v in vb:
+                c = u | v
+                if c.bit_count() <= k_l:
+                    E.add(c)
+        E.discard(1 << n)
+        P[n] = sorted(E, key=key)[:C]
+    return P
+
+
+# ---------------------------------------------------------------------------------------------
+# the flow
+# ---------------------------------------------------------------------------------------------
+
+def _classes(sig: np.ndarray, phase: np.ndarray, num_pis: int) -> List[Tuple[int, int, int]]:
+    """(repr, member, phase) candidate pairs from equal signatures: repr = min id."""
+    order = np.lexsort((np.arange(sig.size), sig))
+    pairs = []
+    i = 0
+    while i < order.size:
+        j = i
+        while j + 1 < order.size and sig[order[j + 1]] == sig[order[i]]:
+            j += 1
+        if j > i:
+            members = order[i:j + 1]
+            r = int(members[0])
+            for mbr in members[1:]:
+                mbr = int(mbr)
+                if mbr > num_pis:  # members are AND nodes; PIs can only be representatives
+                    pairs.append((r, mbr, int(phase[r] ^ phase[mbr])))
+        i = j + 1
+    return pairs
+
+
+def check_miter(aig: Aig, lit_a, lit_b, params: Optional[CecParams] = None) -> CecResult:
+    p = params or CecParams()
+    cur = Miter(aig, lit_a, lit_b)
+    log: List[dict] = []
+    checks: List[dict] = []
+    versions: List[Aig] = []
+    P = cur.lit_a.size
+    po_v = np.full(P, capi.CEC_UNDECIDED, dtype=np.int32)
+
+    def po_status(m: Miter):
+        return np.array([capi.CEC_EQUIVALENT if a == b else capi.CEC_UNDECIDED for a, b in zip(m.lit_a, m.lit_b)],
+                        dtype=np.int32)
+
+    # ---- P phase -------------------------------------------------------------
+    t = time.perf_counter()
+    hctx = capi.Context.from_aig(cur.aig, device=-1, k_max=63)
+    ks = np.array([hctx.pair_k(int(a), int(b)) for a, b in zip(cur.lit_a, cur.lit_b)])
+    hctx.close()
+    thr = p.k_P if (ks <= p.k_P).all() else p.k_p
+    sel = np.nonzero(ks <= thr)[0]
+    subst: Dict[int, int] = {}
+    if sel.size:
+        ctx = _ctx(cur.aig, p, thr)
+        v, cex, k = ctx.sim_exhaustive(cur.lit_a[sel], cur.lit_b[sel])
+        for i, q in enumerate(sel):
+            if v[i] == capi.CEC_NOT_EQUIVALENT:
+                po_v[q] = capi.CEC_NOT_EQUIVALENT
+            elif v[i] == capi.CEC_EQUIVALENT:
+                po_v[q] = capi.CEC_EQUIVALENT
+        neq = [int(q) for i, q in enumerate(sel) if v[i] == capi.CEC_NOT_EQUIVALENT]
+        if neq:
+            q0 = min(neq)
+            i0 = int(np.nonzero(sel == q0)[0][0])
+            vec = ctx.get_cex(i0)
+            log.append({"phase": "P", "threshold": thr, "simulated": int(sel.size), "neq": len(neq),
+                        "s": time.perf_counter() - t})
+            return CecResult(capi.CEC_NOT_EQUIVALENT, po_v, cex=vec, cex_pair=q0, log=log, final_ands=cur.aig.num_ands)
+        for i, q in enumerate(sel):
+            if v[i] == capi.CEC_EQUIVALENT:
+                a, b = int(cur.lit_a[q]), int(cur.lit_b[q])
+                hi, lo = (a, b) if (a >> 1) > (b >> 1) else (b, a)
+                if (hi >> 1) > aig.num_pis:
+                    subst[hi >> 1] = lo ^ (hi & 1)
+        ctx.close()
+    log.append({"phase": "P", "threshold": thr, "simulated": int(sel.size), "s": time.perf_counter() - t})
+    if subst:
+        cur, _ = cur.reduce(subst)
+
+    # ---- G and L phases -----------------------------------------------------------------------
+    tried_global = set()
+    for phase_no in range(p.max_phases):
+        st = po_status(cur)
+        if (st == capi.CEC_EQUIVALENT).all():
+            break
+        t = time.perf_counter()
+        ctx = _ctx(cur.aig, p, p.k_g)
+        N = cur.aig.num_nodes
+        sig, ph = capi.cec_sim_random(ctx.handle, N, p.sim_words, p.seed + phase_no)
+        cand = [(r, m_, f) for r, m_, f in _classes(sig, ph, cur.aig.num_pis)]
+        versions.append(cur.aig)
+        # G phase once per miter version: pairs with support <= k_g
+        gl = [(r, m_, f) for r, m_, f in cand if (r, m_, f) not in tried_global]
+        la = [2 * r for r, m_, f in gl]
+        lb = [2 * m_ ^ f for r, m_, f in gl]
+        subst = {}
+        proved_g = 0
+        if gl:
+            v, _, k = ctx.sim_exhaustive(la, lb)
+            for (r, m_, f), vv in zip(gl, v):
+                if vv == capi.CEC_EQUIVALENT and m_ not in subst:
+                    subst[m_] = 2 * r ^ f
+                    proved_g += 1
+                if vv != capi.CEC_UNDECIDED:
+                    tried_global.add((r, m_, f))
+        remaining = [(r, m_, f) for r, m_, f in cand if m_ not in subst and (r, m_, f) not in tried_global]
+        # L: 3 passes of cut enumeration + local checks (Table I)
+        proved_l = 0
+        for pass_id in range(3):
+            if not remaining:
+                break
+            cuts = enumerate_cuts(cur.aig, p.k_l, p.C, pass_id)
+            ql, qm, off, leaves, who = [], [], [0], [], []
+            for r, m_, f in remaining:
+                if m_ in subst:
+                    continue
+                common = set()
+                for u in cuts[r]:
+                    for v_ in cuts[m_]:
+                        c = u | v_
+                        if c.bit_count() <= p.k_l:
+                            common.add(c)
+                for c in sorted(common, key=lambda x: (x.bit_count(), x))[:p.max_cuts_per_pair]:
+                    ql.append(2 * r)
+                    qm.append(2 * m_ ^ f)
+                    leaves += _bits(c)
+                    off.append(len(leaves))
+                    who.append((r, m_, f))
+            if not ql:
+                continue
+            lv = ctx.check_local_cuts(ql, qm, off, leaves)
+            for q, vv in enumerate(lv):
+                checks.append({"version": len(versions) - 1, "phase": phase_no, "pass": pass_id,
+                               "lit_a": ql[q], "lit_b": qm[q], "leaves": leaves[off[q]:off[q + 1]], "verdict": int(vv)})
+                r, m_, f = who[q]
+                if vv == capi.CEC_EQUIVALENT and m_ not in subst:
+                    subst[m_] = 2 * r ^ f
+                    proved_l += 1
+            remaining = [x for x in remaining if x[1] not in subst]
+        ctx.close()
+        log.append({"phase": f"G+L{phase_no}", "candidates": len(cand), "proved_global": proved_g,
+                    "proved_local": proved_l, "ands": cur.aig.num_ands, "s": time.perf_counter() - t})
+        if not subst:
+            break  # no progress: undecided remainder
+        cur, _ = cur.reduce(subst)
+    st = po_status(cur)
+    po_v = np.where(st == capi.CEC_EQUIVALENT, capi.CEC_EQUIVALENT, po_v)
+    verdict = capi.CEC_EQUIVALENT if (po_v == capi.CEC_EQUIVALENT).all() else capi.CEC_UNDECIDED
+    # the reduced miter's PO pairs that remain can still be refuted exhaustively when small
+    return CecResult(verdict, po_v, log=log, checks=checks, versions=versions, final_ands=cur.aig.num_ands)

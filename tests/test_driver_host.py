@@ -1,0 +1,63 @@
+"""Host logic of the CEC driver (no GPU): Eq. (1) cut enumeration on hand graphs, Table I orders,
+class formation from signatures, and miter reduction preserving PO functions (checked with the
+oracle's evaluator on random assignments)."""
+import numpy as np
+
+import oracle
+from paper_conf_dac_liuy25_b200 import driver
+from workloads import Builder, c4_dp, circuits
+
+
+def test_eq1_cut_enumeration_hand_graph():
+    bd = Builder(3, strash=False)
+    a, b, c = bd.pi(0), bd.pi(1), bd.pi(2)
+    n = bd.raw_and(a, b)      # id 4
+    m = bd.raw_and(n, c)      # id 5
+    aig = bd.finish([m])
+    P = driver.enumerate_cuts(aig, k_l=8, C=8, pass_id=1)
+    as_sets = lambda cuts: sorted(sorted(driver._bits(x)) for x in cuts)
+    assert as_sets(P[4]) == [[1, 2]]
+    assert as_sets(P[5]) == [[1, 2, 3], [3, 4]]   # {u|v : u in P(n)+{{n}}, v in {{c}}}
+    # k_l bound: no cut above 2 leaves survives
+    P2 = driver.enumerate_cuts(aig, k_l=2, C=8, pass_id=1)
+    assert as_sets(P2[5]) == [[3, 4]]
+
+
+def test_table1_orders():
+    bd = Builder(4, strash=False)
+    x = [bd.pi(i) for i in range(4)]
+    n1 = bd.raw_and(x[0], x[1])
+    n2 = bd.raw_and(n1, x[2])
+    n3 = bd.raw_and(n2, x[3])
+    aig = bd.finish([n3])
+    small_level = driver.enumerate_cuts(aig, 8, 1, pass_id=1)[n3 >> 1]
+    large_level = driver.enumerate_cuts(aig, 8, 1, pass_id=2)[n3 >> 1]
+    assert sorted(driver._bits(small_level[0])) == [1, 2, 3, 4]     # PIs: level 0
+    assert sorted(driver._bits(large_level[0])) == [4, n2 >> 1]     # highest-level leaves
+
+
+def test_classes_from_signatures():
+    sig = np.array([7, 5, 9, 5, 9, 9], dtype=np.uint64)
+    ph = np.array([0, 0, 1, 1, 0, 1], dtype=np.uint8)
+    pairs = driver._classes(sig, ph, num_pis=1)
+    assert sorted(pairs) == [(1, 3, 1), (2, 4, 1), (2, 5, 0)]
+
+
+def test_miter_reduction_preserves_functions():
+    m = circuits.random_miter(10, 200, 8, seed=3, window=24)
+    # merge every B-side PO driver into its A-side partner (they are equivalent by construction)
+    cur = driver.Miter(m.aig, m.lit_a, m.lit_b)
+    subst = {}
+    for a, b in zip(m.lit_a, m.lit_b):
+        a, b = int(a), int(b)
+        hi, lo = (a, b) if (a >> 1) > (b >> 1) else (b, a)
+        if (hi >> 1) > m.aig.num_pis and (hi >> 1) not in subst:
+            subst[hi >> 1] = lo ^ (hi & 1)
+    red, _ = cur.reduce(subst)
+    assert all(int(x) == int(y) for x, y in zip(red.lit_a, red.lit_b))
+    o1, o2 = oracle.Oracle.from_aig(m.aig), oracle.Oracle.from_aig(red.aig)
+    rng = np.random.default_rng(0)
+    for _ in range(64):
+        pis = rng.integers(0, 2, size=10).astype(np.uint8)
+        for a_old, a_new in zip(m.lit_a, red.lit_a):
+            assert o1.eval_lit(int(a_old), pis) == o2.eval_lit(int(a_new), pis)

@@ -242,3 +242,51 @@ def test_shard_emulation_matches_single_gpu(world, engine):
         v, c, k = combine_shards(parts)
         assert np.array_equal(v, ref[0]) and np.array_equal(k, ref[2])
         assert [int(x) for x, vv in zip(c, v) if vv == 2] == [int(x) for x, vv in zip(ref[1], ref[0]) if vv == 2]
+
+
+def _replay_checks(res, limit=400):
+    """Every logged local check of the driver, replayed through the oracle on the miter version it
+    ran on: bit-exact per-check parity (the C4 outcome itself is parity-unpinned)."""
+    from collections import defaultdict
+    byv = defaultdict(list)
+    for ch in res.checks[:limit]:
+        byv[ch["version"]].append(ch)
+    for vi, chs in byv.items():
+        orc = Oracle.from_aig(res.versions[vi])
+        off = np.cumsum([0] + [len(c["leaves"]) for c in chs])
+        want = orc.check_local([c["lit_a"] for c in chs], [c["lit_b"] for c in chs], off,
+                               [x for c in chs for x in c["leaves"]])
+        assert [c["verdict"] for c in chs] == [int(w) for w in want]
+
+
+def test_driver_dp8_local_phases_and_bug():
+    from paper_conf_dac_liuy25_b200 import driver
+    from workloads import c4_dp
+    p = driver.CecParams(k_P=6, k_p=6, k_g=6, k_l=8, C=8)
+    m = c4_dp(8)
+    res = driver.check_miter(m.aig, m.lit_a, m.lit_b, p)
+    assert res.checks, "local phases must run"
+    _replay_checks(res)
+    orc = Oracle.from_aig(m.aig)
+    ov, _, _, _ = orc.check_pairs(m.lit_a, m.lit_b)
+    assert all(int(v) == oracle.EQUIVALENT for v in ov)
+    assert res.verdict in (capi.CEC_EQUIVALENT, capi.CEC_UNDECIDED)
+    bug = c4_dp(8, bug=4)
+    rb = driver.check_miter(bug.aig, bug.lit_a, bug.lit_b, p)
+    ov, _, _, _ = Oracle.from_aig(bug.aig).check_pairs(bug.lit_a, bug.lit_b)
+    for q in range(bug.num_pairs):  # soundness: never EQ where the oracle says NEQ
+        if int(ov[q]) == oracle.NOT_EQUIVALENT:
+            assert rb.po_verdicts[q] != capi.CEC_EQUIVALENT
+    _replay_checks(rb)
+
+
+def test_driver_c4_full():
+    from paper_conf_dac_liuy25_b200 import driver
+    from workloads import c4_dp
+    p = driver.CecParams(k_l=16)
+    m = c4_dp(64)
+    res = driver.check_miter(m.aig, m.lit_a, m.lit_b, p)
+    _replay_checks(res, limit=300)
+    bug = c4_dp(64, bug=4)
+    rb = driver.check_miter(bug.aig, bug.lit_a, bug.lit_b, p)
+    assert rb.verdict != capi.CEC_EQUIVALENT  # the C4-bug variant is never reported EQ
