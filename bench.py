@@ -38,7 +38,7 @@ LOP3_PER_CLK_PER_SM = 64  # alu pipe: rt = 2 cycles per warp-instr per SMSP, 4 S
 
 
 def make_workload(name: str):
-    from workloads import c1_add8, c2_mul12, c2_mul12_bug, c5_big
+    from workloads import c1_add8, c2_mul12, c2_mul12_bug, c3_rand, c5_big
 
     if name == "c5":
         m = c5_big()
@@ -49,6 +49,9 @@ def make_workload(name: str):
         return c2_mul12(), "c2_mul12: 12x12 array vs Wallace multiplier miter", None
     if name == "c2bug":
         return c2_mul12_bug(seed=1), "c2_mul12_bug1: C2 with one flipped complement in B's tree", None
+    if name == "c3":
+        return c3_rand(), ("c3_rand100k: 200 random blocks (~100k ANDs) vs rewritten copy over 1024 PIs; "
+                           "1600 PO pairs + 5000 internal (A node, B image) pairs + 64 near-miss pairs"), None
     if name == "c1":
         return c1_add8(), "c1_add8: 8-bit ripple-carry vs Kogge-Stone adder miter", None
     raise SystemExit(f"unknown config {name}")
@@ -165,6 +168,7 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--engine", type=int, default=0, help="0 auto, 1 interpreter, 2 JIT")
     ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--merge", type=int, default=-1, help="0 off, 1 paper (default), 2 cost-aware (default for c3)")
     ap.add_argument("--cpu-log2-patterns", type=int, default=19)
     ap.add_argument("--ref-log2-patterns", type=int, default=17)
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -196,8 +200,9 @@ def main():
         dist.broadcast_object_list(obj, src=0)
         uid = obj[0]
     t_load = time.perf_counter()
+    merge = args.merge if args.merge >= 0 else (capi.CEC_MERGE_COST if args.config == "c3" else capi.CEC_MERGE_PAPER)
     ctx = capi.Context.from_aig(m.aig, device=local, rank=rank, world=world, stream=stream.cuda_stream,
-                                engine=args.engine, nccl_unique_id=uid)
+                                engine=args.engine, merge=merge, nccl_unique_id=uid)
     load_ms = 1e3 * (time.perf_counter() - t_load)
     plan = capi.cec_plan_exhaustive(ctx.handle, m.lit_a, m.lit_b)
     info = capi.cec_plan_info(plan)
@@ -290,7 +295,7 @@ def main():
                        "max_slots": info["max_slots"], "node_patterns_per_step": W_all,
                        "parallelism": f"pattern-space shards x{world}" + (" + NCCL min all-reduce" if world > 1 else ""),
                        "l2": "flushed between timed steps (256 MiB write, outside the events)",
-                       "engine": engine_name, "jit_kernels": st0["jit_kernels"], "jit_compile_ms": st0["jit_ms"],
+                       "merge": ["off", "paper", "cost-aware"][merge], "engine": engine_name, "jit_kernels": st0["jit_kernels"], "jit_compile_ms": st0["jit_ms"],
                        "verdicts": verdicts},
             "clocks": clocks,
             "gpu_launches": int(launches_per_step * args.steps),

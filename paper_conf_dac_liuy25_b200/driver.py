@@ -232,6 +232,7 @@ def check_miter(aig: Aig, lit_a, lit_b, params: Optional[CecParams] = None) -> C
             break
         t = time.perf_counter()
         ctx = _ctx(cur.aig, p, p.k_g)
+        lctx = _ctx(cur.aig, p, max(p.k_l, 1))  # local checks: up to k_l leaves
         N = cur.aig.num_nodes
         sig, ph = capi.cec_sim_random(ctx.handle, N, p.sim_words, p.seed + phase_no)
         cand = [(r, m_, f) for r, m_, f in _classes(sig, ph, cur.aig.num_pis)]
@@ -275,7 +276,7 @@ def check_miter(aig: Aig, lit_a, lit_b, params: Optional[CecParams] = None) -> C
                     who.append((r, m_, f))
             if not ql:
                 continue
-            lv = ctx.check_local_cuts(ql, qm, off, leaves)
+            lv = lctx.check_local_cuts(ql, qm, off, leaves)
             for q, vv in enumerate(lv):
                 checks.append({"version": len(versions) - 1, "phase": phase_no, "pass": pass_id,
                                "lit_a": ql[q], "lit_b": qm[q], "leaves": leaves[off[q]:off[q + 1]], "verdict": int(vv)})
@@ -285,6 +286,7 @@ def check_miter(aig: Aig, lit_a, lit_b, params: Optional[CecParams] = None) -> C
                     proved_l += 1
             remaining = [x for x in remaining if x[1] not in subst]
         ctx.close()
+        lctx.close()
         log.append({"phase": f"G+L{phase_no}", "candidates": len(cand), "proved_global": proved_g,
                     "proved_local": proved_l, "ands": cur.aig.num_ands, "s": time.perf_counter() - t})
         if not subst:

@@ -67,7 +67,7 @@ def concat_miter(a: Aig, b: Aig, name: str = "") -> Miter:
     pb = np.array([int(lit_map[int(l) >> 1]) ^ (int(l) & 1) for l in b.pos], dtype=np.uint32)
     aig = bd.finish(list(a.pos) + list(pb))
     return Miter(aig, a.pos.astype(np.uint32).copy(), pb, name=name,
-                 meta={"a_ands": a_ands, "b_ands": len(bd.ands) - a_ands})
+                 meta={"a_ands": a_ands, "b_ands": len(bd.ands) - a_ands, "b_lit_map": lit_map})
 
 
 def b_image(miter_a_ands: int, num_pis: int, lit_in_b: int) -> int:
@@ -500,3 +500,72 @@ def c5_big(copies: int = 256, n_random: int = 176, seed: int = 5, n_bugs: int = 
     m.meta["bug_copies"] = bug_copies
     m.meta["base_types"] = len(bases)
     return m
+
+
+def c3_rand(seed: int = 3, sample_seed: int = 7, n_blocks: int = 200, block_ands: int = 500, num_pis: int = 1024,
+            n_internal: int = 5000, n_near: int = 64, k_dist=((150, 12, 20), (40, 21, 26), (8, 27, 31), (2, 32, 32)),
+            window: int = 64, p_rw: float = 0.3) -> Miter:
+    """C3: random block AIG A (blocks of ~block_ands ANDs, block b reads a contiguous
+    window of k_b PIs out of num_pis; fanins from the block's last `window` nodes w.p. 0.9 else its
+    PIs; up to 8 dangling nodes per block become POs) vs its rewritten copy B. Pairs: every PO
+    pair, n_internal sampled (A node, B image) pairs and n_near near-miss pairs (A node vs its B
+    image with one fanin complemented: appended nodes, mostly NEQ)."""
+    rng = np.random.default_rng(seed)
+    ks = []
+    for cnt, lo, hi in k_dist:
+        ks += [int(x) for x in rng.integers(lo, hi + 1, size=cnt)]
+    ks = [int(x) for x in rng.permutation(ks)][:n_blocks]
+    bd = Builder(num_pis, strash=True)
+    pos: List[int] = []
+    for kb in ks:
+        start = int(rng.integers(0, num_pis - kb + 1))
+        pis = [bd.pi(start + i) for i in range(kb)]
+        random_block(bd, pis, block_ands, rng, window=window, p_pi=0.1)
+        dang = list(random_block.last_unused)[-8:]
+        pos += [x ^ int(rng.integers(0, 2)) for x in dang]
+    a = bd.finish(pos)
+    img: Dict[int, int] = {}
+    b = rewrite_copy(a, rng, p_rw=p_rw, node_map_out=img)
+    m = concat_miter(a, b, name=f"c3_rand{n_blocks}x{block_ands}")
+    bmap = m.meta["b_lit_map"]
+    I = num_pis
+
+    def b_lit(local_lit: int) -> int:
+        return int(bmap[local_lit >> 1]) ^ (local_lit & 1)
+
+    srng = np.random.default_rng(sample_seed)
+    a_ids = np.arange(1 + I, 1 + I + a.num_ands)
+    la = [int(x) for x in m.lit_a]
+    lb = [int(x) for x in m.lit_b]
+    cand = [int(x) for x in srng.permutation(a_ids)]
+    internal = 0
+    for nid in cand:
+        if internal >= n_internal:
+            break
+        il = b_lit(img[nid])
+        if il == 2 * nid:
+            continue  # hashed onto the A node itself: trivially equal
+        la.append(2 * nid)
+        lb.append(il)
+        internal += 1
+    fan = [tuple(int(v) for v in r) for r in m.aig.fanins]
+    near = 0
+    for nid in cand[::-1]:
+        if near >= n_near:
+            break
+        il = b_lit(img[nid])
+        v = il >> 1
+        if v <= I or il == 2 * nid:
+            continue
+        f0, f1 = fan[v - I - 1]
+        fan.append((f0 ^ 1, f1))
+        new_id = 1 + I + len(fan) - 1
+        la.append(2 * nid)
+        lb.append(2 * new_id ^ (il & 1))
+        near += 1
+    aig = Aig(I, np.asarray(fan, dtype=np.uint32).reshape(-1, 2), m.aig.pos.copy())
+    aig.validate()
+    meta = dict(m.meta)
+    meta.pop("b_lit_map", None)
+    meta.update({"k_blocks": ks, "po_pairs": len(m.lit_a), "internal_pairs": internal, "near_pairs": near})
+    return Miter(aig, np.asarray(la, dtype=np.uint32), np.asarray(lb, dtype=np.uint32), name=m.name, meta=meta)
