@@ -129,7 +129,7 @@ struct cec_plan {
     std::vector<uint32_t> win_nodes;          // AND-node count per window
     std::vector<std::vector<uint32_t>> win_cmps;
     std::vector<DevWin> dwin;
-    std::vector<uint2> prog;
+    std::vector<uint4> prog;
     std::vector<Item> items;
     std::vector<JItem> jitems;
     std::vector<LaunchGroup> groups;
@@ -225,7 +225,7 @@ uint64_t support_of(cec_ctx *c, uint32_t la, uint32_t lb, std::vector<uint32_t> 
 // Schedule builder: topological op order (ascending id, "topological order"), compare
 // ops right after their later root, and linear-scan slot allocation by liveness.
 struct Sched {
-    std::vector<uint2> ops;
+    std::vector<uint4> ops;
     uint32_t nslots = 0;
     uint32_t const_slot = 0xFFFFFFFFu;
 };
@@ -328,13 +328,15 @@ bool build_schedule(cec_ctx *c, const std::vector<uint32_t> &inputs, const std::
             why = "schedule: operand not defined before use";
             return false;
         }
-        uint2 e;
-        e.x = (slot[va] << 1 | (op.la & 1u)) | ((slot[vb] << 1 | (op.lb & 1u)) << 16);
+        uint4 e;
+        e.x = slot[va] * SLOT_BYTES | (op.la & 1u);
+        e.y = slot[vb] * SLOT_BYTES | (op.lb & 1u);
+        e.w = 0;
         // free operands whose last reader is this op (the kernel reads before it writes)
         if (last[va] == o + 1) free_list.push_back(slot[va]);
         if (vb != va && last[vb] == o + 1) free_list.push_back(slot[vb]);
         if (op.cmp) {
-            e.y = OP_CMP | op.id;
+            e.z = OP_CMP | op.id;
         } else {
             uint32_t s;
             if (!free_list.empty()) {
@@ -348,7 +350,7 @@ bool build_schedule(cec_ctx *c, const std::vector<uint32_t> &inputs, const std::
                 return false;
             }
             slot[op.id] = s;
-            e.y = s;
+            e.z = s * SLOT_BYTES;
             if (!last[op.id]) free_list.push_back(s);  // never read (cannot happen in a window)
         }
         out.ops.push_back(e);
@@ -532,10 +534,11 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
     cmps2.reserve(P->cmps.size());
     std::vector<int32_t> remap(P->cmps.size(), -1);
     std::vector<uint32_t> stop_mark;
-    uint32_t max_slot_cap = interp_max_slots_per_warp();
+    const uint32_t max_slot_cap = interp_max_slots_per_warp();
     std::vector<uint32_t> nslots_of;
     std::vector<uint64_t> cost_of;
     std::vector<int32_t> win_jit;                    // JIT structure index per window, -1 = interpreter
+    std::vector<uint64_t> wps_of;                    // words per slice per window
     std::vector<JitProgram> jit_progs;
     std::unordered_map<std::string, uint32_t> jit_index;
     for (size_t w = 0; w < wins.size(); ++w) {
@@ -617,9 +620,6 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
                 nodes.swap(by_id);
             }
         }
-        if (sc.nslots > max_slot_cap)
-            return fail(c, CEC_E_NOMEM, "window %zu needs %u live slots > %u (on-chip capacity)", w, sc.nslots,
-                        max_slot_cap);
         dw.prog_off = (uint32_t)P->prog.size();
         dw.prog_len = (uint32_t)sc.ops.size();
         dw.k = (uint32_t)W.inputs.size();
@@ -639,8 +639,11 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         bool jit = false;
         if (dw.k >= 10 && !nodes.empty()) {
             if (c->opts.engine == CEC_ENGINE_JIT) jit = true;
-            else if (c->opts.engine == CEC_ENGINE_AUTO) jit = node_words >= (1ull << 26);
+            else if (c->opts.engine == CEC_ENGINE_AUTO) jit = node_words >= (1ull << 26) || sc.nslots > max_slot_cap;
         }
+        if (!jit && sc.nslots > max_slot_cap)
+            return fail(c, CEC_E_NOMEM, "window %zu needs %u live slots > %u (shared-memory capacity)", w, sc.nslots,
+                        max_slot_cap);
         if (jit) {
             JitProgram jp;
             jp.k = dw.k;
@@ -670,13 +673,15 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         }
         P->max_k = std::max(P->max_k, dw.k);
         P->max_slots = std::max(P->max_slots, sc.nslots);
+        const uint64_t wps = jit ? 32 : 32 * IV;  // words per slice of this window's engine
+        wps_of.push_back(wps);
         // W accounting: nodes x patterns, per rank and all ranks
-        const uint64_t slices = (ttw + 31) / 32;
+        const uint64_t slices = (ttw + wps - 1) / wps;
         const uint64_t pats_all = dw.k < 5 ? (1ull << dw.k) : ttw * 32;
         P->W_all += (uint64_t)nodes.size() * pats_all;
         uint64_t sb, se;
         cec_shard_range(slices, rank, world, &sb, &se);
-        uint64_t wb = sb * 32, we = std::min<uint64_t>(se * 32, ttw);
+        uint64_t wb = sb * wps, we = std::min<uint64_t>(se * wps, ttw);
         uint64_t pats_rank = we > wb ? (dw.k < 5 ? (1ull << dw.k) : (we - wb) * 32) : 0;
         P->W_rank += (uint64_t)nodes.size() * pats_rank;
         cost_of.push_back((uint64_t)(dw.prog_len + 1) * (se - sb));
@@ -735,7 +740,7 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         uint64_t group_slices = 0;
         for (uint32_t w : ws) {
             uint64_t ttw = tt_words_of(P->dwin[w].k), sb, se;
-            cec_shard_range((ttw + 31) / 32, rank, world, &sb, &se);
+            cec_shard_range((ttw + wps_of[w] - 1) / wps_of[w], rank, world, &sb, &se);
             group_slices += se - sb;
         }
         const uint64_t target = (uint64_t)std::max(c->num_sms, 148) * 16 /*resident warps*/ * 8;
@@ -744,7 +749,7 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
             item_slices = std::max<uint64_t>(jit_pass, (item_slices * 16 + jit_pass - 1) / jit_pass * jit_pass);
         for (uint32_t w : ws) {
             uint64_t ttw = tt_words_of(P->dwin[w].k), sb, se;
-            cec_shard_range((ttw + 31) / 32, rank, world, &sb, &se);
+            cec_shard_range((ttw + wps_of[w] - 1) / wps_of[w], rank, world, &sb, &se);
             for (uint64_t s = sb; s < se; s += item_slices) {
                 const uint32_t e = (uint32_t)std::min<uint64_t>(se, s + item_slices);
                 if (jit)
@@ -783,7 +788,7 @@ cec_status upload(cec_ctx *c, cec_plan *P) {
     DevPlan &d = P->d;
     const size_t ncmp = std::max<size_t>(1, P->cmps.size()), nwin = std::max<size_t>(1, P->dwin.size());
     CUDA_TRY(c, dev_alloc((void **)&d.wins, sizeof(DevWin) * nwin));
-    CUDA_TRY(c, dev_alloc((void **)&d.prog, sizeof(uint2) * std::max<size_t>(1, P->prog.size())));
+    CUDA_TRY(c, dev_alloc((void **)&d.prog, sizeof(uint4) * std::max<size_t>(1, P->prog.size())));
     CUDA_TRY(c, dev_alloc((void **)&d.items, sizeof(Item) * std::max<size_t>(1, P->items.size())));
     CUDA_TRY(c, dev_alloc((void **)&d.first, sizeof(unsigned long long) * ncmp));
     CUDA_TRY(c, dev_alloc((void **)&d.bound, sizeof(unsigned long long) * nwin));
@@ -792,11 +797,11 @@ cec_status upload(cec_ctx *c, cec_plan *P) {
     CUDA_TRY(c, dev_alloc((void **)&d.jitems, sizeof(JItem) * std::max<size_t>(1, P->jitems.size())));
     CUDA_TRY(c, h2d(d.jitems, P->jitems.data(), sizeof(JItem) * P->jitems.size(), c->stream));
     CUDA_TRY(c, h2d(d.wins, P->dwin.data(), sizeof(DevWin) * P->dwin.size(), c->stream));
-    CUDA_TRY(c, h2d(d.prog, P->prog.data(), sizeof(uint2) * P->prog.size(), c->stream));
+    CUDA_TRY(c, h2d(d.prog, P->prog.data(), sizeof(uint4) * P->prog.size(), c->stream));
     CUDA_TRY(c, h2d(d.items, P->items.data(), sizeof(Item) * P->items.size(), c->stream));
     CUDA_TRY(c, event_create(&P->ev0));
     CUDA_TRY(c, event_create(&P->ev1));
-    c->stats.h2d_bytes = sizeof(DevWin) * P->dwin.size() + sizeof(uint2) * P->prog.size() +
+    c->stats.h2d_bytes = sizeof(DevWin) * P->dwin.size() + sizeof(uint4) * P->prog.size() +
                          sizeof(Item) * P->items.size() + sizeof(JItem) * P->jitems.size();
     P->uploaded = true;
     return CEC_OK;

@@ -7,15 +7,17 @@
 
 namespace cec {
 
-// ---- Interpreter program encoding (one uint2 per op) ------------------------------------------
+// ---- Interpreter program encoding (one uint4 = 16 B per op) ------------------------------------
+// Node words live in shared-memory slots; a slot holds IV u32 words per lane of a warp
+// (SLOT_BYTES = 32 * IV * 4). Offsets below are byte offsets of a slot inside the warp's region.
 // AND op  (TT(n)[w] = (TT(f0)[w] ^ m0) & (TT(f1)[w] ^ m1), Alg. 1 l.10-11):
-//   x = (slot0 << 1 | c0) | (slot1 << 1 | c1) << 16 ;  y = out_slot
+//   x = off(f0) | c0 ;  y = off(f1) | c1 ;  z = off(out) ;  w = 0
 // CMP op  (XOR-compare of a pair's root words, Alg. 1 l.12-14):
-//   x = (slotA << 1 | cA) | (slotB << 1 | cB) << 16 ;  y = OP_CMP | cmp_index
-// A slot holds one u32 truth-table word per lane of a warp (32 consecutive words per warp pass).
+//   x = off(a) | ca ;  y = off(b) | cb ;  z = OP_CMP | cmp_index ;  w = 0
+constexpr uint32_t IV = 2;                       // u32 words per lane per slot
+constexpr uint32_t SLOT_BYTES = 32u * IV * 4u;   // 256
 constexpr uint32_t OP_CMP = 0x80000000u;
-constexpr uint32_t MAX_SLOTS = 32767;   // 15-bit slot field
-constexpr uint32_t MAX_CMPS = 0x7FFFFFFFu;
+constexpr uint32_t MAX_SLOTS = 0x7FFFFFFFu / SLOT_BYTES;
 
 struct DevWin {            // one simulation window (§III-B1) after merging
     uint32_t prog_off;     // first op in the program array
@@ -27,8 +29,10 @@ struct DevWin {            // one simulation window (§III-B1) after
     uint32_t tt_words_lo;  // truth-table length in u32 words = max(1, 2^(k-5))
     uint32_t tt_words_hi;
 };
+// A slice = the words one warp carries through the window in one pass: 32 * IV words for the
+// interpreter, 32 words for JIT kernels.
 
-struct Item {              // a contiguous range of 32-word slices of one window
+struct Item {              // a contiguous range of slices of one window
     uint32_t win;
     uint32_t s_begin;
     uint32_t s_end;
@@ -64,7 +68,7 @@ struct LaunchGroup {       // windows sharing one kernel launch
 // Device buffers of one plan.
 struct DevPlan {
     DevWin *wins = nullptr;
-    uint2 *prog = nullptr;
+    uint4 *prog = nullptr;
     Item *items = nullptr;
     unsigned long long *first = nullptr;  // [ncmp] minimum mismatching merged pattern index
     unsigned long long *bound = nullptr;  // [nwin] early-exit bound (all pairs NEQ below it)

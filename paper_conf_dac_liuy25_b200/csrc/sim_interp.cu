@@ -45,6 +45,12 @@ __device__ __forceinline__ uint32_t proj_word(uint32_t j, uint64_t w) {
     }
 }
 
+__device__ __forceinline__ uint32_t lop3_60(uint32_t t, uint32_t b, uint32_t m) {
+    uint32_t r;
+    asm("lop3.b32 %0, %1, %2, %3, 0x60;" : "=r"(r) : "r"(t), "r"(b), "r"(m));
+    return r;
+}
+
 __device__ __noinline__ void record_mismatch(uint32_t c, uint64_t idx, uint32_t win, const DevWin &W,
                                              unsigned long long *first, unsigned long long *bound,
                                              uint32_t *neq_cnt) {
@@ -64,15 +70,28 @@ __device__ __noinline__ void record_mismatch(uint32_t c, uint64_t idx, uint32_t 
     }
 }
 
+__device__ __forceinline__ void report(uint32_t d, uint64_t word_base, uint32_t lane, uint32_t c, uint32_t win,
+                                       const DevWin &W, unsigned long long *first, unsigned long long *bound,
+                                       uint32_t *neq_cnt) {
+    // d = this lane's mismatch bits for word word_base + lane (all lanes of the warp call this)
+    const uint32_t bal = __ballot_sync(FULL, d != 0u);
+    const uint32_t l = (uint32_t)__ffs(bal) - 1u;
+    const uint32_t dl = __shfl_sync(FULL, d, l);
+    if (lane == 0) record_mismatch(c, ((word_base + l) << 5) + (uint32_t)(__ffs(dl) - 1), win, W, first, bound, neq_cnt);
+}
+
+// One warp = one slice of 32*IV consecutive words: lane l holds words base + v*32 + l (v < IV), so
+// a ballot over v = 0 before v = 1 finds mismatches in pattern order.
 __global__ void __launch_bounds__(MAX_WPB * 32)
 interp_kernel(const Item *__restrict__ items, uint32_t nitems, uint32_t *__restrict__ item_ctr,
-              const DevWin *__restrict__ wins, const uint2 *__restrict__ prog, unsigned long long *first,
+              const DevWin *__restrict__ wins, const uint4 *__restrict__ prog, unsigned long long *first,
               unsigned long long *bound, uint32_t *neq_cnt, uint32_t nslots) {
-    extern __shared__ uint32_t smem[];
+    extern __shared__ __align__(16) unsigned char smem[];
     const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31u;
-    uint32_t *vals = smem + (size_t)warp * (nslots * 32u + 64u);
-    uint2 *ibuf = reinterpret_cast<uint2 *>(vals + nslots * 32u);
-    uint32_t *my = vals + lane;  // this lane's column: slot s at my[s * 32]
+    unsigned char *wbase = smem + (size_t)warp * (nslots * SLOT_BYTES + 32u * sizeof(uint4));
+    uint4 *ibuf = reinterpret_cast<uint4 *>(wbase + nslots * SLOT_BYTES);
+    unsigned char *my = wbase + lane * (IV * 4u);  // this lane's uint2 inside every slot
+#define SLOT(off) (*reinterpret_cast<uint2 *>(my + (off)))
 
     for (;;) {
         uint32_t it = 0;
@@ -83,39 +102,42 @@ interp_kernel(const Item *__restrict__ items, uint32_t nitems, uint32_t *__restr
         const DevWin W = wins[item.win];
         const uint64_t tt_words = ((uint64_t)W.tt_words_hi << 32) | W.tt_words_lo;
         for (uint32_t s = item.s_begin; s < item.s_end; ++s) {
-            const uint64_t base_idx = (uint64_t)s << 10;  // first pattern of this 32-word slice
-            if (base_idx >= *((volatile unsigned long long *)&bound[item.win])) break;
-            const uint64_t word = ((uint64_t)s << 5) + lane;
-            const bool active = word < tt_words;
-            for (uint32_t j = 0; j < W.k; ++j) my[j * 32u] = proj_word(j, word);
-            if (W.const_slot != 0xFFFFFFFFu) my[W.const_slot * 32u] = 0u;
+            const uint64_t base = (uint64_t)s * (32u * IV);  // first word of the slice
+            if ((base << 5) >= *((volatile unsigned long long *)&bound[item.win])) break;
+            const uint64_t w0 = base + lane, w1 = base + 32u + lane;
+            const bool act0 = w0 < tt_words, act1 = w1 < tt_words;
+            for (uint32_t j = 0; j < W.k; ++j) SLOT(j * SLOT_BYTES) = make_uint2(proj_word(j, w0), proj_word(j, w1));
+            if (W.const_slot != 0xFFFFFFFFu) SLOT(W.const_slot * SLOT_BYTES) = make_uint2(0u, 0u);
             for (uint32_t p = 0; p < W.prog_len; p += 32u) {
                 const uint32_t n = min(32u, W.prog_len - p);
                 __syncwarp();
                 if (lane < n) ibuf[lane] = prog[W.prog_off + p + lane];
                 __syncwarp();
+#pragma unroll 4
                 for (uint32_t j = 0; j < n; ++j) {
-                    const uint2 ins = ibuf[j];
-                    const uint32_t a = my[(ins.x & 0xFFFEu) << 4] ^ (0u - (ins.x & 1u));
-                    const uint32_t b = my[((ins.x >> 16) & 0xFFFEu) << 4] ^ (0u - ((ins.x >> 16) & 1u));
-                    if (!(ins.y & OP_CMP)) {
-                        my[ins.y << 5] = a & b;
+                    const uint4 ins = ibuf[j];
+                    const uint32_t ma = (uint32_t)((int32_t)(ins.x << 31) >> 31);
+                    const uint32_t mb = (uint32_t)((int32_t)(ins.y << 31) >> 31);
+                    const uint2 a = SLOT(ins.x & ~7u), b = SLOT(ins.y & ~7u);
+                    const uint32_t a0 = a.x ^ ma, a1 = a.y ^ ma;
+                    if (!(ins.z & OP_CMP)) {
+                        // (a ^ ma) & (b ^ mb) as one LOP3 per word on the pre-complemented a:
+                        // inputs (t, b, m) = (0xF0, 0xCC, 0xAA): t & (b ^ m) = 0x60
+                        SLOT(ins.z) = make_uint2(lop3_60(a0, b.x, mb), lop3_60(a1, b.y, mb));
                     } else {
-                        const uint32_t d = active ? (a ^ b) : 0u;
-                        const uint32_t bal = __ballot_sync(FULL, d != 0u);
-                        if (bal) {
-                            const uint32_t l = (uint32_t)__ffs(bal) - 1u;
-                            const uint32_t dl = __shfl_sync(FULL, d, l);
-                            if (lane == 0) {
-                                const uint64_t idx = ((((uint64_t)s << 5) + l) << 5) + (uint32_t)(__ffs(dl) - 1);
-                                record_mismatch(ins.y & ~OP_CMP, idx, item.win, W, first, bound, neq_cnt);
-                            }
+                        const uint32_t d0 = act0 ? (a0 ^ b.x ^ mb) : 0u, d1 = act1 ? (a1 ^ b.y ^ mb) : 0u;
+                        if (__any_sync(FULL, (d0 | d1) != 0u)) {
+                            if (__any_sync(FULL, d0 != 0u))
+                                report(d0, base, lane, ins.z & ~OP_CMP, item.win, W, first, bound, neq_cnt);
+                            else
+                                report(d1, base + 32u, lane, ins.z & ~OP_CMP, item.win, W, first, bound, neq_cnt);
                         }
                     }
                 }
             }
         }
     }
+#undef SLOT
 }
 
 inline const char *ck(cudaError_t e) { return e == cudaSuccess ? nullptr : cudaGetErrorString(e); }
@@ -123,8 +145,8 @@ inline const char *ck(cudaError_t e) { return e == cudaSuccess ? nullptr : cudaG
 }  // namespace
 
 uint32_t interp_max_slots_per_warp() {
-    // one warp per block, whole shared memory: (nslots*32 + 64) * 4 <= 227 KB
-    return (uint32_t)((SMEM_PER_SM / 4 - 64) / 32);
+    // one warp per block, whole shared memory: nslots * SLOT_BYTES + 512 <= 227 KB
+    return (uint32_t)((SMEM_PER_SM - 32 * sizeof(uint4)) / SLOT_BYTES);
 }
 
 const char *launch_run(const DevPlan &d, const std::vector<LaunchGroup> &groups, uint32_t nwin, uint32_t ncmp,
@@ -146,7 +168,7 @@ const char *launch_run(const DevPlan &d, const std::vector<LaunchGroup> &groups,
             ++nl;
             continue;
         }
-        const size_t per_warp = ((size_t)G.nslots * 32 + 64) * 4;
+        const size_t per_warp = (size_t)G.nslots * SLOT_BYTES + 32 * sizeof(uint4);
         // warps per block: the choice that keeps the most warps resident per SM (smem-limited)
         int wpb = 1;
         size_t best = 0;
