@@ -264,10 +264,12 @@ def main():
         e2e = float(t.item())
 
     clocks = clk.summary()
-    sm_clock = clocks.get("sm_max_mhz") or 1965.0
+    sm_clock = clocks.get("sm_mhz") or clocks.get("sm_max_mhz") or 1965.0  # median SM clock seen under load
     props = torch.cuda.get_device_properties(local)
     peak = props.multi_processor_count * LOP3_PER_CLK_PER_SM * sm_clock * 1e6 / 1e12  # TLOP3/s
-    achieved = (W_rank / 32.0) / (ms / 1e3) / 1e12
+    # algorithmic LOP3s of the path: one 3-input LUT per mapped node group per u32 word (JIT), one
+    # per AND (interpreter) — the AND-node count itself is the metric W
+    achieved = stats["lop3_words"] / (ms / 1e3) / 1e12
     traffic = None
     prof = os.path.join(ROOT, "profiles", "ncu_summary.json")
     if os.path.exists(prof):
@@ -304,7 +306,9 @@ def main():
                     "host_prep_ms": st_e2e["host_prep_ms"], "aig_load_ms": load_ms},
             "roofline": {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "TLOP3/s",
                          "frac": achieved / peak, "traffic": traffic,
-                         "peak_basis": f"{props.multi_processor_count} SMs x {LOP3_PER_CLK_PER_SM} LOP3/clk x {sm_clock:.0f} MHz (guide unit counts, max SM clock)"},
+                         "peak_basis": f"{props.multi_processor_count} SMs x {LOP3_PER_CLK_PER_SM} LOP3/clk x {sm_clock:.0f} MHz (guide unit counts, SM clock)",
+                         "lop3_per_word_per_and": stats["lop3_words"] / max(1.0, W_rank / 32.0),
+                         "and_evals_tops": (W_rank / 32.0) / (ms / 1e3) / 1e12},
             "step_ms": step_ms, "wall_s": wall,
         }
         if cpu:

@@ -114,6 +114,9 @@ typedef struct {
     float jit_ms;              /* NVRTC compile + load time spent by the last plan (0 if cached) */
     uint32_t jit_kernels;      /* distinct window structures compiled for the last plan */
     uint32_t jit_windows;      /* windows of the last plan run by JIT kernels (rest: interpreter) */
+    uint64_t lop3_words;       /* LOP3 instructions x u32 words this rank executes per run for the AND
+                                  nodes: mapped 3-input LUTs for JIT windows (a LUT may evaluate
+                                  two ANDs), one per AND for interpreter windows */
 } cec_stats;
 
 /* Fill *opts with the defaults above. */

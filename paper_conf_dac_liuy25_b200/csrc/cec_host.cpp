@@ -65,6 +65,41 @@ NcclApi g_nccl;
 // ------------------------------------------------------------------------------------------------
 // Context and plan
 // ------------------------------------------------------------------------------------------------
+// Per-thread traversal scratch: epoch-stamped flat arrays over node ids (no hashing on the host
+// hot path); one per planning thread.
+struct Scratch {
+    std::vector<uint32_t> stamp, stack;
+    uint32_t epoch = 0;
+    std::vector<uint32_t> sc_stamp, sc_pos, sc_last, sc_slot;
+    uint32_t sc_epoch = 0;
+    std::vector<uint32_t> stop;
+    uint32_t stop_epoch = 0;
+    void init(size_t N) {
+        if (stamp.size() == N) return;
+        stamp.assign(N, 0);
+        sc_stamp.assign(N, 0);
+        sc_pos.assign(N, 0);
+        sc_last.assign(N, 0);
+        sc_slot.assign(N, 0);
+        stop.assign(N, 0);
+        epoch = sc_epoch = stop_epoch = 0;
+    }
+    uint32_t next_epoch() {
+        if (++epoch == 0) {
+            std::fill(stamp.begin(), stamp.end(), 0u);
+            epoch = 1;
+        }
+        return epoch;
+    }
+    uint32_t next_stop() {
+        if (++stop_epoch == 0) {
+            std::fill(stop.begin(), stop.end(), 0u);
+            stop_epoch = 1;
+        }
+        return stop_epoch;
+    }
+};
+
 struct cec_ctx {
     uint32_t I = 0, A = 0, O = 0;
     std::vector<uint32_t> f0, f1;  // fanin literals indexed by node id (valid for AND ids)
@@ -84,23 +119,10 @@ struct cec_ctx {
     // device copy of the AIG for random simulation (lazy)
     uint32_t *d_f0 = nullptr, *d_f1 = nullptr, *d_level_ids = nullptr;
     std::vector<uint32_t> level_off;
-    // scratch for the schedule builder
-    std::vector<uint32_t> sc_stamp, sc_pos, sc_last, sc_slot;
-    uint32_t sc_epoch = 0;
-    // scratch for traversals
-    std::vector<uint32_t> stamp;
-    uint32_t epoch = 0;
-    std::vector<uint32_t> stack;
+    Scratch scratch;  // for serial host work (supports of single pairs, cut validation)
 
     uint32_t N() const { return 1 + I + A; }
     bool is_and(uint32_t id) const { return id > I; }
-    uint32_t next_epoch() {
-        if (++epoch == 0) {
-            std::fill(stamp.begin(), stamp.end(), 0u);
-            epoch = 1;
-        }
-        return epoch;
-    }
 };
 
 struct WinHost {
@@ -135,6 +157,7 @@ struct cec_plan {
     std::vector<LaunchGroup> groups;
     uint32_t jit_windows = 0, jit_kernels = 0;
     float jit_ms = 0.f;
+    uint64_t lop3_words = 0;
     uint64_t W_rank = 0, W_all = 0;
     uint32_t max_k = 0, max_slots = 0;
     float host_ms = 0.f;
@@ -177,15 +200,17 @@ cec_status fail(cec_ctx *c, cec_status s, const char *fmt, ...) {
 // Structural TFI of the roots, stopping at nodes with stop_stamp == stop_epoch
 // (cut leaves) and at PIs/const. Visits every reached node once; calls f(id) for each.
 template <class F>
-void walk_tfi(cec_ctx *c, const uint32_t *roots, int nroots, const std::vector<uint32_t> *stop, uint32_t stop_epoch,
-              F &&f) {
-    const uint32_t ep = c->next_epoch();
-    auto &st = c->stack;
+void walk_tfi(const cec_ctx *c, Scratch &X, const uint32_t *roots, int nroots, const std::vector<uint32_t> *stop,
+              uint32_t stop_epoch, F &&f) {
+    X.init(c->N());
+    const uint32_t ep = X.next_epoch();
+    auto &st = X.stack;
+    auto &stamp = X.stamp;
     st.clear();
     for (int r = 0; r < nroots; ++r) {
         uint32_t v = roots[r];
-        if (c->stamp[v] != ep) {
-            c->stamp[v] = ep;
+        if (stamp[v] != ep) {
+            stamp[v] = ep;
             st.push_back(v);
         }
     }
@@ -196,12 +221,12 @@ void walk_tfi(cec_ctx *c, const uint32_t *roots, int nroots, const std::vector<u
         if (stop && (*stop)[v] == stop_epoch) continue;
         if (!c->is_and(v)) continue;
         uint32_t a = c->f0[v] >> 1, b = c->f1[v] >> 1;
-        if (c->stamp[a] != ep) {
-            c->stamp[a] = ep;
+        if (stamp[a] != ep) {
+            stamp[a] = ep;
             st.push_back(a);
         }
-        if (c->stamp[b] != ep) {
-            c->stamp[b] = ep;
+        if (stamp[b] != ep) {
+            stamp[b] = ep;
             st.push_back(b);
         }
     }
@@ -212,7 +237,7 @@ uint64_t support_of(cec_ctx *c, uint32_t la, uint32_t lb, std::vector<uint32_t> 
     S.clear();
     uint64_t nodes = 0;
     uint32_t roots[2] = {la >> 1, lb >> 1};
-    walk_tfi(c, roots, 2, nullptr, 0, [&](uint32_t v) {
+    walk_tfi(c, c->scratch, roots, 2, nullptr, 0, [&](uint32_t v) {
         if (v >= 1 && v <= c->I)
             S.push_back(v);
         else if (v > c->I)
@@ -230,27 +255,22 @@ struct Sched {
     uint32_t const_slot = 0xFFFFFFFFu;
 };
 
-bool build_schedule(cec_ctx *c, const std::vector<uint32_t> &inputs, const std::vector<uint32_t> &nodes,
-                    const std::vector<Cmp> &cmps, const std::vector<uint32_t> &win_cmps, Sched &out,
-                    std::string &why) {
+bool build_schedule(const cec_ctx *c, Scratch &X, const std::vector<uint32_t> &inputs,
+                    const std::vector<uint32_t> &nodes, const std::vector<Cmp> &cmps,
+                    const std::vector<uint32_t> &win_cmps, Sched &out, std::string &why) {
     const uint32_t k = (uint32_t)inputs.size();
     const uint32_t n = (uint32_t)nodes.size();
     // per-node scratch, valid where sc_stamp == ep (flat arrays: no hashing on the hot host path)
-    if (c->sc_stamp.size() != c->N()) {
-        c->sc_stamp.assign(c->N(), 0);
-        c->sc_pos.assign(c->N(), 0);
-        c->sc_last.assign(c->N(), 0);
-        c->sc_slot.assign(c->N(), 0);
+    X.init(c->N());
+    if (++X.sc_epoch == 0) {
+        std::fill(X.sc_stamp.begin(), X.sc_stamp.end(), 0u);
+        X.sc_epoch = 1;
     }
-    if (++c->sc_epoch == 0) {
-        std::fill(c->sc_stamp.begin(), c->sc_stamp.end(), 0u);
-        c->sc_epoch = 1;
-    }
-    const uint32_t ep = c->sc_epoch;
-    auto &stamp = c->sc_stamp;
-    auto &pos = c->sc_pos;    // 0 = input/const, t+1 = AND node t
-    auto &last = c->sc_last;  // last reading op + 1 (0 = never read)
-    auto &slot = c->sc_slot;
+    const uint32_t ep = X.sc_epoch;
+    auto &stamp = X.sc_stamp;
+    auto &pos = X.sc_pos;    // 0 = input/const, t+1 = AND node t
+    auto &last = X.sc_last;  // last reading op + 1 (0 = never read)
+    auto &slot = X.sc_slot;
     auto touch = [&](uint32_t id) {
         if (stamp[id] != ep) {
             stamp[id] = ep;
@@ -433,7 +453,6 @@ cec_status cec_load_aig(cec_ctx **out, const cec_aig *aig, const cec_opts *opts)
         c->f0.assign(N, 0);
         c->f1.assign(N, 0);
         c->level.assign(N, 0);
-        c->stamp.assign(N, 0);
     } catch (...) {
         return CEC_E_NOMEM;
     }
@@ -512,14 +531,27 @@ JitConfig jit_config() {  // overridable for tuning: CEC_JIT_THREADS / CEC_JIT_M
     if (const char *e = getenv("CEC_JIT_THREADS")) cfg.threads = atoi(e);
     if (const char *e = getenv("CEC_JIT_MINB")) cfg.min_blocks = atoi(e);
     if (const char *e = getenv("CEC_JIT_SYNC")) cfg.sync_every = atoi(e);
+    if (const char *e = getenv("CEC_JIT_FUSE")) cfg.fuse = atoi(e) != 0;
     return cfg;
 }
 
 uint64_t tt_words_of(uint32_t k) { return k <= 5 ? 1ull : (1ull << (k - 5)); }
 
 // Build per-window programs, work items and launch groups; compute W. Common to global and local.
+struct PhaseTimer {  // CEC_TIMING=1: per-phase host timings on stderr
+    bool on = getenv("CEC_TIMING") != nullptr;
+    std::chrono::steady_clock::time_point t = std::chrono::steady_clock::now();
+    void lap(const char *what) {
+        if (!on) return;
+        auto n = std::chrono::steady_clock::now();
+        fprintf(stderr, "[cec] %-28s %8.2f ms\n", what, std::chrono::duration<double, std::milli>(n - t).count());
+        t = n;
+    }
+};
+
 cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, const std::vector<uint32_t> *stop,
                        bool local) {
+    PhaseTimer tm;
     const int32_t rank = c->opts.rank, world = c->opts.world;
     P->dwin.clear();
     P->prog.clear();
@@ -533,47 +565,67 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
     std::vector<Cmp> cmps2;
     cmps2.reserve(P->cmps.size());
     std::vector<int32_t> remap(P->cmps.size(), -1);
-    std::vector<uint32_t> stop_mark;
     const uint32_t max_slot_cap = interp_max_slots_per_warp();
     std::vector<uint32_t> nslots_of;
     std::vector<uint64_t> cost_of;
     std::vector<int32_t> win_jit;                    // JIT structure index per window, -1 = interpreter
     std::vector<uint64_t> wps_of;                    // words per slice per window
+    std::vector<uint64_t> words_rank_of;             // u32 words this rank simulates per window
     std::vector<JitProgram> jit_progs;
     std::unordered_map<std::string, uint32_t> jit_index;
+    // (1) serial: lay out compares window by window (contiguous per window) and own-support masks
+    std::vector<std::vector<uint32_t>> wcs(wins.size());
     for (size_t w = 0; w < wins.size(); ++w) {
-        WinHost &W = wins[w];
-        DevWin dw{};
-        dw.cmp_off = (uint32_t)cmps2.size();
-        std::vector<uint32_t> wc;
-        for (uint32_t ci : W.cmps) {
+        for (uint32_t ci : wins[w].cmps) {
             remap[ci] = (int32_t)cmps2.size();
-            wc.push_back((uint32_t)cmps2.size());
+            wcs[w].push_back((uint32_t)cmps2.size());
             cmps2.push_back(P->cmps[ci]);
         }
-        dw.ncmp = (uint32_t)wc.size();
-        // window nodes: backward traversal from the roots stopping at the inputs (reading Q6)
+        for (uint32_t ci : wcs[w]) {  // a11 pext masks
+            Cmp &cm = cmps2[ci];
+            uint64_t m = 0;
+            size_t j = 0;
+            for (size_t t = 0; t < wins[w].inputs.size() && j < cm.S.size(); ++t) {
+                if (wins[w].inputs[t] == cm.S[j]) {
+                    m |= 1ull << t;
+                    ++j;
+                }
+            }
+            cm.ownmask = m;
+        }
+    }
+    // (2) parallel over windows: node order, schedule, engine choice, JIT program
+    struct WinRes {
+        std::vector<uint32_t> nodes;
+        Sched sc;
+        bool jit = false;
+        JitProgram jp;
+        std::string key, err;
+    };
+    std::vector<WinRes> res(wins.size());
+    auto plan_one = [&](size_t w, Scratch &X) {
+        WinHost &W = wins[w];
+        WinRes &R = res[w];
+        const std::vector<uint32_t> &wc = wcs[w];
         std::vector<uint32_t> roots;
         for (uint32_t ci : wc) {
             roots.push_back(cmps2[ci].la >> 1);
             roots.push_back(cmps2[ci].lb >> 1);
         }
-        // mark inputs as stop nodes
-        // a dedicated stop array (c->stamp is reused by walk_tfi)
-        if (stop_mark.size() != c->N()) stop_mark.assign(c->N(), 0);
-        const uint32_t sep = (uint32_t)w + 1;
-        for (uint32_t x : W.inputs) stop_mark[x] = sep;
+        X.init(c->N());
+        const uint32_t sep = X.next_stop();  // window inputs stop the backward traversal (Q6)
+        for (uint32_t x : W.inputs) X.stop[x] = sep;
         // Node order = a topological order chosen to keep the live set small (it sets the
         // interpreter's shared-memory slots and the JIT kernel's register pressure): depth-first
         // post-order from the roots, compare by compare, deeper fanin first (Sethi-Ullman style).
-        std::vector<uint32_t> nodes;
+        std::vector<uint32_t> &nodes = R.nodes;
         {
-            const uint32_t ep = c->next_epoch();
+            const uint32_t ep = X.next_epoch();
             std::vector<std::pair<uint32_t, uint8_t>> st;
             for (uint32_t r : roots) {
-                if (c->stamp[r] == ep || !c->is_and(r) || stop_mark[r] == sep) continue;
+                if (X.stamp[r] == ep || !c->is_and(r) || X.stop[r] == sep) continue;
                 st.push_back({r, 0});
-                c->stamp[r] = ep;
+                X.stamp[r] = ep;
                 while (!st.empty()) {
                     auto &top = st.back();
                     const uint32_t v = top.first;
@@ -582,8 +634,8 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
                         if (c->level[b] > c->level[a]) std::swap(a, b);  // deeper first
                         const uint32_t nxt = top.second == 0 ? a : b;
                         ++top.second;
-                        if (c->stamp[nxt] != ep && c->is_and(nxt) && stop_mark[nxt] != sep) {
-                            c->stamp[nxt] = ep;
+                        if (X.stamp[nxt] != ep && c->is_and(nxt) && X.stop[nxt] != sep) {
+                            X.stamp[nxt] = ep;
                             st.push_back({nxt, 0});
                         }
                     } else {
@@ -593,33 +645,90 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
                 }
             }
         }
-        for (uint32_t x : W.inputs) stop_mark[x] = 0;
-        // own-support masks (a11 pext)
-        for (uint32_t ci : wc) {
-            Cmp &cm = cmps2[ci];
-            uint64_t m = 0;
-            size_t j = 0;
-            for (size_t t = 0; t < W.inputs.size() && j < cm.S.size(); ++t) {
-                if (W.inputs[t] == cm.S[j]) {
-                    m |= 1ull << t;
-                    ++j;
-                }
-            }
-            cm.ownmask = m;
-        }
-        Sched sc;
         std::string why;
-        if (!build_schedule(c, W.inputs, nodes, cmps2, wc, sc, why)) return fail(c, CEC_E_NOMEM, "%s", why.c_str());
+        if (!build_schedule(c, X, W.inputs, nodes, cmps2, wc, R.sc, why)) {
+            R.err = why;
+            return;
+        }
         {  // the id order (the netlist's own construction order) is often the better one: keep the
            // order with the smaller live set
             std::vector<uint32_t> by_id(nodes);
             std::sort(by_id.begin(), by_id.end());
             Sched sc2;
-            if (build_schedule(c, W.inputs, by_id, cmps2, wc, sc2, why) && sc2.nslots < sc.nslots) {
-                sc = std::move(sc2);
+            if (build_schedule(c, X, W.inputs, by_id, cmps2, wc, sc2, why) && sc2.nslots < R.sc.nslots) {
+                R.sc = std::move(sc2);
                 nodes.swap(by_id);
             }
         }
+        const uint32_t k = (uint32_t)W.inputs.size();
+        // engine choice: straight-line register kernel for big windows (k >= 10 so a 32-word warp
+        // pass is never partial); the interpreter for small ones (JIT compile would dominate)
+        const uint64_t node_words = (uint64_t)nodes.size() * tt_words_of(k);
+        if (k >= 10 && !nodes.empty()) {
+            if (c->opts.engine == CEC_ENGINE_JIT) R.jit = true;
+            else if (c->opts.engine == CEC_ENGINE_AUTO) R.jit = node_words >= (1ull << 26) || R.sc.nslots > max_slot_cap;
+        }
+        if (!R.jit && R.sc.nslots > max_slot_cap) {
+            char b[160];
+            snprintf(b, sizeof b, "window %zu needs %u live slots > %u (shared-memory capacity)", w, R.sc.nslots,
+                     max_slot_cap);
+            R.err = b;
+            return;
+        }
+        if (R.jit) {  // SSA program: refs via the per-thread flat arrays (inputs 1..k, nodes k+1..)
+            JitProgram &jp = R.jp;
+            jp.k = k;
+            if (++X.sc_epoch == 0) {
+                std::fill(X.sc_stamp.begin(), X.sc_stamp.end(), 0u);
+                X.sc_epoch = 1;
+            }
+            const uint32_t ep = X.sc_epoch;
+            auto setref = [&](uint32_t id, uint32_t r) {
+                X.sc_stamp[id] = ep;
+                X.sc_pos[id] = r;
+            };
+            auto ref = [&](uint32_t id) { return id == 0 ? 0u : X.sc_pos[id]; };
+            for (uint32_t j = 0; j < k; ++j) setref(W.inputs[j], j + 1);
+            for (uint32_t t = 0; t < nodes.size(); ++t) setref(nodes[t], k + 1 + t);
+            jp.nodes.reserve(2 * nodes.size());
+            for (uint32_t id : nodes) {
+                jp.nodes.push_back(ref(c->f0[id] >> 1) << 1 | (c->f0[id] & 1u));
+                jp.nodes.push_back(ref(c->f1[id] >> 1) << 1 | (c->f1[id] & 1u));
+            }
+            for (uint32_t ci : wc) {
+                jp.cmps.push_back(ref(cmps2[ci].la >> 1) << 1 | (cmps2[ci].la & 1u));
+                jp.cmps.push_back(ref(cmps2[ci].lb >> 1) << 1 | (cmps2[ci].lb & 1u));
+            }
+            R.key = jit_key(jp);
+        }
+    };
+    {
+        const unsigned hw = std::max(1u, std::min(32u, std::thread::hardware_concurrency()));
+        const unsigned nt = (unsigned)std::min<size_t>(hw, std::max<size_t>(1, wins.size() / 2));
+        if (nt <= 1) {
+            for (size_t w = 0; w < wins.size(); ++w) plan_one(w, c->scratch);
+        } else {
+            std::atomic<size_t> next{0};
+            std::vector<std::thread> pool;
+            for (unsigned t = 0; t < nt; ++t)
+                pool.emplace_back([&]() {
+                    Scratch X;
+                    for (size_t w; (w = next.fetch_add(1)) < wins.size();) plan_one(w, X);
+                });
+            for (auto &th : pool) th.join();
+        }
+    }
+    // (3) serial assembly in window order
+    for (size_t w = 0; w < wins.size(); ++w) {
+        WinHost &W = wins[w];
+        WinRes &R = res[w];
+        if (!R.err.empty()) return fail(c, CEC_E_NOMEM, "%s", R.err.c_str());
+        const std::vector<uint32_t> &wc = wcs[w];
+        const std::vector<uint32_t> &nodes = R.nodes;
+        const Sched &sc = R.sc;
+        DevWin dw{};
+        dw.cmp_off = wc.empty() ? (uint32_t)cmps2.size() : wc[0];
+        dw.ncmp = (uint32_t)wc.size();
         dw.prog_off = (uint32_t)P->prog.size();
         dw.prog_len = (uint32_t)sc.ops.size();
         dw.k = (uint32_t)W.inputs.size();
@@ -633,39 +742,12 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         P->win_nodes.push_back((uint32_t)nodes.size());
         P->win_cmps.push_back(wc);
         nslots_of.push_back(sc.nslots);
-        // engine choice: straight-line register kernel for big windows (k >= 10 so a 32-word warp
-        // pass is never partial); the interpreter for small ones (JIT compile would dominate)
-        const uint64_t node_words = (uint64_t)nodes.size() * ttw;
-        bool jit = false;
-        if (dw.k >= 10 && !nodes.empty()) {
-            if (c->opts.engine == CEC_ENGINE_JIT) jit = true;
-            else if (c->opts.engine == CEC_ENGINE_AUTO) jit = node_words >= (1ull << 26) || sc.nslots > max_slot_cap;
-        }
-        if (!jit && sc.nslots > max_slot_cap)
-            return fail(c, CEC_E_NOMEM, "window %zu needs %u live slots > %u (shared-memory capacity)", w, sc.nslots,
-                        max_slot_cap);
+        const bool jit = R.jit;
         if (jit) {
-            JitProgram jp;
-            jp.k = dw.k;
-            std::unordered_map<uint32_t, uint32_t> ref;
-            ref.reserve(2 * (nodes.size() + W.inputs.size()) + 4);
-            ref[0] = 0;
-            for (uint32_t j = 0; j < dw.k; ++j) ref[W.inputs[j]] = j + 1;
-            for (uint32_t t = 0; t < nodes.size(); ++t) ref[nodes[t]] = dw.k + 1 + t;
-            jp.nodes.reserve(2 * nodes.size());
-            for (uint32_t id : nodes) {
-                jp.nodes.push_back(ref.at(c->f0[id] >> 1) << 1 | (c->f0[id] & 1u));
-                jp.nodes.push_back(ref.at(c->f1[id] >> 1) << 1 | (c->f1[id] & 1u));
-            }
-            for (uint32_t ci : wc) {
-                jp.cmps.push_back(ref.at(cmps2[ci].la >> 1) << 1 | (cmps2[ci].la & 1u));
-                jp.cmps.push_back(ref.at(cmps2[ci].lb >> 1) << 1 | (cmps2[ci].lb & 1u));
-            }
-            std::string key = jit_key(jp);
-            auto it = jit_index.find(key);
+            auto it = jit_index.find(R.key);
             if (it == jit_index.end()) {
-                it = jit_index.emplace(key, (uint32_t)jit_progs.size()).first;
-                jit_progs.push_back(std::move(jp));
+                it = jit_index.emplace(R.key, (uint32_t)jit_progs.size()).first;
+                jit_progs.push_back(std::move(R.jp));
             }
             win_jit.push_back((int32_t)it->second);
         } else {
@@ -684,8 +766,10 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         uint64_t wb = sb * wps, we = std::min<uint64_t>(se * wps, ttw);
         uint64_t pats_rank = we > wb ? (dw.k < 5 ? (1ull << dw.k) : (we - wb) * 32) : 0;
         P->W_rank += (uint64_t)nodes.size() * pats_rank;
+        words_rank_of.push_back(we > wb ? (we - wb) : 0);
         cost_of.push_back((uint64_t)(dw.prog_len + 1) * (se - sb));
     }
+    tm.lap("windows+schedules+jit-progs");
     P->cmps.swap(cmps2);
     for (auto &pc : P->pair_cmp)
         if (pc >= 0) pc = remap[pc];
@@ -717,9 +801,15 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         }
         P->jit_ms = std::chrono::duration<float, std::milli>(std::chrono::steady_clock::now() - t0).count();
     }
+    tm.lap("jit compile/cache");
     P->jit_kernels = (uint32_t)jit_progs.size();
     P->jit_windows = 0;
-    for (int32_t j : win_jit) P->jit_windows += j >= 0;
+    P->lop3_words = 0;
+    for (size_t w = 0; w < win_jit.size(); ++w) {
+        P->jit_windows += win_jit[w] >= 0;
+        const uint64_t per_word = win_jit[w] >= 0 ? jit_kernel_lop3(kernels[win_jit[w]]) : P->win_nodes[w];
+        P->lop3_words += per_word * words_rank_of[w];
+    }
     // work items: slices of each window split into chunks; interpreter windows grouped by slot
     // budget, JIT windows by structure; largest windows first inside a group
     std::map<uint32_t, std::vector<uint32_t>> buckets;   // interpreter: slot budget -> windows
@@ -991,6 +1081,7 @@ cec_status cec_plan_exhaustive(cec_ctx *c, uint32_t n, const uint32_t *la, const
     c->stats.jit_ms = P->jit_ms;
     c->stats.jit_kernels = P->jit_kernels;
     c->stats.jit_windows = P->jit_windows;
+    c->stats.lop3_words = P->lop3_words;
     st = upload(c, P.get());
     if (st != CEC_OK) {
         free_dev(P.get());
@@ -1212,7 +1303,7 @@ cec_status cec_check_local_cuts(cec_ctx *c, uint32_t n, const uint32_t *la, cons
         for (uint32_t x : L) stop[x] = sep;
         bool ok = true;
         uint32_t roots[2] = {la[q] >> 1, lb[q] >> 1};
-        walk_tfi(c, roots, 2, &stop, sep, [&](uint32_t v) {
+        walk_tfi(c, c->scratch, roots, 2, &stop, sep, [&](uint32_t v) {
             if (v >= 1 && v <= c->I && stop[v] != sep) ok = false;
         });
         if (!ok) {

@@ -57,7 +57,8 @@ struct JitKernel;
 struct JitConfig {
     int threads = 512;      // threads per block
     int min_blocks = 1;     // __launch_bounds__ min blocks per SM (registers <= 64K / (threads*min_blocks))
-    int sync_every = 512;   // block-synchronous: __syncthreads() every this many nodes; 0 = warp-independent
+    int sync_every = 512;   // block-synchronous: __syncthreads() every this many LOP3s; 0 = warp-independent
+    bool fuse = true;       // 3-input LUT mapping: absorb single-fanout ANDs into their reader's LOP3
 };
 struct LaunchGroup {       // windows sharing one kernel launch
     uint32_t nslots;       // interpreter: slots per warp in this launch
@@ -84,6 +85,8 @@ const char *jit_compile_cubin(const std::string &src, std::vector<char> &cubin, 
 const char *jit_get_kernel(const JitProgram &p, const JitConfig &cfg, bool load, JitKernel **out);
 double jit_compile_ms(const JitKernel *k);
 int jit_slices_per_pass(const JitKernel *k);
+uint32_t jit_kernel_lop3(const JitKernel *k);
+uint32_t jit_lop3_count(const JitProgram &p, bool fuse);
 const char *jit_launch(JitKernel *K, const JItem *items, uint32_t nitems, uint32_t *ctr, unsigned long long *first,
                        unsigned long long *bound, uint32_t *neq_cnt, void *stream, int num_sms);
 

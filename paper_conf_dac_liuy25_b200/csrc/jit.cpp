@@ -94,6 +94,7 @@ struct JitKernel {
     int block = 128;
     int blocks_per_sm = 0;
     int slices_per_pass = 1;  // block-synchronous kernels: warps per block
+    uint32_t lop3 = 0;        // LOP3 instructions per word of the mapped window
     double compile_ms = 0;
     size_t src_bytes = 0, cubin_bytes = 0;
 };
@@ -108,6 +109,104 @@ std::string jit_key(const JitProgram &p) {
     for (uint32_t v : p.nodes) put(v);
     for (uint32_t v : p.cmps) put(v);
     return key;
+}
+
+// ---- 3-input LUT mapping of the window (one LOP3 per LUT) ----------------------------------------
+// An AND node whose only reader is the next AND up (single fanout inside the window, not a compare
+// root) need not be materialised: the reader's LOP3 can take the absorbed node's fanins directly,
+// as long as the union of leaves stays <= 3 (a LOP3 evaluates ANY 3-input function from an 8-bit
+// LUT). Greedy, in topological order: absorb both fanins if possible, else one, else none. Every AND
+// node is still evaluated exactly (inside the LUT of its reader); only the register write of the
+// absorbed intermediate disappears. The LUT is obtained by evaluating the absorbed expression on
+// the canonical truth tables of the LOP3 inputs (a = 0xF0, b = 0xCC, c = 0xAA).
+struct MappedNode {
+    bool absorbed = false;
+    uint8_t nleaves = 0;
+    uint32_t leaf[3] = {0, 0, 0};  // operand refs
+    uint8_t tt = 0;
+};
+
+std::vector<MappedNode> jit_map(const JitProgram &p, bool fuse) {
+    const uint32_t n = (uint32_t)(p.nodes.size() / 2), ncmp = (uint32_t)(p.cmps.size() / 2);
+    std::vector<uint32_t> uses(p.k + 1 + n, 0);
+    for (uint32_t i = 0; i < 2 * n; ++i) ++uses[p.nodes[i] >> 1];
+    std::vector<bool> root(p.k + 1 + n, false);
+    for (uint32_t i = 0; i < 2 * ncmp; ++i) root[p.cmps[i] >> 1] = true;
+    std::vector<MappedNode> m(n);
+    auto is_node = [&](uint32_t ref) { return ref > p.k; };
+    // value of operand (ref, compl) as an 8-bit truth table over the chosen leaves
+    std::function<uint8_t(uint32_t, uint32_t, const MappedNode &, bool)> eval;
+    for (uint32_t t = 0; t < n; ++t) {
+        const uint32_t oa = p.nodes[2 * t], ob = p.nodes[2 * t + 1];
+        const uint32_t ra = oa >> 1, rb = ob >> 1;
+        auto can = [&](uint32_t r) {
+            return fuse && is_node(r) && uses[r] == 1 && !root[r] && r - p.k - 1 < t;
+        };
+        auto leaves_of = [&](uint32_t r, bool expand, std::vector<uint32_t> &L) {
+            if (expand) {
+                const MappedNode &u = m[r - p.k - 1];
+                for (int i = 0; i < u.nleaves; ++i) L.push_back(u.leaf[i]);
+            } else {
+                L.push_back(r);
+            }
+        };
+        MappedNode best;
+        bool done = false;
+        const bool opts[4][2] = {{true, true}, {true, false}, {false, true}, {false, false}};
+        for (auto &o : opts) {
+            const bool ea = o[0] && can(ra), eb = o[1] && can(rb);
+            if ((o[0] && !ea) || (o[1] && !eb)) continue;
+            std::vector<uint32_t> L;
+            leaves_of(ra, ea, L);
+            leaves_of(rb, eb, L);
+            std::sort(L.begin(), L.end());
+            L.erase(std::unique(L.begin(), L.end()), L.end());
+            if (L.size() > 3) continue;
+            MappedNode cand;
+            cand.nleaves = (uint8_t)L.size();
+            for (size_t i = 0; i < L.size(); ++i) cand.leaf[i] = L[i];
+            static const uint8_t K[3] = {0xF0, 0xCC, 0xAA};
+            auto leaf_tt = [&](uint32_t r) -> uint8_t {
+                for (int i = 0; i < cand.nleaves; ++i)
+                    if (cand.leaf[i] == r) return K[i];
+                return 0;  // unreachable
+            };
+            auto operand_tt = [&](uint32_t r, uint32_t c, bool expand) -> uint8_t {
+                uint8_t v;
+                if (expand) {  // evaluate the absorbed node's own LUT on the new leaf constants
+                    const MappedNode &u = m[r - p.k - 1];
+                    uint8_t in[3] = {0, 0, 0};
+                    for (int i = 0; i < u.nleaves; ++i) in[i] = leaf_tt(u.leaf[i]);
+                    v = 0;
+                    for (int bit = 0; bit < 8; ++bit) {
+                        const int idx = (((in[0] >> bit) & 1) << 2) | (((in[1] >> bit) & 1) << 1) | ((in[2] >> bit) & 1);
+                        // u.tt bit for inputs (x0, x1, x2) sits at position 4*x0 + 2*x1 + x2
+                        v |= (uint8_t)(((u.tt >> idx) & 1) << bit);
+                    }
+                } else {
+                    v = leaf_tt(r);
+                }
+                return c ? (uint8_t)~v : v;
+            };
+            cand.tt = operand_tt(ra, oa & 1u, ea) & operand_tt(rb, ob & 1u, eb);
+            best = cand;
+            if (ea) m[ra - p.k - 1].absorbed = true;
+            if (eb && rb != ra) m[rb - p.k - 1].absorbed = true;
+            done = true;
+            break;
+        }
+        (void)done;
+        m[t].nleaves = best.nleaves;
+        for (int i = 0; i < 3; ++i) m[t].leaf[i] = best.leaf[i];
+        m[t].tt = best.tt;
+    }
+    return m;
+}
+
+uint32_t jit_lop3_count(const JitProgram &p, bool fuse) {
+    uint32_t c = 0;
+    for (const MappedNode &x : jit_map(p, fuse)) c += !x.absorbed;
+    return c;
 }
 
 std::string jit_source(const JitProgram &p, const JitConfig &cfg) {
@@ -195,16 +294,23 @@ std::string jit_source(const JitProgram &p, const JitConfig &cfg) {
                  inv ? "~(" : "", ref_name(p, a >> 1).c_str(), ref_name(p, b >> 1).c_str(), inv ? ")" : "", c, ncmp);
         s += buf;
     };
-    static const unsigned lut[4] = {0xC0, 0x0C, 0x30, 0x03};  // index = ca | cb << 1; a = 0xF0, b = 0xCC
+    const std::vector<MappedNode> map = jit_map(p, cfg.fuse);
     for (uint32_t c : after[0]) emit_cmp(c);
+    uint32_t emitted = 0;
     for (uint32_t t = 0; t < n; ++t) {
-        const uint32_t a = p.nodes[2 * t], b = p.nodes[2 * t + 1];
-        const unsigned L = lut[(a & 1u) | ((b & 1u) << 1)];
-        snprintf(buf, sizeof buf, "      u32 n%u; asm(\"lop3.b32 %%0, %%1, %%2, 0, 0x%02X;\" : \"=r\"(n%u) : \"r\"(%s), \"r\"(%s));\n",
-                 t, L, t, ref_name(p, a >> 1).c_str(), ref_name(p, b >> 1).c_str());
-        s += buf;
+        const MappedNode &x = map[t];
+        if (!x.absorbed) {
+            // LOP3 input order (a, b, c) = leaf[0..2]; the LUT was built for (0xF0, 0xCC, 0xAA)
+            snprintf(buf, sizeof buf,
+                     "      u32 n%u; asm(\"lop3.b32 %%0, %%1, %%2, %%3, 0x%02X;\" : \"=r\"(n%u) : \"r\"(%s), \"r\"(%s), \"r\"(%s));\n",
+                     t, x.tt, t, x.nleaves > 0 ? ref_name(p, x.leaf[0]).c_str() : "0u",
+                     x.nleaves > 1 ? ref_name(p, x.leaf[1]).c_str() : "0u",
+                     x.nleaves > 2 ? ref_name(p, x.leaf[2]).c_str() : "0u");
+            s += buf;
+            ++emitted;
+        }
         for (uint32_t c : after[t + 1]) emit_cmp(c);
-        if (block_sync && (t + 1) % (uint32_t)cfg.sync_every == 0 && t + 1 < n) s += "      __syncthreads();\n";
+        if (block_sync && !x.absorbed && emitted % (uint32_t)cfg.sync_every == 0) s += "      __syncthreads();\n";
     }
     s += block_sync ? "    }\n    __syncthreads();\n  }\n}\n" : "    }\n  }\n}\n";
     return s;
@@ -241,7 +347,7 @@ std::map<std::string, std::unique_ptr<JitKernel>> g_cache;  // process-wide, key
 
 const char *jit_get_kernel(const JitProgram &p, const JitConfig &cfg, bool load, JitKernel **out) {
     char ck[64];
-    snprintf(ck, sizeof ck, "|%d,%d,%d", cfg.threads, cfg.min_blocks, cfg.sync_every);
+    snprintf(ck, sizeof ck, "|%d,%d,%d,%d", cfg.threads, cfg.min_blocks, cfg.sync_every, (int)cfg.fuse);
     const std::string key = jit_key(p) + ck;
     {
         std::lock_guard<std::mutex> g(g_mu);
@@ -277,6 +383,7 @@ const char *jit_get_kernel(const JitProgram &p, const JitConfig &cfg, bool load,
     }
     std::unique_ptr<JitKernel> K(new JitKernel());
     K->block = cfg.threads;
+    K->lop3 = jit_lop3_count(p, cfg.fuse);
     K->slices_per_pass = cfg.sync_every > 0 ? cfg.threads / 32 : 1;
     K->src_bytes = src.size();
     K->cubin_bytes = cubin.size();
@@ -300,6 +407,7 @@ const char *jit_get_kernel(const JitProgram &p, const JitConfig &cfg, bool load,
 
 double jit_compile_ms(const JitKernel *k) { return k ? k->compile_ms : 0.0; }
 int jit_slices_per_pass(const JitKernel *k) { return k ? k->slices_per_pass : 1; }
+uint32_t jit_kernel_lop3(const JitKernel *k) { return k ? k->lop3 : 0; }
 
 const char *jit_launch(JitKernel *K, const JItem *items, uint32_t nitems, uint32_t *ctr, unsigned long long *first,
                        unsigned long long *bound, uint32_t *neq_cnt, void *stream, int num_sms) {
