@@ -1,0 +1,21 @@
+"""Run the CEC driver (P/G/L flow) on C4 and its bug variant; print the phase log as JSON lines."""
+import json
+import os
+import sys
+import time
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+from paper_conf_dac_liuy25_b200 import capi, driver  # noqa: E402
+from workloads import c4_dp  # noqa: E402
+
+for name, m in (("c4_dp64", c4_dp(64)), ("c4_dp64_bug4", c4_dp(64, bug=4))):
+    t = time.perf_counter()
+    r = driver.check_miter(m.aig, m.lit_a, m.lit_b, driver.CecParams(k_l=16))
+    dt = time.perf_counter() - t
+    names = {capi.CEC_EQUIVALENT: "EQ", capi.CEC_NOT_EQUIVALENT: "NEQ", capi.CEC_UNDECIDED: "UND"}
+    print(json.dumps({"miter": name, "verdict": names[r.verdict], "seconds": round(dt, 2),
+                      "po_eq": int((r.po_verdicts == capi.CEC_EQUIVALENT).sum()),
+                      "po_neq": int((r.po_verdicts == capi.CEC_NOT_EQUIVALENT).sum()),
+                      "po_und": int((r.po_verdicts == capi.CEC_UNDECIDED).sum()),
+                      "local_checks": len(r.checks), "final_ands": r.final_ands, "start_ands": int(m.aig.num_ands),
+                      "log": r.log}), flush=True)
