@@ -37,6 +37,7 @@ class CecParams:
     seed: int = 1
     max_phases: int = 64
     max_cuts_per_pair: int = 8
+    final_po_check: bool = True  # after the L phases: exhaustive check of undecided POs with k <= k_P
     device: int = 0
     engine: int = capi.CEC_ENGINE_AUTO
 
@@ -105,11 +106,17 @@ def _bits(mask: int) -> List[int]:
     return out
 
 
-def enumerate_cuts(aig: Aig, k_l: int, C: int, pass_id: int) -> List[List[int]]:
+def enumerate_cuts(aig: Aig, k_l: int, C: int, pass_id: int, repr_of: Optional[Dict[int, int]] = None
+                   ) -> List[List[int]]:
     """P(n) for every node id as bitmasks over node ids. E(n) = {u | v : u in P(n0) + {{n0}},
     v in P(n1) + {{n1}}, |u | v| <= k_l} (Eq. 1); P(n) = the C best of E(n) under the
     Table I order of this pass: pass 1 fanout > size > small level; pass 2 small
-    level > size > fanout; pass 3 large level > size > fanout. PIs: P = {{pi}} (Alg. 2 l.4-5)."""
+    level > size > fanout; pass 3 large level > size > fanout. PIs: P = {{pi}} (Alg. 2 l.4-5).
+    Dominated cuts (supersets of another candidate) are dropped first (priority cuts, ref. [27]).
+    Similarity-guided selection: for a non-representative n (repr_of[n] = r) the
+    candidates are ranked first by s(c, P(r)) = sum_{c' in P(r)} |c & c'| / |c | c'| (larger
+    first), then by the Table I order. Ids ascend, so P(r) is ready before P(n) (r < n), which is
+    what the enumeration levels of Eq. (2) guarantee in the paper's level-wise schedule."""
     I, A = aig.num_pis, aig.num_ands
     N = 1 + I + A
     fan = aig.fanins.astype(np.int64)
@@ -124,6 +131,7 @@ def enumerate_cuts(aig: Aig, k_l: int, C: int, pass_id: int) -> List[List[int]]:
     for i in range(1, I + 1):
         P[i] = [1 << i]
     P[0] = [1]  # constant: treat as its own leaf
+    repr_of = repr_of or {}
 
     def key(mask: int):
         ids = _bits(mask)
@@ -148,7 +156,18 @@ def enumerate_cuts(aig: Aig, k_l: int, C: int, pass_id: int) -> List[List[int]]:
                 if c.bit_count() <= k_l:
                     E.add(c)
         E.discard(1 << n)
-        P[n] = sorted(E, key=key)[:C]
+        # drop dominated cuts (a proper superset of another candidate)
+        Es = sorted(E, key=lambda x: x.bit_count())
+        kept: List[int] = []
+        for c in Es:
+            if not any((c & d) == d for d in kept):
+                kept.append(c)
+        r = repr_of.get(n)
+        if r is not None and P[r]:
+            Pr = P[r]
+            P[n] = sorted(kept, key=lambda c: (-sum((c & d).bit_count() / (c | d).bit_count() for d in Pr),) + key(c))[:C]
+        else:
+            P[n] = sorted(kept, key=key)[:C]
     return P
 
 
@@ -257,7 +276,8 @@ def check_miter(aig: Aig, lit_a, lit_b, params: Optional[CecParams] = None) -> C
         for pass_id in range(3):
             if not remaining:
                 break
-            cuts = enumerate_cuts(cur.aig, p.k_l, p.C, pass_id)
+            repr_of = {m_: r for r, m_, f in remaining}
+            cuts = enumerate_cuts(cur.aig, p.k_l, p.C, pass_id, repr_of)
             ql, qm, off, leaves, who = [], [], [0], [], []
             for r, m_, f in remaining:
                 if m_ in subst:
@@ -294,6 +314,32 @@ def check_miter(aig: Aig, lit_a, lit_b, params: Optional[CecParams] = None) -> C
         cur, _ = cur.reduce(subst)
     st = po_status(cur)
     po_v = np.where(st == capi.CEC_EQUIVALENT, capi.CEC_EQUIVALENT, po_v)
-    verdict = capi.CEC_EQUIVALENT if (po_v == capi.CEC_EQUIVALENT).all() else capi.CEC_UNDECIDED
-    # the reduced miter's PO pairs that remain can still be refuted exhaustively when small
-    return CecResult(verdict, po_v, log=log, checks=checks, versions=versions, final_ands=cur.aig.num_ands)
+    cex_vec, cex_pair = None, -1
+    if p.final_po_check and (po_v != capi.CEC_EQUIVALENT).any():
+        # The P phase only simulated POs with k <= k_p when some PO exceeded k_P.
+        # On the reduced miter, the still-undecided POs with k <= k_P are decided exhaustively
+        # (an extension of the paper's flow, which hands them to ABC instead).
+        t = time.perf_counter()
+        hctx = capi.Context.from_aig(cur.aig, device=-1, k_max=63)
+        und = [q for q in range(P) if po_v[q] != capi.CEC_EQUIVALENT and
+               hctx.pair_k(int(cur.lit_a[q]), int(cur.lit_b[q])) <= p.k_P]
+        hctx.close()
+        if und:
+            ctx = _ctx(cur.aig, p, p.k_P)
+            v, _, _ = ctx.sim_exhaustive(cur.lit_a[und], cur.lit_b[und])
+            for i, q in enumerate(und):
+                if v[i] != capi.CEC_UNDECIDED:
+                    po_v[q] = v[i]
+            neq = [i for i, q in enumerate(und) if v[i] == capi.CEC_NOT_EQUIVALENT]
+            if neq:
+                cex_vec, cex_pair = ctx.get_cex(neq[0]), und[neq[0]]
+            ctx.close()
+        log.append({"phase": "final-P", "threshold": p.k_P, "simulated": len(und), "s": time.perf_counter() - t})
+    if (po_v == capi.CEC_NOT_EQUIVALENT).any():
+        verdict = capi.CEC_NOT_EQUIVALENT
+    elif (po_v == capi.CEC_EQUIVALENT).all():
+        verdict = capi.CEC_EQUIVALENT
+    else:
+        verdict = capi.CEC_UNDECIDED
+    return CecResult(verdict, po_v, cex=cex_vec, cex_pair=cex_pair, log=log, checks=checks, versions=versions,
+                     final_ands=cur.aig.num_ands)

@@ -10,7 +10,7 @@ from workloads import c4_dp  # noqa: E402
 
 for name, m in (("c4_dp64", c4_dp(64)), ("c4_dp64_bug4", c4_dp(64, bug=4))):
     t = time.perf_counter()
-    r = driver.check_miter(m.aig, m.lit_a, m.lit_b, driver.CecParams(k_l=16))
+    r = driver.check_miter(m.aig, m.lit_a, m.lit_b, driver.CecParams(k_l=16, C=16))
     dt = time.perf_counter() - t
     names = {capi.CEC_EQUIVALENT: "EQ", capi.CEC_NOT_EQUIVALENT: "NEQ", capi.CEC_UNDECIDED: "UND"}
     print(json.dumps({"miter": name, "verdict": names[r.verdict], "seconds": round(dt, 2),
