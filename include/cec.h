@@ -155,6 +155,19 @@ cec_status cec_check_local_cuts(cec_ctx *ctx, uint32_t num_checks, const uint32_
  * representative = minimum id); a signature is a filter, never a proof. */
 cec_status cec_sim_random(cec_ctx *ctx, uint32_t num_words, uint64_t seed, uint64_t *sig_out, uint8_t *phase_out);
 
+/* Host cut generator for local checks (Eq. 1, Table I, similarity-guided
+ * selection). For candidate pairs q (repr[q] < member[q], node ids; member equivalent to repr up to
+ * complement), enumerate priority cuts (<= C per node, <= k_l <= 24 leaves, dominated cuts dropped,
+ * Table I order of pass_id in {0,1,2}; members ranked first by similarity to their
+ * representative's cuts) over the TFI of all pairs, and return each pair's common cuts u|v
+ * (<= k_l leaves, smallest first, at most max_cuts): pair q's cuts are [pair_cut_off[q],
+ * pair_cut_off[q+1]) and cut t's leaves (node ids, increasing) are leaves[cut_off[t] ..
+ * cut_off[t+1]). Caller-owned outputs: pair_cut_off[npairs+1], cut_off[npairs*max_cuts+1],
+ * leaves[npairs*max_cuts*k_l]. Host-only (no GPU needed); feed the cuts to cec_check_local_cuts. */
+cec_status cec_common_cuts(cec_ctx *ctx, uint32_t npairs, const uint32_t *repr, const uint32_t *member,
+                           uint32_t k_l, uint32_t C, int32_t pass_id, uint32_t max_cuts, uint32_t *pair_cut_off,
+                           uint32_t *cut_off, uint32_t *leaves);
+
 /* Counter-example of pair `pair_idx` of the most recent cec_sim_exhaustive / cec_plan_results:
  * pi_values_out[i] = value of PI id i+1 (0/1): PI S[j] = bit j of the CEX index, every other PI 0.
  * CEC_E_NOCEX unless that pair was NOT_EQUIVALENT; CEC_E_STATE before any global check. */

@@ -27,7 +27,8 @@ STATUS_NAMES = ["CEC_OK", "CEC_E_ARG", "CEC_E_AIG", "CEC_E_CUT", "CEC_E_NOMEM", 
 EXPORTS = ["cec_default_opts", "cec_load_aig", "cec_sim_exhaustive", "cec_check_local_cuts", "cec_get_cex",
            "cec_pair_support", "cec_plan_exhaustive", "cec_plan_run", "cec_plan_results", "cec_plan_info",
            "cec_plan_window", "cec_plan_free", "cec_stream", "cec_get_stats", "cec_shard_range", "cec_pext64",
-           "cec_free", "cec_last_error", "cec_abi_version", "cec_nccl_unique_id", "cec_sim_random"]
+           "cec_free", "cec_last_error", "cec_abi_version", "cec_nccl_unique_id", "cec_sim_random",
+           "cec_common_cuts"]
 
 
 class CecOpts(ctypes.Structure):
@@ -87,6 +88,7 @@ def _load() -> ctypes.CDLL:
         "cec_abi_version": (ctypes.c_int, []),
         "cec_nccl_unique_id": (ctypes.c_int, [P]),
         "cec_sim_random": (ctypes.c_int, [P, u32, u64, P, P]),
+        "cec_common_cuts": (ctypes.c_int, [P, u32, P, P, u32, u32, i32, u32, P, P, P]),
     }
     for name, (res, args) in sig.items():
         fn = getattr(L, name)
@@ -173,6 +175,18 @@ def cec_sim_random(ctx, num_nodes: int, num_words: int = 64, seed: int = 1):
     ph = np.zeros(max(num_nodes, 1), np.uint8)
     _check(lib.cec_sim_random(ctx, num_words, seed, _p(sig), _p(ph)), ctx)
     return sig[:num_nodes], ph[:num_nodes]
+
+
+def cec_common_cuts(ctx, repr_ids, member_ids, k_l: int, C: int, pass_id: int, max_cuts: int):
+    """Common cuts per candidate pair: (pair_cut_off[n+1], cut_off[ncut+1], leaves[...])."""
+    r, m = _u32(repr_ids), _u32(member_ids)
+    n = r.size
+    pco = np.zeros(n + 1, np.uint32)
+    co = np.zeros(n * max_cuts + 1, np.uint32)
+    lv = np.zeros(max(1, n * max_cuts * k_l), np.uint32)
+    _check(lib.cec_common_cuts(ctx, n, _p(r), _p(m), k_l, C, pass_id, max_cuts, _p(pco), _p(co), _p(lv)), ctx)
+    ncut = int(pco[n])
+    return pco, co[:ncut + 1], lv[:int(co[ncut])]
 
 
 def cec_get_cex(ctx, pair_idx: int, num_pis: int) -> np.ndarray:

@@ -27,6 +27,7 @@
 #include <vector>
 
 #include "../../include/cec.h"
+#include "cec_ctx.hpp"
 #include "cec_internal.hpp"
 
 using namespace cec;
@@ -61,112 +62,6 @@ struct NcclApi {
 };
 NcclApi g_nccl;
 }  // namespace
-
-// ------------------------------------------------------------------------------------------------
-// Context and plan
-// ------------------------------------------------------------------------------------------------
-// Per-thread traversal scratch: epoch-stamped flat arrays over node ids (no hashing on the host
-// hot path); one per planning thread.
-struct Scratch {
-    std::vector<uint32_t> stamp, stack;
-    uint32_t epoch = 0;
-    std::vector<uint32_t> sc_stamp, sc_pos, sc_last, sc_slot;
-    uint32_t sc_epoch = 0;
-    std::vector<uint32_t> stop;
-    uint32_t stop_epoch = 0;
-    void init(size_t N) {
-        if (stamp.size() == N) return;
-        stamp.assign(N, 0);
-        sc_stamp.assign(N, 0);
-        sc_pos.assign(N, 0);
-        sc_last.assign(N, 0);
-        sc_slot.assign(N, 0);
-        stop.assign(N, 0);
-        epoch = sc_epoch = stop_epoch = 0;
-    }
-    uint32_t next_epoch() {
-        if (++epoch == 0) {
-            std::fill(stamp.begin(), stamp.end(), 0u);
-            epoch = 1;
-        }
-        return epoch;
-    }
-    uint32_t next_stop() {
-        if (++stop_epoch == 0) {
-            std::fill(stop.begin(), stop.end(), 0u);
-            stop_epoch = 1;
-        }
-        return stop_epoch;
-    }
-};
-
-struct cec_ctx {
-    uint32_t I = 0, A = 0, O = 0;
-    std::vector<uint32_t> f0, f1;  // fanin literals indexed by node id (valid for AND ids)
-    std::vector<uint32_t> level;   // a1: level(PI)=0, level(AND)=1+max(fanins)
-    cec_opts opts{};
-    bool host_only = true;
-    void *stream = nullptr, *own_stream = nullptr;
-    int num_sms = 0;
-    ncclComm_t comm = nullptr;
-    std::string err;
-    cec_stats stats{};
-    // last global check (for cec_get_cex)
-    bool have_last = false;
-    std::vector<int32_t> last_verdict;
-    std::vector<uint64_t> last_cex;
-    std::vector<std::vector<uint32_t>> last_support;
-    // device copy of the AIG for random simulation (lazy)
-    uint32_t *d_f0 = nullptr, *d_f1 = nullptr, *d_level_ids = nullptr;
-    std::vector<uint32_t> level_off;
-    Scratch scratch;  // for serial host work (supports of single pairs, cut validation)
-
-    uint32_t N() const { return 1 + I + A; }
-    bool is_and(uint32_t id) const { return id > I; }
-};
-
-struct WinHost {
-    std::vector<uint32_t> inputs;  // node ids, increasing
-    std::vector<uint32_t> cmps;    // compare indices of this window
-    uint64_t est_nodes = 0;        // cone-size estimate used by the cost-aware merge
-};
-
-struct Cmp {
-    uint32_t la, lb;
-    uint64_t ownmask = 0;          // bit j set if window input j belongs to this pair's own support
-    std::vector<uint32_t> S;       // own inputs (global: support; local: leaves)
-};
-
-struct cec_plan {
-    bool local = false;
-    uint32_t num_pairs = 0;
-    std::vector<uint32_t> la, lb;      // the caller's pairs
-    std::vector<int32_t> pre_verdict;  // per user pair: -100 = decided by simulation
-    std::vector<uint64_t> pre_cex;
-    std::vector<uint32_t> k;
-    std::vector<int32_t> pair_cmp;
-    std::vector<Cmp> cmps;
-    // windows after merging
-    std::vector<std::vector<uint32_t>> win_inputs;
-    std::vector<uint32_t> win_nodes;          // AND-node count per window
-    std::vector<std::vector<uint32_t>> win_cmps;
-    std::vector<DevWin> dwin;
-    std::vector<uint4> prog;
-    std::vector<Item> items;
-    std::vector<JItem> jitems;
-    std::vector<LaunchGroup> groups;
-    uint32_t jit_windows = 0, jit_kernels = 0;
-    float jit_ms = 0.f;
-    uint64_t lop3_words = 0;
-    uint64_t W_rank = 0, W_all = 0;
-    uint32_t max_k = 0, max_slots = 0;
-    float host_ms = 0.f;
-    // device
-    bool uploaded = false;
-    DevPlan d;
-    void *ev0 = nullptr, *ev1 = nullptr;
-    bool ran = false;
-};
 
 namespace {
 

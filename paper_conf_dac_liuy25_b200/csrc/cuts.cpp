@@ -1,0 +1,245 @@
+// cuts.cpp — host cut generator for local function checking (§III-C1, :132-154).
+//
+// Priority cuts by cut enumeration, Eq. (1):
+//   E(n) = { u | v : u in P(n0) + {{n0}}, v in P(n1) + {{n1}}, |u | v| <= k_l },
+// P(n) = the C best cuts of E(n) after dropping dominated cuts (supersets of another candidate,
+// priority cuts of ref. [27]), ranked by the Table I order of the pass:
+//   pass 0: large average fanout > small size > small average level
+//   pass 1: small average level > small size > large average fanout
+//   pass 2: large average level > small size > large average fanout
+// Non-representatives rank first by similarity to their representative's priority cuts,
+// s(c, P) = sum_{c' in P} |c & c'| / |c | c'|. Nodes are visited in increasing id,
+// a topological order in which every representative (minimum id of its class) precedes its
+// members — the property the enumeration levels of Eq. (2) provide in the paper's level-wise GPU
+// schedule. Common cuts of a pair (repr r, member m) are {u | v : u in P(r), v in P(m),
+// |u | v| <= k_l} without trivial cuts (reading Q14), smallest first.
+//
+// This is the host-minimal stand-in for the paper's GPU cut generator;
+// the checks themselves run on the GPU through cec_check_local_cuts.
+#include <algorithm>
+#include <cstdint>
+#include <cstring>
+#include <vector>
+
+#include "cec_ctx.hpp"
+
+namespace {
+
+constexpr int KMAX = 24;
+
+struct Cut {
+    uint8_t n = 0;
+    uint32_t leaf[KMAX];
+    uint64_t sig = 0;  // bloom signature for fast subset tests
+    // ranking metrics (integers: exact comparisons)
+    uint64_t sum_fanout = 0, sum_level = 0;
+    double sim = 0;
+};
+
+inline uint64_t bit_of(uint32_t id) { return 1ull << (id & 63); }
+
+// merge sorted leaf lists; false if the union exceeds k
+bool merge(const uint32_t *a, int na, const uint32_t *b, int nb, int k, Cut &out) {
+    int i = 0, j = 0, n = 0;
+    while (i < na || j < nb) {
+        uint32_t v;
+        if (j >= nb || (i < na && a[i] < b[j])) {
+            v = a[i++];
+        } else if (i >= na || b[j] < a[i]) {
+            v = b[j++];
+        } else {
+            v = a[i++];
+            ++j;
+        }
+        if (n == k) return false;
+        out.leaf[n++] = v;
+    }
+    out.n = (uint8_t)n;
+    out.sig = 0;
+    for (int t = 0; t < n; ++t) out.sig |= bit_of(out.leaf[t]);
+    return true;
+}
+
+bool subset(const Cut &small, const Cut &big) {  // small ⊆ big
+    if ((small.sig & ~big.sig) != 0 || small.n > big.n) return false;
+    int j = 0;
+    for (int i = 0; i < small.n; ++i) {
+        while (j < big.n && big.leaf[j] < small.leaf[i]) ++j;
+        if (j == big.n || big.leaf[j] != small.leaf[i]) return false;
+        ++j;
+    }
+    return true;
+}
+
+int inter(const Cut &a, const Cut &b) {
+    int i = 0, j = 0, c = 0;
+    while (i < a.n && j < b.n) {
+        if (a.leaf[i] == b.leaf[j]) {
+            ++c;
+            ++i;
+            ++j;
+        } else if (a.leaf[i] < b.leaf[j]) {
+            ++i;
+        } else {
+            ++j;
+        }
+    }
+    return c;
+}
+
+bool same(const Cut &a, const Cut &b) {
+    return a.n == b.n && a.sig == b.sig && std::memcmp(a.leaf, b.leaf, a.n * sizeof(uint32_t)) == 0;
+}
+
+// a < b in the Table I order of the pass (cross-multiplied averages: exact)
+bool table1_less(const Cut &a, const Cut &b, int pass) {
+    const uint64_t fa = a.sum_fanout * b.n, fb = b.sum_fanout * a.n;  // avg fanout a vs b
+    const uint64_t la = a.sum_level * b.n, lb = b.sum_level * a.n;    // avg level a vs b
+    if (pass == 0) {
+        if (fa != fb) return fa > fb;
+        if (a.n != b.n) return a.n < b.n;
+        if (la != lb) return la < lb;
+    } else if (pass == 1) {
+        if (la != lb) return la < lb;
+        if (a.n != b.n) return a.n < b.n;
+        if (fa != fb) return fa > fb;
+    } else {
+        if (la != lb) return la > lb;
+        if (a.n != b.n) return a.n < b.n;
+        if (fa != fb) return fa > fb;
+    }
+    return std::lexicographical_compare(a.leaf, a.leaf + a.n, b.leaf, b.leaf + b.n);
+}
+
+}  // namespace
+
+extern "C" cec_status cec_common_cuts(cec_ctx *c, uint32_t npairs, const uint32_t *repr, const uint32_t *member,
+                                      uint32_t k_l, uint32_t C, int32_t pass_id, uint32_t max_cuts,
+                                      uint32_t *pair_cut_off, uint32_t *cut_off, uint32_t *leaves) {
+    if (!c || (npairs && (!repr || !member || !pair_cut_off || !cut_off || !leaves)) || k_l == 0 || k_l > KMAX ||
+        C == 0 || max_cuts == 0 || pass_id < 0 || pass_id > 2)
+        return CEC_E_ARG;
+    const uint32_t N = c->N();
+    for (uint32_t q = 0; q < npairs; ++q)
+        if (repr[q] >= N || member[q] >= N || repr[q] >= member[q]) return CEC_E_ARG;
+    // levels and fanouts over the whole AIG (Table I metrics)
+    std::vector<uint32_t> fanout(N, 0);
+    for (uint32_t id = c->I + 1; id < N; ++id) {
+        ++fanout[c->f0[id] >> 1];
+        ++fanout[c->f1[id] >> 1];
+    }
+    // nodes that need cuts: the TFI of every pair node
+    std::vector<uint8_t> need(N, 0);
+    {
+        std::vector<uint32_t> st;
+        for (uint32_t q = 0; q < npairs; ++q)
+            for (uint32_t r : {repr[q], member[q]})
+                if (!need[r]) {
+                    need[r] = 1;
+                    st.push_back(r);
+                }
+        while (!st.empty()) {
+            const uint32_t v = st.back();
+            st.pop_back();
+            if (v <= c->I) continue;
+            for (uint32_t f : {c->f0[v] >> 1, c->f1[v] >> 1})
+                if (!need[f]) {
+                    need[f] = 1;
+                    st.push_back(f);
+                }
+        }
+    }
+    std::vector<uint32_t> repr_of(N, 0xFFFFFFFFu);
+    for (uint32_t q = 0; q < npairs; ++q) repr_of[member[q]] = repr[q];
+    std::vector<std::vector<Cut>> P(N);
+    auto trivial = [&](uint32_t id) {
+        Cut t;
+        t.n = 1;
+        t.leaf[0] = id;
+        t.sig = bit_of(id);
+        return t;
+    };
+    for (uint32_t id = 1; id <= c->I; ++id)
+        if (need[id]) P[id].push_back(trivial(id));
+    if (need[0]) P[0].push_back(trivial(0));
+    std::vector<Cut> E;
+    for (uint32_t id = c->I + 1; id < N; ++id) {
+        if (!need[id]) continue;
+        const uint32_t a = c->f0[id] >> 1, b = c->f1[id] >> 1;
+        std::vector<Cut> ua(P[a]), vb(P[b]);
+        ua.push_back(trivial(a));
+        vb.push_back(trivial(b));
+        E.clear();
+        Cut m;
+        for (const Cut &u : ua)
+            for (const Cut &v : vb)
+                if (merge(u.leaf, u.n, v.leaf, v.n, (int)k_l, m)) {
+                    if (m.n == 1 && m.leaf[0] == id) continue;
+                    E.push_back(m);
+                }
+        // dedupe + drop dominated: process by size, keep a cut unless a kept cut is its subset
+        std::sort(E.begin(), E.end(), [](const Cut &x, const Cut &y) {
+            if (x.n != y.n) return x.n < y.n;
+            return std::lexicographical_compare(x.leaf, x.leaf + x.n, y.leaf, y.leaf + y.n);
+        });
+        std::vector<Cut> kept;
+        for (const Cut &x : E) {
+            bool dom = false;
+            for (const Cut &k : kept)
+                if (same(k, x) || subset(k, x)) {
+                    dom = true;
+                    break;
+                }
+            if (!dom) kept.push_back(x);
+        }
+        for (Cut &x : kept) {
+            x.sum_fanout = x.sum_level = 0;
+            for (int t = 0; t < x.n; ++t) {
+                x.sum_fanout += fanout[x.leaf[t]];
+                x.sum_level += c->level[x.leaf[t]];
+            }
+            x.sim = 0;
+        }
+        const uint32_t r = repr_of[id];
+        if (r != 0xFFFFFFFFu && !P[r].empty()) {
+            for (Cut &x : kept) {
+                double s = 0;
+                for (const Cut &y : P[r]) {
+                    const int in = inter(x, y);
+                    s += (double)in / (double)(x.n + y.n - in);
+                }
+                x.sim = s;
+            }
+            std::sort(kept.begin(), kept.end(), [&](const Cut &x, const Cut &y) {
+                if (x.sim != y.sim) return x.sim > y.sim;
+                return table1_less(x, y, pass_id);
+            });
+        } else {
+            std::sort(kept.begin(), kept.end(), [&](const Cut &x, const Cut &y) { return table1_less(x, y, pass_id); });
+        }
+        if (kept.size() > C) kept.resize(C);
+        P[id].swap(kept);
+    }
+    // common cuts per pair
+    uint32_t ncut = 0, nleaf = 0;
+    cut_off[0] = 0;
+    for (uint32_t q = 0; q < npairs; ++q) {
+        pair_cut_off[q] = ncut;
+        std::vector<Cut> common;
+        Cut m;
+        for (const Cut &u : P[repr[q]])
+            for (const Cut &v : P[member[q]])
+                if (merge(u.leaf, u.n, v.leaf, v.n, (int)k_l, m)) common.push_back(m);
+        std::sort(common.begin(), common.end(), [](const Cut &x, const Cut &y) {
+            if (x.n != y.n) return x.n < y.n;
+            return std::lexicographical_compare(x.leaf, x.leaf + x.n, y.leaf, y.leaf + y.n);
+        });
+        common.erase(std::unique(common.begin(), common.end(), same), common.end());
+        for (size_t i = 0; i < common.size() && i < max_cuts; ++i) {
+            for (int t = 0; t < common[i].n; ++t) leaves[nleaf++] = common[i].leaf[t];
+            cut_off[++ncut] = nleaf;
+        }
+    }
+    pair_cut_off[npairs] = ncut;
+    return CEC_OK;
+}

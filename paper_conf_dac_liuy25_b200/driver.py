@@ -38,6 +38,7 @@ class CecParams:
     max_phases: int = 64
     max_cuts_per_pair: int = 8
     final_po_check: bool = True  # after the L phases: exhaustive check of undecided POs with k <= k_P
+    native_cuts: bool = True     # C++ cut generator (cec_common_cuts); False = the Python reference
     device: int = 0
     engine: int = capi.CEC_ENGINE_AUTO
 
@@ -276,24 +277,34 @@ def check_miter(aig: Aig, lit_a, lit_b, params: Optional[CecParams] = None) -> C
         for pass_id in range(3):
             if not remaining:
                 break
-            repr_of = {m_: r for r, m_, f in remaining}
-            cuts = enumerate_cuts(cur.aig, p.k_l, p.C, pass_id, repr_of)
+            todo = [x for x in remaining if x[1] not in subst]
             ql, qm, off, leaves, who = [], [], [0], [], []
-            for r, m_, f in remaining:
-                if m_ in subst:
-                    continue
-                common = set()
-                for u in cuts[r]:
-                    for v_ in cuts[m_]:
-                        c = u | v_
-                        if c.bit_count() <= p.k_l:
-                            common.add(c)
-                for c in sorted(common, key=lambda x: (x.bit_count(), x))[:p.max_cuts_per_pair]:
-                    ql.append(2 * r)
-                    qm.append(2 * m_ ^ f)
-                    leaves += _bits(c)
-                    off.append(len(leaves))
-                    who.append((r, m_, f))
+            if p.native_cuts and todo:
+                pco, co, lvs = capi.cec_common_cuts(lctx.handle, [x[0] for x in todo], [x[1] for x in todo],
+                                                     p.k_l, p.C, pass_id, p.max_cuts_per_pair)
+                for i, (r, m_, f) in enumerate(todo):
+                    for ct in range(int(pco[i]), int(pco[i + 1])):
+                        ql.append(2 * r)
+                        qm.append(2 * m_ ^ f)
+                        leaves += [int(x) for x in lvs[co[ct]:co[ct + 1]]]
+                        off.append(len(leaves))
+                        who.append((r, m_, f))
+            elif todo:
+                repr_of = {m_: r for r, m_, f in todo}
+                cuts = enumerate_cuts(cur.aig, p.k_l, p.C, pass_id, repr_of)
+                for r, m_, f in todo:
+                    common = set()
+                    for u in cuts[r]:
+                        for v_ in cuts[m_]:
+                            c = u | v_
+                            if c.bit_count() <= p.k_l:
+                                common.add(c)
+                    for c in sorted(common, key=lambda x: (x.bit_count(), x))[:p.max_cuts_per_pair]:
+                        ql.append(2 * r)
+                        qm.append(2 * m_ ^ f)
+                        leaves += _bits(c)
+                        off.append(len(leaves))
+                        who.append((r, m_, f))
             if not ql:
                 continue
             lv = lctx.check_local_cuts(ql, qm, off, leaves)

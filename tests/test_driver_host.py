@@ -61,3 +61,33 @@ def test_miter_reduction_preserves_functions():
         pis = rng.integers(0, 2, size=10).astype(np.uint8)
         for a_old, a_new in zip(m.lit_a, red.lit_a):
             assert o1.eval_lit(int(a_old), pis) == o2.eval_lit(int(a_new), pis)
+
+
+def test_native_common_cuts_are_valid_cuts():
+    """cec_common_cuts (C++, host-only): every returned common cut is a real cut of both roots
+    (the oracle's cut validation accepts it), has <= k_l leaves in increasing id, and no pair gets
+    more than max_cuts cuts."""
+    from paper_conf_dac_liuy25_b200 import capi
+    from workloads import c4_dp
+    m = c4_dp(8)
+    ctx = capi.Context.from_aig(m.aig, device=-1)
+    # candidate pairs: the PO pairs whose B driver has a higher id (repr = A side)
+    pairs = [(int(a) >> 1, int(b) >> 1, (int(a) ^ int(b)) & 1) for a, b in zip(m.lit_a, m.lit_b)
+             if (int(a) >> 1) < (int(b) >> 1) and (int(a) >> 1) > m.aig.num_pis]
+    orc = oracle.Oracle.from_aig(m.aig)
+    for pass_id in range(3):
+        pco, co, lv = capi.cec_common_cuts(ctx.handle, [r for r, _, _ in pairs], [x for _, x, _ in pairs], 10, 8,
+                                           pass_id, 6)
+        la, lb, off, leaves = [], [], [0], []
+        for i, (r, mm, f) in enumerate(pairs):
+            assert pco[i + 1] - pco[i] <= 6
+            for t in range(int(pco[i]), int(pco[i + 1])):
+                L = [int(x) for x in lv[co[t]:co[t + 1]]]
+                assert 1 <= len(L) <= 10 and L == sorted(L)
+                la.append(2 * r)
+                lb.append(2 * mm ^ f)
+                leaves += L
+                off.append(len(leaves))
+        assert la, "some common cuts expected"
+        v = orc.check_local(la, lb, off, leaves)
+        assert all(int(x) != oracle.BADCUT for x in v)
