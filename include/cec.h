@@ -155,6 +155,12 @@ cec_status cec_check_local_cuts(cec_ctx *ctx, uint32_t num_checks, const uint32_
  * representative = minimum id); a signature is a filter, never a proof. */
 cec_status cec_sim_random(cec_ctx *ctx, uint32_t num_words, uint64_t seed, uint64_t *sig_out, uint8_t *phase_out);
 
+/* Same as cec_sim_random with caller-chosen patterns (e.g. counter-examples, "CEX
+ * patterns for splitting the class of a disproved pair"): PI id i+1 takes the num_words u32 words
+ * pi_words[i*num_words .. (i+1)*num_words). */
+cec_status cec_sim_patterns(cec_ctx *ctx, uint32_t num_words, const uint32_t *pi_words, uint64_t *sig_out,
+                            uint8_t *phase_out);
+
 /* Host cut generator for local checks (Eq. 1, Table I, similarity-guided
  * selection). For candidate pairs q (repr[q] < member[q], node ids; member equivalent to repr up to
  * complement), enumerate priority cuts (<= C per node, <= k_l <= 24 leaves, dominated cuts dropped,

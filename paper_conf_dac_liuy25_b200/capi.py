@@ -28,7 +28,7 @@ EXPORTS = ["cec_default_opts", "cec_load_aig", "cec_sim_exhaustive", "cec_check_
            "cec_pair_support", "cec_plan_exhaustive", "cec_plan_run", "cec_plan_results", "cec_plan_info",
            "cec_plan_window", "cec_plan_free", "cec_stream", "cec_get_stats", "cec_shard_range", "cec_pext64",
            "cec_free", "cec_last_error", "cec_abi_version", "cec_nccl_unique_id", "cec_sim_random",
-           "cec_common_cuts"]
+           "cec_common_cuts", "cec_sim_patterns"]
 
 
 class CecOpts(ctypes.Structure):
@@ -89,6 +89,7 @@ def _load() -> ctypes.CDLL:
         "cec_nccl_unique_id": (ctypes.c_int, [P]),
         "cec_sim_random": (ctypes.c_int, [P, u32, u64, P, P]),
         "cec_common_cuts": (ctypes.c_int, [P, u32, P, P, u32, u32, i32, u32, P, P, P]),
+        "cec_sim_patterns": (ctypes.c_int, [P, u32, P, P, P]),
     }
     for name, (res, args) in sig.items():
         fn = getattr(L, name)
@@ -174,6 +175,15 @@ def cec_sim_random(ctx, num_nodes: int, num_words: int = 64, seed: int = 1):
     sig = np.zeros(max(num_nodes, 1), np.uint64)
     ph = np.zeros(max(num_nodes, 1), np.uint8)
     _check(lib.cec_sim_random(ctx, num_words, seed, _p(sig), _p(ph)), ctx)
+    return sig[:num_nodes], ph[:num_nodes]
+
+
+def cec_sim_patterns(ctx, num_nodes: int, pi_words: np.ndarray):
+    """Signatures for caller patterns: pi_words uint32 [num_pis, num_words] (PI id i+1 = row i)."""
+    w = np.ascontiguousarray(pi_words, dtype=np.uint32)
+    sig = np.zeros(max(num_nodes, 1), np.uint64)
+    ph = np.zeros(max(num_nodes, 1), np.uint8)
+    _check(lib.cec_sim_patterns(ctx, w.shape[1], _p(w), _p(sig), _p(ph)), ctx)
     return sig[:num_nodes], ph[:num_nodes]
 
 

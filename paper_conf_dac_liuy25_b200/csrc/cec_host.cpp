@@ -1109,7 +1109,20 @@ cec_status cec_sim_exhaustive(cec_ctx *c, uint32_t n, const uint32_t *la, const 
     return st;
 }
 
+static cec_status sim_signatures(cec_ctx *c, uint32_t W, uint64_t seed, const uint32_t *pi_words, uint64_t *sig_out,
+                                 uint8_t *phase_out);
+
 cec_status cec_sim_random(cec_ctx *c, uint32_t W, uint64_t seed, uint64_t *sig_out, uint8_t *phase_out) {
+    return sim_signatures(c, W, seed, nullptr, sig_out, phase_out);
+}
+
+cec_status cec_sim_patterns(cec_ctx *c, uint32_t W, const uint32_t *pi_words, uint64_t *sig_out, uint8_t *phase_out) {
+    if (!pi_words) return fail(c, CEC_E_ARG, "null pi_words");
+    return sim_signatures(c, W, 0, pi_words, sig_out, phase_out);
+}
+
+static cec_status sim_signatures(cec_ctx *c, uint32_t W, uint64_t seed, const uint32_t *pi_words, uint64_t *sig_out,
+                                 uint8_t *phase_out) {
     if (!c || !sig_out || W == 0) return fail(c, CEC_E_ARG, "null argument or num_words == 0");
     if (c->host_only) return fail(c, CEC_E_CUDA, "host-only context: no CUDA device (no CPU fallback)");
     const uint32_t N = c->N();
@@ -1142,8 +1155,12 @@ cec_status cec_sim_random(cec_ctx *c, uint32_t W, uint64_t seed, uint64_t *sig_o
     CUDA_TRY(c, dev_alloc((void **)&sig, sizeof(unsigned long long) * N));
     CUDA_TRY(c, dev_alloc((void **)&ph, N));
     uint32_t nl = 0;
+    if (pi_words) {  // caller patterns: PI id i+1 takes words pi_words[i*W .. i*W+W)
+        CUDA_TRY(c, dev_memset(tt, 0, sizeof(uint32_t) * W, c->stream));
+        CUDA_TRY(c, h2d(tt + W, pi_words, sizeof(uint32_t) * (size_t)c->I * W, c->stream));
+    }
     const char *e = random_sim(c->d_f0, c->d_f1, c->d_level_ids, c->level_off, c->I, N, W, seed, tt, sig, ph, c->stream,
-                               c->num_sms, &nl);
+                               c->num_sms, &nl, pi_words != nullptr);
     if (e) return fail(c, CEC_E_CUDA, "CUDA: %s (random simulation)", e);
     CUDA_TRY(c, d2h(sig_out, sig, sizeof(unsigned long long) * N, c->stream));
     std::vector<uint8_t> phase(N);

@@ -94,7 +94,7 @@ const char *jit_launch(JitKernel *K, const JItem *items, uint32_t nitems, uint32
 const char *random_sim(const uint32_t *d_f0, const uint32_t *d_f1, const uint32_t *d_level_ids,
                        const std::vector<uint32_t> &level_off, uint32_t I, uint32_t N, uint32_t W, uint64_t seed,
                        uint32_t *d_tt, unsigned long long *d_sig, uint8_t *d_phase, void *stream, int num_sms,
-                       uint32_t *launches);
+                       uint32_t *launches, bool pi_words_given);
 
 // sim_interp.cu
 const char *launch_run(const DevPlan &d, const std::vector<LaunchGroup> &groups, uint32_t nwin, uint32_t ncmp,

@@ -70,16 +70,18 @@ inline const char *ck(cudaError_t e) { return e == cudaSuccess ? nullptr : cudaG
 const char *random_sim(const uint32_t *d_f0, const uint32_t *d_f1, const uint32_t *d_level_ids,
                        const std::vector<uint32_t> &level_off, uint32_t I, uint32_t N, uint32_t W, uint64_t seed,
                        uint32_t *d_tt, unsigned long long *d_sig, uint8_t *d_phase, void *stream, int num_sms,
-                       uint32_t *launches) {
+                       uint32_t *launches, bool pi_words_given) {
     cudaStream_t st = (cudaStream_t)stream;
     const int T = 256;
     const uint64_t grid_cap = (uint64_t)num_sms * 8;
     auto grid_for = [&](uint64_t work) { return (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(grid_cap, (work + T - 1) / T)); };
     uint32_t nl = 0;
-    rs_pis<<<grid_for((uint64_t)I * W + W), T, 0, st>>>(d_tt, I, W, seed);
-    ++nl;
     const char *e;
-    if ((e = ck(cudaGetLastError()))) return e;
+    if (!pi_words_given) {
+        rs_pis<<<grid_for((uint64_t)I * W + W), T, 0, st>>>(d_tt, I, W, seed);
+        ++nl;
+        if ((e = ck(cudaGetLastError()))) return e;
+    }
     for (size_t l = 1; l + 1 < level_off.size(); ++l) {
         const uint32_t n = level_off[l + 1] - level_off[l];
         if (!n) continue;

@@ -39,6 +39,7 @@ class CecParams:
     max_cuts_per_pair: int = 8
     final_po_check: bool = True  # after the L phases: exhaustive check of undecided POs with k <= k_P
     native_cuts: bool = True     # C++ cut generator (cec_common_cuts); False = the Python reference
+    max_cex_patterns: int = 1024  # CEX patterns kept for class refinement
     device: int = 0
     engine: int = capi.CEC_ENGINE_AUTO
 
@@ -176,6 +177,15 @@ def enumerate_cuts(aig: Aig, k_l: int, C: int, pass_id: int, repr_of: Optional[D
 # the flow
 # ---------------------------------------------------------------------------------------------
 
+def pack_patterns(patterns: List[np.ndarray], num_pis: int) -> np.ndarray:
+    """Pack PI assignments (uint8[num_pis] each) into u32 words: pattern j is bit j%32 of word j//32."""
+    W = max(1, (len(patterns) + 31) // 32)
+    words = np.zeros((num_pis, W), dtype=np.uint32)
+    for j, pat in enumerate(patterns):
+        words[:, j // 32] |= (np.asarray(pat[:num_pis], dtype=np.uint32) & 1) << np.uint32(j % 32)
+    return words
+
+
 def _classes(sig: np.ndarray, phase: np.ndarray, num_pis: int) -> List[Tuple[int, int, int]]:
     """(repr, member, phase) candidate pairs from equal signatures: repr = min id."""
     order = np.lexsort((np.arange(sig.size), sig))
@@ -246,6 +256,7 @@ def check_miter(aig: Aig, lit_a, lit_b, params: Optional[CecParams] = None) -> C
 
     # ---- G and L phases -----------------------------------------------------------------------
     tried_global = set()
+    cex_patterns: List[np.ndarray] = []  # CEXs of refuted candidate pairs (class refinement)
     for phase_no in range(p.max_phases):
         st = po_status(cur)
         if (st == capi.CEC_EQUIVALENT).all():
@@ -255,6 +266,12 @@ def check_miter(aig: Aig, lit_a, lit_b, params: Optional[CecParams] = None) -> C
         lctx = _ctx(cur.aig, p, max(p.k_l, 1))  # local checks: up to k_l leaves
         N = cur.aig.num_nodes
         sig, ph = capi.cec_sim_random(ctx.handle, N, p.sim_words, p.seed + phase_no)
+        if cex_patterns:
+            # CEX patterns split the classes of disproved pairs: combine
+            # the random-pattern and CEX-pattern signatures; the relative phase must agree in both
+            sig_c, ph_c = capi.cec_sim_patterns(ctx.handle, N, pack_patterns(cex_patterns, cur.aig.num_pis))
+            sig = np.array([hash((int(a), int(b), int(x) ^ int(y))) & ((1 << 63) - 1)
+                            for a, b, x, y in zip(sig, sig_c, ph, ph_c)], dtype=np.uint64)
         cand = [(r, m_, f) for r, m_, f in _classes(sig, ph, cur.aig.num_pis)]
         versions.append(cur.aig)
         # G phase once per miter version: pairs with support <= k_g
@@ -265,6 +282,9 @@ def check_miter(aig: Aig, lit_a, lit_b, params: Optional[CecParams] = None) -> C
         proved_g = 0
         if gl:
             v, _, k = ctx.sim_exhaustive(la, lb)
+            for i in np.nonzero(v == capi.CEC_NOT_EQUIVALENT)[0][:p.max_cex_patterns]:
+                if len(cex_patterns) < p.max_cex_patterns:
+                    cex_patterns.append(ctx.get_cex(int(i)))
             for (r, m_, f), vv in zip(gl, v):
                 if vv == capi.CEC_EQUIVALENT and m_ not in subst:
                     subst[m_] = 2 * r ^ f

@@ -91,3 +91,11 @@ def test_native_common_cuts_are_valid_cuts():
         assert la, "some common cuts expected"
         v = orc.check_local(la, lb, off, leaves)
         assert all(int(x) != oracle.BADCUT for x in v)
+
+
+def test_pack_patterns():
+    pats = [np.array([1, 0, 1], np.uint8), np.array([0, 1, 1], np.uint8)] + [np.zeros(3, np.uint8)] * 30 + \
+           [np.array([1, 1, 0], np.uint8)]
+    w = driver.pack_patterns(pats, 3)
+    assert w.shape == (3, 2)
+    assert [int(x) for x in w[:, 0]] == [0b01, 0b10, 0b11] and [int(x) for x in w[:, 1]] == [0b1, 0b1, 0]
