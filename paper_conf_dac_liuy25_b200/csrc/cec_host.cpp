@@ -489,6 +489,9 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
             cm.ownmask = m;
         }
     }
+    // AUTO engine: a window is compiled when its sweep is at least this many node-words
+    uint64_t jit_min_node_words = 1ull << 26;
+    if (const char *e = getenv("CEC_JIT_MIN_NODE_WORDS")) jit_min_node_words = strtoull(e, nullptr, 10);
     // (2) parallel over windows: node order, schedule, engine choice, JIT program
     struct WinRes {
         std::vector<uint32_t> nodes;
@@ -561,7 +564,7 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         const uint64_t node_words = (uint64_t)nodes.size() * tt_words_of(k);
         if (k >= 10 && !nodes.empty()) {
             if (c->opts.engine == CEC_ENGINE_JIT) R.jit = true;
-            else if (c->opts.engine == CEC_ENGINE_AUTO) R.jit = node_words >= (1ull << 26) || R.sc.nslots > max_slot_cap;
+            else if (c->opts.engine == CEC_ENGINE_AUTO) R.jit = node_words >= jit_min_node_words || R.sc.nslots > max_slot_cap;
         }
         if (!R.jit && R.sc.nslots > max_slot_cap) {
             char b[160];

@@ -297,3 +297,28 @@ def test_driver_c4_full():
     q = rb.cex_pair
     assert orc.eval_lit(int(bug.lit_a[q]), rb.cex) != orc.eval_lit(int(bug.lit_b[q]), rb.cex)
     _replay_checks(rb, limit=300)
+
+
+def test_sim_patterns_and_random_classes_vs_oracle():
+    """cec_sim_patterns / cec_sim_random (partial simulation for ECs): nodes get
+    equal signatures iff their complement-canonical value vectors on the patterns are equal (checked
+    node by node with the oracle's evaluator), and the phase bit is the node's value on pattern 0."""
+    from paper_conf_dac_liuy25_b200 import driver
+    m = circuits.c2_mul12_bug(seed=1, n=5)
+    aig = m.aig
+    ctx = gpu_ctx(aig)
+    N, I = aig.num_nodes, aig.num_pis
+    rng = np.random.default_rng(3)
+    pats = [rng.integers(0, 2, size=I).astype(np.uint8) for _ in range(40)]
+    sig, ph = capi.cec_sim_patterns(ctx.handle, N, driver.pack_patterns(pats, I))
+    orc = Oracle.from_aig(aig)
+    W = (len(pats) + 31) // 32 * 32  # padded patterns are all-zero assignments
+    allp = pats + [np.zeros(I, np.uint8)] * (W - len(pats))
+    vec = {}
+    for nid in range(N):
+        v = tuple(orc.eval_lit(2 * nid, p) for p in allp)
+        assert int(ph[nid]) == v[0]
+        vec[nid] = tuple(x ^ v[0] for x in v)
+    for a in range(N):
+        for b in range(a + 1, N, 7):
+            assert (int(sig[a]) == int(sig[b])) == (vec[a] == vec[b])
