@@ -628,13 +628,13 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         dw.cmp_off = wc.empty() ? (uint32_t)cmps2.size() : wc[0];
         dw.ncmp = (uint32_t)wc.size();
         dw.prog_off = (uint32_t)P->prog.size();
-        dw.prog_len = (uint32_t)sc.ops.size();
+        dw.prog_len = R.jit ? 0u : (uint32_t)sc.ops.size();  // JIT windows need no interpreter ops
         dw.k = (uint32_t)W.inputs.size();
         dw.const_slot = sc.const_slot;
         const uint64_t ttw = tt_words_of(dw.k);
         dw.tt_words_lo = (uint32_t)ttw;
         dw.tt_words_hi = (uint32_t)(ttw >> 32);
-        P->prog.insert(P->prog.end(), sc.ops.begin(), sc.ops.end());
+        if (!R.jit) P->prog.insert(P->prog.end(), sc.ops.begin(), sc.ops.end());
         P->dwin.push_back(dw);
         P->win_inputs.push_back(W.inputs);
         P->win_nodes.push_back((uint32_t)nodes.size());
@@ -665,7 +665,7 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         uint64_t pats_rank = we > wb ? (dw.k < 5 ? (1ull << dw.k) : (we - wb) * 32) : 0;
         P->W_rank += (uint64_t)nodes.size() * pats_rank;
         words_rank_of.push_back(we > wb ? (we - wb) : 0);
-        cost_of.push_back((uint64_t)(dw.prog_len + 1) * (se - sb));
+        cost_of.push_back((uint64_t)(sc.ops.size() + 1) * (se - sb));
     }
     tm.lap("windows+schedules+jit-progs");
     P->cmps.swap(cmps2);
