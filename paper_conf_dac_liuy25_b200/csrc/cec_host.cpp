@@ -373,7 +373,7 @@ cec_status cec_load_aig(cec_ctx **out, const cec_aig *aig, const cec_opts *opts)
             return CEC_E_CUDA;
         }
         c->stream = c->opts.stream ? c->opts.stream : c->own_stream;
-        if (c->opts.world > 1 && c->opts.nccl_unique_id) {  // NULL id: shard-only mode, no collective
+        if (c->opts.nccl_unique_id) {  // NULL id with world > 1: shard-only mode, no collective
             if (!g_nccl.load()) return fail(nullptr, CEC_E_NCCL, "NCCL library not found");
             ncclUniqueId uid;
             std::memcpy(&uid, c->opts.nccl_unique_id, sizeof uid);

@@ -40,6 +40,7 @@ class CecParams:
     final_po_check: bool = True  # after the L phases: exhaustive check of undecided POs with k <= k_P
     native_cuts: bool = True     # C++ cut generator (cec_common_cuts); False = the Python reference
     max_cex_patterns: int = 1024  # CEX patterns kept for class refinement
+    distance1: bool = True        # also simulate every distance-1 neighbour of each CEX
     device: int = 0
     engine: int = capi.CEC_ENGINE_AUTO
 
@@ -177,6 +178,14 @@ def enumerate_cuts(aig: Aig, k_l: int, C: int, pass_id: int, repr_of: Optional[D
 # the flow
 # ---------------------------------------------------------------------------------------------
 
+def hctx_support(aig: Aig, la: int, lb: int) -> List[int]:
+    h = capi.Context.from_aig(aig, device=-1, k_max=63)
+    try:
+        return capi.cec_pair_support(h.handle, int(la), int(lb))
+    finally:
+        h.close()
+
+
 def pack_patterns(patterns: List[np.ndarray], num_pis: int) -> np.ndarray:
     """Pack PI assignments (uint8[num_pis] each) into u32 words: pattern j is bit j%32 of word j//32."""
     W = max(1, (len(patterns) + 31) // 32)
@@ -283,8 +292,17 @@ def check_miter(aig: Aig, lit_a, lit_b, params: Optional[CecParams] = None) -> C
         if gl:
             v, _, k = ctx.sim_exhaustive(la, lb)
             for i in np.nonzero(v == capi.CEC_NOT_EQUIVALENT)[0][:p.max_cex_patterns]:
-                if len(cex_patterns) < p.max_cex_patterns:
-                    cex_patterns.append(ctx.get_cex(int(i)))
+                if len(cex_patterns) >= p.max_cex_patterns:
+                    break
+                cx = ctx.get_cex(int(i))
+                cex_patterns.append(cx)
+                if p.distance1:  # distance-1 simulation of the CEX over the pair's support
+                    for pi in hctx_support(cur.aig, la[i], lb[i]):
+                        if len(cex_patterns) >= p.max_cex_patterns:
+                            break
+                        nb = cx.copy()
+                        nb[pi - 1] ^= 1
+                        cex_patterns.append(nb)
             for (r, m_, f), vv in zip(gl, v):
                 if vv == capi.CEC_EQUIVALENT and m_ not in subst:
                     subst[m_] = 2 * r ^ f

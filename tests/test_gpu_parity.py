@@ -322,3 +322,14 @@ def test_sim_patterns_and_random_classes_vs_oracle():
     for a in range(N):
         for b in range(a + 1, N, 7):
             assert (int(sig[a]) == int(sig[b])) == (vec[a] == vec[b])
+
+
+def test_nccl_min_allreduce_single_rank():
+    """The NCCL path of a10 on one GPU: a 1-rank communicator from cec_nccl_unique_id, the min
+    all-reduce runs inside cec_plan_run and the results equal the no-NCCL run."""
+    m = c2_mul12_bug(seed=1, n=10)
+    uid = capi.cec_nccl_unique_id()
+    got = gpu_ctx(m.aig, rank=0, world=1, nccl_unique_id=uid).sim_exhaustive(m.lit_a, m.lit_b)
+    ref = gpu_ctx(m.aig).sim_exhaustive(m.lit_a, m.lit_b)
+    for a, b in zip(got, ref):
+        assert np.array_equal(a, b)
