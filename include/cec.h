@@ -84,7 +84,7 @@ typedef struct {
     int32_t rank, world;       /* world > 1: SPMD over `world` GPUs; every rank passes the same
                                   AIG, pairs and options; rank r simulates its contiguous share of
                                   every window's pattern slices */
-    const void *nccl_unique_id;/* 128-byte ncclUniqueId for world > 1 (the caller bootstraps it,
+    const void *nccl_unique_id;/* 128-byte ncclUniqueId for world >= 1 (the caller bootstraps it,
                                   e.g. through torch.distributed): one ncclAllReduce(min) of the
                                   per-pair first-mismatch indices makes the results identical on
                                   every rank. NULL with world > 1 = shard-only mode: no collective;
@@ -130,7 +130,8 @@ cec_status cec_load_aig(cec_ctx **ctx, const cec_aig *aig, const cec_opts *opts)
 /* Global exhaustive check of num_pairs literal pairs (Alg. 1 :89-108).
  * For a pair with k = |supp(a) U supp(b)| <= k_max the verdict is exact: EQUIVALENT, or
  * NOT_EQUIVALENT with cex_index_out = the minimum mismatching pattern in the pair's own support
- * order. k > k_max gives UNDECIDED and CEC_NO_CEX (the caller may fall back to local cuts).
+ * order. k > k_max (or k > 41: more than 2^41 patterns) gives UNDECIDED and CEC_NO_CEX (the caller
+ * may fall back to local cuts).
  * lit_a == lit_b -> EQUIVALENT; lit_a == lit_b ^ 1 -> NOT_EQUIVALENT at index 0.
  * verdict_out / cex_index_out / k_out are caller-owned host arrays of num_pairs (cex_index_out and
  * k_out may be NULL). Blocking: returns after the kernels, the cross-GPU reduction and the copy
@@ -139,8 +140,8 @@ cec_status cec_sim_exhaustive(cec_ctx *ctx, uint32_t num_pairs, const uint32_t *
                               int32_t *verdict_out, uint64_t *cex_index_out, uint32_t *k_out);
 
 /* Local function checks (§III-C1). Check q compares lit_a[q] and lit_b[q] as
- * functions of the leaves cut_leaves[cut_off[q] .. cut_off[q+1]) (node ids, any order, taken in
- * increasing id; at most k_max and at most 24 leaves). verdict_out[q] = EQUIVALENT if the two local
+ * functions of the leaves cut_leaves[cut_off[q] .. cut_off[q+1]) (node ids > 0, any order, taken in
+ * increasing id; at most k_max and at most 24 leaves; CEC_E_ARG otherwise). verdict_out[q] = EQUIVALENT if the two local
  * functions are identical; UNDECIDED if they differ (the difference may be an SDC, so
  * no CEX is produced); CEC_BAD_CUT if the backward traversal from a root reaches a PI that is not a
  * leaf, in which case the call returns CEC_E_CUT after filling every other verdict. */

@@ -421,6 +421,9 @@ cec_status cec_pair_support(cec_ctx *ctx, uint32_t la, uint32_t lb, uint32_t *su
 namespace {
 
 constexpr int32_t DECIDED_BY_SIM = -100;
+// Slice indices are 32-bit (2^(k-10) JIT slices): windows above 2^41 patterns are never enumerated
+// (they would take days even at the LOP3 peak); such pairs are UNDECIDED like k > k_max.
+constexpr size_t MAX_K_ENUM = 41;
 JitConfig jit_config() {  // overridable for tuning: CEC_JIT_THREADS / CEC_JIT_MINB / CEC_JIT_SYNC
     JitConfig cfg;
     if (const char *e = getenv("CEC_JIT_THREADS")) cfg.threads = atoi(e);
@@ -909,7 +912,7 @@ cec_status cec_plan_exhaustive(cec_ctx *c, uint32_t n, const uint32_t *la, const
             P->pre_cex[p] = 0;
             continue;
         }
-        if (S.size() > kmax) {
+        if (S.size() > kmax || S.size() > MAX_K_ENUM) {
             P->pre_verdict[p] = CEC_UNDECIDED;
             continue;
         }
@@ -1208,7 +1211,7 @@ cec_status cec_check_local_cuts(cec_ctx *c, uint32_t n, const uint32_t *la, cons
             return fail(c, CEC_E_ARG, "check %u: bad literal or cut offsets", q);
         std::vector<uint32_t> L(leaves + cut_off[q], leaves + cut_off[q + 1]);
         for (uint32_t x : L)
-            if (x >= c->N()) return fail(c, CEC_E_ARG, "check %u: leaf out of range", q);
+            if (x == 0 || x >= c->N()) return fail(c, CEC_E_ARG, "check %u: leaf out of range (or constant)", q);
         std::sort(L.begin(), L.end());  // increasing id (reading Q15)
         L.erase(std::unique(L.begin(), L.end()), L.end());
         if (L.size() > kcap) return fail(c, CEC_E_ARG, "check %u: %zu leaves > %u", q, L.size(), kcap);

@@ -152,8 +152,9 @@ extern "C" cec_status cec_common_cuts(cec_ctx *c, uint32_t npairs, const uint32_
     std::vector<uint32_t> repr_of(N, 0xFFFFFFFFu);
     for (uint32_t q = 0; q < npairs; ++q) repr_of[member[q]] = repr[q];
     std::vector<std::vector<Cut>> P(N);
-    auto trivial = [&](uint32_t id) {
+    auto trivial = [&](uint32_t id) {  // the constant needs no leaf: its cut is empty
         Cut t;
+        if (id == 0) return t;
         t.n = 1;
         t.leaf[0] = id;
         t.sig = bit_of(id);
@@ -174,7 +175,7 @@ extern "C" cec_status cec_common_cuts(cec_ctx *c, uint32_t npairs, const uint32_
         for (const Cut &u : ua)
             for (const Cut &v : vb)
                 if (merge(u.leaf, u.n, v.leaf, v.n, (int)k_l, m)) {
-                    if (m.n == 1 && m.leaf[0] == id) continue;
+                    if (m.n == 0 || (m.n == 1 && m.leaf[0] == id)) continue;
                     E.push_back(m);
                 }
         // dedupe + drop dominated: process by size, keep a cut unless a kept cut is its subset
@@ -229,7 +230,7 @@ extern "C" cec_status cec_common_cuts(cec_ctx *c, uint32_t npairs, const uint32_
         Cut m;
         for (const Cut &u : P[repr[q]])
             for (const Cut &v : P[member[q]])
-                if (merge(u.leaf, u.n, v.leaf, v.n, (int)k_l, m)) common.push_back(m);
+                if (merge(u.leaf, u.n, v.leaf, v.n, (int)k_l, m) && m.n > 0) common.push_back(m);
         std::sort(common.begin(), common.end(), [](const Cut &x, const Cut &y) {
             if (x.n != y.n) return x.n < y.n;
             return std::lexicographical_compare(x.leaf, x.leaf + x.n, y.leaf, y.leaf + y.n);
