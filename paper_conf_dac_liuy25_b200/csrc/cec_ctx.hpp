@@ -58,6 +58,7 @@ struct cec_ctx {
     cec_opts opts{};
     bool host_only = true;
     void *stream = nullptr, *own_stream = nullptr;
+    AuxStreams aux;  // side streams for concurrent launch groups
     int num_sms = 0;
     ncclComm_t comm = nullptr;
     std::string err;

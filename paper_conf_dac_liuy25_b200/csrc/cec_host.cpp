@@ -373,6 +373,10 @@ cec_status cec_load_aig(cec_ctx **out, const cec_aig *aig, const cec_opts *opts)
             return CEC_E_CUDA;
         }
         c->stream = c->opts.stream ? c->opts.stream : c->own_stream;
+        if (getenv("CEC_NO_SIDE_STREAMS") == nullptr) {
+            const char *ea = aux_create(c->aux);
+            if (ea) return fail(nullptr, CEC_E_CUDA, "CUDA: %s (side streams)", ea);
+        }
         if (c->opts.nccl_unique_id) {  // NULL id with world > 1: shard-only mode, no collective
             if (!g_nccl.load()) return fail(nullptr, CEC_E_NCCL, "NCCL library not found");
             ncclUniqueId uid;
@@ -391,6 +395,7 @@ void cec_free(cec_ctx *ctx) {
     dev_free(ctx->d_f1);
     dev_free(ctx->d_level_ids);
     if (ctx->comm && g_nccl.destroy) g_nccl.destroy(ctx->comm);
+    aux_destroy(ctx->aux);
     if (ctx->own_stream) stream_destroy(ctx->own_stream);
     delete ctx;
 }
@@ -493,7 +498,7 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         }
     }
     // AUTO engine: a window is compiled when its sweep is at least this many node-words
-    uint64_t jit_min_node_words = 1ull << 26;
+    uint64_t jit_min_node_words = 1ull << 23;
     if (const char *e = getenv("CEC_JIT_MIN_NODE_WORDS")) jit_min_node_words = strtoull(e, nullptr, 10);
     // (2) parallel over windows: node order, schedule, engine choice, JIT program
     struct WinRes {
@@ -999,7 +1004,7 @@ cec_status cec_plan_run(cec_ctx *c, cec_plan *P) {
     CUDA_TRY(c, event_record(P->ev0, c->stream));
     uint32_t nl = 0;
     const char *e = launch_run(P->d, P->groups, (uint32_t)P->dwin.size(), (uint32_t)P->cmps.size(), c->stream,
-                                  c->num_sms, &nl);
+                                  c->num_sms, &nl, &c->aux);
     if (e) return fail(c, CEC_E_CUDA, "CUDA: %s (kernel launch)", e);
     if (c->comm && !P->cmps.empty()) {  // a10: one NCCL min all-reduce of first_idx
         ncclResult_t r = g_nccl.all_reduce(P->d.first, P->d.first, P->cmps.size(), ncclUint64, ncclMin, c->comm,

@@ -97,8 +97,19 @@ const char *random_sim(const uint32_t *d_f0, const uint32_t *d_f1, const uint32_
                        uint32_t *launches, bool pi_words_given);
 
 // sim_interp.cu
+// Side streams: independent launch groups (different window structures) run concurrently, so the
+// tail of one persistent grid overlaps the next and small groups do not serialise.
+constexpr int NAUX = 4;
+struct AuxStreams {
+    void *s[NAUX] = {};
+    void *fork = nullptr;
+    void *join[NAUX] = {};
+    bool ok = false;
+};
+const char *aux_create(AuxStreams &a);
+void aux_destroy(AuxStreams &a);
 const char *launch_run(const DevPlan &d, const std::vector<LaunchGroup> &groups, uint32_t nwin, uint32_t ncmp,
-                       void *stream, int num_sms, uint32_t *launches);
+                       void *stream, int num_sms, uint32_t *launches, AuxStreams *aux);
 const char *dev_alloc(void **p, size_t bytes);
 const char *dev_free(void *p);
 const char *h2d(void *dst, const void *src, size_t bytes, void *stream);

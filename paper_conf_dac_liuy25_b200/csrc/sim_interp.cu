@@ -149,18 +149,55 @@ uint32_t interp_max_slots_per_warp() {
     return (uint32_t)((SMEM_PER_SM - 32 * sizeof(uint4)) / SLOT_BYTES);
 }
 
+const char *aux_create(AuxStreams &a) {
+    if (a.ok) return nullptr;
+    const char *e;
+    for (int i = 0; i < NAUX; ++i) {
+        cudaStream_t s;
+        if ((e = ck(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking)))) return e;
+        a.s[i] = s;
+        cudaEvent_t ev;
+        if ((e = ck(cudaEventCreateWithFlags(&ev, cudaEventDisableTiming)))) return e;
+        a.join[i] = ev;
+    }
+    cudaEvent_t f;
+    if ((e = ck(cudaEventCreateWithFlags(&f, cudaEventDisableTiming)))) return e;
+    a.fork = f;
+    a.ok = true;
+    return nullptr;
+}
+
+void aux_destroy(AuxStreams &a) {
+    for (int i = 0; i < NAUX; ++i) {
+        if (a.s[i]) cudaStreamDestroy((cudaStream_t)a.s[i]);
+        if (a.join[i]) cudaEventDestroy((cudaEvent_t)a.join[i]);
+    }
+    if (a.fork) cudaEventDestroy((cudaEvent_t)a.fork);
+    a = AuxStreams{};
+}
+
 const char *launch_run(const DevPlan &d, const std::vector<LaunchGroup> &groups, uint32_t nwin, uint32_t ncmp,
-                       void *stream, int num_sms, uint32_t *launches) {
-    cudaStream_t st = (cudaStream_t)stream;
+                       void *stream, int num_sms, uint32_t *launches, AuxStreams *aux) {
+    cudaStream_t main_st = (cudaStream_t)stream;
+    cudaStream_t st = main_st;
     const char *e;
     if ((e = ck(cudaMemsetAsync(d.first, 0xFF, sizeof(unsigned long long) * (ncmp ? ncmp : 1), st)))) return e;
     if ((e = ck(cudaMemsetAsync(d.bound, 0xFF, sizeof(unsigned long long) * (nwin ? nwin : 1), st)))) return e;
     if ((e = ck(cudaMemsetAsync(d.neq_cnt, 0, sizeof(uint32_t) * (nwin ? nwin : 1), st)))) return e;
     if ((e = ck(cudaMemsetAsync(d.item_ctr, 0, sizeof(uint32_t) * (groups.size() ? groups.size() : 1), st)))) return e;
+    const bool multi = aux && aux->ok && groups.size() > 1;
+    if (multi) {
+        if ((e = ck(cudaEventRecord((cudaEvent_t)aux->fork, main_st)))) return e;
+        for (int i = 0; i < NAUX; ++i)
+            if ((e = ck(cudaStreamWaitEvent((cudaStream_t)aux->s[i], (cudaEvent_t)aux->fork, 0)))) return e;
+    }
     uint32_t nl = 0;
     for (size_t g = 0; g < groups.size(); ++g) {
         const LaunchGroup &G = groups[g];
         if (G.nitems == 0) continue;
+        // the biggest group stays on the caller's stream; the others round-robin on side streams
+        st = (multi && g > 0) ? (cudaStream_t)aux->s[(g - 1) % NAUX] : main_st;
+        stream = st;
         if (G.jit) {
             if ((e = jit_launch(G.jit, d.jitems + G.item_off, G.nitems, d.item_ctr + g, d.first, d.bound, d.neq_cnt,
                                 stream, num_sms)))
@@ -194,6 +231,12 @@ const char *launch_run(const DevPlan &d, const std::vector<LaunchGroup> &groups,
                                                               d.prog, d.first, d.bound, d.neq_cnt, G.nslots);
         if ((e = ck(cudaGetLastError()))) return e;
         ++nl;
+    }
+    if (multi) {  // join: the caller's stream waits for every side stream
+        for (int i = 0; i < NAUX; ++i) {
+            if ((e = ck(cudaEventRecord((cudaEvent_t)aux->join[i], (cudaStream_t)aux->s[i])))) return e;
+            if ((e = ck(cudaStreamWaitEvent(main_st, (cudaEvent_t)aux->join[i], 0)))) return e;
+        }
     }
     if (launches) *launches = nl;
     return nullptr;
