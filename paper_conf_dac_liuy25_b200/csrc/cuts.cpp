@@ -33,8 +33,22 @@ struct Cut {
     uint64_t sig = 0;  // bloom signature for fast subset tests
     // ranking metrics (integers: exact comparisons)
     uint64_t sum_fanout = 0, sum_level = 0;
-    double sim = 0;
+    unsigned __int128 sim = 0;  // similarity x lcm(1..2*KMAX): exact, so ties are unambiguous
 };
+
+unsigned __int128 lcm_upto(int n) {
+    unsigned __int128 l = 1;
+    for (int i = 2; i <= n; ++i) {
+        unsigned __int128 a = l, b = (unsigned __int128)i;
+        while (b) {
+            unsigned __int128 t = a % b;
+            a = b;
+            b = t;
+        }
+        l = l / a * (unsigned __int128)i;
+    }
+    return l;
+}
 
 inline uint64_t bit_of(uint32_t id) { return 1ull << (id & 63); }
 
@@ -203,11 +217,12 @@ extern "C" cec_status cec_common_cuts(cec_ctx *c, uint32_t npairs, const uint32_
         }
         const uint32_t r = repr_of[id];
         if (r != 0xFFFFFFFFu && !P[r].empty()) {
+            static const unsigned __int128 L = lcm_upto(2 * KMAX);
             for (Cut &x : kept) {
-                double s = 0;
+                unsigned __int128 s = 0;
                 for (const Cut &y : P[r]) {
                     const int in = inter(x, y);
-                    s += (double)in / (double)(x.n + y.n - in);
+                    s += (unsigned __int128)in * (L / (unsigned __int128)(x.n + y.n - in));
                 }
                 x.sim = s;
             }

@@ -99,3 +99,45 @@ def test_pack_patterns():
     w = driver.pack_patterns(pats, 3)
     assert w.shape == (3, 2)
     assert [int(x) for x in w[:, 0]] == [0b01, 0b10, 0b11] and [int(x) for x in w[:, 1]] == [0b1, 0b1, 0]
+
+
+import pytest  # noqa: E402
+
+
+@pytest.mark.parametrize("case", range(10))
+def test_native_common_cuts_match_cut_oracle(case):
+    """cec_common_cuts (C++) == oracle/cuts.py (plain Python, exact arithmetic) cut for cut."""
+    from oracle import cuts as cut_oracle
+    from paper_conf_dac_liuy25_b200 import capi
+    from workloads import c4_dp
+    rng = np.random.default_rng(case)
+    if case < 4:
+        m = c4_dp(6 + 2 * case)
+    else:
+        m = circuits.random_miter(12, 150 + 40 * case, 10, seed=900 + case, window=24)
+    aig = m.aig
+    # candidate pairs: (lower id, higher id) of the PO pairs and of random node pairs
+    pairs = set()
+    for a, b in zip(m.lit_a, m.lit_b):
+        x, y = sorted((int(a) >> 1, int(b) >> 1))
+        if x < y:
+            pairs.add((x, y))
+    N = aig.num_nodes
+    for _ in range(20):
+        x, y = sorted(int(v) for v in rng.integers(1, N, size=2))
+        if x < y:
+            pairs.add((x, y))
+    pairs = sorted(pairs)
+    # a member may have one representative only
+    seen, P = set(), []
+    for x, y in pairs:
+        if y not in seen:
+            seen.add(y)
+            P.append((x, y))
+    k_l, C, pass_id, mc = int(rng.integers(4, 13)), int(rng.integers(2, 9)), case % 3, int(rng.integers(1, 7))
+    ctx = capi.Context.from_aig(aig, device=-1)
+    pco, co, lv = capi.cec_common_cuts(ctx.handle, [x for x, _ in P], [y for _, y in P], k_l, C, pass_id, mc)
+    want = cut_oracle.common_cuts(aig.num_pis, aig.fanins, [x for x, _ in P], [y for _, y in P], k_l, C, pass_id, mc)
+    for i in range(len(P)):
+        got = [tuple(int(v) for v in lv[co[t]:co[t + 1]]) for t in range(int(pco[i]), int(pco[i + 1]))]
+        assert got == want[i], (i, P[i], got, want[i])
