@@ -120,3 +120,6 @@ struct cec_plan {
     bool ran = false;
 };
 
+
+// device copy of the AIG (fanin literals + level CSR), uploaded on first use (cec_host.cpp)
+extern "C" cec_status cec_ensure_device_aig(cec_ctx *c);  // internal (not in include/cec.h)

@@ -1123,19 +1123,8 @@ cec_status cec_sim_exhaustive(cec_ctx *c, uint32_t n, const uint32_t *la, const 
 static cec_status sim_signatures(cec_ctx *c, uint32_t W, uint64_t seed, const uint32_t *pi_words, uint64_t *sig_out,
                                  uint8_t *phase_out);
 
-cec_status cec_sim_random(cec_ctx *c, uint32_t W, uint64_t seed, uint64_t *sig_out, uint8_t *phase_out) {
-    return sim_signatures(c, W, seed, nullptr, sig_out, phase_out);
-}
-
-cec_status cec_sim_patterns(cec_ctx *c, uint32_t W, const uint32_t *pi_words, uint64_t *sig_out, uint8_t *phase_out) {
-    if (!pi_words) return fail(c, CEC_E_ARG, "null pi_words");
-    return sim_signatures(c, W, 0, pi_words, sig_out, phase_out);
-}
-
-static cec_status sim_signatures(cec_ctx *c, uint32_t W, uint64_t seed, const uint32_t *pi_words, uint64_t *sig_out,
-                                 uint8_t *phase_out) {
-    if (!c || !sig_out || W == 0) return fail(c, CEC_E_ARG, "null argument or num_words == 0");
-    if (c->host_only) return fail(c, CEC_E_CUDA, "host-only context: no CUDA device (no CPU fallback)");
+cec_status cec_ensure_device_aig(cec_ctx *c) {
+    if (c->host_only) return fail(c, CEC_E_CUDA, "host-only context");
     const uint32_t N = c->N();
     if (!c->d_f0) {  // AIG and level CSR on the device (a1)
         uint32_t maxl = 0;
@@ -1152,6 +1141,27 @@ static cec_status sim_signatures(cec_ctx *c, uint32_t W, uint64_t seed, const ui
         CUDA_TRY(c, h2d(c->d_f1, c->f1.data(), sizeof(uint32_t) * N, c->stream));
         CUDA_TRY(c, h2d(c->d_level_ids, ids.data(), sizeof(uint32_t) * ids.size(), c->stream));
         CUDA_TRY(c, stream_sync(c->stream));
+    }
+    return CEC_OK;
+}
+
+cec_status cec_sim_random(cec_ctx *c, uint32_t W, uint64_t seed, uint64_t *sig_out, uint8_t *phase_out) {
+    return sim_signatures(c, W, seed, nullptr, sig_out, phase_out);
+}
+
+cec_status cec_sim_patterns(cec_ctx *c, uint32_t W, const uint32_t *pi_words, uint64_t *sig_out, uint8_t *phase_out) {
+    if (!pi_words) return fail(c, CEC_E_ARG, "null pi_words");
+    return sim_signatures(c, W, 0, pi_words, sig_out, phase_out);
+}
+
+static cec_status sim_signatures(cec_ctx *c, uint32_t W, uint64_t seed, const uint32_t *pi_words, uint64_t *sig_out,
+                                 uint8_t *phase_out) {
+    if (!c || !sig_out || W == 0) return fail(c, CEC_E_ARG, "null argument or num_words == 0");
+    if (c->host_only) return fail(c, CEC_E_CUDA, "host-only context: no CUDA device (no CPU fallback)");
+    const uint32_t N = c->N();
+    {
+        cec_status st = cec_ensure_device_aig(c);
+        if (st != CEC_OK) return st;
     }
     uint32_t *tt = nullptr;
     unsigned long long *sig = nullptr;

@@ -90,6 +90,16 @@ uint32_t jit_lop3_count(const JitProgram &p, bool fuse);
 const char *jit_launch(JitKernel *K, const JItem *items, uint32_t nitems, uint32_t *ctr, unsigned long long *first,
                        unsigned long long *bound, uint32_t *neq_cnt, void *stream, int num_sms);
 
+// cuts_gpu.cu
+uint32_t gpu_cuts_max_C();
+const char *gpu_common_cuts(const uint32_t *d_f0, const uint32_t *d_f1, uint32_t N,
+                            const std::vector<uint32_t> &fanout, const std::vector<uint32_t> &level,
+                            const std::vector<uint32_t> &repr_of, const std::vector<uint32_t> &pis_needed,
+                            const std::vector<std::vector<uint32_t>> &el_lists, const std::vector<uint32_t> &repr,
+                            const std::vector<uint32_t> &member, uint32_t k_l, uint32_t C, int pass, uint32_t max_cuts,
+                            void *stream, int num_sms, std::vector<uint32_t> &cut_counts,
+                            std::vector<uint32_t> &cut_leaves_flat);
+
 // sim_random.cu
 const char *random_sim(const uint32_t *d_f0, const uint32_t *d_f1, const uint32_t *d_level_ids,
                        const std::vector<uint32_t> &level_off, uint32_t I, uint32_t N, uint32_t W, uint64_t seed,

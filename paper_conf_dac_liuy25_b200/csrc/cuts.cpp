@@ -18,6 +18,7 @@
 // the checks themselves run on the GPU through cec_check_local_cuts.
 #include <algorithm>
 #include <cstdint>
+#include <cstdlib>
 #include <cstring>
 #include <vector>
 
@@ -165,6 +166,41 @@ extern "C" cec_status cec_common_cuts(cec_ctx *c, uint32_t npairs, const uint32_
     }
     std::vector<uint32_t> repr_of(N, 0xFFFFFFFFu);
     for (uint32_t q = 0; q < npairs; ++q) repr_of[member[q]] = repr[q];
+    if (!c->host_only && C <= gpu_cuts_max_C() && getenv("CEC_CUTS_HOST") == nullptr) {
+        // GPU cut generator: nodes grouped by enumeration level (Eq. 2)
+        cec_status st = cec_ensure_device_aig(c);
+        if (st != CEC_OK) return st;
+        std::vector<uint32_t> el(N, 0), pis;
+        std::vector<std::vector<uint32_t>> lists;
+        for (uint32_t id = 1; id <= c->I; ++id)
+            if (need[id]) pis.push_back(id);
+        for (uint32_t id = c->I + 1; id < N; ++id) {
+            if (!need[id]) continue;
+            uint32_t e = 1 + std::max(el[c->f0[id] >> 1], el[c->f1[id] >> 1]);
+            if (repr_of[id] != 0xFFFFFFFFu) e = std::max(e, 1 + el[repr_of[id]]);
+            el[id] = e;
+            if (lists.size() <= e) lists.resize(e + 1);
+            lists[e].push_back(id);
+        }
+        std::vector<uint32_t> lvl(c->level.begin(), c->level.end());
+        std::vector<uint32_t> R(repr, repr + npairs), M(member, member + npairs), counts, flat;
+        const char *e = gpu_common_cuts(c->d_f0, c->d_f1, N, fanout, lvl, repr_of, pis, lists, R, M, k_l, C, pass_id,
+                                        max_cuts, c->stream, c->num_sms, counts, flat);
+        if (e) return CEC_E_CUDA;
+        uint32_t ncut = 0, nleaf = 0;
+        size_t pos = 0;
+        cut_off[0] = 0;
+        for (uint32_t q = 0; q < npairs; ++q) {
+            pair_cut_off[q] = ncut;
+            for (uint32_t t = 0; t < counts[q]; ++t) {
+                const uint32_t n = flat[pos++];
+                for (uint32_t i = 0; i < n; ++i) leaves[nleaf++] = flat[pos++];
+                cut_off[++ncut] = nleaf;
+            }
+        }
+        pair_cut_off[npairs] = ncut;
+        return CEC_OK;
+    }
     std::vector<std::vector<Cut>> P(N);
     auto trivial = [&](uint32_t id) {  // the constant needs no leaf: its cut is empty
         Cut t;

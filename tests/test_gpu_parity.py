@@ -333,3 +333,35 @@ def test_nccl_min_allreduce_single_rank():
     ref = gpu_ctx(m.aig).sim_exhaustive(m.lit_a, m.lit_b)
     for a, b in zip(got, ref):
         assert np.array_equal(a, b)
+
+
+@pytest.mark.parametrize("case", range(8))
+def test_gpu_cut_generator_matches_cut_oracle(case):
+    """NEXT-1: the GPU cut generator (level-parallel by Eq. 2, warp per node) returns exactly the cuts
+    of oracle/cuts.py (Eq. 1 + Table I + dominance + similarity, exact arithmetic)."""
+    from oracle import cuts as cut_oracle
+    from workloads import c4_dp
+    rng = np.random.default_rng(50 + case)
+    m = c4_dp(6 + 2 * case) if case < 4 else circuits.random_miter(12, 150 + 60 * case, 10, seed=950 + case, window=24)
+    aig = m.aig
+    pairs = set()
+    for a, b in zip(m.lit_a, m.lit_b):
+        x, y = sorted((int(a) >> 1, int(b) >> 1))
+        if x < y:
+            pairs.add((x, y))
+    for _ in range(30):
+        x, y = sorted(int(v) for v in rng.integers(1, aig.num_nodes, size=2))
+        if x < y:
+            pairs.add((x, y))
+    seen, P = set(), []
+    for x, y in sorted(pairs):
+        if y not in seen:
+            seen.add(y)
+            P.append((x, y))
+    k_l, C, pass_id, mc = int(rng.integers(4, 17)), int(rng.integers(2, 17)), case % 3, int(rng.integers(1, 9))
+    ctx = gpu_ctx(aig)
+    pco, co, lv = capi.cec_common_cuts(ctx.handle, [x for x, _ in P], [y for _, y in P], k_l, C, pass_id, mc)
+    want = cut_oracle.common_cuts(aig.num_pis, aig.fanins, [x for x, _ in P], [y for _, y in P], k_l, C, pass_id, mc)
+    for i in range(len(P)):
+        got = [tuple(int(v) for v in lv[co[t]:co[t + 1]]) for t in range(int(pco[i]), int(pco[i + 1]))]
+        assert got == want[i], (i, P[i], got, want[i])
