@@ -20,6 +20,7 @@
 #include <cstdint>
 #include <cstdlib>
 #include <cstring>
+#include <string>
 #include <vector>
 
 #include "cec_ctx.hpp"
@@ -166,7 +167,12 @@ extern "C" cec_status cec_common_cuts(cec_ctx *c, uint32_t npairs, const uint32_
     }
     std::vector<uint32_t> repr_of(N, 0xFFFFFFFFu);
     for (uint32_t q = 0; q < npairs; ++q) repr_of[member[q]] = repr[q];
-    if (!c->host_only && C <= gpu_cuts_max_C() && getenv("CEC_CUTS_HOST") == nullptr) {
+    size_t n_need = 0;
+    for (uint32_t id = c->I + 1; id < N; ++id) n_need += need[id];
+    // GPU generator for large cones (one launch per enumeration level pays off only at scale);
+    // CEC_CUTS_GPU=1 / CEC_CUTS_HOST=1 force a side (tests pin both against oracle/cuts.py)
+    const bool force_gpu = getenv("CEC_CUTS_GPU") != nullptr, force_host = getenv("CEC_CUTS_HOST") != nullptr;
+    if (!c->host_only && C <= gpu_cuts_max_C() && !force_host && (force_gpu || n_need >= 20000)) {
         // GPU cut generator: nodes grouped by enumeration level (Eq. 2)
         cec_status st = cec_ensure_device_aig(c);
         if (st != CEC_OK) return st;
@@ -186,7 +192,10 @@ extern "C" cec_status cec_common_cuts(cec_ctx *c, uint32_t npairs, const uint32_
         std::vector<uint32_t> R(repr, repr + npairs), M(member, member + npairs), counts, flat;
         const char *e = gpu_common_cuts(c->d_f0, c->d_f1, N, fanout, lvl, repr_of, pis, lists, R, M, k_l, C, pass_id,
                                         max_cuts, c->stream, c->num_sms, counts, flat);
-        if (e) return CEC_E_CUDA;
+        if (e) {
+            c->err = std::string("CUDA: ") + e + " (GPU cut generator)";
+            return CEC_E_CUDA;
+        }
         uint32_t ncut = 0, nleaf = 0;
         size_t pos = 0;
         cut_off[0] = 0;

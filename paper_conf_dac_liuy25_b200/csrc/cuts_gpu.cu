@@ -151,6 +151,10 @@ __device__ __forceinline__ void load_list(const GCut *P, const uint32_t *cnt, ui
     n = c + 1;
 }
 
+__host__ __device__ constexpr size_t level_smem_per_warp() {
+    return (sizeof(Keys) * EMAX + sizeof(GCut) * (2 * (CMAX + 1) + EMAX) + sizeof(uint32_t) * EMAX + 15) / 16 * 16;
+}
+
 __global__ void __launch_bounds__(WPB * 32)
 cut_level_kernel(const uint32_t *__restrict__ nodes, uint32_t nnodes, const uint32_t *__restrict__ f0,
                  const uint32_t *__restrict__ f1, const uint32_t *__restrict__ fanout,
@@ -158,13 +162,12 @@ cut_level_kernel(const uint32_t *__restrict__ nodes, uint32_t nnodes, const uint
                  uint32_t k_l, uint32_t C, int pass) {
     extern __shared__ __align__(16) unsigned char sm[];
     const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31u;
-    const size_t per_warp = sizeof(GCut) * (2 * (CMAX + 1) + EMAX) + sizeof(Keys) * EMAX + sizeof(uint32_t) * EMAX;
-    unsigned char *base = sm + per_warp * warp;
-    GCut *Ua = reinterpret_cast<GCut *>(base);
+    unsigned char *base = sm + level_smem_per_warp() * warp;
+    Keys *K = reinterpret_cast<Keys *>(base);  // first: 16-byte aligned (__int128 member)
+    GCut *Ua = reinterpret_cast<GCut *>(K + EMAX);
     GCut *Vb = Ua + (CMAX + 1);
     GCut *E = Vb + (CMAX + 1);
-    Keys *K = reinterpret_cast<Keys *>(E + EMAX);
-    uint32_t *rank = reinterpret_cast<uint32_t *>(K + EMAX);
+    uint32_t *rank = reinterpret_cast<uint32_t *>(E + EMAX);
     const unsigned __int128 L = d_lcm48();
     for (uint32_t w = blockIdx.x * WPB + warp; w < nnodes; w += gridDim.x * WPB) {
         const uint32_t id = nodes[w];
@@ -359,7 +362,7 @@ const char *gpu_common_cuts(const uint32_t *d_f0, const uint32_t *d_f1, uint32_t
             return e;
         }
     }
-    const size_t smem_lvl = WPB * (sizeof(GCut) * (2 * (CMAX + 1) + EMAX) + sizeof(Keys) * EMAX + sizeof(uint32_t) * EMAX);
+    const size_t smem_lvl = WPB * level_smem_per_warp();
     CK(cudaFuncSetAttribute(cut_level_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_lvl));
     size_t off = 0;
     for (auto &l : el_lists) {

@@ -360,7 +360,11 @@ def test_gpu_cut_generator_matches_cut_oracle(case):
             P.append((x, y))
     k_l, C, pass_id, mc = int(rng.integers(4, 17)), int(rng.integers(2, 17)), case % 3, int(rng.integers(1, 9))
     ctx = gpu_ctx(aig)
-    pco, co, lv = capi.cec_common_cuts(ctx.handle, [x for x, _ in P], [y for _, y in P], k_l, C, pass_id, mc)
+    os.environ["CEC_CUTS_GPU"] = "1"  # small cones would otherwise use the host generator
+    try:
+        pco, co, lv = capi.cec_common_cuts(ctx.handle, [x for x, _ in P], [y for _, y in P], k_l, C, pass_id, mc)
+    finally:
+        del os.environ["CEC_CUTS_GPU"]
     want = cut_oracle.common_cuts(aig.num_pis, aig.fanins, [x for x, _ in P], [y for _, y in P], k_l, C, pass_id, mc)
     for i in range(len(P)):
         got = [tuple(int(v) for v in lv[co[t]:co[t + 1]]) for t in range(int(pco[i]), int(pco[i + 1]))]
