@@ -166,7 +166,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--config", default="c5")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--engine", type=int, default=0, help="0 auto, 1 interpreter, 2 JIT")
+    ap.add_argument("--engine", type=int, default=0, help="0 auto, 1 interpreter, 2 JIT, 3 paper Alg. 1 (simt in HBM)")
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--merge", type=int, default=-1, help="0 off, 1 paper (default), 2 cost-aware (default for c3)")
     ap.add_argument("--cpu-log2-patterns", type=int, default=19)
@@ -207,7 +207,8 @@ def main():
     plan = capi.cec_plan_exhaustive(ctx.handle, m.lit_a, m.lit_b)
     info = capi.cec_plan_info(plan)
     st0 = ctx.stats()
-    engine_name = ("jit" if st0["jit_windows"] == info["num_windows"] else
+    engine_name = ("simt (paper Alg. 1)" if args.engine == capi.CEC_ENGINE_SIMT else
+                   "jit" if st0["jit_windows"] == info["num_windows"] else
                    "interp" if st0["jit_windows"] == 0 else f"jit({st0['jit_windows']} windows)+interp")
 
     for _ in range(args.warmup):
@@ -270,6 +271,7 @@ def main():
     # algorithmic LOP3s of the path: one 3-input LUT per mapped node group per u32 word (JIT), one
     # per AND (interpreter) — the AND-node count itself is the metric W
     achieved = stats["lop3_words"] / (ms / 1e3) / 1e12
+    simt = args.engine == capi.CEC_ENGINE_SIMT
     traffic = None
     prof = os.path.join(ROOT, "profiles", "ncu_summary.json")
     if os.path.exists(prof):
@@ -278,6 +280,14 @@ def main():
         except Exception:
             traffic = None
 
+    hbm_peak = 6453.7
+    mp = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(mp):
+        try:
+            hbm_peak = float(json.load(open(mp)).get("hbm_gbs", hbm_peak))
+        except Exception:
+            pass
+    simt_gbs = 12.0 * (W_rank / 32.0) / (ms / 1e3) / 1e9
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         import oracle
@@ -304,11 +314,16 @@ def main():
             "e2e": {"value": W_all / (e2e / 1e3), "unit": UNIT, "ms_per_miter": e2e,
                     "h2d_bytes_per_step": int(st_e2e["h2d_bytes"]), "d2h_bytes_per_step": int(st_e2e["d2h_bytes"]),
                     "host_prep_ms": st_e2e["host_prep_ms"], "aig_load_ms": load_ms},
-            "roofline": {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "TLOP3/s",
+            "roofline": ({"bound": "hbm", "achieved": simt_gbs, "peak": hbm_peak, "unit": "GB/s",
+                          "frac": simt_gbs / hbm_peak, "traffic": None,
+                          "peak_basis": "MEASURED_PEAKS.json hbm_gbs (copy bandwidth)",
+                          "algorithmic_bytes": "12 B per node per u32 word (2 fanin reads + 1 write of the simulation table)"}
+                         if simt else
+                         {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "TLOP3/s",
                          "frac": achieved / peak, "traffic": traffic,
                          "peak_basis": f"{props.multi_processor_count} SMs x {LOP3_PER_CLK_PER_SM} LOP3/clk x {sm_clock:.0f} MHz (guide unit counts, SM clock)",
                          "lop3_per_word_per_and": stats["lop3_words"] / max(1.0, W_rank / 32.0),
-                         "and_evals_tops": (W_rank / 32.0) / (ms / 1e3) / 1e12},
+                         "and_evals_tops": (W_rank / 32.0) / (ms / 1e3) / 1e12}),
             "step_ms": step_ms, "wall_s": wall,
         }
         if cpu:

@@ -68,7 +68,10 @@ typedef enum {
 typedef enum {
     CEC_ENGINE_AUTO = 0,
     CEC_ENGINE_INTERP = 1, /* schedule interpreter: values in shared memory slots */
-    CEC_ENGINE_JIT = 2     /* per-window-structure register-resident kernel compiled with NVRTC */
+    CEC_ENGINE_JIT = 2,    /* per-window-structure register-resident kernel compiled with NVRTC */
+    CEC_ENGINE_SIMT = 3    /* the paper's Alg. 1: simulation table in HBM, rounds of
+                              E words, one launch per topological level; global checks on one GPU
+                              only (world = 1); table size M from env CEC_SIMT_MB (default 16384) */
 } cec_engine;
 
 typedef struct {

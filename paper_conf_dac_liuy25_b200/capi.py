@@ -18,7 +18,7 @@ LIB_PATH = os.path.join(HERE, "libcec.so")
 CEC_OK, CEC_E_ARG, CEC_E_AIG, CEC_E_CUT, CEC_E_NOMEM, CEC_E_CUDA, CEC_E_NCCL, CEC_E_NOCEX, CEC_E_STATE = range(9)
 CEC_BAD_CUT, CEC_UNDECIDED, CEC_EQUIVALENT, CEC_NOT_EQUIVALENT = -1, 0, 1, 2
 CEC_MERGE_OFF, CEC_MERGE_PAPER, CEC_MERGE_COST = 0, 1, 2
-CEC_ENGINE_AUTO, CEC_ENGINE_INTERP, CEC_ENGINE_JIT = 0, 1, 2
+CEC_ENGINE_AUTO, CEC_ENGINE_INTERP, CEC_ENGINE_JIT, CEC_ENGINE_SIMT = 0, 1, 2, 3
 CEC_NO_CEX = (1 << 64) - 1
 STATUS_NAMES = ["CEC_OK", "CEC_E_ARG", "CEC_E_AIG", "CEC_E_CUT", "CEC_E_NOMEM", "CEC_E_CUDA", "CEC_E_NCCL",
                 "CEC_E_NOCEX", "CEC_E_STATE"]

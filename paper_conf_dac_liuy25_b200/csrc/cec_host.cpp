@@ -572,9 +572,10 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         const uint64_t node_words = (uint64_t)nodes.size() * tt_words_of(k);
         if (k >= 10 && !nodes.empty()) {
             if (c->opts.engine == CEC_ENGINE_JIT) R.jit = true;
+            else if (c->opts.engine == CEC_ENGINE_SIMT && !local) R.jit = false;
             else if (c->opts.engine == CEC_ENGINE_AUTO) R.jit = node_words >= jit_min_node_words || R.sc.nslots > max_slot_cap;
         }
-        if (!R.jit && R.sc.nslots > max_slot_cap) {
+        if (!R.jit && R.sc.nslots > max_slot_cap && !(c->opts.engine == CEC_ENGINE_SIMT && !local)) {
             char b[160];
             snprintf(b, sizeof b, "window %zu needs %u live slots > %u (shared-memory capacity)", w, R.sc.nslots,
                      max_slot_cap);
@@ -675,11 +676,72 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         words_rank_of.push_back(we > wb ? (we - wb) : 0);
         cost_of.push_back((uint64_t)(sc.ops.size() + 1) * (se - sb));
     }
+    if (c->opts.engine == CEC_ENGINE_SIMT && !local) {  // the paper's Alg. 1 layout (sim_simt.cu)
+        if (world != 1) return fail(c, CEC_E_ARG, "CEC_ENGINE_SIMT runs on one GPU (world = 1)");
+        SimtPlan &S = P->simt;
+        S = SimtPlan{};
+        std::vector<uint32_t> row_of(c->N(), 0), lvl_of(c->N(), 0);
+        uint64_t rows = 1;  // row 0 = constant 0
+        std::vector<std::vector<uint4>> by_level;
+        uint64_t max_ttw = 1;
+        for (size_t w = 0; w < wins.size(); ++w) {
+            const WinHost &W = wins[w];
+            const uint32_t k = (uint32_t)W.inputs.size();
+            max_ttw = std::max<uint64_t>(max_ttw, tt_words_of(k));
+            S.h_ttw.push_back(tt_words_of(k));
+            row_of[0] = 0;
+            lvl_of[0] = 0;
+            for (uint32_t j = 0; j < k; ++j) {
+                row_of[W.inputs[j]] = (uint32_t)rows;
+                lvl_of[W.inputs[j]] = 0;
+                S.h_inputs.push_back(make_uint4((uint32_t)rows++, (uint32_t)w, j, 0));
+            }
+            for (uint32_t id : res[w].nodes) {  // topological: fanins are inputs, 0 or earlier nodes
+                const uint32_t a = c->f0[id] >> 1, b = c->f1[id] >> 1;
+                const uint32_t l = 1 + std::max(lvl_of[a], lvl_of[b]);  // window level, inputs at 0
+                lvl_of[id] = l;
+                row_of[id] = (uint32_t)rows++;
+                if (by_level.size() <= l) by_level.resize(l + 1);
+                by_level[l].push_back(make_uint4(row_of[id], row_of[a] | (c->f0[id] & 1u) << 31,
+                                                 row_of[b] | (c->f1[id] & 1u) << 31, (uint32_t)w));
+            }
+            for (uint32_t ci : wcs[w]) {
+                const Cmp &cm = cmps2[ci];
+                S.h_pairs.push_back(make_uint4(row_of[cm.la >> 1] | (cm.la & 1u) << 31,
+                                               row_of[cm.lb >> 1] | (cm.lb & 1u) << 31, (uint32_t)w, ci));
+            }
+        }
+        for (auto &l : by_level) {
+            S.level_off.push_back((uint32_t)S.h_nodes.size());
+            S.h_nodes.insert(S.h_nodes.end(), l.begin(), l.end());
+        }
+        S.level_off.push_back((uint32_t)S.h_nodes.size());
+        uint64_t M = 16384ull << 18;  // words (16 GiB)
+        if (const char *e = getenv("CEC_SIMT_MB")) M = strtoull(e, nullptr, 10) << 18;
+        uint64_t E = 4;  // Alg. 1 l.2: the largest power of two with E x rows <= M
+        while (E * 2 * rows <= M && E < max_ttw) E *= 2;
+        if (E * rows > M) return fail(c, CEC_E_NOMEM, "simulation table: %llu rows do not fit M", (unsigned long long)rows);
+        S.E = (uint32_t)E;
+        S.rows = rows;
+        S.rounds = (max_ttw + E - 1) / E;  // Alg. 1 l.4, with the ceiling (reading Q5)
+        S.n_inputs = (uint32_t)S.h_inputs.size();
+        S.n_pairs = (uint32_t)S.h_pairs.size();
+        P->groups.clear();
+        P->items.clear();
+        P->jitems.clear();
+    }
     tm.lap("windows+schedules+jit-progs");
     P->cmps.swap(cmps2);
     for (auto &pc : P->pair_cmp)
         if (pc >= 0) pc = remap[pc];
     // compile the distinct JIT structures (in parallel; cached process-wide by structure)
+    if (P->simt.E) {  // no JIT kernels / work items for Alg. 1 plans
+        P->jit_kernels = 0;
+        P->jit_windows = 0;
+        P->lop3_words = 0;
+        for (size_t w = 0; w < wins.size(); ++w) P->lop3_words += (uint64_t)P->win_nodes[w] * words_rank_of[w];
+        return CEC_OK;
+    }
     std::vector<JitKernel *> kernels(jit_progs.size(), nullptr);
     const JitConfig jcfg = jit_config();
     const uint64_t jit_pass = jcfg.sync_every > 0 ? (uint64_t)jcfg.threads / 32 : 1;
@@ -795,6 +857,18 @@ cec_status upload(cec_ctx *c, cec_plan *P) {
     CUDA_TRY(c, h2d(d.wins, P->dwin.data(), sizeof(DevWin) * P->dwin.size(), c->stream));
     CUDA_TRY(c, h2d(d.prog, P->prog.data(), sizeof(uint4) * P->prog.size(), c->stream));
     CUDA_TRY(c, h2d(d.items, P->items.data(), sizeof(Item) * P->items.size(), c->stream));
+    if (P->simt.E) {
+        SimtPlan &S = P->simt;
+        CUDA_TRY(c, dev_alloc((void **)&S.d_simt, sizeof(uint32_t) * (size_t)S.E * S.rows));
+        CUDA_TRY(c, dev_alloc((void **)&S.d_inputs, sizeof(uint4) * std::max<size_t>(1, S.h_inputs.size())));
+        CUDA_TRY(c, dev_alloc((void **)&S.d_nodes, sizeof(uint4) * std::max<size_t>(1, S.h_nodes.size())));
+        CUDA_TRY(c, dev_alloc((void **)&S.d_pairs, sizeof(uint4) * std::max<size_t>(1, S.h_pairs.size())));
+        CUDA_TRY(c, dev_alloc((void **)&S.d_ttw, sizeof(unsigned long long) * std::max<size_t>(1, S.h_ttw.size())));
+        CUDA_TRY(c, h2d(S.d_inputs, S.h_inputs.data(), sizeof(uint4) * S.h_inputs.size(), c->stream));
+        CUDA_TRY(c, h2d(S.d_nodes, S.h_nodes.data(), sizeof(uint4) * S.h_nodes.size(), c->stream));
+        CUDA_TRY(c, h2d(S.d_pairs, S.h_pairs.data(), sizeof(uint4) * S.h_pairs.size(), c->stream));
+        CUDA_TRY(c, h2d(S.d_ttw, S.h_ttw.data(), sizeof(unsigned long long) * S.h_ttw.size(), c->stream));
+    }
     CUDA_TRY(c, event_create(&P->ev0));
     CUDA_TRY(c, event_create(&P->ev1));
     c->stats.h2d_bytes = sizeof(DevWin) * P->dwin.size() + sizeof(uint4) * P->prog.size() +
@@ -814,6 +888,14 @@ void free_dev(cec_plan *P) {
     dev_free(d.item_ctr);
     dev_free(d.jitems);
     d = DevPlan{};
+    dev_free(P->simt.d_simt);
+    dev_free(P->simt.d_inputs);
+    dev_free(P->simt.d_nodes);
+    dev_free(P->simt.d_pairs);
+    dev_free(P->simt.d_ttw);
+    P->simt.d_simt = nullptr;
+    P->simt.d_inputs = P->simt.d_nodes = P->simt.d_pairs = nullptr;
+    P->simt.d_ttw = nullptr;
     event_destroy(P->ev0);
     event_destroy(P->ev1);
     P->ev0 = P->ev1 = nullptr;
@@ -1003,8 +1085,9 @@ cec_status cec_plan_run(cec_ctx *c, cec_plan *P) {
     if (!P->uploaded) return fail(c, CEC_E_STATE, "plan not uploaded");
     CUDA_TRY(c, event_record(P->ev0, c->stream));
     uint32_t nl = 0;
-    const char *e = launch_run(P->d, P->groups, (uint32_t)P->dwin.size(), (uint32_t)P->cmps.size(), c->stream,
-                                  c->num_sms, &nl, &c->aux);
+    const char *e = P->simt.E ? launch_simt(P->simt, P->d.first, (uint32_t)P->cmps.size(), c->stream, c->num_sms, &nl)
+                              : launch_run(P->d, P->groups, (uint32_t)P->dwin.size(), (uint32_t)P->cmps.size(),
+                                           c->stream, c->num_sms, &nl, &c->aux);
     if (e) return fail(c, CEC_E_CUDA, "CUDA: %s (kernel launch)", e);
     if (c->comm && !P->cmps.empty()) {  // a10: one NCCL min all-reduce of first_idx
         ncclResult_t r = g_nccl.all_reduce(P->d.first, P->d.first, P->cmps.size(), ncclUint64, ncclMin, c->comm,

@@ -100,6 +100,23 @@ const char *gpu_common_cuts(const uint32_t *d_f0, const uint32_t *d_f1, uint32_t
                             void *stream, int num_sms, std::vector<uint32_t> &cut_counts,
                             std::vector<uint32_t> &cut_leaves_flat);
 
+// sim_simt.cu — the paper's Alg. 1 (simulation table in HBM, rounds x levels) for comparison
+struct SimtPlan {
+    uint32_t E = 0;                 // words per row per round (0 = plan does not use this engine)
+    uint64_t rounds = 0, rows = 0;
+    uint4 *d_simt = nullptr;        // rows x E words
+    uint4 *d_inputs = nullptr;      // {row, window, j, 0}
+    uint4 *d_nodes = nullptr;       // by level: {row, row_f0 | c0 << 31, row_f1 | c1 << 31, window}
+    uint4 *d_pairs = nullptr;       // {row_a | ca << 31, row_b | cb << 31, window, cmp}
+    unsigned long long *d_ttw = nullptr;  // words of each window's truth table
+    uint32_t n_inputs = 0, n_pairs = 0;
+    std::vector<uint32_t> level_off;
+    std::vector<uint4> h_inputs, h_nodes, h_pairs;
+    std::vector<unsigned long long> h_ttw;
+};
+const char *launch_simt(const SimtPlan &S, unsigned long long *first, uint32_t ncmp, void *stream, int num_sms,
+                        uint32_t *launches);
+
 // sim_random.cu
 const char *random_sim(const uint32_t *d_f0, const uint32_t *d_f1, const uint32_t *d_level_ids,
                        const std::vector<uint32_t> &level_off, uint32_t I, uint32_t N, uint32_t W, uint64_t seed,

@@ -69,7 +69,8 @@ def test_paper_examples_on_gpu():
     assert list(lv) == [capi.CEC_UNDECIDED, capi.CEC_EQUIVALENT]  # PAPER.md:35/:130 SDC; cut = support
 
 
-ENGINES = [capi.CEC_ENGINE_INTERP, capi.CEC_ENGINE_JIT]
+ENGINES = [capi.CEC_ENGINE_INTERP, capi.CEC_ENGINE_JIT, capi.CEC_ENGINE_SIMT]
+SHARD_ENGINES = [capi.CEC_ENGINE_INTERP, capi.CEC_ENGINE_JIT]
 
 
 @pytest.mark.parametrize("seed", range(60))
@@ -79,7 +80,7 @@ def test_fuzz_tiny_random(seed):
     m = tiny_random(I, int(rng.integers(1, 120)), 24, 7000 + seed)
     kmax = int(rng.integers(0, 13))
     merge = int(rng.integers(0, 3))
-    check_vs_oracle(m, k_max=kmax, merge=merge, engine=ENGINES[seed % 2])
+    check_vs_oracle(m, k_max=kmax, merge=merge, engine=ENGINES[seed % 3])
 
 
 @pytest.mark.parametrize("engine", ENGINES)
@@ -232,7 +233,7 @@ def combine_shards(results):
 
 
 @pytest.mark.parametrize("world", [2, 3, 8])
-@pytest.mark.parametrize("engine", ENGINES)
+@pytest.mark.parametrize("engine", SHARD_ENGINES)
 def test_shard_emulation_matches_single_gpu(world, engine):
     """rank g of G simulates its slices; min over ranks == the 1-GPU result."""
     for m in (c2_mul12_bug(seed=1, n=10), c5_big(copies=8, n_random=5, n_bugs=3, rand_pis=16, rand_ands=1500, mul_n=8)):
