@@ -434,7 +434,7 @@ JitConfig jit_config() {  // overridable for tuning: CEC_JIT_THREADS / CEC_JIT_M
     if (const char *e = getenv("CEC_JIT_THREADS")) cfg.threads = atoi(e);
     if (const char *e = getenv("CEC_JIT_MINB")) cfg.min_blocks = atoi(e);
     if (const char *e = getenv("CEC_JIT_SYNC")) cfg.sync_every = atoi(e);
-    if (const char *e = getenv("CEC_JIT_FUSE")) cfg.fuse = atoi(e) != 0;
+    if (const char *e = getenv("CEC_JIT_FUSE")) cfg.fuse = atoi(e);
     return cfg;
 }
 

@@ -58,7 +58,8 @@ struct JitConfig {
     int threads = 512;      // threads per block
     int min_blocks = 1;     // __launch_bounds__ min blocks per SM (registers <= 64K / (threads*min_blocks))
     int sync_every = 512;   // block-synchronous: __syncthreads() every this many LOP3s; 0 = warp-independent
-    bool fuse = true;       // 3-input LUT mapping: absorb single-fanout ANDs into their reader's LOP3
+    int fuse = 2;           // 3-input LUT mapping: 0 none, 1 greedy (absorb single-fanout ANDs into the
+                            // reader's LOP3), 2 area-flow mapping over 3-feasible cuts
 };
 struct LaunchGroup {       // windows sharing one kernel launch
     uint32_t nslots;       // interpreter: slots per warp in this launch
@@ -86,7 +87,7 @@ const char *jit_get_kernel(const JitProgram &p, const JitConfig &cfg, bool load,
 double jit_compile_ms(const JitKernel *k);
 int jit_slices_per_pass(const JitKernel *k);
 uint32_t jit_kernel_lop3(const JitKernel *k);
-uint32_t jit_lop3_count(const JitProgram &p, bool fuse);
+uint32_t jit_lop3_count(const JitProgram &p, int mode);
 const char *jit_launch(JitKernel *K, const JItem *items, uint32_t nitems, uint32_t *ctr, unsigned long long *first,
                        unsigned long long *bound, uint32_t *neq_cnt, void *stream, int num_sms);
 

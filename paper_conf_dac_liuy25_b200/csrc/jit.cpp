@@ -203,9 +203,145 @@ std::vector<MappedNode> jit_map(const JitProgram &p, bool fuse) {
     return m;
 }
 
-uint32_t jit_lop3_count(const JitProgram &p, bool fuse) {
+// ---- area-oriented 3-LUT mapping (fuse mode 2) -----------------------------------------------------
+// Every node gets its 3-feasible cuts (merged from its fanins' cuts, like Eq. (1) with k = 3); the
+// best cut minimises the area flow AF(n) = 1 + sum_{leaf l} AF(l) / fanout(l) (inputs: 0). Mapping
+// then walks from the compare roots down: a node is materialised (one LOP3) iff it is a root or a
+// leaf of a chosen cut; every other AND is evaluated inside the LUT of the node that covers it
+// (possibly inside several LUTs — duplication is what lets multi-fanout logic be absorbed too).
+std::vector<MappedNode> jit_map_area(const JitProgram &p) {
+    const uint32_t n = (uint32_t)(p.nodes.size() / 2), ncmp = (uint32_t)(p.cmps.size() / 2);
+    const uint32_t R = p.k + 1 + n;
+    struct C3 {
+        uint8_t m;
+        uint32_t l[3];
+    };
+    std::vector<uint32_t> fanout(R, 0);
+    for (uint32_t i = 0; i < 2 * n; ++i) ++fanout[p.nodes[i] >> 1];
+    std::vector<bool> root(R, false);
+    for (uint32_t i = 0; i < 2 * ncmp; ++i) root[p.cmps[i] >> 1] = true;
+    for (uint32_t r = 0; r < R; ++r)
+        if (root[r]) ++fanout[r];
+    std::vector<std::vector<C3>> cuts(R);
+    std::vector<double> af(R, 0.0);
+    std::vector<C3> best(R);
+    std::vector<bool> req(R, false);
+    std::vector<double> est(fanout.begin(), fanout.end());  // fanout estimate used by area flow
+    const size_t CAP = 16;
+    const int ITER = 3;  // area flow, then re-estimate fanouts from the mapping's references
+    for (int iter = 0; iter < ITER; ++iter) {
+        for (uint32_t r = 0; r < R; ++r) cuts[r].clear();
+        for (uint32_t r = 0; r <= p.k; ++r) {
+            cuts[r].push_back(C3{1, {r, 0, 0}});
+            best[r] = cuts[r][0];
+            af[r] = 0.0;
+        }
+        auto cost = [&](const C3 &c) {
+            double a = 1.0;
+            for (int i = 0; i < c.m; ++i) a += af[c.l[i]] / std::max(1.0, est[c.l[i]]);
+            return a;
+        };
+        for (uint32_t t = 0; t < n; ++t) {
+            const uint32_t me = p.k + 1 + t;
+            const uint32_t a = p.nodes[2 * t] >> 1, b = p.nodes[2 * t + 1] >> 1;
+            std::vector<C3> cand;
+            for (const C3 &u : cuts[a])
+                for (const C3 &v : cuts[b]) {
+                    uint32_t L[6];
+                    int m = 0;
+                    for (int i = 0; i < u.m; ++i) L[m++] = u.l[i];
+                    for (int i = 0; i < v.m; ++i) L[m++] = v.l[i];
+                    std::sort(L, L + m);
+                    m = (int)(std::unique(L, L + m) - L);
+                    if (m > 3) continue;
+                    C3 c{(uint8_t)m, {0, 0, 0}};
+                    for (int i = 0; i < m; ++i) c.l[i] = L[i];
+                    bool dup = false;
+                    for (const C3 &d : cand)
+                        if (d.m == c.m && std::equal(d.l, d.l + d.m, c.l)) dup = true;
+                    if (!dup) cand.push_back(c);
+                }
+            std::sort(cand.begin(), cand.end(), [&](const C3 &x, const C3 &y) {
+                const double cx = cost(x), cy = cost(y);
+                if (cx != cy) return cx < cy;
+                if (x.m != y.m) return x.m < y.m;
+                return std::lexicographical_compare(x.l, x.l + x.m, y.l, y.l + y.m);
+            });
+            if (cand.size() > CAP) cand.resize(CAP);
+            best[me] = cand[0];  // the trivial {a, b} merge always exists
+            af[me] = cost(cand[0]);
+            cuts[me] = cand;
+            cuts[me].push_back(C3{1, {me, 0, 0}});  // the trivial cut, for readers
+        }
+        // cover from the roots
+        std::fill(req.begin(), req.end(), false);
+        std::vector<double> refs(R, 0.0);
+        for (uint32_t r = 0; r < R; ++r)
+            if (root[r]) {
+                req[r] = true;
+                refs[r] += 1.0;
+            }
+        for (uint32_t t = n; t-- > 0;) {
+            const uint32_t me = p.k + 1 + t;
+            if (!req[me]) continue;
+            for (int i = 0; i < best[me].m; ++i) {
+                req[best[me].l[i]] = true;
+                refs[best[me].l[i]] += 1.0;
+            }
+        }
+        for (uint32_t r = 0; r < R; ++r) est[r] = 0.5 * est[r] + 0.5 * std::max(1.0, refs[r]);
+    }
+    // LUT truth tables: evaluate the cone between the leaves and the node on (0xF0, 0xCC, 0xAA)
+    std::vector<MappedNode> out(n);
+    std::vector<uint8_t> val(R, 0);
+    std::vector<uint32_t> stamp(R, 0);
+    uint32_t ep = 0;
+    static const uint8_t K[3] = {0xF0, 0xCC, 0xAA};
+    std::function<uint8_t(uint32_t)> ev = [&](uint32_t r) -> uint8_t {
+        if (stamp[r] == ep) return val[r];
+        uint8_t v;
+        if (r == 0) {
+            v = 0;
+        } else if (r <= p.k) {
+            v = 0;  // unreachable for a valid cut (inputs are always leaves)
+        } else {
+            const uint32_t t = r - p.k - 1;
+            const uint32_t oa = p.nodes[2 * t], ob = p.nodes[2 * t + 1];
+            const uint8_t va = ev(oa >> 1) ^ (uint8_t)((oa & 1u) ? 0xFF : 0), vb = ev(ob >> 1) ^ (uint8_t)((ob & 1u) ? 0xFF : 0);
+            v = va & vb;
+        }
+        stamp[r] = ep;
+        val[r] = v;
+        return v;
+    };
+    for (uint32_t t = 0; t < n; ++t) {
+        const uint32_t me = p.k + 1 + t;
+        MappedNode &x = out[t];
+        x.absorbed = !req[me];
+        if (x.absorbed) continue;
+        const C3 &c = best[me];
+        ++ep;
+        for (int i = 0; i < c.m; ++i) {
+            stamp[c.l[i]] = ep;
+            val[c.l[i]] = c.l[i] == 0 ? 0 : K[i];
+        }
+        // evaluate node me itself over its cut (its own value is not a leaf)
+        const uint32_t oa = p.nodes[2 * t], ob = p.nodes[2 * t + 1];
+        const uint8_t va = ev(oa >> 1) ^ (uint8_t)((oa & 1u) ? 0xFF : 0), vb = ev(ob >> 1) ^ (uint8_t)((ob & 1u) ? 0xFF : 0);
+        x.tt = va & vb;
+        x.nleaves = c.m;
+        for (int i = 0; i < 3; ++i) x.leaf[i] = i < c.m ? c.l[i] : 0;
+    }
+    return out;
+}
+
+std::vector<MappedNode> jit_map_mode(const JitProgram &p, int mode) {
+    return mode == 2 ? jit_map_area(p) : jit_map(p, mode != 0);
+}
+
+uint32_t jit_lop3_count(const JitProgram &p, int mode) {
     uint32_t c = 0;
-    for (const MappedNode &x : jit_map(p, fuse)) c += !x.absorbed;
+    for (const MappedNode &x : jit_map_mode(p, mode)) c += !x.absorbed;
     return c;
 }
 
@@ -294,7 +430,7 @@ std::string jit_source(const JitProgram &p, const JitConfig &cfg) {
                  inv ? "~(" : "", ref_name(p, a >> 1).c_str(), ref_name(p, b >> 1).c_str(), inv ? ")" : "", c, ncmp);
         s += buf;
     };
-    const std::vector<MappedNode> map = jit_map(p, cfg.fuse);
+    const std::vector<MappedNode> map = jit_map_mode(p, cfg.fuse);
     for (uint32_t c : after[0]) emit_cmp(c);
     uint32_t emitted = 0;
     for (uint32_t t = 0; t < n; ++t) {
