@@ -150,6 +150,81 @@ struct Sched {
     uint32_t const_slot = 0xFFFFFFFFu;
 };
 
+// Peak number of simultaneously live values of the schedule build_schedule would produce for this
+// node order (= its slot count), computed without allocating slots or encoding ops.
+uint32_t live_peak(const cec_ctx *c, Scratch &X, const std::vector<uint32_t> &inputs, const std::vector<uint32_t> &nodes,
+                   const std::vector<Cmp> &cmps, const std::vector<uint32_t> &win_cmps) {
+    X.init(c->N());
+    if (++X.sc_epoch == 0) {
+        std::fill(X.sc_stamp.begin(), X.sc_stamp.end(), 0u);
+        X.sc_epoch = 1;
+    }
+    const uint32_t ep = X.sc_epoch;
+    auto &stamp = X.sc_stamp;
+    auto &pos = X.sc_pos;    // 0 = input/const, t+1 = AND node t
+    auto &last = X.sc_last;  // last reader position (op index + 1), 0 = never read
+    const uint32_t n = (uint32_t)nodes.size(), k = (uint32_t)inputs.size();
+    auto touch = [&](uint32_t id) {
+        if (stamp[id] != ep) {
+            stamp[id] = ep;
+            pos[id] = 0;
+            last[id] = 0;
+        }
+    };
+    touch(0);
+    for (uint32_t id : inputs) touch(id);
+    for (uint32_t t = 0; t < n; ++t) {
+        touch(nodes[t]);
+        pos[nodes[t]] = t + 1;
+    }
+    // a compare reads its roots right after the later one (op position = that node's position)
+    std::vector<uint32_t> cmp_last_reads;  // reader positions of compares, in node-position units
+    bool uses_const = false;
+    for (uint32_t t = 0; t < n; ++t) {
+        const uint32_t id = nodes[t];
+        for (uint32_t f : {c->f0[id] >> 1, c->f1[id] >> 1}) {
+            touch(f);
+            last[f] = std::max(last[f], 2 * (t + 1));  // node t reads at 2(t+1)
+            uses_const |= f == 0;
+        }
+    }
+    for (uint32_t ci : win_cmps) {
+        const Cmp &cm = cmps[ci];
+        touch(cm.la >> 1);
+        touch(cm.lb >> 1);
+        const uint32_t at = 2 * std::max(pos[cm.la >> 1], pos[cm.lb >> 1]) + 1;  // right after the later root
+        last[cm.la >> 1] = std::max(last[cm.la >> 1], at);
+        last[cm.lb >> 1] = std::max(last[cm.lb >> 1], at);
+        uses_const |= (cm.la >> 1) == 0 || (cm.lb >> 1) == 0;
+    }
+    // sweep: values die at their last read; an output is born at its node
+    std::vector<uint32_t> deaths(2 * n + 3, 0);
+    uint32_t live = 0;
+    bool const_is_input = false;
+    for (uint32_t id : inputs) {
+        const_is_input |= id == 0;
+        if (last[id]) {
+            ++live;
+            ++deaths[last[id]];
+        }
+    }
+    uint32_t slots = k + ((uses_const && !const_is_input) ? 1 : 0);  // inputs occupy slots 0..k-1 at pass start
+    if (uses_const && !const_is_input) ++live, ++deaths[last[0]];
+    uint32_t peak = live;
+    for (uint32_t t = 0; t < n; ++t) {
+        const uint32_t rd = 2 * (t + 1);
+        live -= deaths[rd];  // operands whose last reader is node t are freed before its output
+        deaths[rd] = 0;
+        ++live;              // node t's output
+        if (last[nodes[t]]) ++deaths[last[nodes[t]]];
+        else --live;         // never read (cannot happen in a window)
+        peak = std::max(peak, live);
+        live -= deaths[rd + 1];  // compares placed after node t
+        deaths[rd + 1] = 0;
+    }
+    return std::max(std::max(peak, slots), 1u);
+}
+
 bool build_schedule(const cec_ctx *c, Scratch &X, const std::vector<uint32_t> &inputs,
                     const std::vector<uint32_t> &nodes, const std::vector<Cmp> &cmps,
                     const std::vector<uint32_t> &win_cmps, Sched &out, std::string &why) {
@@ -551,20 +626,16 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
                 }
             }
         }
+        // the id order (the netlist's own construction order) is often the better one: keep the
+        // order with the smaller live set (counted without building the schedule)
         std::string why;
-        if (!build_schedule(c, X, W.inputs, nodes, cmps2, wc, R.sc, why)) {
-            R.err = why;
-            return;
-        }
-        {  // the id order (the netlist's own construction order) is often the better one: keep the
-           // order with the smaller live set
+        {
             std::vector<uint32_t> by_id(nodes);
             std::sort(by_id.begin(), by_id.end());
-            Sched sc2;
-            if (build_schedule(c, X, W.inputs, by_id, cmps2, wc, sc2, why) && sc2.nslots < R.sc.nslots) {
-                R.sc = std::move(sc2);
-                nodes.swap(by_id);
-            }
+            const uint32_t l_id = live_peak(c, X, W.inputs, by_id, cmps2, wc);
+            const uint32_t l_dfs = live_peak(c, X, W.inputs, nodes, cmps2, wc);
+            if (l_id < l_dfs) nodes.swap(by_id);
+            R.sc.nslots = std::min(l_id, l_dfs);
         }
         const uint32_t k = (uint32_t)W.inputs.size();
         // engine choice: straight-line register kernel for big windows (k >= 10 so a 32-word warp
@@ -574,6 +645,12 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
             if (c->opts.engine == CEC_ENGINE_JIT) R.jit = true;
             else if (c->opts.engine == CEC_ENGINE_SIMT && !local) R.jit = false;
             else if (c->opts.engine == CEC_ENGINE_AUTO) R.jit = node_words >= jit_min_node_words || R.sc.nslots > max_slot_cap;
+        }
+        if (!R.jit && !(c->opts.engine == CEC_ENGINE_SIMT && !local)) {  // interpreter program
+            if (!build_schedule(c, X, W.inputs, nodes, cmps2, wc, R.sc, why)) {
+                R.err = why;
+                return;
+            }
         }
         if (!R.jit && R.sc.nslots > max_slot_cap && !(c->opts.engine == CEC_ENGINE_SIMT && !local)) {
             char b[160];
@@ -770,6 +847,7 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         P->jit_ms = std::chrono::duration<float, std::milli>(std::chrono::steady_clock::now() - t0).count();
     }
     tm.lap("jit compile/cache");
+    PhaseTimer tm2;
     P->jit_kernels = (uint32_t)jit_progs.size();
     P->jit_windows = 0;
     P->lop3_words = 0;
@@ -919,6 +997,7 @@ double est_cost(uint64_t nodes, size_t k) { return (double)nodes * (double)(k <=
 extern "C" {
 
 cec_status cec_plan_exhaustive(cec_ctx *c, uint32_t n, const uint32_t *la, const uint32_t *lb, cec_plan **out) {
+    PhaseTimer tm;
     if (!c || !out || (n && (!la || !lb))) return fail(c, CEC_E_ARG, "null argument");
     *out = nullptr;
     auto t0 = std::chrono::steady_clock::now();
@@ -986,6 +1065,7 @@ cec_status cec_plan_exhaustive(cec_ctx *c, uint32_t n, const uint32_t *la, const
             for (auto &th : pool) th.join();
         }
     }
+    tm.lap("supports");
     for (uint32_t p = 0; p < n; ++p) {
         const std::vector<uint32_t> &S = supp[p];
         const uint64_t cone = cones[p];
@@ -1058,8 +1138,10 @@ cec_status cec_plan_exhaustive(cec_ctx *c, uint32_t n, const uint32_t *la, const
         }
         wins.push_back(std::move(w));
     }
+    tm.lap("routing+merging");
     cec_status st = finish_plan(c, P.get(), wins, nullptr, false);
     if (st != CEC_OK) return st;
+    tm.lap("finish_plan");
     auto t1 = std::chrono::steady_clock::now();
     P->host_ms = std::chrono::duration<float, std::milli>(t1 - t0).count();
     c->stats.host_prep_ms = P->host_ms;
@@ -1075,6 +1157,7 @@ cec_status cec_plan_exhaustive(cec_ctx *c, uint32_t n, const uint32_t *la, const
         free_dev(P.get());
         return st;
     }
+    tm.lap("upload");
     *out = P.release();
     return CEC_OK;
 }
