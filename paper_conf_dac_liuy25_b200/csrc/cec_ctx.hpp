@@ -72,6 +72,7 @@ struct cec_ctx {
     uint32_t *d_f0 = nullptr, *d_f1 = nullptr, *d_level_ids = nullptr;
     std::vector<uint32_t> level_off;
     Scratch scratch;  // for serial host work (supports of single pairs, cut validation)
+    std::vector<Scratch> pool;  // one per planning thread, kept across calls (allocated once)
 
     uint32_t N() const { return 1 + I + A; }
     bool is_and(uint32_t id) const { return id > I; }

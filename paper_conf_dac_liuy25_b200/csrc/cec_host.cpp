@@ -694,9 +694,10 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         } else {
             std::atomic<size_t> next{0};
             std::vector<std::thread> pool;
+            if (c->pool.size() < nt) c->pool.resize(nt);
             for (unsigned t = 0; t < nt; ++t)
-                pool.emplace_back([&]() {
-                    Scratch X;
+                pool.emplace_back([&, t]() {
+                    Scratch &X = c->pool[t];  // persistent per-thread scratch (no per-call allocation)
                     for (size_t w; (w = next.fetch_add(1)) < wins.size();) plan_one(w, X);
                 });
             for (auto &th : pool) th.join();
@@ -1025,11 +1026,17 @@ cec_status cec_plan_exhaustive(cec_ctx *c, uint32_t n, const uint32_t *la, const
         const unsigned hw = std::max(1u, std::min(16u, std::thread::hardware_concurrency()));
         const unsigned nt = (unsigned)std::min<uint64_t>(hw, (n + 63) / 64);
         std::atomic<uint32_t> next{0};
-        auto work = [&]() {
-            std::vector<uint32_t> stamp(c->N(), 0), st;
-            uint32_t ep = 0;
-            for (uint32_t p; (p = next.fetch_add(1)) < n;) {
-                ++ep;
+        if (c->pool.size() < nt + 1) c->pool.resize(nt + 1);
+        auto work = [&](unsigned tid) {
+            Scratch &X = c->pool[tid];
+            X.init(c->N());
+            std::vector<uint32_t> &stamp = X.stamp, &st = X.stack;
+            uint32_t &ep = X.epoch;
+            // chunks of consecutive pairs per thread: pairs of one PO group share their cone, so a
+            // thread walks the same (cache-resident) nodes again
+            for (uint32_t p0; (p0 = next.fetch_add(64)) < n;)
+            for (uint32_t p = p0; p < std::min(n, p0 + 64); ++p) {
+                ep = X.next_epoch();
                 auto &S = supp[p];
                 uint64_t nodes = 0;
                 st.clear();
@@ -1058,10 +1065,10 @@ cec_status cec_plan_exhaustive(cec_ctx *c, uint32_t n, const uint32_t *la, const
             }
         };
         if (nt <= 1) {
-            work();
+            work(0);
         } else {
             std::vector<std::thread> pool;
-            for (unsigned t = 0; t < nt; ++t) pool.emplace_back(work);
+            for (unsigned t = 0; t < nt; ++t) pool.emplace_back(work, t);
             for (auto &th : pool) th.join();
         }
     }
