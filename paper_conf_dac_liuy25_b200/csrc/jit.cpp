@@ -400,10 +400,12 @@ std::string jit_source(const JitProgram &p, const JitConfig &cfg) {
                  "    const u32 it = s_it;\n"
                  "    if (it >= nitems) return;\n"
                  "    const JItem I = s_item;\n"
+                 "    u64 bnd = *((volatile u64 *)&bound[I.win]);\n"
                  "    for (u32 s0 = I.s_begin; s0 < I.s_end; s0 += %du) {\n"
                  "      const u32 s = s0 + warp;\n"
-                 "      const bool live = s < I.s_end && ((u64)s << 10) < *((volatile u64 *)&bound[I.win]);\n"
-                 "      if (!__syncthreads_or(live)) break;\n",
+                 "      const bool live = s < I.s_end && ((u64)s << 10) < bnd;\n"
+                 "      if (!__syncthreads_or(live)) break;\n"
+                 "      const u64 bnd_next = *((volatile u64 *)&bound[I.win]);  // used next pass: latency hidden\n",
                  nw);
         s += buf;
     }
@@ -431,6 +433,8 @@ std::string jit_source(const JitProgram &p, const JitConfig &cfg) {
         s += buf;
     };
     const std::vector<MappedNode> map = jit_map_mode(p, cfg.fuse);
+    uint32_t lut_total = 0;
+    for (const MappedNode &x : map) lut_total += !x.absorbed;
     for (uint32_t c : after[0]) emit_cmp(c);
     uint32_t emitted = 0;
     for (uint32_t t = 0; t < n; ++t) {
@@ -446,9 +450,12 @@ std::string jit_source(const JitProgram &p, const JitConfig &cfg) {
             ++emitted;
         }
         for (uint32_t c : after[t + 1]) emit_cmp(c);
-        if (block_sync && !x.absorbed && emitted % (uint32_t)cfg.sync_every == 0) s += "      __syncthreads();\n";
+        // keep the block's warps in one stretch of a large body (shared I-cache lines); a small body
+        // (<= 2048 LUTs, <= 32 KB of SASS) fits the caches and needs no mid-body barrier
+        if (block_sync && !x.absorbed && lut_total > 2048 && emitted % (uint32_t)cfg.sync_every == 0)
+            s += "      __syncthreads();\n";
     }
-    s += block_sync ? "    }\n    __syncthreads();\n  }\n}\n" : "    }\n  }\n}\n";
+    s += block_sync ? "      bnd = bnd_next;\n    }\n    __syncthreads();\n  }\n}\n" : "    }\n  }\n}\n";
     return s;
 }
 
