@@ -142,6 +142,17 @@ interp_kernel(const Item *__restrict__ items, uint32_t nitems, uint32_t *__restr
 
 inline const char *ck(cudaError_t e) { return e == cudaSuccess ? nullptr : cudaGetErrorString(e); }
 
+__global__ void reset_run(unsigned long long *first, uint32_t ncmp, unsigned long long *bound, uint32_t *neq_cnt,
+                          uint32_t nwin, uint32_t *item_ctr, uint32_t ngroups) {
+    const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i < ncmp) first[i] = ~0ull;
+    if (i < nwin) {
+        bound[i] = ~0ull;
+        neq_cnt[i] = 0u;
+    }
+    if (i < ngroups) item_ctr[i] = 0u;
+}
+
 }  // namespace
 
 uint32_t interp_max_slots_per_warp() {
@@ -181,10 +192,12 @@ const char *launch_run(const DevPlan &d, const std::vector<LaunchGroup> &groups,
     cudaStream_t main_st = (cudaStream_t)stream;
     cudaStream_t st = main_st;
     const char *e;
-    if ((e = ck(cudaMemsetAsync(d.first, 0xFF, sizeof(unsigned long long) * (ncmp ? ncmp : 1), st)))) return e;
-    if ((e = ck(cudaMemsetAsync(d.bound, 0xFF, sizeof(unsigned long long) * (nwin ? nwin : 1), st)))) return e;
-    if ((e = ck(cudaMemsetAsync(d.neq_cnt, 0, sizeof(uint32_t) * (nwin ? nwin : 1), st)))) return e;
-    if ((e = ck(cudaMemsetAsync(d.item_ctr, 0, sizeof(uint32_t) * (groups.size() ? groups.size() : 1), st)))) return e;
+    {  // one launch resets the run state (first-mismatch indices, bounds, counters)
+        const uint32_t ng = (uint32_t)(groups.size() ? groups.size() : 1);
+        const uint32_t n = std::max(std::max(ncmp, nwin), ng);
+        reset_run<<<(n + 255) / 256, 256, 0, st>>>(d.first, ncmp, d.bound, d.neq_cnt, nwin, d.item_ctr, ng);
+        if ((e = ck(cudaGetLastError()))) return e;
+    }
     const bool multi = aux && aux->ok && groups.size() > 1;
     if (multi) {
         if ((e = ck(cudaEventRecord((cudaEvent_t)aux->fork, main_st)))) return e;
