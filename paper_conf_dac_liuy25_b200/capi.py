@@ -119,7 +119,7 @@ def cec_default_opts(**kw) -> CecOpts:
 
 def cec_last_error(ctx) -> str:
     s = lib.cec_last_error(ctx)
-    return s.decode() if s else ""
+    return s.decode(errors="replace") if s else ""
 
 
 def _check(st: int, ctx=None):

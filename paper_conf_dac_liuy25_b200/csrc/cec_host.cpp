@@ -510,6 +510,7 @@ JitConfig jit_config() {  // overridable for tuning: CEC_JIT_THREADS / CEC_JIT_M
     if (const char *e = getenv("CEC_JIT_MINB")) cfg.min_blocks = atoi(e);
     if (const char *e = getenv("CEC_JIT_SYNC")) cfg.sync_every = atoi(e);
     if (const char *e = getenv("CEC_JIT_FUSE")) cfg.fuse = atoi(e);
+    if (const char *e = getenv("CEC_JIT_SPLICE")) cfg.splice = atoi(e) != 0;
     return cfg;
 }
 
@@ -826,7 +827,7 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
     P->jit_ms = 0.f;
     if (!jit_progs.empty()) {
         auto t0 = std::chrono::steady_clock::now();
-        std::vector<const char *> errs(jit_progs.size(), nullptr);
+        std::vector<std::string> errs(jit_progs.size());  // copied in the worker (messages are thread-local)
         const bool load = !c->host_only;
         // compile (CPU-heavy, thread-safe) in parallel without loading, then load serially
         const unsigned hw = std::max(1u, std::min(16u, std::thread::hardware_concurrency()));
@@ -835,11 +836,14 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         for (unsigned t = 0; t < std::min<size_t>(hw, jit_progs.size()); ++t)
             pool.emplace_back([&]() {
                 for (size_t i; (i = next.fetch_add(1)) < jit_progs.size();)
-                    errs[i] = jit_get_kernel(jit_progs[i], jcfg, false, &kernels[i]);
+                {
+                    const char *e = jit_get_kernel(jit_progs[i], jcfg, false, &kernels[i]);
+                    if (e) errs[i] = e;
+                }
             });
         for (auto &th : pool) th.join();
         for (size_t i = 0; i < jit_progs.size(); ++i) {
-            if (errs[i]) return fail(c, CEC_E_CUDA, "JIT: %s", errs[i]);
+            if (!errs[i].empty()) return fail(c, CEC_E_CUDA, "JIT: %s", errs[i].c_str());
             if (load) {
                 const char *e = jit_get_kernel(jit_progs[i], jcfg, true, &kernels[i]);
                 if (e) return fail(c, CEC_E_CUDA, "JIT load: %s", e);

@@ -60,6 +60,7 @@ struct JitConfig {
     int sync_every = 512;   // block-synchronous: __syncthreads() every this many LOP3s; 0 = warp-independent
     int fuse = 2;           // 3-input LUT mapping: 0 none, 1 greedy (absorb single-fanout ANDs into the
                             // reader's LOP3), 2 area-flow mapping over 3-feasible cuts
+    bool splice = true;     // body as generated PTX spliced into an NVRTC skeleton (skips NVVM on it)
 };
 struct LaunchGroup {       // windows sharing one kernel launch
     uint32_t nslots;       // interpreter: slots per warp in this launch

@@ -49,6 +49,8 @@ struct Nvrtc {
     nvrtcResult_t (*cubin_size)(nvrtcProgram_t, size_t *) = nullptr;
     nvrtcResult_t (*cubin)(nvrtcProgram_t, char *) = nullptr;
     nvrtcResult_t (*destroy)(nvrtcProgram_t *) = nullptr;
+    nvrtcResult_t (*ptx_size)(nvrtcProgram_t, size_t *) = nullptr;
+    nvrtcResult_t (*ptx)(nvrtcProgram_t, char *) = nullptr;
     std::string why;
     bool load() {
         if (h) return true;
@@ -68,7 +70,9 @@ struct Nvrtc {
         cubin_size = (decltype(cubin_size))dlsym(h, "nvrtcGetCUBINSize");
         cubin = (decltype(cubin))dlsym(h, "nvrtcGetCUBIN");
         destroy = (decltype(destroy))dlsym(h, "nvrtcDestroyProgram");
-        if (!(create && compile && log_size && log && cubin_size && cubin && destroy)) {
+        ptx_size = (decltype(ptx_size))dlsym(h, "nvrtcGetPTXSize");
+        ptx = (decltype(ptx))dlsym(h, "nvrtcGetPTX");
+        if (!(create && compile && log_size && log && cubin_size && cubin && destroy && ptx_size && ptx)) {
             why = "libnvrtc is missing symbols";
             return false;
         }
@@ -432,31 +436,225 @@ std::string jit_source(const JitProgram &p, const JitConfig &cfg) {
                  inv ? "~(" : "", ref_name(p, a >> 1).c_str(), ref_name(p, b >> 1).c_str(), inv ? ")" : "", c, ncmp);
         s += buf;
     };
+    if (cfg.splice && block_sync) {
+        // PTX-splice mode: the whole LUT network is ONE inline-asm statement whose text is a marker
+        // with its operands (compare outputs, then input words); the body PTX is generated directly
+        // and spliced in after NVRTC (jit_body_ptx), so NVVM never sees the thousands of LUTs
+        for (uint32_t c = 0; c < ncmp; ++c) {
+            snprintf(buf, sizeof buf, "      u32 d%u;\n", c);
+            s += buf;
+        }
+        s += "      asm volatile(\"//@@BODY@@";
+        for (uint32_t i = 0; i < ncmp + p.k; ++i) {
+            snprintf(buf, sizeof buf, " %%%u", i);
+            s += buf;
+        }
+        s += "\"";
+        s += " :";
+        for (uint32_t c = 0; c < ncmp; ++c) {
+            snprintf(buf, sizeof buf, "%s \"=r\"(d%u)", c ? "," : "", c);
+            s += buf;
+        }
+        s += " :";
+        for (uint32_t j = 0; j < p.k; ++j) {
+            snprintf(buf, sizeof buf, "%s \"r\"(x%u)", j ? "," : "", j);
+            s += buf;
+        }
+        s += " : \"memory\");\n";
+        for (uint32_t c = 0; c < ncmp; ++c) {
+            snprintf(buf, sizeof buf,
+                     "      { const u32 d = live ? d%u : 0u; if (__any_sync(0xFFFFFFFFu, d != 0u)) rep(d, %uu, I.win, s, lane, %uu, I.cmp_off, first, bound, neq_cnt); }\n",
+                     c, c, ncmp);
+            s += buf;
+        }
+    } else {
+        const std::vector<MappedNode> map = jit_map_mode(p, cfg.fuse);
+        uint32_t lut_total = 0;
+        for (const MappedNode &x : map) lut_total += !x.absorbed;
+        for (uint32_t c : after[0]) emit_cmp(c);
+        uint32_t emitted = 0;
+        for (uint32_t t = 0; t < n; ++t) {
+            const MappedNode &x = map[t];
+            if (!x.absorbed) {
+                // LOP3 input order (a, b, c) = leaf[0..2]; the LUT was built for (0xF0, 0xCC, 0xAA)
+                snprintf(buf, sizeof buf,
+                         "      u32 n%u; asm(\"lop3.b32 %%0, %%1, %%2, %%3, 0x%02X;\" : \"=r\"(n%u) : \"r\"(%s), \"r\"(%s), \"r\"(%s));\n",
+                         t, x.tt, t, x.nleaves > 0 ? ref_name(p, x.leaf[0]).c_str() : "0u",
+                         x.nleaves > 1 ? ref_name(p, x.leaf[1]).c_str() : "0u",
+                         x.nleaves > 2 ? ref_name(p, x.leaf[2]).c_str() : "0u");
+                s += buf;
+                ++emitted;
+            }
+            for (uint32_t c : after[t + 1]) emit_cmp(c);
+            // keep the block's warps in one stretch of a large body (shared I-cache lines); a small body
+            // (<= 2048 LUTs, <= 32 KB of SASS) fits the caches and needs no mid-body barrier
+            if (block_sync && !x.absorbed && lut_total > 2048 && emitted % (uint32_t)cfg.sync_every == 0)
+                s += "      __syncthreads();\n";
+        }
+    }
+    s += block_sync ? "      bnd = bnd_next;\n    }\n    __syncthreads();\n  }\n}\n" : "    }\n  }\n}\n";
+    return s;
+}
+
+// PTX of the LUT network for splice mode: out_regs[c] receive the compare diffs, in_regs[j] hold
+// the input words. One lop3.b32 per materialised LUT (mapping of jit_map_mode), a bar.sync every
+// sync_every LUTs for large bodies, and d_c = a ^ b (^ ~0) right after the later root.
+std::string jit_body_ptx(const JitProgram &p, const JitConfig &cfg, const std::vector<std::string> &out_regs,
+                         const std::vector<std::string> &in_regs) {
+    const uint32_t n = (uint32_t)(p.nodes.size() / 2), ncmp = (uint32_t)(p.cmps.size() / 2);
     const std::vector<MappedNode> map = jit_map_mode(p, cfg.fuse);
     uint32_t lut_total = 0;
     for (const MappedNode &x : map) lut_total += !x.absorbed;
+    std::string s;
+    s.reserve(64 * (size_t)n + 4096);
+    char buf[256];
+    snprintf(buf, sizeof buf, "{\n.reg .b32 %%cz;\n.reg .b32 %%cn<%u>;\nmov.b32 %%cz, 0;\n", std::max<uint32_t>(n, 1));
+    s += buf;
+    auto reg = [&](uint32_t ref) -> std::string {
+        if (ref == 0) return "%cz";
+        if (ref <= p.k) return in_regs[ref - 1];
+        return "%cn" + std::to_string(ref - p.k - 1);
+    };
+    std::vector<std::vector<uint32_t>> after(n + 1);
+    for (uint32_t c = 0; c < ncmp; ++c) {
+        const uint32_t m = std::max(p.cmps[2 * c] >> 1, p.cmps[2 * c + 1] >> 1);
+        after[m > p.k ? m - p.k : 0].push_back(c);
+    }
+    auto emit_cmp = [&](uint32_t c) {
+        const uint32_t a = p.cmps[2 * c], b = p.cmps[2 * c + 1];
+        const unsigned lut = ((a ^ b) & 1u) ? 0xC3u : 0x3Cu;  // ~(a ^ b) : a ^ b on (0xF0, 0xCC)
+        snprintf(buf, sizeof buf, "lop3.b32 %s, %s, %s, %%cz, 0x%02X;\n", out_regs[c].c_str(), reg(a >> 1).c_str(),
+                 reg(b >> 1).c_str(), lut);
+        s += buf;
+    };
     for (uint32_t c : after[0]) emit_cmp(c);
     uint32_t emitted = 0;
     for (uint32_t t = 0; t < n; ++t) {
         const MappedNode &x = map[t];
         if (!x.absorbed) {
-            // LOP3 input order (a, b, c) = leaf[0..2]; the LUT was built for (0xF0, 0xCC, 0xAA)
-            snprintf(buf, sizeof buf,
-                     "      u32 n%u; asm(\"lop3.b32 %%0, %%1, %%2, %%3, 0x%02X;\" : \"=r\"(n%u) : \"r\"(%s), \"r\"(%s), \"r\"(%s));\n",
-                     t, x.tt, t, x.nleaves > 0 ? ref_name(p, x.leaf[0]).c_str() : "0u",
-                     x.nleaves > 1 ? ref_name(p, x.leaf[1]).c_str() : "0u",
-                     x.nleaves > 2 ? ref_name(p, x.leaf[2]).c_str() : "0u");
+            snprintf(buf, sizeof buf, "lop3.b32 %%cn%u, %s, %s, %s, 0x%02X;\n", t,
+                     x.nleaves > 0 ? reg(x.leaf[0]).c_str() : "%cz", x.nleaves > 1 ? reg(x.leaf[1]).c_str() : "%cz",
+                     x.nleaves > 2 ? reg(x.leaf[2]).c_str() : "%cz", x.tt);
             s += buf;
             ++emitted;
         }
         for (uint32_t c : after[t + 1]) emit_cmp(c);
-        // keep the block's warps in one stretch of a large body (shared I-cache lines); a small body
-        // (<= 2048 LUTs, <= 32 KB of SASS) fits the caches and needs no mid-body barrier
-        if (block_sync && !x.absorbed && lut_total > 2048 && emitted % (uint32_t)cfg.sync_every == 0)
-            s += "      __syncthreads();\n";
+        if (!x.absorbed && lut_total > 2048 && emitted % (uint32_t)cfg.sync_every == 0) s += "bar.sync 0;\n";
     }
-    s += block_sync ? "      bnd = bnd_next;\n    }\n    __syncthreads();\n  }\n}\n" : "    }\n  }\n}\n";
+    s += "}\n";
     return s;
+}
+
+namespace {
+// ---- nvJitLink (PTX -> cubin, thread-safe per handle), loaded on demand -------------------------
+struct JitLink {
+    void *h = nullptr;
+    int (*create)(void **, uint32_t, const char **) = nullptr;
+    int (*add)(void *, int, const void *, size_t, const char *) = nullptr;
+    int (*complete)(void *) = nullptr;
+    int (*cubin_size)(void *, size_t *) = nullptr;
+    int (*cubin)(void *, void *) = nullptr;
+    int (*log_size)(void *, size_t *) = nullptr;
+    int (*log)(void *, char *) = nullptr;
+    int (*destroy)(void **) = nullptr;
+    bool tried = false, ok = false;
+    bool load() {
+        if (tried) return ok;
+        tried = true;
+        const char *cands[] = {"/usr/local/cuda/lib64/libnvJitLink.so.12", "libnvJitLink.so.12"};
+        for (const char *c : cands) {
+            h = dlopen(c, RTLD_NOW | RTLD_LOCAL);
+            if (!h) continue;
+            create = (decltype(create))dlsym(h, "__nvJitLinkCreate_12_9");
+            add = (decltype(add))dlsym(h, "__nvJitLinkAddData_12_9");
+            complete = (decltype(complete))dlsym(h, "__nvJitLinkComplete_12_9");
+            cubin_size = (decltype(cubin_size))dlsym(h, "__nvJitLinkGetLinkedCubinSize_12_9");
+            cubin = (decltype(cubin))dlsym(h, "__nvJitLinkGetLinkedCubin_12_9");
+            log_size = (decltype(log_size))dlsym(h, "__nvJitLinkGetErrorLogSize_12_9");
+            log = (decltype(log))dlsym(h, "__nvJitLinkGetErrorLog_12_9");
+            destroy = (decltype(destroy))dlsym(h, "__nvJitLinkDestroy_12_9");
+            ok = create && add && complete && cubin_size && cubin && log_size && log && destroy;
+            if (ok) break;
+        }
+        return ok;
+    }
+};
+JitLink g_link;
+}  // namespace
+
+// Splice-mode compile: NVRTC turns the small skeleton into PTX, the generated body replaces the
+// marker line, nvJitLink assembles the result for sm_100a.
+const char *jit_compile_splice(const JitProgram &p, const JitConfig &cfg, const std::string &src,
+                               std::vector<char> &cubin, std::string &log) {
+    {
+        std::lock_guard<std::mutex> g(g_mu);
+        if (!g_nvrtc.load()) return g_nvrtc.why.c_str();
+        if (!g_link.load()) return "nvJitLink (12.9) not available";
+    }
+    nvrtcProgram_t prog = nullptr;
+    if (g_nvrtc.create(&prog, src.c_str(), "cecjit.cu", 0, nullptr, nullptr) != 0) return "nvrtcCreateProgram failed";
+    const char *opts[] = {"--gpu-architecture=compute_100a", "--std=c++17", "-default-device"};
+    const int rc = g_nvrtc.compile(prog, 3, opts);
+    size_t ls = 0;
+    g_nvrtc.log_size(prog, &ls);
+    log.assign(ls, '\0');
+    if (ls) g_nvrtc.log(prog, &log[0]);
+    if (rc != 0) {
+        g_nvrtc.destroy(&prog);
+        return "NVRTC compilation failed (skeleton)";
+    }
+    size_t ps = 0;
+    g_nvrtc.ptx_size(prog, &ps);
+    std::string ptx(ps, '\0');
+    g_nvrtc.ptx(prog, &ptx[0]);
+    g_nvrtc.destroy(&prog);
+    const size_t m = ptx.find("//@@BODY@@");
+    if (m == std::string::npos) return "splice marker not found in PTX";
+    const size_t eol = ptx.find('\n', m);
+    std::vector<std::string> regs;
+    {
+        size_t i = m + 10;
+        while (i < eol) {
+            while (i < eol && ptx[i] == ' ') ++i;
+            size_t j = i;
+            while (j < eol && ptx[j] != ' ' && ptx[j] != '\r') ++j;
+            if (j > i) regs.emplace_back(ptx.substr(i, j - i));
+            i = j + 1;
+        }
+    }
+    const uint32_t ncmp = (uint32_t)(p.cmps.size() / 2);
+    if (regs.size() != ncmp + p.k) return "splice: operand count mismatch";
+    std::vector<std::string> outs(regs.begin(), regs.begin() + ncmp), ins(regs.begin() + ncmp, regs.end());
+    ptx.replace(m, eol - m, jit_body_ptx(p, cfg, outs, ins));
+    while (!ptx.empty() && ptx.back() == '\0') ptx.pop_back();
+    if (const char *dir = getenv("CEC_JIT_DUMP")) {
+        char path[512];
+        snprintf(path, sizeof path, "%s/cecjit_%016zx.ptx", dir, std::hash<std::string>()(ptx));
+        if (FILE *f = fopen(path, "w")) {
+            fwrite(ptx.data(), 1, ptx.size(), f);
+            fclose(f);
+        }
+    }
+    void *h = nullptr;
+    const char *lopts[] = {"-arch=sm_100a"};
+    if (g_link.create(&h, 1, lopts) != 0) return "nvJitLinkCreate failed";
+    int r = g_link.add(h, 2 /* NVJITLINK_INPUT_PTX */, ptx.data(), ptx.size(), "cecjit.ptx");
+    if (r == 0) r = g_link.complete(h);
+    if (r != 0) {
+        size_t es = 0;
+        g_link.log_size(h, &es);
+        std::string el(es, '\0');
+        if (es) g_link.log(h, &el[0]);
+        log += el;
+        g_link.destroy(&h);
+        return "nvJitLink failed";
+    }
+    size_t cs = 0;
+    g_link.cubin_size(h, &cs);
+    cubin.resize(cs);
+    g_link.cubin(h, cubin.data());
+    g_link.destroy(&h);
+    return nullptr;
 }
 
 const char *jit_compile_cubin(const std::string &src, std::vector<char> &cubin, std::string &log) {
@@ -490,7 +688,8 @@ std::map<std::string, std::unique_ptr<JitKernel>> g_cache;  // process-wide, key
 
 const char *jit_get_kernel(const JitProgram &p, const JitConfig &cfg, bool load, JitKernel **out) {
     char ck[64];
-    snprintf(ck, sizeof ck, "|%d,%d,%d,%d", cfg.threads, cfg.min_blocks, cfg.sync_every, (int)cfg.fuse);
+    snprintf(ck, sizeof ck, "|%d,%d,%d,%d,%d", cfg.threads, cfg.min_blocks, cfg.sync_every, (int)cfg.fuse,
+             (int)cfg.splice);
     const std::string key = jit_key(p) + ck;
     {
         std::lock_guard<std::mutex> g(g_mu);
@@ -504,7 +703,8 @@ const char *jit_get_kernel(const JitProgram &p, const JitConfig &cfg, bool load,
     const std::string src = jit_source(p, cfg);
     std::vector<char> cubin;
     std::string log;
-    const char *e = jit_compile_cubin(src, cubin, log);
+    const char *e = (cfg.splice && cfg.sync_every > 0) ? jit_compile_splice(p, cfg, src, cubin, log)
+                                                       : jit_compile_cubin(src, cubin, log);
     if (e) {
         static thread_local std::string msg;
         msg = std::string(e) + ": " + log.substr(0, 400);
