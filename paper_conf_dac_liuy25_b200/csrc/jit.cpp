@@ -438,21 +438,27 @@ std::string jit_source(const JitProgram &p, const JitConfig &cfg) {
     };
     if (cfg.splice && block_sync) {
         // PTX-splice mode: the whole LUT network is ONE inline-asm statement whose text is a marker
-        // with its operands (compare outputs, then input words); the body PTX is generated directly
-        // and spliced in after NVRTC (jit_body_ptx), so NVVM never sees the thousands of LUTs
-        for (uint32_t c = 0; c < ncmp; ++c) {
-            snprintf(buf, sizeof buf, "      u32 d%u;\n", c);
+        // with its operands; the body PTX is generated directly and spliced in after NVRTC
+        // (jit_body_ptx), so NVVM never sees the thousands of LUTs. Compares inside the body vote
+        // per warp; a mismatching compare sets its bit in the warp masks m* and stores the lanes'
+        // diff words to dbuf (rare path), so only the masks stay live through the body.
+        const uint32_t M = (ncmp + 31) / 32;
+        if (ncmp) {
+            snprintf(buf, sizeof buf, "      u32 dbuf[%u];\n", ncmp);
+            s += buf;
+        }
+        for (uint32_t w = 0; w < M; ++w) {
+            snprintf(buf, sizeof buf, "      u32 m%u;\n", w);
             s += buf;
         }
         s += "      asm volatile(\"//@@BODY@@";
-        for (uint32_t i = 0; i < ncmp + p.k; ++i) {
+        for (uint32_t i = 0; i < M + p.k + (ncmp ? 1 : 0); ++i) {
             snprintf(buf, sizeof buf, " %%%u", i);
             s += buf;
         }
-        s += "\"";
-        s += " :";
-        for (uint32_t c = 0; c < ncmp; ++c) {
-            snprintf(buf, sizeof buf, "%s \"=r\"(d%u)", c ? "," : "", c);
+        s += "\" :";
+        for (uint32_t w = 0; w < M; ++w) {
+            snprintf(buf, sizeof buf, "%s \"=r\"(m%u)", w ? "," : "", w);
             s += buf;
         }
         s += " :";
@@ -460,11 +466,14 @@ std::string jit_source(const JitProgram &p, const JitConfig &cfg) {
             snprintf(buf, sizeof buf, "%s \"r\"(x%u)", j ? "," : "", j);
             s += buf;
         }
+        if (ncmp) s += ", \"l\"(dbuf)";
         s += " : \"memory\");\n";
-        for (uint32_t c = 0; c < ncmp; ++c) {
+        for (uint32_t w = 0; w < M; ++w) {
             snprintf(buf, sizeof buf,
-                     "      { const u32 d = live ? d%u : 0u; if (__any_sync(0xFFFFFFFFu, d != 0u)) rep(d, %uu, I.win, s, lane, %uu, I.cmp_off, first, bound, neq_cnt); }\n",
-                     c, c, ncmp);
+                     "      for (u32 mk = m%u; mk; mk &= mk - 1u) { const u32 c = %uu + (u32)__ffs(mk) - 1u;\n"
+                     "        const u32 d = live ? dbuf[c] : 0u;\n"
+                     "        if (__any_sync(0xFFFFFFFFu, d != 0u)) rep(d, c, I.win, s, lane, %uu, I.cmp_off, first, bound, neq_cnt); }\n",
+                     w, 32 * w, ncmp);
             s += buf;
         }
     } else {
@@ -499,17 +508,20 @@ std::string jit_source(const JitProgram &p, const JitConfig &cfg) {
 // PTX of the LUT network for splice mode: out_regs[c] receive the compare diffs, in_regs[j] hold
 // the input words. One lop3.b32 per materialised LUT (mapping of jit_map_mode), a bar.sync every
 // sync_every LUTs for large bodies, and d_c = a ^ b (^ ~0) right after the later root.
-std::string jit_body_ptx(const JitProgram &p, const JitConfig &cfg, const std::vector<std::string> &out_regs,
-                         const std::vector<std::string> &in_regs) {
+std::string jit_body_ptx(const JitProgram &p, const JitConfig &cfg, const std::vector<std::string> &masks,
+                         const std::vector<std::string> &in_regs, const std::string &dbuf) {
     const uint32_t n = (uint32_t)(p.nodes.size() / 2), ncmp = (uint32_t)(p.cmps.size() / 2);
     const std::vector<MappedNode> map = jit_map_mode(p, cfg.fuse);
     uint32_t lut_total = 0;
     for (const MappedNode &x : map) lut_total += !x.absorbed;
     std::string s;
-    s.reserve(64 * (size_t)n + 4096);
-    char buf[256];
-    snprintf(buf, sizeof buf, "{\n.reg .b32 %%cz;\n.reg .b32 %%cn<%u>;\nmov.b32 %%cz, 0;\n", std::max<uint32_t>(n, 1));
+    s.reserve(64 * (size_t)n + 160 * (size_t)ncmp + 4096);
+    char buf[320];
+    snprintf(buf, sizeof buf,
+             "{\n.reg .b32 %%cz;\n.reg .b32 %%cd;\n.reg .pred %%cp;\n.reg .pred %%cq;\n.reg .b32 %%cn<%u>;\nmov.b32 %%cz, 0;\n",
+             std::max<uint32_t>(n, 1));
     s += buf;
+    for (const std::string &m : masks) s += "mov.b32 " + m + ", 0;\n";
     auto reg = [&](uint32_t ref) -> std::string {
         if (ref == 0) return "%cz";
         if (ref <= p.k) return in_regs[ref - 1];
@@ -523,8 +535,11 @@ std::string jit_body_ptx(const JitProgram &p, const JitConfig &cfg, const std::v
     auto emit_cmp = [&](uint32_t c) {
         const uint32_t a = p.cmps[2 * c], b = p.cmps[2 * c + 1];
         const unsigned lut = ((a ^ b) & 1u) ? 0xC3u : 0x3Cu;  // ~(a ^ b) : a ^ b on (0xF0, 0xCC)
-        snprintf(buf, sizeof buf, "lop3.b32 %s, %s, %s, %%cz, 0x%02X;\n", out_regs[c].c_str(), reg(a >> 1).c_str(),
-                 reg(b >> 1).c_str(), lut);
+        snprintf(buf, sizeof buf,
+                 "lop3.b32 %%cd, %s, %s, %%cz, 0x%02X;\nsetp.ne.b32 %%cp, %%cd, 0;\nvote.sync.any.pred %%cq, %%cp, 0xffffffff;\n"
+                 "@%%cq st.u32 [%s+%u], %%cd;\n@%%cq or.b32 %s, %s, %u;\n",
+                 reg(a >> 1).c_str(), reg(b >> 1).c_str(), lut, dbuf.c_str(), 4 * c, masks[c / 32].c_str(),
+                 masks[c / 32].c_str(), 1u << (c % 32));
         s += buf;
     };
     for (uint32_t c : after[0]) emit_cmp(c);
@@ -622,10 +637,11 @@ const char *jit_compile_splice(const JitProgram &p, const JitConfig &cfg, const 
             i = j + 1;
         }
     }
-    const uint32_t ncmp = (uint32_t)(p.cmps.size() / 2);
-    if (regs.size() != ncmp + p.k) return "splice: operand count mismatch";
-    std::vector<std::string> outs(regs.begin(), regs.begin() + ncmp), ins(regs.begin() + ncmp, regs.end());
-    ptx.replace(m, eol - m, jit_body_ptx(p, cfg, outs, ins));
+    const uint32_t ncmp = (uint32_t)(p.cmps.size() / 2), M = (ncmp + 31) / 32;
+    if (regs.size() != M + p.k + (ncmp ? 1 : 0)) return "splice: operand count mismatch";
+    std::vector<std::string> masks(regs.begin(), regs.begin() + M), ins(regs.begin() + M, regs.begin() + M + p.k);
+    const std::string dbuf = ncmp ? regs.back() : std::string("%cz");
+    ptx.replace(m, eol - m, jit_body_ptx(p, cfg, masks, ins, dbuf));
     while (!ptx.empty() && ptx.back() == '\0') ptx.pop_back();
     if (const char *dir = getenv("CEC_JIT_DUMP")) {
         char path[512];
