@@ -23,9 +23,7 @@ import argparse
 import json
 import os
 import statistics
-import subprocess
 import sys
-import tempfile
 import threading
 import time
 
@@ -81,50 +79,76 @@ def oracle_sample(m, copy_idx, log2_patterns):
 
 
 class ClockSampler:
-    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
-              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
-              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+    """SM clock + throttle reasons sampled DURING the timed region: an NVML polling thread (every
+    5 ms, plus one sample on entry and one on exit so even a sub-millisecond region has readings)."""
+    REASONS = {0x8: "hw_slowdown", 0x40: "hw_thermal_slowdown", 0x20: "sw_thermal_slowdown",
+               0x4: "sw_power_cap", 0x80: "hw_power_brake_slowdown"}
 
     def __init__(self, gpu: int):
         self.gpu = gpu
-        self.proc = None
-        self.path = None
+        self.rows = []
+        self.stop = None
+        self.thread = None
+        self.h = None
+        self.nvml = None
+
+    def _handle(self):
+        import pynvml as nv
+        nv.nvmlInit()
+        self.nvml = nv
+        try:  # the torch device's own PCI bus id (CUDA_VISIBLE_DEVICES may renumber)
+            import torch
+            p = torch.cuda.get_device_properties(self.gpu)
+            bus = f"{p.pci_domain_id:08x}:{p.pci_bus_id:02x}:{p.pci_device_id:02x}.0"
+            return nv.nvmlDeviceGetHandleByPciBusId(bus)
+        except Exception:
+            return nv.nvmlDeviceGetHandleByIndex(self.gpu)
+
+    def _sample(self):
+        nv = self.nvml
+        sm = nv.nvmlDeviceGetClockInfo(self.h, nv.NVML_CLOCK_SM)
+        try:
+            r = nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+        except Exception:
+            r = nv.nvmlDeviceGetCurrentClocksThrottleReasons(self.h)
+        try:
+            pw = nv.nvmlDeviceGetPowerUsage(self.h) / 1e3
+        except Exception:
+            pw = None
+        self.rows.append((sm, r, pw))
 
     def __enter__(self):
-        fd, self.path = tempfile.mkstemp(suffix=".csv")
-        os.close(fd)
         try:
-            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.FIELDS}",
-                                          "--format=csv,noheader,nounits", "-lms", "100"],
-                                         stdout=open(self.path, "w"), stderr=subprocess.DEVNULL)
-        except OSError:
-            self.proc = None
+            self.h = self._handle()
+            self.max_mhz = self.nvml.nvmlDeviceGetMaxClockInfo(self.h, self.nvml.NVML_CLOCK_SM)
+            self._sample()
+        except Exception:
+            self.h = None
+            return self
+        self.stop = threading.Event()
+
+        def loop():
+            while not self.stop.wait(0.005):
+                self._sample()
+
+        self.thread = threading.Thread(target=loop, daemon=True)
+        self.thread.start()
         return self
 
     def __exit__(self, *a):
-        if self.proc:
-            self.proc.terminate()
-            try:
-                self.proc.wait(timeout=5)
-            except subprocess.TimeoutExpired:
-                self.proc.kill()
+        if self.thread:
+            self._sample()
+            self.stop.set()
+            self.thread.join()
 
     def summary(self):
-        if not self.path or not os.path.exists(self.path):
-            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
-        rows = []
-        for line in open(self.path):
-            f = [x.strip() for x in line.split(",")]
-            if len(f) >= 9 and f[1].replace(".", "").isdigit():
-                rows.append(f)
-        os.unlink(self.path)
-        if not rows:
-            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["no samples"]}
-        sm = [float(r[1]) for r in rows]
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        reasons = sorted({names[i] for r in rows for i in range(4) if r[5 + i].lower() == "active"})
-        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": float(rows[0][2]), "reasons": reasons,
-                "samples": len(rows), "power_w_max": max(float(r[3]) for r in rows if r[3].replace(".", "").isdigit())}
+        if self.h is None or not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvml unavailable"]}
+        sm = [r[0] for r in self.rows]
+        reasons = sorted({name for _, bits, _ in self.rows for b, name in self.REASONS.items() if bits & b})
+        pw = [r[2] for r in self.rows if r[2] is not None]
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": float(self.max_mhz), "reasons": reasons,
+                "samples": len(self.rows), "source": "nvml 5 ms", "power_w_max": max(pw) if pw else None}
 
 
 def run_reference(args):
@@ -321,7 +345,7 @@ def main():
                          if simt else
                          {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "TLOP3/s",
                          "frac": achieved / peak, "traffic": traffic,
-                         "peak_basis": f"{props.multi_processor_count} SMs x {LOP3_PER_CLK_PER_SM} LOP3/clk x {sm_clock:.0f} MHz (guide unit counts, SM clock)",
+                         "peak_basis": f"{props.multi_processor_count} SMs x {LOP3_PER_CLK_PER_SM} LOP3/clk x {sm_clock:.0f} MHz (guide unit counts, SM clock; microbenchmark scripts/peaks.cu measured 64.00 LOP3/clk/SM = 18.53 TLOP3/s at 1957 MHz, profiles/round1_peaks.json)",
                          "lop3_per_word_per_and": stats["lop3_words"] / max(1.0, W_rank / 32.0),
                          "and_evals_tops": (W_rank / 32.0) / (ms / 1e3) / 1e12}),
             "step_ms": step_ms, "wall_s": wall,

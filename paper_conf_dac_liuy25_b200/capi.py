@@ -327,4 +327,7 @@ class Context:
             self._ctx = None
 
     def __del__(self):
-        self.close()
+        try:
+            self.close()
+        except TypeError:  # interpreter shutdown: module globals already torn down
+            pass

@@ -5,6 +5,7 @@
 
 #include <algorithm>
 #include <cstdint>
+#include <memory>
 #include <string>
 #include <vector>
 
@@ -71,6 +72,7 @@ struct cec_ctx {
     // device copy of the AIG for random simulation (lazy)
     uint32_t *d_f0 = nullptr, *d_f1 = nullptr, *d_level_ids = nullptr;
     std::vector<uint32_t> level_off;
+    std::shared_ptr<DevPool> devpool;  // plan device blocks + pinned staging (device contexts)
     Scratch scratch;  // for serial host work (supports of single pairs, cut validation)
     std::vector<Scratch> pool;  // one per planning thread, kept across calls (allocated once)
 
@@ -118,8 +120,14 @@ struct cec_plan {
     // device
     bool uploaded = false;
     DevPlan d;
+    std::shared_ptr<DevPool> pool;  // owner of the block below
+    void *arena = nullptr;          // one device block holding every DevPlan buffer
+    size_t arena_cap = 0;
     void *ev0 = nullptr, *ev1 = nullptr;
     bool ran = false;
+    uint32_t runs = 0;                     // completed cec_plan_run calls
+    void *graph = nullptr, *graph_stream = nullptr;  // captured run (replayed from the 2nd run on)
+    uint32_t graph_launches = 0;
 };
 
 

@@ -471,6 +471,7 @@ void cec_free(cec_ctx *ctx) {
     dev_free(ctx->d_level_ids);
     if (ctx->comm && g_nccl.destroy) g_nccl.destroy(ctx->comm);
     aux_destroy(ctx->aux);
+    ctx->devpool.reset();  // freed here unless a live plan still holds it
     if (ctx->own_stream) stream_destroy(ctx->own_stream);
     delete ctx;
 }
@@ -876,8 +877,14 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
     }
     // Each launch is a persistent grid pulling items; size items per GROUP so even a one-window
     // group (e.g. a bug-variant structure) splits into enough items to fill every SM.
-    auto add_items = [&](std::vector<uint32_t> ws, bool jit) {
+    auto add_items = [&](std::vector<uint32_t> ws, bool jit, LaunchGroup &g) {
         std::stable_sort(ws.begin(), ws.end(), [&](uint32_t a, uint32_t b) { return cost_of[a] > cost_of[b]; });
+        g.nwin = (uint32_t)ws.size();
+        for (uint32_t w : ws) {
+            g.lop3_words += (win_jit[w] >= 0 ? jit_kernel_lop3(kernels[win_jit[w]]) : P->win_nodes[w]) * words_rank_of[w];
+            g.max_k = std::max(g.max_k, P->dwin[w].k);
+            g.nodes = std::max(g.nodes, P->win_nodes[w]);
+        }
         uint64_t group_slices = 0;
         for (uint32_t w : ws) {
             uint64_t ttw = tt_words_of(P->dwin[w].k), sb, se;
@@ -904,7 +911,7 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         LaunchGroup g{};
         g.jit = kernels[kv.first];
         g.item_off = (uint32_t)P->jitems.size();
-        add_items(kv.second, true);
+        add_items(kv.second, true, g);
         g.nitems = (uint32_t)(P->jitems.size() - g.item_off);
         P->groups.push_back(g);
     }
@@ -912,7 +919,7 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         LaunchGroup g{};
         g.nslots = kv.first;
         g.item_off = (uint32_t)P->items.size();
-        add_items(kv.second, false);
+        add_items(kv.second, false, g);
         g.nitems = (uint32_t)(P->items.size() - g.item_off);
         P->groups.push_back(g);
     }
@@ -928,18 +935,44 @@ cec_status upload(cec_ctx *c, cec_plan *P) {
     if (c->host_only) return CEC_OK;
     DevPlan &d = P->d;
     const size_t ncmp = std::max<size_t>(1, P->cmps.size()), nwin = std::max<size_t>(1, P->dwin.size());
-    CUDA_TRY(c, dev_alloc((void **)&d.wins, sizeof(DevWin) * nwin));
-    CUDA_TRY(c, dev_alloc((void **)&d.prog, sizeof(uint4) * std::max<size_t>(1, P->prog.size())));
-    CUDA_TRY(c, dev_alloc((void **)&d.items, sizeof(Item) * std::max<size_t>(1, P->items.size())));
-    CUDA_TRY(c, dev_alloc((void **)&d.first, sizeof(unsigned long long) * ncmp));
-    CUDA_TRY(c, dev_alloc((void **)&d.bound, sizeof(unsigned long long) * nwin));
-    CUDA_TRY(c, dev_alloc((void **)&d.neq_cnt, sizeof(uint32_t) * nwin));
-    CUDA_TRY(c, dev_alloc((void **)&d.item_ctr, sizeof(uint32_t) * std::max<size_t>(1, P->groups.size())));
-    CUDA_TRY(c, dev_alloc((void **)&d.jitems, sizeof(JItem) * std::max<size_t>(1, P->jitems.size())));
-    CUDA_TRY(c, h2d(d.jitems, P->jitems.data(), sizeof(JItem) * P->jitems.size(), c->stream));
-    CUDA_TRY(c, h2d(d.wins, P->dwin.data(), sizeof(DevWin) * P->dwin.size(), c->stream));
-    CUDA_TRY(c, h2d(d.prog, P->prog.data(), sizeof(uint4) * P->prog.size(), c->stream));
-    CUDA_TRY(c, h2d(d.items, P->items.data(), sizeof(Item) * P->items.size(), c->stream));
+    // one device block: [wins | prog | items | jitems] (uploaded by one H2D from pinned staging)
+    // then [first | bound | neq_cnt | item_ctr] (initialised on the device by the reset kernel)
+    auto al = [](size_t x) { return (x + 255) / 256 * 256; };
+    const size_t b_wins = sizeof(DevWin) * P->dwin.size(), b_prog = sizeof(uint4) * P->prog.size(),
+                 b_items = sizeof(Item) * P->items.size(), b_jitems = sizeof(JItem) * P->jitems.size();
+    size_t off = 0;
+    const size_t o_wins = off; off += al(std::max<size_t>(b_wins, 1));
+    const size_t o_prog = off; off += al(std::max<size_t>(b_prog, 1));
+    const size_t o_items = off; off += al(std::max<size_t>(b_items, 1));
+    const size_t o_jitems = off; off += al(std::max<size_t>(b_jitems, 1));
+    const size_t up_bytes = off;
+    const size_t o_first = off; off += al(sizeof(unsigned long long) * ncmp);
+    const size_t o_bound = off; off += al(sizeof(unsigned long long) * nwin);
+    const size_t o_neq = off; off += al(sizeof(uint32_t) * nwin);
+    const size_t o_ctr = off; off += al(sizeof(uint32_t) * std::max<size_t>(1, P->groups.size()));
+    if (!c->devpool) c->devpool = std::make_shared<DevPool>();
+    P->pool = c->devpool;
+    CUDA_TRY(c, P->pool->get(off, &P->arena, &P->arena_cap));
+    char *base = (char *)P->arena;
+    d.wins = (DevWin *)(base + o_wins);
+    d.prog = (uint4 *)(base + o_prog);
+    d.items = (Item *)(base + o_items);
+    d.jitems = (JItem *)(base + o_jitems);
+    d.first = (unsigned long long *)(base + o_first);
+    d.bound = (unsigned long long *)(base + o_bound);
+    d.neq_cnt = (uint32_t *)(base + o_neq);
+    d.item_ctr = (uint32_t *)(base + o_ctr);
+    {
+        void *hst = nullptr;
+        CUDA_TRY(c, P->pool->staging(up_bytes, &hst));
+        char *h = (char *)hst;
+        if (b_wins) memcpy(h + o_wins, P->dwin.data(), b_wins);
+        if (b_prog) memcpy(h + o_prog, P->prog.data(), b_prog);
+        if (b_items) memcpy(h + o_items, P->items.data(), b_items);
+        if (b_jitems) memcpy(h + o_jitems, P->jitems.data(), b_jitems);
+        CUDA_TRY(c, h2d(base, h, o_jitems + b_jitems, c->stream));
+        CUDA_TRY(c, P->pool->staged(c->stream));
+    }
     if (P->simt.E) {
         SimtPlan &S = P->simt;
         CUDA_TRY(c, dev_alloc((void **)&S.d_simt, sizeof(uint32_t) * (size_t)S.E * S.rows));
@@ -961,16 +994,11 @@ cec_status upload(cec_ctx *c, cec_plan *P) {
 }
 
 void free_dev(cec_plan *P) {
-    DevPlan &d = P->d;
-    dev_free(d.wins);
-    dev_free(d.prog);
-    dev_free(d.items);
-    dev_free(d.first);
-    dev_free(d.bound);
-    dev_free(d.neq_cnt);
-    dev_free(d.item_ctr);
-    dev_free(d.jitems);
-    d = DevPlan{};
+    if (P->pool && P->arena) P->pool->put(P->arena, P->arena_cap);
+    P->arena = nullptr;
+    P->arena_cap = 0;
+    P->pool.reset();
+    P->d = DevPlan{};
     dev_free(P->simt.d_simt);
     dev_free(P->simt.d_inputs);
     dev_free(P->simt.d_nodes);
@@ -982,6 +1010,8 @@ void free_dev(cec_plan *P) {
     event_destroy(P->ev0);
     event_destroy(P->ev1);
     P->ev0 = P->ev1 = nullptr;
+    graph_destroy(P->graph);
+    P->graph = P->graph_stream = nullptr;
 }
 
 bool lex_less(const std::vector<uint32_t> &a, const std::vector<uint32_t> &b) {
@@ -1026,7 +1056,31 @@ cec_status cec_plan_exhaustive(cec_ctx *c, uint32_t n, const uint32_t *la, const
     // a2: structural supports of all pairs, in parallel (independent TFI walks, own scratch each)
     std::vector<std::vector<uint32_t>> supp(n);
     std::vector<uint64_t> cones(n, 0);
-    {
+    // On a device context the supports come from the GPU (supp_gpu.cu: one launch per level over
+    // the whole AIG, lists saturating at k_max + 1); only pairs above k_max (exact k) and the
+    // cost-aware merge (which needs cone sizes) walk cones on the host.
+    std::vector<uint8_t> need_walk(n, 1);
+    bool gpu_supp = !c->host_only && c->opts.merge != CEC_MERGE_COST && n >= 64 && c->N() >= (1u << 16);
+    if (const char *e = getenv("CEC_SUPP_GPU")) gpu_supp = !c->host_only && c->opts.merge != CEC_MERGE_COST && atoi(e) != 0;
+    if (gpu_supp) {
+        cec_status st = cec_ensure_device_aig(c);
+        if (st != CEC_OK) return st;
+        if (!c->devpool) c->devpool = std::make_shared<DevPool>();
+        const uint32_t cap = kmax + 1;
+        std::vector<uint2> roots(n);
+        for (uint32_t p = 0; p < n; ++p) roots[p] = make_uint2(la[p] >> 1, lb[p] >> 1);
+        std::vector<uint32_t> lists, cnt;
+        uint32_t nl = 0;
+        CUDA_TRY(c, gpu_supports(*c->devpool, c->d_f0, c->d_f1, c->d_level_ids, c->level_off, c->I, c->N(), cap, roots,
+                                 lists, cnt, c->stream, &nl));
+        for (uint32_t p = 0; p < n; ++p)
+            if (cnt[p] < cap) {
+                supp[p].assign(lists.begin() + (size_t)p * cap, lists.begin() + (size_t)p * cap + cnt[p]);
+                need_walk[p] = 0;
+            }
+        tm.lap("supports (gpu)");
+    }
+    if (std::find(need_walk.begin(), need_walk.end(), (uint8_t)1) != need_walk.end()) {
         const unsigned hw = std::max(1u, std::min(16u, std::thread::hardware_concurrency()));
         const unsigned nt = (unsigned)std::min<uint64_t>(hw, (n + 63) / 64);
         std::atomic<uint32_t> next{0};
@@ -1040,6 +1094,7 @@ cec_status cec_plan_exhaustive(cec_ctx *c, uint32_t n, const uint32_t *la, const
             // thread walks the same (cache-resident) nodes again
             for (uint32_t p0; (p0 = next.fetch_add(64)) < n;)
             for (uint32_t p = p0; p < std::min(n, p0 + 64); ++p) {
+                if (!need_walk[p]) continue;
                 ep = X.next_epoch();
                 auto &S = supp[p];
                 uint64_t nodes = 0;
@@ -1177,11 +1232,30 @@ cec_status cec_plan_run(cec_ctx *c, cec_plan *P) {
     if (!c || !P) return CEC_E_ARG;
     if (c->host_only) return fail(c, CEC_E_CUDA, "host-only context: no CUDA device (no CPU fallback)");
     if (!P->uploaded) return fail(c, CEC_E_STATE, "plan not uploaded");
-    CUDA_TRY(c, event_record(P->ev0, c->stream));
     uint32_t nl = 0;
-    const char *e = P->simt.E ? launch_simt(P->simt, P->d.first, (uint32_t)P->cmps.size(), c->stream, c->num_sms, &nl)
-                              : launch_run(P->d, P->groups, (uint32_t)P->dwin.size(), (uint32_t)P->cmps.size(),
-                                           c->stream, c->num_sms, &nl, &c->aux);
+    const char *e = nullptr;
+    // a plan that is run again is replayed as a CUDA graph (captured on its second run)
+    const bool use_graph = !P->simt.E && P->runs >= 1 && getenv("CEC_NO_GRAPH") == nullptr &&
+                           getenv("CEC_PROFILE_GROUPS") == nullptr;
+    if (use_graph && P->graph && P->graph_stream != c->stream) {
+        graph_destroy(P->graph);
+        P->graph = nullptr;
+    }
+    if (use_graph && !P->graph) {
+        e = graph_capture_run(P->d, P->groups, (uint32_t)P->dwin.size(), (uint32_t)P->cmps.size(), c->stream,
+                              c->num_sms, &P->graph_launches, &c->aux, &P->graph);
+        P->graph_stream = c->stream;
+        if (e) return fail(c, CEC_E_CUDA, "CUDA: %s (graph capture)", e);
+    }
+    CUDA_TRY(c, event_record(P->ev0, c->stream));
+    if (use_graph) {
+        e = graph_launch(P->graph, c->stream);
+        nl = P->graph_launches;
+    } else {
+        e = P->simt.E ? launch_simt(P->simt, P->d.first, (uint32_t)P->cmps.size(), c->stream, c->num_sms, &nl)
+                      : launch_run(P->d, P->groups, (uint32_t)P->dwin.size(), (uint32_t)P->cmps.size(), c->stream,
+                                   c->num_sms, &nl, &c->aux);
+    }
     if (e) return fail(c, CEC_E_CUDA, "CUDA: %s (kernel launch)", e);
     if (c->comm && !P->cmps.empty()) {  // a10: one NCCL min all-reduce of first_idx
         ncclResult_t r = g_nccl.all_reduce(P->d.first, P->d.first, P->cmps.size(), ncclUint64, ncclMin, c->comm,
@@ -1196,6 +1270,7 @@ cec_status cec_plan_run(cec_ctx *c, cec_plan *P) {
     c->stats.max_k = P->max_k;
     c->stats.max_slots = P->max_slots;
     P->ran = true;
+    ++P->runs;
     return CEC_OK;
 }
 
@@ -1288,12 +1363,17 @@ cec_status cec_sim_exhaustive(cec_ctx *c, uint32_t n, const uint32_t *la, const 
                               uint64_t *cex, uint32_t *k_out) {
     if (!c) return CEC_E_ARG;
     if (c->host_only) return fail(c, CEC_E_CUDA, "host-only context: no CUDA device (no CPU fallback)");
+    PhaseTimer tm;
     cec_plan *P = nullptr;
     cec_status st = cec_plan_exhaustive(c, n, la, lb, &P);
     if (st != CEC_OK) return st;
+    tm.lap("call: plan+upload");
     if (!P->cmps.empty()) st = cec_plan_run(c, P);
+    tm.lap("call: launch");
     if (st == CEC_OK) st = cec_plan_results(c, P, verdict, cex, k_out);
+    tm.lap("call: sync+results");
     cec_plan_free(P);
+    tm.lap("call: free");
     return st;
 }
 

@@ -3,6 +3,8 @@
 #pragma once
 #include <cstdint>
 #include <string>
+#include <mutex>
+#include <utility>
 #include <vector>
 
 namespace cec {
@@ -66,6 +68,8 @@ struct LaunchGroup {       // windows sharing one kernel launch
     uint32_t nslots;       // interpreter: slots per warp in this launch
     uint32_t item_off, nitems;
     JitKernel *jit = nullptr;  // non-null: a JIT structure group (items index DevPlan::jitems)
+    uint64_t lop3_words = 0;   // executed LOP3 x u32 words of the group (CEC_PROFILE_GROUPS report)
+    uint32_t nwin = 0, max_k = 0, nodes = 0;
 };
 
 // Device buffers of one plan.
@@ -79,6 +83,29 @@ struct DevPlan {
     uint32_t *item_ctr = nullptr;         // [ngroups]
     JItem *jitems = nullptr;
 };
+
+// Per-context cache of device blocks and one pinned host staging buffer (sim_interp.cu): a plan takes
+// one device block for all its buffers and returns it on free, so repeated calls do no
+// cudaMalloc/cudaFree (cudaFree synchronises the device). Shared (refcounted) by the context and
+// its live plans, so a plan may outlive the context.
+struct DevPool {
+    std::mutex mu;
+    std::vector<std::pair<void *, size_t>> free_blocks;
+    void *pinned = nullptr;
+    size_t pinned_bytes = 0;
+    void *pinned_ev = nullptr;  // last H2D out of the staging buffer
+    const char *get(size_t bytes, void **p, size_t *cap);
+    void put(void *p, size_t cap);
+    const char *staging(size_t bytes, void **host);  // waits for the previous H2D out of it
+    const char *staged(void *stream);                // records the H2D just issued
+    ~DevPool();
+};
+
+// supp_gpu.cu: a2 supports of all pairs (sorted PI lists saturating at cap = k_max + 1)
+const char *gpu_supports(DevPool &pool, const uint32_t *d_f0, const uint32_t *d_f1, const uint32_t *d_level_ids,
+                         const std::vector<uint32_t> &level_off, uint32_t I, uint32_t N, uint32_t cap,
+                         const std::vector<uint2> &roots, std::vector<uint32_t> &lists_out,
+                         std::vector<uint32_t> &cnt_out, void *stream, uint32_t *launches);
 
 // jit.cpp
 std::string jit_key(const JitProgram &p);
@@ -128,17 +155,22 @@ const char *random_sim(const uint32_t *d_f0, const uint32_t *d_f1, const uint32_
 // sim_interp.cu
 // Side streams: independent launch groups (different window structures) run concurrently, so the
 // tail of one persistent grid overlaps the next and small groups do not serialise.
-constexpr int NAUX = 4;
+constexpr int NAUX_MAX = 32;
 struct AuxStreams {
-    void *s[NAUX] = {};
+    int n = 0;                 // side streams in use (CEC_SIDE_STREAMS, default 4)
+    void *s[NAUX_MAX] = {};
     void *fork = nullptr;
-    void *join[NAUX] = {};
+    void *join[NAUX_MAX] = {};
     bool ok = false;
 };
 const char *aux_create(AuxStreams &a);
 void aux_destroy(AuxStreams &a);
 const char *launch_run(const DevPlan &d, const std::vector<LaunchGroup> &groups, uint32_t nwin, uint32_t ncmp,
                        void *stream, int num_sms, uint32_t *launches, AuxStreams *aux);
+const char *graph_capture_run(const DevPlan &d, const std::vector<LaunchGroup> &groups, uint32_t nwin, uint32_t ncmp,
+                              void *stream, int num_sms, uint32_t *launches, AuxStreams *aux, void **exec_out);
+const char *graph_launch(void *exec, void *stream);
+void graph_destroy(void *exec);
 const char *dev_alloc(void **p, size_t bytes);
 const char *dev_free(void *p);
 const char *h2d(void *dst, const void *src, size_t bytes, void *stream);

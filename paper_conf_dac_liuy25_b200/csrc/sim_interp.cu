@@ -18,6 +18,9 @@
 //    refuted publishes a bound and later slices above it are skipped (bounded early exit, Q9).
 #include <cuda_runtime.h>
 
+#include <cstdio>
+#include <cstdlib>
+
 #include <algorithm>
 #include <cstdint>
 #include <vector>
@@ -163,7 +166,9 @@ uint32_t interp_max_slots_per_warp() {
 const char *aux_create(AuxStreams &a) {
     if (a.ok) return nullptr;
     const char *e;
-    for (int i = 0; i < NAUX; ++i) {
+    a.n = 4;
+    if (const char *v = getenv("CEC_SIDE_STREAMS")) a.n = std::max(1, std::min(NAUX_MAX, atoi(v)));
+    for (int i = 0; i < a.n; ++i) {
         cudaStream_t s;
         if ((e = ck(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking)))) return e;
         a.s[i] = s;
@@ -179,7 +184,7 @@ const char *aux_create(AuxStreams &a) {
 }
 
 void aux_destroy(AuxStreams &a) {
-    for (int i = 0; i < NAUX; ++i) {
+    for (int i = 0; i < a.n; ++i) {
         if (a.s[i]) cudaStreamDestroy((cudaStream_t)a.s[i]);
         if (a.join[i]) cudaEventDestroy((cudaEvent_t)a.join[i]);
     }
@@ -198,18 +203,27 @@ const char *launch_run(const DevPlan &d, const std::vector<LaunchGroup> &groups,
         reset_run<<<(n + 255) / 256, 256, 0, st>>>(d.first, ncmp, d.bound, d.neq_cnt, nwin, d.item_ctr, ng);
         if ((e = ck(cudaGetLastError()))) return e;
     }
-    const bool multi = aux && aux->ok && groups.size() > 1;
+    const bool multi = aux && aux->ok && groups.size() > 1 && getenv("CEC_PROFILE_GROUPS") == nullptr;
     if (multi) {
         if ((e = ck(cudaEventRecord((cudaEvent_t)aux->fork, main_st)))) return e;
-        for (int i = 0; i < NAUX; ++i)
+        for (int i = 0; i < aux->n; ++i)
             if ((e = ck(cudaStreamWaitEvent((cudaStream_t)aux->s[i], (cudaEvent_t)aux->fork, 0)))) return e;
     }
     uint32_t nl = 0;
+    // CEC_PROFILE_GROUPS=1: serial launches, each group timed with events, one line per group on stderr
+    static const bool prof = getenv("CEC_PROFILE_GROUPS") != nullptr;
+    std::vector<cudaEvent_t> pev;
+    if (prof && !multi) {
+        pev.resize(groups.size() + 1);
+        for (auto &x : pev) cudaEventCreate(&x);
+        cudaEventRecord(pev[0], main_st);
+    }
     for (size_t g = 0; g < groups.size(); ++g) {
         const LaunchGroup &G = groups[g];
+        if (!pev.empty() && g > 0) cudaEventRecord(pev[g], main_st);
         if (G.nitems == 0) continue;
         // the biggest group stays on the caller's stream; the others round-robin on side streams
-        st = (multi && g > 0) ? (cudaStream_t)aux->s[(g - 1) % NAUX] : main_st;
+        st = (multi && g > 0) ? (cudaStream_t)aux->s[(g - 1) % aux->n] : main_st;
         stream = st;
         if (G.jit) {
             if ((e = jit_launch(G.jit, d.jitems + G.item_off, G.nitems, d.item_ctr + g, d.first, d.bound, d.neq_cnt,
@@ -245,14 +259,126 @@ const char *launch_run(const DevPlan &d, const std::vector<LaunchGroup> &groups,
         if ((e = ck(cudaGetLastError()))) return e;
         ++nl;
     }
+    if (!pev.empty()) {
+        cudaEventRecord(pev[groups.size()], main_st);
+        cudaEventSynchronize(pev[groups.size()]);
+        for (size_t g = 0; g < groups.size(); ++g) {
+            float ms = 0.f;
+            cudaEventElapsedTime(&ms, pev[g], pev[g + 1]);
+            const LaunchGroup &G = groups[g];
+            fprintf(stderr, "group %zu %s win=%u max_k=%u nodes=%u items=%u lop3_words=%llu ms=%.4f tlop3=%.3f\n", g,
+                    G.jit ? "jit" : "interp", G.nwin, G.max_k, G.nodes, G.nitems, (unsigned long long)G.lop3_words,
+                    ms, ms > 0 ? G.lop3_words / (ms * 1e9) : 0.0);
+        }
+        for (auto &x : pev) cudaEventDestroy(x);
+    }
     if (multi) {  // join: the caller's stream waits for every side stream
-        for (int i = 0; i < NAUX; ++i) {
+        for (int i = 0; i < aux->n; ++i) {
             if ((e = ck(cudaEventRecord((cudaEvent_t)aux->join[i], (cudaStream_t)aux->s[i])))) return e;
             if ((e = ck(cudaStreamWaitEvent(main_st, (cudaEvent_t)aux->join[i], 0)))) return e;
         }
     }
     if (launches) *launches = nl;
     return nullptr;
+}
+
+// CUDA graph of one plan run (the reset kernel plus every window launch with its side-stream
+// fork/join): captured once per (plan, stream) and replayed, so a re-run costs one graph launch
+// instead of one host launch per group (C3: ~1.6k launches per run).
+const char *graph_capture_run(const DevPlan &d, const std::vector<LaunchGroup> &groups, uint32_t nwin, uint32_t ncmp,
+                              void *stream, int num_sms, uint32_t *launches, AuxStreams *aux, void **exec_out) {
+    cudaStream_t st = (cudaStream_t)stream;
+    const char *e;
+    *exec_out = nullptr;
+    if ((e = ck(cudaStreamBeginCapture(st, cudaStreamCaptureModeRelaxed)))) return e;
+    const char *le = launch_run(d, groups, nwin, ncmp, stream, num_sms, launches, aux);
+    cudaGraph_t g = nullptr;
+    const char *ee = ck(cudaStreamEndCapture(st, &g));
+    if (le || ee) {
+        if (g) cudaGraphDestroy(g);
+        return le ? le : ee;
+    }
+    cudaGraphExec_t x = nullptr;
+    e = ck(cudaGraphInstantiate(&x, g, 0));
+    cudaGraphDestroy(g);
+    if (e) return e;
+    *exec_out = x;
+    return nullptr;
+}
+const char *graph_launch(void *exec, void *stream) {
+    return ck(cudaGraphLaunch((cudaGraphExec_t)exec, (cudaStream_t)stream));
+}
+void graph_destroy(void *exec) {
+    if (exec) cudaGraphExecDestroy((cudaGraphExec_t)exec);
+}
+
+const char *DevPool::get(size_t bytes, void **p, size_t *cap) {
+    {
+        std::lock_guard<std::mutex> g(mu);
+        size_t best = free_blocks.size();
+        for (size_t i = 0; i < free_blocks.size(); ++i)
+            if (free_blocks[i].second >= bytes && (best == free_blocks.size() || free_blocks[i].second < free_blocks[best].second))
+                best = i;
+        if (best < free_blocks.size()) {
+            *p = free_blocks[best].first;
+            *cap = free_blocks[best].second;
+            free_blocks.erase(free_blocks.begin() + best);
+            return nullptr;
+        }
+    }
+    const size_t c = (std::max<size_t>(bytes, 1) + (2u << 20) - 1) / (2u << 20) * (2u << 20);
+    const char *e = ck(cudaMalloc(p, c));
+    *cap = e ? 0 : c;
+    return e;
+}
+void DevPool::put(void *p, size_t cap) {
+    if (!p) return;
+    std::lock_guard<std::mutex> g(mu);
+    free_blocks.emplace_back(p, cap);
+    size_t total = 0;
+    for (auto &b : free_blocks) total += b.second;
+    while (total > (1ull << 30) && free_blocks.size() > 1) {  // keep at most ~1 GiB cached
+        auto it = std::max_element(free_blocks.begin(), free_blocks.end(),
+                                   [](const std::pair<void *, size_t> &a, const std::pair<void *, size_t> &b) {
+                                       return a.second < b.second;
+                                   });
+        total -= it->second;
+        cudaFree(it->first);
+        free_blocks.erase(it);
+    }
+}
+const char *DevPool::staging(size_t bytes, void **host) {
+    const char *e;
+    if (pinned_ev && (e = ck(cudaEventSynchronize((cudaEvent_t)pinned_ev)))) return e;
+    if (bytes > pinned_bytes) {
+        if (pinned) cudaFreeHost(pinned);
+        pinned = nullptr;
+        const size_t c = (bytes + (1u << 20) - 1) / (1u << 20) * (1u << 20);
+        if ((e = ck(cudaMallocHost(&pinned, c)))) {
+            pinned_bytes = 0;
+            return e;
+        }
+        pinned_bytes = c;
+    }
+    *host = pinned;
+    return nullptr;
+}
+const char *DevPool::staged(void *stream) {
+    const char *e;
+    if (!pinned_ev) {
+        cudaEvent_t ev;
+        if ((e = ck(cudaEventCreateWithFlags(&ev, cudaEventDisableTiming)))) return e;
+        pinned_ev = ev;
+    }
+    return ck(cudaEventRecord((cudaEvent_t)pinned_ev, (cudaStream_t)stream));
+}
+DevPool::~DevPool() {
+    if (pinned_ev) {
+        cudaEventSynchronize((cudaEvent_t)pinned_ev);
+        cudaEventDestroy((cudaEvent_t)pinned_ev);
+    }
+    if (pinned) cudaFreeHost(pinned);
+    for (auto &b : free_blocks) cudaFree(b.first);
 }
 
 const char *dev_alloc(void **p, size_t bytes) { return ck(cudaMalloc(p, bytes ? bytes : 16)); }

@@ -205,18 +205,25 @@ def test_local_checks_vs_oracle(seed):
     assert list(map(int, got)) == list(map(int, want))
 
 
-def test_plan_rerun_is_deterministic():
-    m = c2_mul12_bug(seed=1, n=10)
-    ctx = gpu_ctx(m.aig)
-    plan = capi.cec_plan_exhaustive(ctx.handle, m.lit_a, m.lit_b)
-    outs = []
-    for _ in range(3):
-        capi.cec_plan_run(ctx.handle, plan)
-        outs.append(capi.cec_plan_results(ctx.handle, plan, m.num_pairs))
-    for o in outs[1:]:
-        for a, b in zip(outs[0], o):
+@pytest.mark.parametrize("engine", ENGINES)
+def test_plan_rerun_is_deterministic(engine):
+    """Runs 2+ of a plan replay a captured CUDA graph (side-stream groups included); every run must
+    reproduce the eager first run, which the other tests pin to the oracle."""
+    for m in (c2_mul12_bug(seed=1, n=10),
+              c5_big(copies=8, n_random=5, n_bugs=3, rand_pis=16, rand_ands=1500, mul_n=8)):
+        ctx = gpu_ctx(m.aig, engine=engine)
+        plan = capi.cec_plan_exhaustive(ctx.handle, m.lit_a, m.lit_b)
+        outs = []
+        for _ in range(4):
+            capi.cec_plan_run(ctx.handle, plan)
+            outs.append(capi.cec_plan_results(ctx.handle, plan, m.num_pairs))
+        for o in outs[1:]:
+            for a, b in zip(outs[0], o):
+                assert np.array_equal(a, b)
+        capi.cec_plan_free(plan)
+        eager = gpu_ctx(m.aig, engine=engine).sim_exhaustive(m.lit_a, m.lit_b)
+        for a, b in zip(eager, outs[-1]):
             assert np.array_equal(a, b)
-    capi.cec_plan_free(plan)
 
 
 def combine_shards(results):
@@ -370,3 +377,21 @@ def test_gpu_cut_generator_matches_cut_oracle(case):
     for i in range(len(P)):
         got = [tuple(int(v) for v in lv[co[t]:co[t + 1]]) for t in range(int(pco[i]), int(pco[i + 1]))]
         assert got == want[i], (i, P[i], got, want[i])
+
+
+@pytest.mark.parametrize("k_max", [8, 16, 32])
+def test_gpu_supports_match_host_walk(k_max, monkeypatch):
+    """a2 on the device (supp_gpu.cu, lists saturating at k_max + 1) gives the same k, verdicts and
+    CEX as the host cone walk, including pairs above k_max (exact k recomputed on the host)."""
+    from workloads import c4_dp
+
+    saturated = False
+    for m in (c4_dp(16), c5_big(copies=6, n_random=4, n_bugs=3, rand_pis=14, rand_ands=700, mul_n=7)):
+        outs = []
+        for flag in ("0", "1"):
+            monkeypatch.setenv("CEC_SUPP_GPU", flag)
+            outs.append(gpu_ctx(m.aig, k_max=k_max, merge=capi.CEC_MERGE_PAPER).sim_exhaustive(m.lit_a, m.lit_b))
+        for a, b in zip(*outs):
+            assert np.array_equal(a, b)
+        saturated |= bool((outs[0][2] > k_max).any())
+    assert saturated  # the saturated-list path (host re-walk) was exercised
