@@ -93,6 +93,7 @@ struct Cmp {
 };
 
 struct cec_plan {
+    ~cec_plan();  // returns the device block (cec_host.cpp)
     bool local = false;
     uint32_t num_pairs = 0;
     std::vector<uint32_t> la, lb;      // the caller's pairs

@@ -17,6 +17,7 @@
 #include <cstdarg>
 #include <cstdlib>
 #include <cstdio>
+#include <cmath>
 #include <cstring>
 #include <map>
 #include <memory>
@@ -1014,6 +1015,7 @@ void free_dev(cec_plan *P) {
     P->graph = P->graph_stream = nullptr;
 }
 
+
 bool lex_less(const std::vector<uint32_t> &a, const std::vector<uint32_t> &b) {
     return std::lexicographical_compare(a.begin(), a.end(), b.begin(), b.end());
 }
@@ -1029,15 +1031,15 @@ double est_cost(uint64_t nodes, size_t k) { return (double)nodes * (double)(k <=
 
 }  // namespace
 
+cec_plan::~cec_plan() { free_dev(this); }
+
 extern "C" {
 
-cec_status cec_plan_exhaustive(cec_ctx *c, uint32_t n, const uint32_t *la, const uint32_t *lb, cec_plan **out) {
-    PhaseTimer tm;
-    if (!c || !out || (n && (!la || !lb))) return fail(c, CEC_E_ARG, "null argument");
-    *out = nullptr;
-    auto t0 = std::chrono::steady_clock::now();
-    std::unique_ptr<cec_plan> P(new (std::nothrow) cec_plan());
-    if (!P) return CEC_E_NOMEM;
+}  // extern "C"
+
+// a2-a5 of a global check: supports, trivial pairs, routing by k, compares, windows and merging.
+static cec_status plan_route(cec_ctx *c, uint32_t n, const uint32_t *la, const uint32_t *lb, cec_plan *P,
+                             std::vector<WinHost> &wins, PhaseTimer &tm) {
     P->num_pairs = n;
     P->la.assign(la, la + n);
     P->lb.assign(lb, lb + n);
@@ -1184,7 +1186,6 @@ cec_status cec_plan_exhaustive(cec_ctx *c, uint32_t n, const uint32_t *la, const
     for (uint32_t i = 0; i < order.size(); ++i) order[i] = i;
     std::stable_sort(order.begin(), order.end(),
                      [&](uint32_t a, uint32_t b) { return lex_less(wins0[a].inputs, wins0[b].inputs); });
-    std::vector<WinHost> wins;
     const uint32_t ks = std::min(c->opts.k_s, kmax);
     for (uint32_t oi : order) {
         WinHost &w = wins0[oi];
@@ -1205,7 +1206,22 @@ cec_status cec_plan_exhaustive(cec_ctx *c, uint32_t n, const uint32_t *la, const
         wins.push_back(std::move(w));
     }
     tm.lap("routing+merging");
-    cec_status st = finish_plan(c, P.get(), wins, nullptr, false);
+    return CEC_OK;
+}
+
+extern "C" {
+
+cec_status cec_plan_exhaustive(cec_ctx *c, uint32_t n, const uint32_t *la, const uint32_t *lb, cec_plan **out) {
+    PhaseTimer tm;
+    if (!c || !out || (n && (!la || !lb))) return fail(c, CEC_E_ARG, "null argument");
+    *out = nullptr;
+    auto t0 = std::chrono::steady_clock::now();
+    std::unique_ptr<cec_plan> P(new (std::nothrow) cec_plan());
+    if (!P) return CEC_E_NOMEM;
+    std::vector<WinHost> wins;
+    cec_status st = plan_route(c, n, la, lb, P.get(), wins, tm);
+    if (st != CEC_OK) return st;
+    st = finish_plan(c, P.get(), wins, nullptr, false);
     if (st != CEC_OK) return st;
     tm.lap("finish_plan");
     auto t1 = std::chrono::steady_clock::now();
@@ -1274,6 +1290,11 @@ cec_status cec_plan_run(cec_ctx *c, cec_plan *P) {
     return CEC_OK;
 }
 
+}  // extern "C"
+static void resolve_results(cec_ctx *c, cec_plan *P, const std::vector<unsigned long long> &first, int32_t *verdict,
+                            uint64_t *cex, uint32_t *k_out);
+extern "C" {
+
 cec_status cec_plan_results(cec_ctx *c, cec_plan *P, int32_t *verdict, uint64_t *cex, uint32_t *k_out) {
     if (!c || !P || (P->num_pairs && !verdict)) return fail(c, CEC_E_ARG, "null argument");
     std::vector<unsigned long long> first(P->cmps.size(), ~0ull);
@@ -1288,6 +1309,15 @@ cec_status cec_plan_results(cec_ctx *c, cec_plan *P, int32_t *verdict, uint64_t 
         CUDA_TRY(c, event_elapsed(&ms, P->ev0, P->ev1));
         c->stats.kernel_ms = ms;
     }
+    resolve_results(c, P, first, verdict, cex, k_out);
+    return CEC_OK;
+}
+
+}  // extern "C"
+
+// a11: per user pair, verdict and own-order CEX (pext of the merged index) from first[cmp].
+static void resolve_results(cec_ctx *c, cec_plan *P, const std::vector<unsigned long long> &first, int32_t *verdict,
+                            uint64_t *cex, uint32_t *k_out) {
     if (!P->local) {
         c->last_verdict.assign(P->num_pairs, CEC_UNDECIDED);
         c->last_cex.assign(P->num_pairs, CEC_NO_CEX);
@@ -1320,8 +1350,9 @@ cec_status cec_plan_results(cec_ctx *c, cec_plan *P, int32_t *verdict, uint64_t 
         }
     }
     if (!P->local) c->have_last = true;
-    return CEC_OK;
 }
+
+extern "C" {
 
 cec_status cec_plan_info(const cec_plan *P, uint32_t *nw, uint64_t *W, uint32_t *mk, uint32_t *ms) {
     if (!P) return CEC_E_ARG;
@@ -1363,18 +1394,134 @@ cec_status cec_sim_exhaustive(cec_ctx *c, uint32_t n, const uint32_t *la, const 
                               uint64_t *cex, uint32_t *k_out) {
     if (!c) return CEC_E_ARG;
     if (c->host_only) return fail(c, CEC_E_CUDA, "host-only context: no CUDA device (no CPU fallback)");
+    if (n && (!la || !lb || !verdict)) return fail(c, CEC_E_ARG, "null argument");
     PhaseTimer tm;
-    cec_plan *P = nullptr;
-    cec_status st = cec_plan_exhaustive(c, n, la, lb, &P);
+    auto t0 = std::chrono::steady_clock::now();
+    std::unique_ptr<cec_plan> P(new (std::nothrow) cec_plan());
+    if (!P) return CEC_E_NOMEM;
+    std::vector<WinHost> wins;
+    cec_status st = plan_route(c, n, la, lb, P.get(), wins, tm);
     if (st != CEC_OK) return st;
-    tm.lap("call: plan+upload");
-    if (!P->cmps.empty()) st = cec_plan_run(c, P);
-    tm.lap("call: launch");
-    if (st == CEC_OK) st = cec_plan_results(c, P, verdict, cex, k_out);
+    // Pipelined execution: the merged windows are cut into K chunks; chunk i is planned (node
+    // orders, programs, work items), uploaded and launched while the GPU still runs chunk i-1, so
+    // the host's per-window planning hides behind the sweep. Each chunk is an independent sub-plan
+    // (own compares, bounds, launch groups); results are gathered per compare at the end.
+    int K = 4;
+    if (const char *e = getenv("CEC_PIPELINE")) K = std::max(1, atoi(e));
+    if (c->opts.engine == CEC_ENGINE_SIMT || wins.size() < (size_t)2 * K) K = 1;
+    std::vector<double> wcost(wins.size());
+    double total = 0;
+    for (size_t w = 0; w < wins.size(); ++w) {
+        const uint32_t k = (uint32_t)std::min<size_t>(wins[w].inputs.size(), 40);
+        wcost[w] = std::ldexp(1.0, (int)k) * (double)(1 + std::max<uint64_t>(wins[w].est_nodes, wins[w].cmps.size()));
+        total += wcost[w];
+    }
+    std::vector<size_t> cut{0};  // contiguous window ranges of about equal cost
+    {
+        double acc = 0;
+        for (size_t w = 0; w < wins.size(); ++w) {
+            acc += wcost[w];
+            if ((int)cut.size() < K && acc >= total * (double)cut.size() / K && w + 1 < wins.size()) cut.push_back(w + 1);
+        }
+        cut.push_back(wins.size());
+    }
+    struct Sub {
+        std::unique_ptr<cec_plan> p;
+        std::vector<uint32_t> gcmp;  // local compare j (before finish_plan's renumbering) -> global
+    };
+    std::vector<Sub> subs;
+    cec_stats agg{};
+    float jit_ms = 0.f;
+    for (size_t ch = 0; ch + 1 < cut.size(); ++ch) {
+        if (cut[ch] == cut[ch + 1]) continue;
+        Sub S;
+        S.p.reset(new (std::nothrow) cec_plan());
+        if (!S.p) return CEC_E_NOMEM;
+        std::vector<WinHost> cw;
+        for (size_t w = cut[ch]; w < cut[ch + 1]; ++w) {
+            WinHost h;
+            h.inputs = wins[w].inputs;
+            h.est_nodes = wins[w].est_nodes;
+            for (uint32_t ci : wins[w].cmps) {
+                h.cmps.push_back((uint32_t)S.gcmp.size());
+                S.gcmp.push_back(ci);
+                S.p->cmps.push_back(P->cmps[ci]);
+            }
+            cw.push_back(std::move(h));
+        }
+        S.p->pair_cmp.resize(S.gcmp.size());
+        for (uint32_t j = 0; j < S.gcmp.size(); ++j) S.p->pair_cmp[j] = (int32_t)j;
+        if ((st = finish_plan(c, S.p.get(), cw, nullptr, false)) != CEC_OK) return st;
+        if ((st = upload(c, S.p.get())) != CEC_OK) {
+            free_dev(S.p.get());
+            return st;
+        }
+        if (!S.p->cmps.empty() && (st = cec_plan_run(c, S.p.get())) != CEC_OK) {
+            free_dev(S.p.get());
+            return st;
+        }
+        agg.num_launches += c->stats.num_launches;
+        agg.node_patterns += S.p->W_rank;
+        agg.node_patterns_all += S.p->W_all;
+        agg.num_windows += (uint32_t)S.p->dwin.size();
+        agg.max_k = std::max(agg.max_k, S.p->max_k);
+        agg.max_slots = std::max(agg.max_slots, S.p->max_slots);
+        agg.jit_kernels += S.p->jit_kernels;
+        agg.jit_windows += S.p->jit_windows;
+        agg.lop3_words += S.p->lop3_words;
+        agg.h2d_bytes += c->stats.h2d_bytes;
+        jit_ms += S.p->jit_ms;
+        subs.push_back(std::move(S));
+    }
+    P->host_ms = std::chrono::duration<float, std::milli>(std::chrono::steady_clock::now() - t0).count();
+    tm.lap("call: plan+launch (pipelined)");
+    // gather: first[] of every chunk into the global compare order, with the chunk's pext masks
+    std::vector<unsigned long long> first(P->cmps.size(), ~0ull);
+    std::vector<std::vector<unsigned long long>> part(subs.size());
+    for (size_t i = 0; i < subs.size(); ++i) {
+        part[i].assign(subs[i].p->cmps.size(), ~0ull);
+        if (!part[i].empty()) {
+            cec_status s2 = CEC_OK;
+            const char *e = d2h(part[i].data(), subs[i].p->d.first, sizeof(unsigned long long) * part[i].size(), c->stream);
+            if (e) s2 = fail(c, CEC_E_CUDA, "CUDA: %s", e);
+            if (s2 != CEC_OK) {
+                for (auto &x : subs) free_dev(x.p.get());
+                return s2;
+            }
+        }
+    }
+    const char *se = stream_sync(c->stream);
+    float kms = 0.f;
+    if (!se && !subs.empty() && subs.front().p->ran && subs.back().p->ran)
+        se = event_elapsed(&kms, subs.front().p->ev0, subs.back().p->ev1);
+    for (size_t i = 0; i < subs.size(); ++i) {
+        const Sub &S = subs[i];
+        for (uint32_t j = 0; j < S.gcmp.size(); ++j) {
+            const int32_t lj = S.p->pair_cmp[j];  // finish_plan's renumbering of local compare j
+            P->cmps[S.gcmp[j]].ownmask = S.p->cmps[lj].ownmask;
+            first[S.gcmp[j]] = part[i][lj];
+        }
+        free_dev(S.p.get());
+    }
+    if (se) return fail(c, CEC_E_CUDA, "CUDA: %s", se);
+    resolve_results(c, P.get(), first, verdict, cex, k_out);
+    const float host_ms = P->host_ms;
+    c->stats.num_launches = agg.num_launches;
+    c->stats.node_patterns = agg.node_patterns;
+    c->stats.node_patterns_all = agg.node_patterns_all;
+    c->stats.num_windows = agg.num_windows;
+    c->stats.max_k = agg.max_k;
+    c->stats.max_slots = agg.max_slots;
+    c->stats.jit_kernels = agg.jit_kernels;
+    c->stats.jit_windows = agg.jit_windows;
+    c->stats.lop3_words = agg.lop3_words;
+    c->stats.h2d_bytes = agg.h2d_bytes;
+    c->stats.d2h_bytes = sizeof(unsigned long long) * first.size();
+    c->stats.jit_ms = jit_ms;
+    c->stats.kernel_ms = kms;
+    c->stats.host_prep_ms = host_ms;
     tm.lap("call: sync+results");
-    cec_plan_free(P);
-    tm.lap("call: free");
-    return st;
+    return CEC_OK;
 }
 
 static cec_status sim_signatures(cec_ctx *c, uint32_t W, uint64_t seed, const uint32_t *pi_words, uint64_t *sig_out,
