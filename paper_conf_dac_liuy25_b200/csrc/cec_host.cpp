@@ -1068,7 +1068,7 @@ static cec_status plan_route(cec_ctx *c, uint32_t n, const uint32_t *la, const u
         cec_status st = cec_ensure_device_aig(c);
         if (st != CEC_OK) return st;
         if (!c->devpool) c->devpool = std::make_shared<DevPool>();
-        const uint32_t cap = kmax + 1;
+        const uint32_t cap = std::min<uint32_t>(kmax, MAX_K_ENUM) + 1;  // k above either is routed away
         std::vector<uint2> roots(n);
         for (uint32_t p = 0; p < n; ++p) roots[p] = make_uint2(la[p] >> 1, lb[p] >> 1);
         std::vector<uint32_t> lists, cnt;
@@ -1406,7 +1406,15 @@ cec_status cec_sim_exhaustive(cec_ctx *c, uint32_t n, const uint32_t *la, const 
     // orders, programs, work items), uploaded and launched while the GPU still runs chunk i-1, so
     // the host's per-window planning hides behind the sweep. Each chunk is an independent sub-plan
     // (own compares, bounds, launch groups); results are gathered per compare at the end.
-    int K = 4;
+    // It pays when the sweep dominates per-window planning (median window k >= 20, e.g. C5); with
+    // many small windows (C3) chunking only fragments the launch groups.
+    int K = 1;
+    if (!wins.empty()) {
+        std::vector<uint32_t> ks(wins.size());
+        for (size_t w = 0; w < wins.size(); ++w) ks[w] = (uint32_t)wins[w].inputs.size();
+        std::nth_element(ks.begin(), ks.begin() + ks.size() / 2, ks.end());
+        if (ks[ks.size() / 2] >= 20) K = 4;
+    }
     if (const char *e = getenv("CEC_PIPELINE")) K = std::max(1, atoi(e));
     if (c->opts.engine == CEC_ENGINE_SIMT || wins.size() < (size_t)2 * K) K = 1;
     std::vector<double> wcost(wins.size());
@@ -1416,12 +1424,13 @@ cec_status cec_sim_exhaustive(cec_ctx *c, uint32_t n, const uint32_t *la, const 
         wcost[w] = std::ldexp(1.0, (int)k) * (double)(1 + std::max<uint64_t>(wins[w].est_nodes, wins[w].cmps.size()));
         total += wcost[w];
     }
-    std::vector<size_t> cut{0};  // contiguous window ranges of about equal cost
-    {
+    std::vector<size_t> cut{0};  // contiguous window ranges of about equal cost; the first chunk is
+    {                            // half-size so the GPU starts early
         double acc = 0;
+        const double unit = total / (K - 0.5);
         for (size_t w = 0; w < wins.size(); ++w) {
             acc += wcost[w];
-            if ((int)cut.size() < K && acc >= total * (double)cut.size() / K && w + 1 < wins.size()) cut.push_back(w + 1);
+            if ((int)cut.size() < K && acc >= unit * ((double)cut.size() - 0.5) && w + 1 < wins.size()) cut.push_back(w + 1);
         }
         cut.push_back(wins.size());
     }

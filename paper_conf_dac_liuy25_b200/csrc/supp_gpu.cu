@@ -1,11 +1,11 @@
 // supp_gpu.cu — a2 structural supports on the device (PAPER.md:23 "support", :81 window inputs).
 //
 // supp(PI) = {PI}, supp(const0) = {}, supp(AND n) = supp(f0) U supp(f1), as sorted PI-id lists
-// saturating at `cap` = k_max + 1 entries (a list of cap entries means "more than k_max": the pair
-// is routed away from exhaustive simulation, and the host recomputes its exact k by a cone walk).
-// One launch per topological level, one thread per node (the level CSR of cec_ensure_device_aig);
-// then one thread per pair merges the two root lists. Lists live in one device block of
-// N x cap u32 (C5: 2M nodes x 33 = 270 MB, written once and read twice per call: ~0.3 ms of HBM).
+// saturating at `cap` = min(k_max, 41) + 1 <= 42 entries (a list of cap entries means "more than
+// k_max": the pair is routed away from exhaustive simulation, and the host recomputes its exact k
+// by a cone walk). One launch per topological level (cec_ensure_device_aig's CSR), one warp per
+// node; then one warp per pair merges the two root lists (C5: 247 levels, 1.8 ms in total). Lists live in one
+// device block of N x cap u32 (C5: 2M nodes x 33 = 270 MB, written once and read twice per call).
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -17,25 +17,6 @@
 namespace cec {
 namespace {
 
-__device__ __forceinline__ uint32_t merge_capped(const uint32_t *__restrict__ a, uint32_t na,
-                                                 const uint32_t *__restrict__ b, uint32_t nb, uint32_t *__restrict__ out,
-                                                 uint32_t cap) {
-    uint32_t i = 0, j = 0, n = 0;
-    while (n < cap && (i < na || j < nb)) {
-        uint32_t v;
-        if (j >= nb || (i < na && a[i] < b[j])) {
-            v = a[i++];
-        } else if (i >= na || b[j] < a[i]) {
-            v = b[j++];
-        } else {
-            v = a[i++];
-            ++j;
-        }
-        out[n++] = v;
-    }
-    return n;
-}
-
 __global__ void supp_init(uint32_t *lists, uint32_t *cnt, uint32_t I, uint32_t cap) {
     const uint32_t id = blockIdx.x * blockDim.x + threadIdx.x;
     if (id > I) return;
@@ -43,26 +24,92 @@ __global__ void supp_init(uint32_t *lists, uint32_t *cnt, uint32_t I, uint32_t c
     lists[(size_t)id * cap] = id;
 }
 
-__global__ void supp_level(const uint32_t *__restrict__ ids, uint32_t n, const uint32_t *__restrict__ f0,
-                           const uint32_t *__restrict__ f1, uint32_t *lists, uint32_t *cnt, uint32_t cap) {
-    const uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
-    if (t >= n) return;
-    const uint32_t id = ids[t], a = f0[id] >> 1, b = f1[id] >> 1;
-    const uint32_t na = cnt[a], nb = cnt[b];
-    cnt[id] = (na >= cap || nb >= cap) ? cap
-                                       : merge_capped(lists + (size_t)a * cap, na, lists + (size_t)b * cap, nb,
-                                                      lists + (size_t)id * cap, cap);
+// One warp per node: both fanin lists are staged in shared memory (one coalesced load each) and
+// every element's output rank comes from a binary search in the other list:
+// rank(x in A) = i + lb(B, x) - #{dup b < x},  rank(y in B, not in A) = lb(A, y) + j - #{dup b < y}
+__device__ __forceinline__ uint32_t lower_bound_s(const uint32_t *s, uint32_t n, uint32_t v) {
+    uint32_t lo = 0, hi = n;
+    while (lo < hi) {
+        const uint32_t mid = (lo + hi) >> 1;
+        if (s[mid] < v) lo = mid + 1;
+        else hi = mid;
+    }
+    return lo;
+}
+__device__ __forceinline__ uint32_t warp_union_smem(const uint32_t *__restrict__ A, uint32_t na,
+                                                    const uint32_t *__restrict__ B, uint32_t nb, uint32_t *__restrict__ out,
+                                                    uint32_t cap, uint32_t lane, uint32_t *sa, uint32_t *sb) {
+    if (lane < na) sa[lane] = A[lane];
+    if (lane + 32 < na) sa[lane + 32] = A[lane + 32];
+    if (lane < nb) sb[lane] = B[lane];
+    if (lane + 32 < nb) sb[lane + 32] = B[lane + 32];
+    __syncwarp();
+    bool d0 = false, d1 = false;
+    uint32_t y0 = 0, y1 = 0, la0 = 0, la1 = 0;
+    if (lane < nb) {
+        y0 = sb[lane];
+        la0 = lower_bound_s(sa, na, y0);
+        d0 = la0 < na && sa[la0] == y0;
+    }
+    if (lane + 32 < nb) {
+        y1 = sb[lane + 32];
+        la1 = lower_bound_s(sa, na, y1);
+        d1 = la1 < na && sa[la1] == y1;
+    }
+    const unsigned long long dm =
+        (unsigned long long)__ballot_sync(0xFFFFFFFFu, d0) | ((unsigned long long)__ballot_sync(0xFFFFFFFFu, d1) << 32);
+    const uint32_t total = na + nb - (uint32_t)__popcll(dm);
+    auto dups_below = [&](uint32_t pos) {  // duplicate b elements at positions < pos
+        return (uint32_t)__popcll(pos >= 64 ? dm : (dm & ((1ull << pos) - 1ull)));
+    };
+    for (uint32_t i = lane; i < na; i += 32) {
+        const uint32_t x = sa[i], lb = lower_bound_s(sb, nb, x);
+        const uint32_t r = i + lb - dups_below(lb);
+        if (r < cap) out[r] = x;
+    }
+    if (lane < nb && !d0) {
+        const uint32_t r = la0 + lane - dups_below(lane);
+        if (r < cap) out[r] = y0;
+    }
+    if (lane + 32 < nb && !d1) {
+        const uint32_t r = la1 + lane + 32 - dups_below(lane + 32);
+        if (r < cap) out[r] = y1;
+    }
+    __syncwarp();
+    return total < cap ? total : cap;
 }
 
+__global__ void supp_level_smem(const uint32_t *__restrict__ ids, uint32_t n, const uint32_t *__restrict__ f0,
+                                const uint32_t *__restrict__ f1, uint32_t *lists, uint32_t *cnt, uint32_t cap) {
+    __shared__ uint32_t sh[8][128];
+    const uint32_t lane = threadIdx.x & 31u, wib = threadIdx.x >> 5;
+    const uint32_t nw = gridDim.x * blockDim.x / 32;
+    for (uint32_t t = (blockIdx.x * blockDim.x + threadIdx.x) / 32; t < n; t += nw) {
+        const uint32_t id = ids[t], a = f0[id] >> 1, b = f1[id] >> 1;
+        const uint32_t na = cnt[a], nb = cnt[b];
+        uint32_t r = cap;
+        if (na < cap && nb < cap)
+            r = warp_union_smem(lists + (size_t)a * cap, na, lists + (size_t)b * cap, nb, lists + (size_t)id * cap, cap,
+                                lane, sh[wib], sh[wib] + 64);
+        if (lane == 0) cnt[id] = r;
+    }
+}
+
+// one warp per pair: union of the two root lists
 __global__ void supp_pairs(const uint2 *__restrict__ roots, uint32_t n, const uint32_t *__restrict__ lists,
                            const uint32_t *__restrict__ cnt, uint32_t cap, uint32_t *out, uint32_t *out_cnt) {
-    const uint32_t p = blockIdx.x * blockDim.x + threadIdx.x;
-    if (p >= n) return;
-    const uint2 r = roots[p];
-    const uint32_t na = cnt[r.x], nb = cnt[r.y];
-    out_cnt[p] = (na >= cap || nb >= cap)
-                     ? cap
-                     : merge_capped(lists + (size_t)r.x * cap, na, lists + (size_t)r.y * cap, nb, out + (size_t)p * cap, cap);
+    __shared__ uint32_t sh[8][128];
+    const uint32_t lane = threadIdx.x & 31u, wib = threadIdx.x >> 5;
+    const uint32_t nw = gridDim.x * blockDim.x / 32;
+    for (uint32_t p = (blockIdx.x * blockDim.x + threadIdx.x) / 32; p < n; p += nw) {
+        const uint2 r = roots[p];
+        const uint32_t na = cnt[r.x], nb = cnt[r.y];
+        uint32_t c = cap;
+        if (na < cap && nb < cap)
+            c = warp_union_smem(lists + (size_t)r.x * cap, na, lists + (size_t)r.y * cap, nb, out + (size_t)p * cap, cap, lane,
+                                sh[wib], sh[wib] + 64);
+        if (lane == 0) out_cnt[p] = c;
+    }
 }
 
 inline const char *ck(cudaError_t e) { return e == cudaSuccess ? nullptr : cudaGetErrorString(e); }
@@ -96,16 +143,18 @@ const char *gpu_supports(DevPool &pool, const uint32_t *d_f0, const uint32_t *d_
         return m;
     };
     if ((e = ck(cudaMemcpyAsync(d_roots, roots.data(), sizeof(uint2) * n, cudaMemcpyHostToDevice, st)))) return fail(e);
+    if (cap > 64) return fail("support cap above 64");
     supp_init<<<(I + 1 + T - 1) / T, T, 0, st>>>(lists, cnt, I, cap);
     ++nl;
-    for (size_t l = 1; l + 1 < level_off.size(); ++l) {
+    auto wgrid = [&](uint32_t m) { return (unsigned)std::min<uint64_t>(148ull * 16, ((uint64_t)m * 32 + T - 1) / T); };
+    for (size_t l = 1; l + 1 < level_off.size(); ++l) {  // one launch per topological level
         const uint32_t b = level_off[l], m = level_off[l + 1] - b;
         if (!m) continue;
-        supp_level<<<(m + T - 1) / T, T, 0, st>>>(d_level_ids + b, m, d_f0, d_f1, lists, cnt, cap);
+        supp_level_smem<<<wgrid(m), T, 0, st>>>(d_level_ids + b, m, d_f0, d_f1, lists, cnt, cap);
         ++nl;
     }
     if (n) {
-        supp_pairs<<<(n + T - 1) / T, T, 0, st>>>(d_roots, n, lists, cnt, cap, out, ocnt);
+        supp_pairs<<<wgrid(n), T, 0, st>>>(d_roots, n, lists, cnt, cap, out, ocnt);
         ++nl;
     }
     if ((e = ck(cudaGetLastError()))) return fail(e);
