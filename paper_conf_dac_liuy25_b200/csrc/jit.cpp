@@ -231,8 +231,8 @@ std::vector<MappedNode> jit_map_area(const JitProgram &p) {
     std::vector<C3> best(R);
     std::vector<bool> req(R, false);
     std::vector<double> est(fanout.begin(), fanout.end());  // fanout estimate used by area flow
-    const size_t CAP = 16;
-    const int ITER = 3;  // area flow, then re-estimate fanouts from the mapping's references
+    static const size_t CAP = getenv("CEC_MAP_CAP") ? (size_t)atoi(getenv("CEC_MAP_CAP")) : 16;
+    static const int ITER = getenv("CEC_MAP_ITER") ? atoi(getenv("CEC_MAP_ITER")) : 3;  // area flow, then re-estimate fanouts from the mapping's references
     for (int iter = 0; iter < ITER; ++iter) {
         for (uint32_t r = 0; r < R; ++r) cuts[r].clear();
         for (uint32_t r = 0; r <= p.k; ++r) {
@@ -295,6 +295,55 @@ std::vector<MappedNode> jit_map_area(const JitProgram &p) {
         }
         for (uint32_t r = 0; r < R; ++r) est[r] = 0.5 * est[r] + 0.5 * std::max(1.0, refs[r]);
     }
+    // exact local area recovery: with the cover's reference counts, each node in topological order
+    // takes the cut whose LUTs NOT already shared with the rest of the cover are fewest (the area
+    // it adds if referenced = LUTs that become live; dereferencing gives it back). Two passes.
+    std::vector<int32_t> nref(R, 0);
+    for (uint32_t r = 0; r < R; ++r)
+        if (root[r]) ++nref[r];
+    for (uint32_t t = n; t-- > 0;) {
+        const uint32_t me = p.k + 1 + t;
+        if (nref[me] > 0)
+            for (int i = 0; i < best[me].m; ++i) ++nref[best[me].l[i]];
+    }
+    std::function<uint32_t(uint32_t)> ref_cut = [&](uint32_t r) -> uint32_t {
+        uint32_t a = 1;
+        for (int i = 0; i < best[r].m; ++i) {
+            const uint32_t l = best[r].l[i];
+            if (l > p.k && nref[l]++ == 0) a += ref_cut(l);
+        }
+        return a;
+    };
+    std::function<uint32_t(uint32_t)> deref_cut = [&](uint32_t r) -> uint32_t {
+        uint32_t a = 1;
+        for (int i = 0; i < best[r].m; ++i) {
+            const uint32_t l = best[r].l[i];
+            if (l > p.k && --nref[l] == 0) a += deref_cut(l);
+        }
+        return a;
+    };
+    static const int EA = getenv("CEC_MAP_EA") ? atoi(getenv("CEC_MAP_EA")) : 2;
+    for (int pass = 0; pass < EA; ++pass)
+        for (uint32_t t = 0; t < n; ++t) {
+            const uint32_t me = p.k + 1 + t;
+            const bool mapped = nref[me] > 0;
+            if (mapped) deref_cut(me);
+            C3 keep = best[me];
+            uint32_t best_a = UINT32_MAX;
+            for (const C3 &c : cuts[me]) {
+                if (c.m == 1 && c.l[0] == me) continue;  // the trivial cut
+                best[me] = c;
+                const uint32_t a = ref_cut(me);
+                deref_cut(me);
+                if (a < best_a) {
+                    best_a = a;
+                    keep = c;
+                }
+            }
+            best[me] = keep;
+            if (mapped) ref_cut(me);
+        }
+    for (uint32_t r = 0; r < R; ++r) req[r] = nref[r] > 0;
     // LUT truth tables: evaluate the cone between the leaves and the node on (0xF0, 0xCC, 0xAA)
     std::vector<MappedNode> out(n);
     std::vector<uint8_t> val(R, 0);
