@@ -67,6 +67,8 @@ def _load():
         L.oracle_cex_vector.argtypes = [P, ctypes.c_uint32, ctypes.c_uint32, ctypes.c_uint64, P]
         L.oracle_eval_lit.restype = ctypes.c_int
         L.oracle_eval_lit.argtypes = [P, ctypes.c_uint32, P]
+        L.oracle_eval_all.restype = None
+        L.oracle_eval_all.argtypes = [P, P, P]
         L.oracle_check_local.restype = ctypes.c_int
         L.oracle_check_local.argtypes = [P, ctypes.c_uint32, P, P, P, P, P]
         _lib = L
@@ -131,6 +133,13 @@ class Oracle:
     def eval_lit(self, lit: int, pis: np.ndarray) -> int:
         p = np.ascontiguousarray(pis, dtype=np.uint8)
         return int(_lib.oracle_eval_lit(self._h, lit, _ptr(p)))
+
+    def eval_all(self, pis: np.ndarray) -> np.ndarray:
+        """Value (0/1) of every node id under one PI assignment (PI id i+1 = pis[i])."""
+        p = np.ascontiguousarray(pis, dtype=np.uint8)
+        out = np.zeros(1 + self.num_pis + self.num_ands, dtype=np.uint8)
+        _lib.oracle_eval_all(self._h, _ptr(p), _ptr(out))
+        return out
 
     def check_local(self, lit_a, lit_b, cut_off, leaves) -> np.ndarray:
         la = np.ascontiguousarray(lit_a, dtype=np.uint32)

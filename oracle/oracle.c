@@ -309,6 +309,15 @@ int oracle_eval_lit(const oaig *g, uint32_t lit, const uint8_t *pis) {
     return r;
 }
 
+/* Value of every node id (const 0 = 0) under one PI assignment; val_out[1 + num_pis + num_ands]. */
+void oracle_eval_all(const oaig *g, const uint8_t *pis, uint8_t *val) {
+    uint32_t N = 1 + g->num_pis + g->num_ands;
+    val[0] = 0;
+    for (uint32_t i = 0; i < g->num_pis; i++) val[1 + i] = pis[i] & 1u;
+    for (uint32_t id = g->num_pis + 1; id < N; id++)
+        val[id] = (uint8_t)((val[g->f0[id] >> 1] ^ (g->f0[id] & 1u)) & (val[g->f1[id] >> 1] ^ (g->f1[id] & 1u)));
+}
+
 /* ------------------------------------------------------------------------------------------ */
 /* Local checks (SURVEY.md §8(c) "Local check of a pair on cut L")                             */
 /* ------------------------------------------------------------------------------------------ */
