@@ -165,6 +165,21 @@ cec_status cec_sim_random(cec_ctx *ctx, uint32_t num_words, uint64_t seed, uint6
 cec_status cec_sim_patterns(cec_ctx *ctx, uint32_t num_words, const uint32_t *pi_words, uint64_t *sig_out,
                             uint8_t *phase_out);
 
+/* Equivalence classes from partial simulation, on the GPU (§II-B "nodes with identical
+ * partial truth tables are put into the same equivalence class"; :61/:183; :187 counter-example
+ * patterns split classes). Every node is simulated on 32*(num_words +
+ * num_pattern_words) patterns: first num_words random words per PI (PI id i, word w: low 32 bits
+ * of splitmix64(seed ^ (i << 32) ^ w), as in cec_sim_random), then the caller's words (PI id i+1
+ * takes pi_words[i*num_pattern_words .. (i+1)*num_pattern_words), e.g. CEXs packed LSB-first).
+ * Nodes whose value vectors are equal or complementary form one class (exactly: rows are compared,
+ * a signature collision never merges classes); representative = minimum id (const 0 and PIs may
+ * represent, only AND nodes are members). Output, ordered by member id: (repr_out[q], member_out[q],
+ * phase_out[q] = 1 if the member is the representative's complement); *num_pairs_out = the total
+ * number of pairs, of which the first min(total, cap) are written to the caller-owned arrays. */
+cec_status cec_sim_classes(cec_ctx *ctx, uint32_t num_words, uint64_t seed, uint32_t num_pattern_words,
+                           const uint32_t *pi_words, uint32_t cap, uint32_t *num_pairs_out, uint32_t *repr_out,
+                           uint32_t *member_out, uint8_t *phase_out);
+
 /* Host cut generator for local checks (Eq. 1, Table I, similarity-guided
  * selection). For candidate pairs q (repr[q] < member[q], node ids; member equivalent to repr up to
  * complement), enumerate priority cuts (<= C per node, <= k_l <= 24 leaves, dominated cuts dropped,
@@ -177,6 +192,22 @@ cec_status cec_sim_patterns(cec_ctx *ctx, uint32_t num_words, const uint32_t *pi
 cec_status cec_common_cuts(cec_ctx *ctx, uint32_t npairs, const uint32_t *repr, const uint32_t *member,
                            uint32_t k_l, uint32_t C, int32_t pass_id, uint32_t max_cuts, uint32_t *pair_cut_off,
                            uint32_t *cut_off, uint32_t *leaves);
+
+/* Miter reduction on the GPU ("reduces the miter by merging the proved equivalent
+ * pairs", :185, :187). Merge q redirects every fanout of AND node member[q]
+ * to the literal repr_lit[q] (a proved equivalence; repr_lit[q] >> 1 < member[q], representative =
+ * lower id; each member listed once); then the AIG is rebuilt with structural hashing: every
+ * AND in increasing id gets image = new(repr) if merged, else AND(new(f0), new(f1)) with
+ * x&0 = 0, x&1 = x, x&x = x, x&!x = 0 and one node per normalised fanin pair (a < b), new ids in
+ * creation order (AIGER-binary order again). Outputs (caller-owned host arrays):
+ * *new_num_ands; new_fanin_lits[2 * new_num_ands] (capacity 2 * num_ands suffices: the result never
+ * grows); image_out[1 + num_pis + num_ands] (NULL allowed) = the new literal of every old node id;
+ * lits[num_lits] (in/out, NULL allowed when num_lits = 0): old literals mapped to new ones (e.g.
+ * the PO pairs). PIs keep their ids. CEC_E_ARG for a bad merge list; CEC_E_CUDA without a device.
+ * The context keeps the old AIG: load the result with cec_load_aig. */
+cec_status cec_reduce(cec_ctx *ctx, uint32_t num_subst, const uint32_t *member, const uint32_t *repr_lit,
+                      uint32_t *new_num_ands, uint32_t *new_fanin_lits, uint32_t *image_out, uint32_t num_lits,
+                      uint32_t *lits);
 
 /* Counter-example of pair `pair_idx` of the most recent cec_sim_exhaustive / cec_plan_results:
  * pi_values_out[i] = value of PI id i+1 (0/1): PI S[j] = bit j of the CEX index, every other PI 0.

@@ -28,7 +28,7 @@ EXPORTS = ["cec_default_opts", "cec_load_aig", "cec_sim_exhaustive", "cec_check_
            "cec_pair_support", "cec_plan_exhaustive", "cec_plan_run", "cec_plan_results", "cec_plan_info",
            "cec_plan_window", "cec_plan_free", "cec_stream", "cec_get_stats", "cec_shard_range", "cec_pext64",
            "cec_free", "cec_last_error", "cec_abi_version", "cec_nccl_unique_id", "cec_sim_random",
-           "cec_common_cuts", "cec_sim_patterns"]
+           "cec_common_cuts", "cec_sim_patterns", "cec_reduce", "cec_sim_classes"]
 
 
 class CecOpts(ctypes.Structure):
@@ -90,6 +90,8 @@ def _load() -> ctypes.CDLL:
         "cec_sim_random": (ctypes.c_int, [P, u32, u64, P, P]),
         "cec_common_cuts": (ctypes.c_int, [P, u32, P, P, u32, u32, i32, u32, P, P, P]),
         "cec_sim_patterns": (ctypes.c_int, [P, u32, P, P, P]),
+        "cec_reduce": (ctypes.c_int, [P, u32, P, P, P, P, P, u32, P]),
+        "cec_sim_classes": (ctypes.c_int, [P, u32, u64, u32, P, u32, P, P, P, P]),
     }
     for name, (res, args) in sig.items():
         fn = getattr(L, name)
@@ -199,6 +201,34 @@ def cec_common_cuts(ctx, repr_ids, member_ids, k_l: int, C: int, pass_id: int, m
     return pco, co[:ncut + 1], lv[:int(co[ncut])]
 
 
+def cec_sim_classes(ctx, num_words: int, seed: int, pi_words: Optional[np.ndarray] = None, cap: Optional[int] = None):
+    """GPU equivalence classes: (repr uint32[P], member uint32[P], phase uint8[P]) ordered by member.
+    pi_words: optional uint32 [num_pis, Wc] caller patterns (PI id i+1 = row i)."""
+    w = None if pi_words is None else np.ascontiguousarray(pi_words, dtype=np.uint32)
+    wc = 0 if w is None else int(w.shape[1])
+    total = ctypes.c_uint32()
+    if cap is None:  # ask for the count first, then fetch
+        _check(lib.cec_sim_classes(ctx, num_words, seed, wc, _p(w), 0, ctypes.byref(total), None, None, None), ctx)
+        cap = int(total.value)
+    r = np.zeros(max(cap, 1), np.uint32)
+    m = np.zeros(max(cap, 1), np.uint32)
+    ph = np.zeros(max(cap, 1), np.uint8)
+    _check(lib.cec_sim_classes(ctx, num_words, seed, wc, _p(w), cap, ctypes.byref(total), _p(r), _p(m), _p(ph)), ctx)
+    n = min(cap, int(total.value))
+    return r[:n], m[:n], ph[:n]
+
+
+def cec_reduce(ctx, num_pis: int, num_ands: int, member_ids, repr_lits, lits=()):
+    """GPU miter reduction: returns (new_fanins uint32 [A', 2], image uint32 [N], mapped lits)."""
+    m, r, lv = _u32(member_ids), _u32(repr_lits), _u32(lits).copy()
+    fan = np.zeros(max(2 * num_ands, 2), np.uint32)
+    img = np.zeros(1 + num_pis + num_ands, np.uint32)
+    na = ctypes.c_uint32()
+    _check(lib.cec_reduce(ctx, m.size, _p(m), _p(r), ctypes.byref(na), _p(fan), _p(img), lv.size,
+                          _p(lv) if lv.size else None), ctx)
+    return fan[:2 * na.value].reshape(-1, 2), img, lv
+
+
 def cec_get_cex(ctx, pair_idx: int, num_pis: int) -> np.ndarray:
     out = np.zeros(max(num_pis, 1), np.uint8)
     _check(lib.cec_get_cex(ctx, pair_idx, _p(out)), ctx)
@@ -296,6 +326,7 @@ class Context:
         uid = opt.pop("nccl_unique_id", None)
         self.opts = cec_default_opts(**opt)
         self.num_pis = num_pis
+        self.num_ands = int(np.asarray(fanins).reshape(-1, 2).shape[0])
         self._ctx = cec_load_aig(num_pis, fanins, pos, self.opts, nccl_unique_id=uid)
 
     @classmethod
@@ -314,6 +345,12 @@ class Context:
 
     def get_cex(self, pair_idx: int) -> np.ndarray:
         return cec_get_cex(self._ctx, pair_idx, self.num_pis)
+
+    def sim_classes(self, num_words: int, seed: int, pi_words=None, cap=None):
+        return cec_sim_classes(self._ctx, num_words, seed, pi_words, cap)
+
+    def reduce(self, member_ids, repr_lits, lits=()):
+        return cec_reduce(self._ctx, self.num_pis, self.num_ands, member_ids, repr_lits, lits)
 
     def pair_k(self, lit_a: int, lit_b: int) -> int:
         return cec_pair_k(self._ctx, lit_a, lit_b)

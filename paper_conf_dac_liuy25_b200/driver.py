@@ -1,17 +1,17 @@
 """Host driver above the C ABI: the simulation-based CEC flow of PAPER.md §III-D (Fig. 5, :179-187).
 
   P phase  PO pairs with support <= k_P (all) or <= k_p (subset) -> cec_sim_exhaustive
-  ECs partial random simulation on the GPU (cec_sim_random) -> classes,
-            representative = minimum id, pairs (repr, member)
+  ECs partial simulation of random + CEX patterns and exact classes on the
+            GPU (cec_sim_classes) -> pairs (repr = minimum id, member, phase)
   G phase  candidate pairs with support <= k_g -> cec_sim_exhaustive
   L phases  (§III-C) 3 passes of cut enumeration (Eq. 1, Table I orders) and local
             checks (cec_check_local_cuts); reduce the miter after each phase; repeat until no progress
   reduction proved pairs are merged (member -> representative) and the miter is
-            rebuilt with structural hashing
+            rebuilt with structural hashing on the GPU (cec_reduce)
 
-Every simulation runs in libcec.so's CUDA kernels. The host part here is graph bookkeeping: cut
-enumeration (a host-minimal stand-in for the GPU cut generator), class
-formation from GPU signatures, and miter rebuilding. Undecided pairs remain undecided (the paper
+Every simulation, the class formation and the miter rebuild run in libcec.so's CUDA kernels; cuts
+come from the native cut generator (cec_common_cuts, GPU for large cones). The host part here is
+the phase policy and its bookkeeping. Undecided pairs remain undecided (the paper
 then hands the reduced miter to ABC, which is out of scope).
 """
 from __future__ import annotations
@@ -23,7 +23,7 @@ from typing import Dict, List, Optional, Tuple
 import numpy as np
 
 from . import capi
-from workloads.aig import Aig, Builder  # structural builder (strash) used for miter reduction
+from workloads.aig import Aig  # plain container (num_pis, fanins, pos); no graph building here
 
 
 @dataclasses.dataclass
@@ -69,27 +69,20 @@ class Miter:
         self.lit_a = np.asarray(lit_a, dtype=np.uint32).copy()
         self.lit_b = np.asarray(lit_b, dtype=np.uint32).copy()
 
-    def reduce(self, subst: Dict[int, int]) -> "Miter":
+    def reduce(self, subst: Dict[int, int], device: int = 0) -> Tuple["Miter", np.ndarray]:
         """Merge proved pairs: node id -> literal of its (lower-id) representative,
-        then rebuild with structural hashing so merged fanouts collapse."""
-        I, A = self.aig.num_pis, self.aig.num_ands
-        fan = self.aig.fanins.astype(np.int64)
-        new = np.zeros(1 + I + A, dtype=np.int64)
-        new[1:1 + I] = 2 * np.arange(1, I + 1)
-        bd = Builder(I, strash=True)
-
-        def m(lit):
-            return int(new[lit >> 1]) ^ (lit & 1)
-
-        for j in range(A):
-            nid = 1 + I + j
-            if nid in subst:
-                new[nid] = m(subst[nid])
-            else:
-                new[nid] = bd.AND(m(int(fan[j, 0])), m(int(fan[j, 1])))
-        la = np.array([m(int(x)) for x in self.lit_a], dtype=np.uint32)
-        lb = np.array([m(int(x)) for x in self.lit_b], dtype=np.uint32)
-        return Miter(bd.finish(list(la) + list(lb)), la, lb), new
+        rebuilt with structural hashing so merged fanouts collapse — on the GPU (cec_reduce).
+        Returns the reduced miter and the image (new literal) of every old node id."""
+        ctx = capi.Context.from_aig(self.aig, device=device)
+        try:
+            mem = np.fromiter(subst.keys(), dtype=np.uint32, count=len(subst))
+            rep = np.fromiter(subst.values(), dtype=np.uint32, count=len(subst))
+            fan, image, lits = ctx.reduce(mem, rep, np.concatenate([self.lit_a, self.lit_b]))
+        finally:
+            ctx.close()
+        P = self.lit_a.size
+        aig = Aig(self.aig.num_pis, np.ascontiguousarray(fan, dtype=np.uint32), lits.astype(np.uint32))
+        return Miter(aig, lits[:P], lits[P:]), image
 
 
 def _ctx(aig: Aig, p: CecParams, k_max: int, k_s: Optional[int] = None) -> capi.Context:
@@ -195,26 +188,6 @@ def pack_patterns(patterns: List[np.ndarray], num_pis: int) -> np.ndarray:
     return words
 
 
-def _classes(sig: np.ndarray, phase: np.ndarray, num_pis: int) -> List[Tuple[int, int, int]]:
-    """(repr, member, phase) candidate pairs from equal signatures: repr = min id."""
-    order = np.lexsort((np.arange(sig.size), sig))
-    pairs = []
-    i = 0
-    while i < order.size:
-        j = i
-        while j + 1 < order.size and sig[order[j + 1]] == sig[order[i]]:
-            j += 1
-        if j > i:
-            members = order[i:j + 1]
-            r = int(members[0])
-            for mbr in members[1:]:
-                mbr = int(mbr)
-                if mbr > num_pis:  # members are AND nodes; PIs can only be representatives
-                    pairs.append((r, mbr, int(phase[r] ^ phase[mbr])))
-        i = j + 1
-    return pairs
-
-
 def check_miter(aig: Aig, lit_a, lit_b, params: Optional[CecParams] = None) -> CecResult:
     p = params or CecParams()
     cur = Miter(aig, lit_a, lit_b)
@@ -256,12 +229,14 @@ def check_miter(aig: Aig, lit_a, lit_b, params: Optional[CecParams] = None) -> C
             if v[i] == capi.CEC_EQUIVALENT:
                 a, b = int(cur.lit_a[q]), int(cur.lit_b[q])
                 hi, lo = (a, b) if (a >> 1) > (b >> 1) else (b, a)
-                if (hi >> 1) > aig.num_pis:
+                # an identical node pair (a >> 1 == b >> 1) needs no merge (and merging a node
+                # into itself is not a reduction)
+                if (hi >> 1) > aig.num_pis and (hi >> 1) != (lo >> 1):
                     subst[hi >> 1] = lo ^ (hi & 1)
         ctx.close()
     log.append({"phase": "P", "threshold": thr, "simulated": int(sel.size), "s": time.perf_counter() - t})
     if subst:
-        cur, _ = cur.reduce(subst)
+        cur, _ = cur.reduce(subst, p.device)
 
     # ---- G and L phases -----------------------------------------------------------------------
     tried_global = set()
@@ -273,15 +248,11 @@ def check_miter(aig: Aig, lit_a, lit_b, params: Optional[CecParams] = None) -> C
         t = time.perf_counter()
         ctx = _ctx(cur.aig, p, p.k_g)
         lctx = _ctx(cur.aig, p, max(p.k_l, 1))  # local checks: up to k_l leaves
-        N = cur.aig.num_nodes
-        sig, ph = capi.cec_sim_random(ctx.handle, N, p.sim_words, p.seed + phase_no)
-        if cex_patterns:
-            # CEX patterns split the classes of disproved pairs: combine
-            # the random-pattern and CEX-pattern signatures; the relative phase must agree in both
-            sig_c, ph_c = capi.cec_sim_patterns(ctx.handle, N, pack_patterns(cex_patterns, cur.aig.num_pis))
-            sig = np.array([hash((int(a), int(b), int(x) ^ int(y))) & ((1 << 63) - 1)
-                            for a, b, x, y in zip(sig, sig_c, ph, ph_c)], dtype=np.uint64)
-        cand = [(r, m_, f) for r, m_, f in _classes(sig, ph, cur.aig.num_pis)]
+        # equivalence classes on the GPU: random patterns plus the CEX patterns
+        # of disproved pairs, which split their classes
+        words = pack_patterns(cex_patterns, cur.aig.num_pis) if cex_patterns else None
+        cr, cm, cf = ctx.sim_classes(p.sim_words, p.seed + phase_no, words)
+        cand = [(int(r), int(m_), int(f)) for r, m_, f in zip(cr, cm, cf)]
         versions.append(cur.aig)
         # G phase once per miter version: pairs with support <= k_g
         gl = [(r, m_, f) for r, m_, f in cand if (r, m_, f) not in tried_global]
@@ -360,7 +331,7 @@ def check_miter(aig: Aig, lit_a, lit_b, params: Optional[CecParams] = None) -> C
                     "proved_local": proved_l, "ands": cur.aig.num_ands, "s": time.perf_counter() - t})
         if not subst:
             break  # no progress: undecided remainder
-        cur, _ = cur.reduce(subst)
+        cur, _ = cur.reduce(subst, p.device)
     st = po_status(cur)
     po_v = np.where(st == capi.CEC_EQUIVALENT, capi.CEC_EQUIVALENT, po_v)
     cex_vec, cex_pair = None, -1

@@ -2,6 +2,7 @@
 class formation from signatures, and miter reduction preserving PO functions (checked with the
 oracle's evaluator on random assignments)."""
 import numpy as np
+import pytest
 
 import oracle
 from paper_conf_dac_liuy25_b200 import driver
@@ -36,14 +37,9 @@ def test_table1_orders():
     assert sorted(driver._bits(large_level[0])) == [4, n2 >> 1]     # highest-level leaves
 
 
-def test_classes_from_signatures():
-    sig = np.array([7, 5, 9, 5, 9, 9], dtype=np.uint64)
-    ph = np.array([0, 0, 1, 1, 0, 1], dtype=np.uint8)
-    pairs = driver._classes(sig, ph, num_pis=1)
-    assert sorted(pairs) == [(1, 3, 1), (2, 4, 1), (2, 5, 0)]
-
-
+@pytest.mark.gpu
 def test_miter_reduction_preserves_functions():
+    """The driver's reduction (GPU cec_reduce) keeps every PO function (oracle evaluator)."""
     m = circuits.random_miter(10, 200, 8, seed=3, window=24)
     # merge every B-side PO driver into its A-side partner (they are equivalent by construction)
     cur = driver.Miter(m.aig, m.lit_a, m.lit_b)
@@ -51,7 +47,7 @@ def test_miter_reduction_preserves_functions():
     for a, b in zip(m.lit_a, m.lit_b):
         a, b = int(a), int(b)
         hi, lo = (a, b) if (a >> 1) > (b >> 1) else (b, a)
-        if (hi >> 1) > m.aig.num_pis and (hi >> 1) not in subst:
+        if (hi >> 1) > m.aig.num_pis and (hi >> 1) != (lo >> 1) and (hi >> 1) not in subst:
             subst[hi >> 1] = lo ^ (hi & 1)
     red, _ = cur.reduce(subst)
     assert all(int(x) == int(y) for x, y in zip(red.lit_a, red.lit_b))
