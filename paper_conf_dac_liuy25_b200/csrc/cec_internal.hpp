@@ -149,14 +149,16 @@ const char *launch_simt(const SimtPlan &S, unsigned long long *first, uint32_t n
 // reduce_gpu.cu: miter reduction (merge + strash rebuild) over a host topological batch schedule
 const char *gpu_reduce(const uint32_t *d_f0, const uint32_t *d_f1, uint32_t I, uint32_t N, const std::vector<uint32_t> &sub,
                        const std::vector<uint32_t> &batch_ids, const std::vector<uint32_t> &batch_off, void *stream,
-                       int num_sms, std::vector<uint32_t> &new_fanins, std::vector<uint32_t> &image, uint32_t *launches);
+                       int num_sms, DevPool *pool, std::vector<uint32_t> &new_fanins, std::vector<uint32_t> &image,
+                       uint32_t *launches, float *kernel_ms);
 
 // classes_gpu.cu: partial simulation -> exact equivalence classes -> (repr, member, phase) pairs
 const char *gpu_classes(const uint32_t *d_f0, const uint32_t *d_f1, const uint32_t *d_level_ids,
                         const std::vector<uint32_t> &level_off, uint32_t I, uint32_t N, uint32_t Wr, uint64_t seed,
                         uint32_t Wc, const uint32_t *h_words, uint32_t cap, void *stream, int num_sms,
-                        uint32_t *total_out, std::vector<uint32_t> &repr, std::vector<uint32_t> &member,
-                        std::vector<uint8_t> &phase, uint32_t *launches);
+                        DevPool *pool, uint32_t *total_out, std::vector<uint32_t> &repr,
+                        std::vector<uint32_t> &member, std::vector<uint8_t> &phase, uint32_t *launches,
+                        float *kernel_ms);
 
 // sim_random.cu
 const char *random_sim(const uint32_t *d_f0, const uint32_t *d_f1, const uint32_t *d_level_ids,

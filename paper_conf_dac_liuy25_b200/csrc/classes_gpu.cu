@@ -27,6 +27,7 @@
 #include <vector>
 
 #include "cec_internal.hpp"
+#include "dev_util.cuh"
 
 namespace cec {
 namespace {
@@ -106,8 +107,9 @@ inline const char *ck(cudaError_t e) { return e == cudaSuccess ? nullptr : cudaG
 const char *gpu_classes(const uint32_t *d_f0, const uint32_t *d_f1, const uint32_t *d_level_ids,
                         const std::vector<uint32_t> &level_off, uint32_t I, uint32_t N, uint32_t Wr, uint64_t seed,
                         uint32_t Wc, const uint32_t *h_words, uint32_t cap, void *stream, int num_sms,
-                        uint32_t *total_out, std::vector<uint32_t> &repr, std::vector<uint32_t> &member,
-                        std::vector<uint8_t> &phase, uint32_t *launches) {
+                        DevPool *pool, uint32_t *total_out, std::vector<uint32_t> &repr,
+                        std::vector<uint32_t> &member, std::vector<uint8_t> &phase, uint32_t *launches,
+                        float *kernel_ms) {
     cudaStream_t st = (cudaStream_t)stream;
     const uint32_t W = Wr + Wc;
     size_t sort_bytes = 0, scan_bytes = 0, mscan_bytes = 0;
@@ -129,13 +131,12 @@ const char *gpu_classes(const uint32_t *d_f0, const uint32_t *d_f1, const uint32
                  o_ids = take(4ull * N), o_ids2 = take(4ull * N), o_seg = take(4ull * N), o_flag = take(4ull * N),
                  o_pos = take(4ull * N), o_rep = take(4ull * N), o_rph = take(N), o_cw = take(4ull * I * Wc + 4),
                  o_or = take(4ull * ocap), o_om = take(4ull * ocap), o_op = take(ocap), o_tmp = take(tmp_bytes);
-    char *blk = nullptr;
     const char *e;
-    if ((e = ck(cudaMalloc((void **)&blk, off)))) return e;
-    struct Free {
-        char *p;
-        ~Free() { cudaFree(p); }
-    } guard{blk};
+    DevBlock B{pool, st};
+    if ((e = B.alloc(off))) return e;
+    char *blk = (char *)B.p;
+    EventPair ev;
+    if ((e = ev.create())) return e;
     uint32_t *tt = (uint32_t *)(blk + o_tt), *ids = (uint32_t *)(blk + o_ids), *ids2 = (uint32_t *)(blk + o_ids2);
     unsigned long long *sig = (unsigned long long *)(blk + o_sig), *sig2 = (unsigned long long *)(blk + o_sig2);
     uint8_t *ph = (uint8_t *)(blk + o_ph), *rph = (uint8_t *)(blk + o_rph), *op = (uint8_t *)(blk + o_op);
@@ -148,6 +149,7 @@ const char *gpu_classes(const uint32_t *d_f0, const uint32_t *d_f1, const uint32
     auto grid = [&](uint64_t work) { return (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(gcap, (work + T - 1) / T)); };
     uint32_t nl = 0;
     if (Wc && (e = ck(cudaMemcpyAsync(cw, h_words, 4ull * I * Wc, cudaMemcpyHostToDevice, st)))) return e;
+    if ((e = ck(cudaEventRecord(ev.a, st)))) return e;
     cl_pis<<<grid((uint64_t)(I + 1) * W), T, 0, st>>>(tt, I, W, Wr, seed, cw, Wc);
     ++nl;
     uint32_t nsim = 0;
@@ -167,6 +169,7 @@ const char *gpu_classes(const uint32_t *d_f0, const uint32_t *d_f1, const uint32
     cl_scatter<<<grid(N), T, 0, st>>>(flag, pos, rep, rph, N, cap, orr, om, op);
     nl += 6;
     if ((e = ck(cudaGetLastError()))) return e;
+    if ((e = ck(cudaEventRecord(ev.b, st)))) return e;
     uint32_t tail[2] = {0, 0};
     if ((e = ck(cudaMemcpyAsync(&tail[0], pos + (N - 1), 4, cudaMemcpyDeviceToHost, st)))) return e;
     if ((e = ck(cudaMemcpyAsync(&tail[1], flag + (N - 1), 4, cudaMemcpyDeviceToHost, st)))) return e;
@@ -183,6 +186,7 @@ const char *gpu_classes(const uint32_t *d_f0, const uint32_t *d_f1, const uint32
     }
     *total_out = total;
     if (launches) *launches = nl;
+    if (kernel_ms) cudaEventElapsedTime(kernel_ms, ev.a, ev.b);
     return nullptr;
 }
 

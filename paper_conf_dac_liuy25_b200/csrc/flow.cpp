@@ -5,7 +5,9 @@
 //                   builds the topological batch schedule on the host (O(N): batch(member) =
 //                   batch(repr) + 1, batch(AND) = 1 + max over fanins) and runs reduce_gpu.cu on
 //                   the context's device copy of the AIG.
+#include <chrono>
 #include <cstring>
+#include <memory>
 #include <string>
 #include <vector>
 
@@ -19,6 +21,7 @@ extern "C" cec_status cec_reduce(cec_ctx *c, uint32_t num_subst, const uint32_t 
         c->err = "null argument";
         return CEC_E_ARG;
     }
+    const auto t0 = std::chrono::steady_clock::now();
     const uint32_t N = c->N();
     constexpr uint32_t NONE = 0xFFFFFFFFu;
     std::vector<uint32_t> sub(N, NONE);
@@ -60,7 +63,11 @@ extern "C" cec_status cec_reduce(cec_ctx *c, uint32_t num_subst, const uint32_t 
     if (st != CEC_OK) return st;
     std::vector<uint32_t> fan, image;
     uint32_t nl = 0;
-    if (const char *e = gpu_reduce(c->d_f0, c->d_f1, c->I, N, sub, ids, boff, c->stream, c->num_sms, fan, image, &nl)) {
+    if (!c->devpool) c->devpool = std::make_shared<DevPool>();
+    float kms = 0.f;
+    const float host_ms = std::chrono::duration<float, std::milli>(std::chrono::steady_clock::now() - t0).count();
+    if (const char *e = gpu_reduce(c->d_f0, c->d_f1, c->I, N, sub, ids, boff, c->stream, c->num_sms, c->devpool.get(),
+                                   fan, image, &nl, &kms)) {
         c->err = std::string("CUDA: ") + e + " (miter reduction)";
         return CEC_E_CUDA;
     }
@@ -69,6 +76,8 @@ extern "C" cec_status cec_reduce(cec_ctx *c, uint32_t num_subst, const uint32_t 
     if (image_out) std::memcpy(image_out, image.data(), 4 * (size_t)N);
     for (uint32_t i = 0; i < num_lits; ++i) lits[i] = image[lits[i] >> 1] ^ (lits[i] & 1u);
     c->stats.num_launches = nl;
+    c->stats.kernel_ms = kms;
+    c->stats.host_prep_ms = host_ms;
     return CEC_OK;
 }
 
@@ -90,8 +99,11 @@ extern "C" cec_status cec_sim_classes(cec_ctx *c, uint32_t num_words, uint64_t s
     std::vector<uint32_t> r, m;
     std::vector<uint8_t> ph;
     uint32_t total = 0, nl = 0;
+    float kms = 0.f;
+    if (!c->devpool) c->devpool = std::make_shared<DevPool>();
     if (const char *e = gpu_classes(c->d_f0, c->d_f1, c->d_level_ids, c->level_off, c->I, c->N(), num_words, seed,
-                                    num_pattern_words, pi_words, cap, c->stream, c->num_sms, &total, r, m, ph, &nl)) {
+                                    num_pattern_words, pi_words, cap, c->stream, c->num_sms, c->devpool.get(), &total,
+                                    r, m, ph, &nl, &kms)) {
         c->err = std::string("CUDA: ") + e + " (equivalence classes)";
         return CEC_E_CUDA;
     }
@@ -102,5 +114,6 @@ extern "C" cec_status cec_sim_classes(cec_ctx *c, uint32_t num_words, uint64_t s
         std::memcpy(phase_out, ph.data(), ph.size());
     }
     c->stats.num_launches = nl;
+    c->stats.kernel_ms = kms;
     return CEC_OK;
 }

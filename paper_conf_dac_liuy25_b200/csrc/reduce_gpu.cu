@@ -27,6 +27,7 @@
 #include <vector>
 
 #include "cec_internal.hpp"
+#include "dev_util.cuh"
 
 namespace cec {
 namespace {
@@ -134,7 +135,8 @@ inline const char *ck(cudaError_t e) { return e == cudaSuccess ? nullptr : cudaG
 
 const char *gpu_reduce(const uint32_t *d_f0, const uint32_t *d_f1, uint32_t I, uint32_t N, const std::vector<uint32_t> &sub,
                        const std::vector<uint32_t> &batch_ids, const std::vector<uint32_t> &batch_off, void *stream,
-                       int num_sms, std::vector<uint32_t> &new_fanins, std::vector<uint32_t> &image, uint32_t *launches) {
+                       int num_sms, DevPool *pool, std::vector<uint32_t> &new_fanins, std::vector<uint32_t> &image,
+                       uint32_t *launches, float *kernel_ms) {
     cudaStream_t st = (cudaStream_t)stream;
     const uint32_t A = N - 1 - I;
     uint32_t cap = 1024;
@@ -144,13 +146,12 @@ const char *gpu_reduce(const uint32_t *d_f0, const uint32_t *d_f1, uint32_t I, u
     cub::DeviceScan::ExclusiveSum(nullptr, scan_bytes, (uint32_t *)nullptr, (uint32_t *)nullptr, (int)N, st);
     const size_t n32 = 6 * (size_t)N + cap + 1 + 2 * (size_t)A + 4;
     const size_t bytes = 8 * (size_t)cap + 4 * n32 + scan_bytes + 256;
-    char *blk = nullptr;
     const char *e;
-    if ((e = ck(cudaMalloc((void **)&blk, bytes)))) return e;
-    struct Free {
-        char *p;
-        ~Free() { cudaFree(p); }
-    } guard{blk};
+    DevBlock B{pool, st};
+    if ((e = B.alloc(bytes))) return e;
+    char *blk = (char *)B.p;
+    EventPair ev;
+    if ((e = ev.create())) return e;
     unsigned long long *keys = (unsigned long long *)blk;
     uint32_t *p = (uint32_t *)(blk + 8 * (size_t)cap);
     uint32_t *d_sub = p, *d_ids = p + N, *lab = p + 2 * (size_t)N, *surv = p + 3 * (size_t)N, *rank = p + 4 * (size_t)N;
@@ -166,6 +167,7 @@ const char *gpu_reduce(const uint32_t *d_f0, const uint32_t *d_f1, uint32_t I, u
     const int T = 256;
     const unsigned gcap = (unsigned)std::max(1, num_sms * 8);
     auto grid = [&](uint64_t work) { return (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(gcap, (work + T - 1) / T)); };
+    if ((e = ck(cudaEventRecord(ev.a, st)))) return e;
     rd_init<<<grid(std::max<uint64_t>(cap, I + 1)), T, 0, st>>>(keys, minid, cap, lab, I);
     ++nl;
     for (size_t b = 0; b + 1 < batch_off.size(); ++b) {
@@ -184,6 +186,7 @@ const char *gpu_reduce(const uint32_t *d_f0, const uint32_t *d_f1, uint32_t I, u
     rd_image<<<grid(N), T, 0, st>>>(lab, N, I, minid, rank, img);
     nl += 2;
     if ((e = ck(cudaGetLastError()))) return e;
+    if ((e = ck(cudaEventRecord(ev.b, st)))) return e;
     uint32_t tail[2] = {0, 0}, ovf = 0;  // survivors = rank[N-1] + surv[N-1]
     if ((e = ck(cudaMemcpyAsync(&tail[0], rank + (N - 1), 4, cudaMemcpyDeviceToHost, st)))) return e;
     if ((e = ck(cudaMemcpyAsync(&tail[1], surv + (N - 1), 4, cudaMemcpyDeviceToHost, st)))) return e;
@@ -199,6 +202,7 @@ const char *gpu_reduce(const uint32_t *d_f0, const uint32_t *d_f1, uint32_t I, u
         return e;
     if ((e = ck(cudaStreamSynchronize(st)))) return e;
     if (launches) *launches = nl;
+    if (kernel_ms) cudaEventElapsedTime(kernel_ms, ev.a, ev.b);
     return nullptr;
 }
 

@@ -3,9 +3,10 @@
   NEXT-2  cec_sim_classes : partial simulation (random words) + exact equivalence classes + pairs
   NEXT-3  cec_reduce      : miter reduction (merge + strash rebuild)
 
-Each GPU number is the median wall time of the blocking C-ABI call (its small H2D of the merge list
-/ D2H of the results included) over --reps calls after one warm-up, on the configuration's full
-AIG. `roofline` is the HBM bound of the algorithmic bytes (classes: every node row of W words is
+Each row reports the median wall time of the blocking C-ABI call (host schedule, H2D of the merge
+list / D2H of the results included) and the median device time of its kernels (CUDA events on the
+launch stream, stats.kernel_ms) over --reps calls after one warm-up, on the configuration's full
+AIG; the roofline fraction uses the device time. `roofline` is the HBM bound of the algorithmic bytes (classes: every node row of W words is
 written once and its two fanin rows read once, then read again for the signature: 16 B per
 node-word; reduce: per AND 8 B fanins + 4 B merge entry + 2 x 4 B fanin images + 4 B image + a
 16 B table probe ~= 40 B) against MEASURED_PEAKS' HBM copy bandwidth. The oracle
@@ -42,14 +43,16 @@ def hbm_peak():
     return 6453.7, "SURVEY.md §8(d) copy bandwidth"
 
 
-def timed(fn, reps):
+def timed(fn, ctx, reps):
+    """(median call wall time, median device time of the call's kernels from stats.kernel_ms)."""
     fn()
-    ts = []
+    ts, ks = [], []
     for _ in range(reps):
         t = time.perf_counter()
         fn()
         ts.append(time.perf_counter() - t)
-    return statistics.median(ts)
+        ks.append(ctx.stats()["kernel_ms"] / 1e3)
+    return statistics.median(ts), statistics.median(ks)
 
 
 def po_merges(m):
@@ -80,13 +83,14 @@ def main():
         ctx = capi.Context.from_aig(m.aig, device=0)
         # ---- NEXT-2: classes
         out = {}
-        t = timed(lambda: out.__setitem__("c", ctx.sim_classes(a.words, 1)), a.reps)
+        t, tk = timed(lambda: out.__setitem__("c", ctx.sim_classes(a.words, 1)), ctx, a.reps)
         npairs = int(out["c"][0].size)
         bytes_alg = 16.0 * N * a.words * 1.0
         rec = {"row": "NEXT-2 cec_sim_classes", "config": name, "nodes": N, "words": a.words,
-               "pairs": npairs, "gpu_ms": round(1e3 * t, 3), "launches": ctx.stats()["num_launches"],
-               "roofline": {"bound": "hbm", "algorithmic_bytes": bytes_alg, "achieved_GBps": bytes_alg / t / 1e9,
-                            "peak_GBps": peak, "peak_source": peak_src, "frac": bytes_alg / t / 1e9 / peak}}
+               "pairs": npairs, "call_ms": round(1e3 * t, 3), "kernel_ms": round(1e3 * tk, 3),
+               "launches": ctx.stats()["num_launches"],
+               "roofline": {"bound": "hbm", "algorithmic_bytes": bytes_alg, "achieved_GBps": bytes_alg / tk / 1e9,
+                            "peak_GBps": peak, "peak_source": peak_src, "frac": bytes_alg / tk / 1e9 / peak}}
         if not a.no_oracle:
             orc = oracle.Oracle.from_aig(m.aig)
             W_or = max(1, a.words // 16) if N > 1_000_000 else a.words
@@ -103,14 +107,14 @@ def main():
         mem = np.fromiter(subst.keys(), dtype=np.uint32, count=len(subst))
         rep = np.fromiter(subst.values(), dtype=np.uint32, count=len(subst))
         lits = np.concatenate([m.lit_a, m.lit_b])
-        t = timed(lambda: out.__setitem__("r", ctx.reduce(mem, rep, lits)), a.reps)
+        t, tk = timed(lambda: out.__setitem__("r", ctx.reduce(mem, rep, lits)), ctx, a.reps)
         A = m.aig.num_ands
         bytes_alg = 40.0 * A
         rec = {"row": "NEXT-3 cec_reduce", "config": name, "ands": A, "merges": len(subst),
-               "new_ands": int(out["r"][0].shape[0]), "gpu_ms": round(1e3 * t, 3),
-               "launches": ctx.stats()["num_launches"],
-               "roofline": {"bound": "hbm", "algorithmic_bytes": bytes_alg, "achieved_GBps": bytes_alg / t / 1e9,
-                            "peak_GBps": peak, "peak_source": peak_src, "frac": bytes_alg / t / 1e9 / peak}}
+               "new_ands": int(out["r"][0].shape[0]), "call_ms": round(1e3 * t, 3), "kernel_ms": round(1e3 * tk, 3),
+               "host_schedule_ms": round(ctx.stats()["host_prep_ms"], 3), "launches": ctx.stats()["num_launches"],
+               "roofline": {"bound": "hbm", "algorithmic_bytes": bytes_alg, "achieved_GBps": bytes_alg / tk / 1e9,
+                            "peak_GBps": peak, "peak_source": peak_src, "frac": bytes_alg / tk / 1e9 / peak}}
         if not a.no_oracle:
             fan = [(int(x), int(y)) for x, y in m.aig.fanins]
             t0 = time.perf_counter()
