@@ -823,53 +823,108 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         for (size_t w = 0; w < wins.size(); ++w) P->lop3_words += (uint64_t)P->win_nodes[w] * words_rank_of[w];
         return CEC_OK;
     }
-    std::vector<JitKernel *> kernels(jit_progs.size(), nullptr);
     const JitConfig jcfg = jit_config();
     const uint64_t jit_pass = jcfg.sync_every > 0 ? (uint64_t)jcfg.threads / 32 : 1;
+    // Compile units: a structure whose windows fill the GPU on their own gets its own kernel; the
+    // others (typically single small windows) are packed into bundle kernels (jit_source_bundle)
+    // so one persistent grid runs all of them instead of many tiny launches.
+    std::vector<std::vector<uint32_t>> units;  // program indices per compiled kernel
+    std::vector<uint32_t> unit_of(jit_progs.size(), 0), sid_of(jit_progs.size(), 0);
+    {
+        // a structure runs standalone when its sweep is long next to a launch's ramp and tail:
+        // >= 2^34 node-words (~0.5 ms at the LOP3 peak), e.g. C5's copy types; else it is bundled
+        std::vector<uint64_t> work(jit_progs.size(), 0);
+        std::vector<uint64_t> nodes_of(jit_progs.size(), 0);
+        for (size_t i = 0; i < jit_progs.size(); ++i) nodes_of[i] = jit_progs[i].nodes.size() / 2;
+        for (size_t w = 0; w < win_jit.size(); ++w)
+            if (win_jit[w] >= 0) work[win_jit[w]] += nodes_of[win_jit[w]] * words_rank_of[w];
+        uint64_t fill = 1ull << 34;
+        if (const char *e = getenv("CEC_BUNDLE_BELOW")) fill = strtoull(e, nullptr, 10);
+        const bool can_bundle = jcfg.splice && jcfg.sync_every > 0 && P->dwin.size() < (1u << 20) &&
+                                getenv("CEC_NO_BUNDLE") == nullptr;
+        uint32_t max_per = 24;
+        uint64_t max_nodes = 24000;
+        if (const char *e = getenv("CEC_BUNDLE_MAX")) max_per = std::max(1, atoi(e));
+        std::vector<uint32_t> cur;
+        uint64_t cur_nodes = 0;
+        auto flush = [&]() {
+            if (cur.empty()) return;
+            for (uint32_t t = 0; t < cur.size(); ++t) {
+                unit_of[cur[t]] = (uint32_t)units.size();
+                sid_of[cur[t]] = t;
+            }
+            units.push_back(cur);
+            cur.clear();
+            cur_nodes = 0;
+        };
+        for (uint32_t i = 0; i < jit_progs.size(); ++i) {
+            if (!can_bundle || work[i] >= fill) {
+                unit_of[i] = (uint32_t)units.size();
+                sid_of[i] = 0;
+                units.push_back({i});
+                continue;
+            }
+            if (cur.size() >= max_per || cur_nodes + nodes_of[i] > max_nodes) flush();
+            cur.push_back(i);
+            cur_nodes += nodes_of[i];
+        }
+        flush();
+    }
+    std::vector<JitKernel *> kernels(units.size(), nullptr);
     P->jit_ms = 0.f;
-    if (!jit_progs.empty()) {
+    if (!units.empty()) {
         auto t0 = std::chrono::steady_clock::now();
-        std::vector<std::string> errs(jit_progs.size());  // copied in the worker (messages are thread-local)
+        std::vector<std::string> errs(units.size());  // copied in the worker (messages are thread-local)
         const bool load = !c->host_only;
+        std::vector<std::vector<const JitProgram *>> uprogs(units.size());
+        for (size_t u = 0; u < units.size(); ++u)
+            for (uint32_t i : units[u]) uprogs[u].push_back(&jit_progs[i]);
         // compile (CPU-heavy, thread-safe) in parallel without loading, then load serially
         const unsigned hw = std::max(1u, std::min(16u, std::thread::hardware_concurrency()));
         std::vector<std::thread> pool;
         std::atomic<size_t> next{0};
-        for (unsigned t = 0; t < std::min<size_t>(hw, jit_progs.size()); ++t)
+        for (unsigned t = 0; t < std::min<size_t>(hw, units.size()); ++t)
             pool.emplace_back([&]() {
-                for (size_t i; (i = next.fetch_add(1)) < jit_progs.size();)
+                for (size_t i; (i = next.fetch_add(1)) < units.size();)
                 {
-                    const char *e = jit_get_kernel(jit_progs[i], jcfg, false, &kernels[i]);
+                    const char *e = jit_get_unit(uprogs[i], jcfg, false, &kernels[i]);
                     if (e) errs[i] = e;
                 }
             });
         for (auto &th : pool) th.join();
-        for (size_t i = 0; i < jit_progs.size(); ++i) {
+        for (size_t i = 0; i < units.size(); ++i) {
             if (!errs[i].empty()) return fail(c, CEC_E_CUDA, "JIT: %s", errs[i].c_str());
             if (load) {
-                const char *e = jit_get_kernel(jit_progs[i], jcfg, true, &kernels[i]);
+                const char *e = jit_get_unit(uprogs[i], jcfg, true, &kernels[i]);
                 if (e) return fail(c, CEC_E_CUDA, "JIT load: %s", e);
             }
         }
         P->jit_ms = std::chrono::duration<float, std::milli>(std::chrono::steady_clock::now() - t0).count();
     }
+    auto lop3_of = [&](uint32_t w) -> uint64_t {
+        const int32_t pi = win_jit[w];
+        return pi >= 0 ? jit_kernel_lop3_sid(kernels[unit_of[pi]], sid_of[pi]) : P->win_nodes[w];
+    };
+    auto jwin = [&](uint32_t w) -> uint32_t {  // item window field: window | sid << 20 in bundles
+        const int32_t pi = win_jit[w];
+        return units[unit_of[pi]].size() > 1 ? (w | sid_of[pi] << 20) : w;
+    };
     tm.lap("jit compile/cache");
     PhaseTimer tm2;
-    P->jit_kernels = (uint32_t)jit_progs.size();
+    P->jit_kernels = (uint32_t)units.size();
     P->jit_windows = 0;
     P->lop3_words = 0;
-    for (size_t w = 0; w < win_jit.size(); ++w) {
+    for (uint32_t w = 0; w < win_jit.size(); ++w) {
         P->jit_windows += win_jit[w] >= 0;
-        const uint64_t per_word = win_jit[w] >= 0 ? jit_kernel_lop3(kernels[win_jit[w]]) : P->win_nodes[w];
-        P->lop3_words += per_word * words_rank_of[w];
+        P->lop3_words += lop3_of(w) * words_rank_of[w];
     }
     // work items: slices of each window split into chunks; interpreter windows grouped by slot
     // budget, JIT windows by structure; largest windows first inside a group
     std::map<uint32_t, std::vector<uint32_t>> buckets;   // interpreter: slot budget -> windows
-    std::map<int32_t, std::vector<uint32_t>> jgroups;    // JIT: structure -> windows
+    std::map<int32_t, std::vector<uint32_t>> jgroups;    // JIT: compiled unit -> windows
     for (uint32_t w = 0; w < P->dwin.size(); ++w) {
         if (win_jit[w] >= 0) {
-            jgroups[win_jit[w]].push_back(w);
+            jgroups[(int32_t)unit_of[win_jit[w]]].push_back(w);
             continue;
         }
         uint32_t b = (nslots_of[w] + 31) / 32 * 32;
@@ -882,7 +937,7 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         std::stable_sort(ws.begin(), ws.end(), [&](uint32_t a, uint32_t b) { return cost_of[a] > cost_of[b]; });
         g.nwin = (uint32_t)ws.size();
         for (uint32_t w : ws) {
-            g.lop3_words += (win_jit[w] >= 0 ? jit_kernel_lop3(kernels[win_jit[w]]) : P->win_nodes[w]) * words_rank_of[w];
+            g.lop3_words += lop3_of(w) * words_rank_of[w];
             g.max_k = std::max(g.max_k, P->dwin[w].k);
             g.nodes = std::max(g.nodes, P->win_nodes[w]);
         }
@@ -902,7 +957,7 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
             for (uint64_t s = sb; s < se; s += item_slices) {
                 const uint32_t e = (uint32_t)std::min<uint64_t>(se, s + item_slices);
                 if (jit)
-                    P->jitems.push_back(JItem{w, (uint32_t)s, e, P->dwin[w].cmp_off});
+                    P->jitems.push_back(JItem{jwin(w), (uint32_t)s, e, P->dwin[w].cmp_off});
                 else
                     P->items.push_back(Item{w, (uint32_t)s, e, 0});
             }

@@ -112,6 +112,9 @@ std::string jit_key(const JitProgram &p);
 std::string jit_source(const JitProgram &p, const JitConfig &cfg);
 const char *jit_compile_cubin(const std::string &src, std::vector<char> &cubin, std::string &log);
 const char *jit_get_kernel(const JitProgram &p, const JitConfig &cfg, bool load, JitKernel **out);
+// several structures in one kernel (items carry window | sid << 20), see jit_source_bundle
+const char *jit_get_unit(const std::vector<const JitProgram *> &ps, const JitConfig &cfg, bool load, JitKernel **out);
+uint32_t jit_kernel_lop3_sid(const JitKernel *k, uint32_t sid);
 double jit_compile_ms(const JitKernel *k);
 int jit_slices_per_pass(const JitKernel *k);
 uint32_t jit_kernel_lop3(const JitKernel *k);

@@ -98,7 +98,8 @@ struct JitKernel {
     int block = 128;
     int blocks_per_sm = 0;
     int slices_per_pass = 1;  // block-synchronous kernels: warps per block
-    uint32_t lop3 = 0;        // LOP3 instructions per word of the mapped window
+    uint32_t lop3 = 0;        // LOP3 instructions per word of the mapped window (structure 0)
+    std::vector<uint32_t> lop3s;  // per structure of a bundle (sid order)
     double compile_ms = 0;
     size_t src_bytes = 0, cubin_bytes = 0;
 };
@@ -429,6 +430,12 @@ std::string jit_source(const JitProgram &p, const JitConfig &cfg) {
              "  const u32 lane = threadIdx.x & 31u;\n",
              cfg.threads, cfg.min_blocks);
     s += buf;
+    // input (projection) words: word index = 32 s + lane, so inputs 5..9 depend on the
+    // lane only (computed once per thread) and inputs >= 10 on the slice only (warp-uniform)
+    for (uint32_t j = 5; j < std::min<uint32_t>(p.k, 10); ++j) {
+        snprintf(buf, sizeof buf, "  const u32 x%u = 0u - ((lane >> %u) & 1u);\n", j, j - 5);
+        s += buf;
+    }
     if (!block_sync) {
         // every warp independent: pulls items itself, one 32-word slice per pass
         s += "  for (;;) {\n"
@@ -462,12 +469,13 @@ std::string jit_source(const JitProgram &p, const JitConfig &cfg) {
                  nw);
         s += buf;
     }
-    s += "      const u64 word = ((u64)s << 5) + lane;\n";
     for (uint32_t j = 0; j < p.k; ++j) {
         if (j < 5)
             snprintf(buf, sizeof buf, "      const u32 x%u = %s;\n", j, kMask[j]);
+        else if (j < 10)
+            continue;  // lane-only, hoisted above
         else
-            snprintf(buf, sizeof buf, "      const u32 x%u = 0u - (u32)((word >> %u) & 1ull);\n", j, j - 5);
+            snprintf(buf, sizeof buf, "      const u32 x%u = 0u - ((s >> %u) & 1u);\n", j, j - 10);
         s += buf;
     }
     // compares are placed right after their later root so roots die early (fewer live registers)
@@ -500,7 +508,7 @@ std::string jit_source(const JitProgram &p, const JitConfig &cfg) {
             snprintf(buf, sizeof buf, "      u32 m%u;\n", w);
             s += buf;
         }
-        s += "      asm volatile(\"//@@BODY@@";
+        s += "      asm volatile(\"//@@BODY0@@";
         for (uint32_t i = 0; i < M + p.k + (ncmp ? 1 : 0); ++i) {
             snprintf(buf, sizeof buf, " %%%u", i);
             s += buf;
@@ -551,6 +559,112 @@ std::string jit_source(const JitProgram &p, const JitConfig &cfg) {
         }
     }
     s += block_sync ? "      bnd = bnd_next;\n    }\n    __syncthreads();\n  }\n}\n" : "    }\n  }\n}\n";
+    return s;
+}
+
+// Bundle kernel: several window STRUCTURES in one kernel (splice + block-synchronous mode only).
+// Items carry (window | sid << 20); the block takes an item, every warp computes the input words
+// of its slice once and the item's structure body runs from a switch. Used for structures whose own
+// launch could not fill the GPU (single small windows, e.g. most of C3's): one persistent grid pulls
+// the items of all of them, instead of hundreds of tiny launches serialised over a few streams.
+std::string jit_source_bundle(const std::vector<const JitProgram *> &ps, const JitConfig &cfg) {
+    const int nw = cfg.threads / 32;
+    uint32_t kmax = 0;
+    for (const JitProgram *p : ps) kmax = std::max(kmax, p->k);
+    std::string s;
+    char buf[1024];
+    s += "typedef unsigned int u32; typedef unsigned long long u64;\n"
+         "struct JItem { u32 win, s_begin, s_end, cmp_off; };\n"
+         "__device__ __noinline__ void rep(u32 d, u32 c, u32 win, u32 s, u32 lane, u32 ncmp, u32 cmp_off,\n"
+         "    u64 *first, u64 *bound, u32 *neq_cnt) {\n"
+         "  const u32 bal = __ballot_sync(0xFFFFFFFFu, d != 0u);\n"
+         "  const u32 l = (u32)__ffs(bal) - 1u;\n"
+         "  const u32 dl = __shfl_sync(0xFFFFFFFFu, d, l);\n"
+         "  if (lane != 0u) return;\n"
+         "  const u64 idx = ((((u64)s << 5) + l) << 5) + (u32)(__ffs(dl) - 1);\n"
+         "  const u64 old = atomicMin(&first[cmp_off + c], idx);\n"
+         "  if (old != ~0ull) return;\n"
+         "  __threadfence();\n"
+         "  if (atomicAdd(&neq_cnt[win], 1u) + 1u != ncmp) return;\n"
+         "  __threadfence();\n"
+         "  u64 mx = 0;\n"
+         "  for (u32 t = 0; t < ncmp; ++t) { u64 v = atomicAdd(&first[cmp_off + t], 0ull); mx = v > mx ? v : mx; }\n"
+         "  atomicMin(&bound[win], mx);\n"
+         "}\n";
+    snprintf(buf, sizeof buf,
+             "extern \"C\" __global__ void __launch_bounds__(%d, %d) cecjit(const JItem *__restrict__ items, u32 nitems,\n"
+             "    u32 *ctr, u64 *first, u64 *bound, u32 *neq_cnt) {\n"
+             "  const u32 lane = threadIdx.x & 31u;\n"
+             "  const u32 warp = threadIdx.x >> 5;\n"
+             "  __shared__ u32 s_it; __shared__ JItem s_item;\n"
+             "  for (;;) {\n"
+             "    if (threadIdx.x == 0u) { const u32 t = atomicAdd(ctr, 1u); s_it = t; if (t < nitems) s_item = items[t]; }\n"
+             "    __syncthreads();\n"
+             "    const u32 it = s_it;\n"
+             "    if (it >= nitems) return;\n"
+             "    JItem I = s_item;\n"
+             "    const u32 sid = I.win >> 20;\n"
+             "    I.win &= 0xFFFFFu;\n"
+             "    u64 bnd = *((volatile u64 *)&bound[I.win]);\n"
+             "    for (u32 s0 = I.s_begin; s0 < I.s_end; s0 += %du) {\n"
+             "      const u32 s = s0 + warp;\n"
+             "      const bool live = s < I.s_end && ((u64)s << 10) < bnd;\n"
+             "      if (!__syncthreads_or(live)) break;\n"
+             "      const u64 bnd_next = *((volatile u64 *)&bound[I.win]);\n",
+             cfg.threads, cfg.min_blocks, nw);
+    s += buf;
+    for (uint32_t j = 0; j < kmax; ++j) {
+        if (j < 5)
+            snprintf(buf, sizeof buf, "      const u32 x%u = %s;\n", j, kMask[j]);
+        else if (j < 10)
+            snprintf(buf, sizeof buf, "      const u32 x%u = 0u - ((lane >> %u) & 1u);\n", j, j - 5);
+        else
+            snprintf(buf, sizeof buf, "      const u32 x%u = 0u - ((s >> %u) & 1u);\n", j, j - 10);
+        s += buf;
+    }
+    s += "      switch (sid) {\n";
+    for (size_t i = 0; i < ps.size(); ++i) {
+        const JitProgram &p = *ps[i];
+        const uint32_t ncmp = (uint32_t)(p.cmps.size() / 2), M = (ncmp + 31) / 32;
+        snprintf(buf, sizeof buf, "      case %zuu: {\n", i);
+        s += buf;
+        if (ncmp) {
+            snprintf(buf, sizeof buf, "        u32 dbuf[%u];\n", ncmp);
+            s += buf;
+        }
+        for (uint32_t w = 0; w < M; ++w) {
+            snprintf(buf, sizeof buf, "        u32 m%u;\n", w);
+            s += buf;
+        }
+        snprintf(buf, sizeof buf, "        asm volatile(\"//@@BODY%zu@@", i);
+        s += buf;
+        for (uint32_t t = 0; t < M + p.k + (ncmp ? 1 : 0); ++t) {
+            snprintf(buf, sizeof buf, " %%%u", t);
+            s += buf;
+        }
+        s += "\" :";
+        for (uint32_t w = 0; w < M; ++w) {
+            snprintf(buf, sizeof buf, "%s \"=r\"(m%u)", w ? "," : "", w);
+            s += buf;
+        }
+        s += " :";
+        for (uint32_t j = 0; j < p.k; ++j) {
+            snprintf(buf, sizeof buf, "%s \"r\"(x%u)", j ? "," : "", j);
+            s += buf;
+        }
+        if (ncmp) s += ", \"l\"(dbuf)";
+        s += " : \"memory\");\n";
+        for (uint32_t w = 0; w < M; ++w) {
+            snprintf(buf, sizeof buf,
+                     "        for (u32 mk = m%u; mk; mk &= mk - 1u) { const u32 c = %uu + (u32)__ffs(mk) - 1u;\n"
+                     "          const u32 d = live ? dbuf[c] : 0u;\n"
+                     "          if (__any_sync(0xFFFFFFFFu, d != 0u)) rep(d, c, I.win, s, lane, %uu, I.cmp_off, first, bound, neq_cnt); }\n",
+                     w, 32 * w, ncmp);
+            s += buf;
+        }
+        s += "      } break;\n";
+    }
+    s += "      default: break;\n      }\n      bnd = bnd_next;\n    }\n    __syncthreads();\n  }\n}\n";
     return s;
 }
 
@@ -648,7 +762,7 @@ JitLink g_link;
 
 // Splice-mode compile: NVRTC turns the small skeleton into PTX, the generated body replaces the
 // marker line, nvJitLink assembles the result for sm_100a.
-const char *jit_compile_splice(const JitProgram &p, const JitConfig &cfg, const std::string &src,
+const char *jit_compile_splice(const std::vector<const JitProgram *> &ps, const JitConfig &cfg, const std::string &src,
                                std::vector<char> &cubin, std::string &log) {
     {
         std::lock_guard<std::mutex> g(g_mu);
@@ -667,30 +781,34 @@ const char *jit_compile_splice(const JitProgram &p, const JitConfig &cfg, const 
         g_nvrtc.destroy(&prog);
         return "NVRTC compilation failed (skeleton)";
     }
-    size_t ps = 0;
-    g_nvrtc.ptx_size(prog, &ps);
-    std::string ptx(ps, '\0');
+    size_t ptx_bytes = 0;
+    g_nvrtc.ptx_size(prog, &ptx_bytes);
+    std::string ptx(ptx_bytes, '\0');
     g_nvrtc.ptx(prog, &ptx[0]);
     g_nvrtc.destroy(&prog);
-    const size_t m = ptx.find("//@@BODY@@");
-    if (m == std::string::npos) return "splice marker not found in PTX";
-    const size_t eol = ptx.find('\n', m);
-    std::vector<std::string> regs;
-    {
-        size_t i = m + 10;
-        while (i < eol) {
-            while (i < eol && ptx[i] == ' ') ++i;
-            size_t j = i;
-            while (j < eol && ptx[j] != ' ' && ptx[j] != '\r') ++j;
-            if (j > i) regs.emplace_back(ptx.substr(i, j - i));
-            i = j + 1;
+    for (size_t i = 0; i < ps.size(); ++i) {
+        const JitProgram &p = *ps[i];
+        const std::string marker = "//@@BODY" + std::to_string(i) + "@@";
+        const size_t m = ptx.find(marker);
+        if (m == std::string::npos) return "splice marker not found in PTX";
+        const size_t eol = ptx.find('\n', m);
+        std::vector<std::string> regs;
+        {
+            size_t q = m + marker.size();
+            while (q < eol) {
+                while (q < eol && ptx[q] == ' ') ++q;
+                size_t j = q;
+                while (j < eol && ptx[j] != ' ' && ptx[j] != '\r') ++j;
+                if (j > q) regs.emplace_back(ptx.substr(q, j - q));
+                q = j + 1;
+            }
         }
+        const uint32_t ncmp = (uint32_t)(p.cmps.size() / 2), M = (ncmp + 31) / 32;
+        if (regs.size() != M + p.k + (ncmp ? 1 : 0)) return "splice: operand count mismatch";
+        std::vector<std::string> masks(regs.begin(), regs.begin() + M), ins(regs.begin() + M, regs.begin() + M + p.k);
+        const std::string dbuf = ncmp ? regs.back() : std::string("%cz");
+        ptx.replace(m, eol - m, jit_body_ptx(p, cfg, masks, ins, dbuf));
     }
-    const uint32_t ncmp = (uint32_t)(p.cmps.size() / 2), M = (ncmp + 31) / 32;
-    if (regs.size() != M + p.k + (ncmp ? 1 : 0)) return "splice: operand count mismatch";
-    std::vector<std::string> masks(regs.begin(), regs.begin() + M), ins(regs.begin() + M, regs.begin() + M + p.k);
-    const std::string dbuf = ncmp ? regs.back() : std::string("%cz");
-    ptx.replace(m, eol - m, jit_body_ptx(p, cfg, masks, ins, dbuf));
     while (!ptx.empty() && ptx.back() == '\0') ptx.pop_back();
     if (const char *dir = getenv("CEC_JIT_DUMP")) {
         char path[512];
@@ -751,11 +869,16 @@ namespace {
 std::map<std::string, std::unique_ptr<JitKernel>> g_cache;  // process-wide, keyed by structure
 }
 
-const char *jit_get_kernel(const JitProgram &p, const JitConfig &cfg, bool load, JitKernel **out) {
+const char *jit_get_unit(const std::vector<const JitProgram *> &ps, const JitConfig &cfg, bool load, JitKernel **out) {
+    if (ps.empty()) return "empty JIT unit";
+    const bool bundle = ps.size() > 1;
+    if (bundle && !(cfg.splice && cfg.sync_every > 0)) return "JIT bundles need the block-synchronous splice mode";
     char ck[64];
     snprintf(ck, sizeof ck, "|%d,%d,%d,%d,%d", cfg.threads, cfg.min_blocks, cfg.sync_every, (int)cfg.fuse,
              (int)cfg.splice);
-    const std::string key = jit_key(p) + ck;
+    std::string key;
+    for (const JitProgram *p : ps) key += jit_key(*p) + "#";
+    key += ck;
     {
         std::lock_guard<std::mutex> g(g_mu);
         auto it = g_cache.find(key);
@@ -765,10 +888,10 @@ const char *jit_get_kernel(const JitProgram &p, const JitConfig &cfg, bool load,
         }
     }
     auto t0 = std::chrono::steady_clock::now();
-    const std::string src = jit_source(p, cfg);
+    const std::string src = bundle ? jit_source_bundle(ps, cfg) : jit_source(*ps[0], cfg);
     std::vector<char> cubin;
     std::string log;
-    const char *e = (cfg.splice && cfg.sync_every > 0) ? jit_compile_splice(p, cfg, src, cubin, log)
+    const char *e = (cfg.splice && cfg.sync_every > 0) ? jit_compile_splice(ps, cfg, src, cubin, log)
                                                        : jit_compile_cubin(src, cubin, log);
     if (e) {
         static thread_local std::string msg;
@@ -791,7 +914,8 @@ const char *jit_get_kernel(const JitProgram &p, const JitConfig &cfg, bool load,
     }
     std::unique_ptr<JitKernel> K(new JitKernel());
     K->block = cfg.threads;
-    K->lop3 = jit_lop3_count(p, cfg.fuse);
+    for (const JitProgram *p : ps) K->lop3s.push_back(jit_lop3_count(*p, cfg.fuse));
+    K->lop3 = K->lop3s[0];
     K->slices_per_pass = cfg.sync_every > 0 ? cfg.threads / 32 : 1;
     K->src_bytes = src.size();
     K->cubin_bytes = cubin.size();
@@ -813,9 +937,16 @@ const char *jit_get_kernel(const JitProgram &p, const JitConfig &cfg, bool load,
     return nullptr;
 }
 
+const char *jit_get_kernel(const JitProgram &p, const JitConfig &cfg, bool load, JitKernel **out) {
+    return jit_get_unit({&p}, cfg, load, out);
+}
+
 double jit_compile_ms(const JitKernel *k) { return k ? k->compile_ms : 0.0; }
 int jit_slices_per_pass(const JitKernel *k) { return k ? k->slices_per_pass : 1; }
 uint32_t jit_kernel_lop3(const JitKernel *k) { return k ? k->lop3 : 0; }
+uint32_t jit_kernel_lop3_sid(const JitKernel *k, uint32_t sid) {
+    return k && sid < k->lop3s.size() ? k->lop3s[sid] : 0;
+}
 
 const char *jit_launch(JitKernel *K, const JItem *items, uint32_t nitems, uint32_t *ctr, unsigned long long *first,
                        unsigned long long *bound, uint32_t *neq_cnt, void *stream, int num_sms) {

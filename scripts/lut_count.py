@@ -12,7 +12,7 @@ from paper_conf_dac_liuy25_b200 import capi  # noqa: E402
 name = sys.argv[1] if len(sys.argv) > 1 else "c5"
 m, _, _ = bench.make_workload(name)
 merge = capi.CEC_MERGE_COST if name == "c3" else capi.CEC_MERGE_PAPER
-ctx = capi.Context.from_aig(m.aig, device=-1, merge=merge, engine=capi.CEC_ENGINE_JIT)
+ctx = capi.Context.from_aig(m.aig, device=-1, merge=merge, engine=int(os.environ.get("CEC_ENGINE", capi.CEC_ENGINE_JIT)))
 t = time.perf_counter()
 plan = capi.cec_plan_exhaustive(ctx.handle, m.lit_a, m.lit_b)
 dt = time.perf_counter() - t

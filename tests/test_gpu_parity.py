@@ -417,3 +417,28 @@ def test_pipelined_call_matches_single_plan(engine, monkeypatch):
         for p in np.flatnonzero(got[0] == capi.CEC_NOT_EQUIVALENT)[:3]:
             pis = ctx.get_cex(int(p))  # the CEX vector of the pipelined call distinguishes the pair
             assert orc.eval_lit(int(m.lit_a[p]), pis) != orc.eval_lit(int(m.lit_b[p]), pis)
+
+
+def _c3_small():
+    """A reduced C3: 30 random blocks with supports 10..16 over 256 PIs (oracle in seconds) — many
+    distinct small window structures, i.e. the JIT bundle kernels (jit_source_bundle)."""
+    return circuits.c3_rand(n_blocks=30, block_ands=300, num_pis=256, n_internal=600, n_near=32,
+                            k_dist=((30, 10, 16),))
+
+
+def test_jit_bundles_vs_oracle_and_unbundled(monkeypatch):
+    m = _c3_small()
+    ctx, gv, gc, gk = check_vs_oracle(m, engine=capi.CEC_ENGINE_JIT, merge=capi.CEC_MERGE_COST)
+    st = ctx.stats()
+    assert st["jit_windows"] > st["jit_kernels"]  # structures were bundled
+    monkeypatch.setenv("CEC_NO_BUNDLE", "1")
+    ctx2 = gpu_ctx(m.aig, engine=capi.CEC_ENGINE_JIT, merge=capi.CEC_MERGE_COST)
+    got = ctx2.sim_exhaustive(m.lit_a, m.lit_b)
+    for a, b in zip((gv, gc, gk), got):
+        assert np.array_equal(a, b)
+    monkeypatch.setenv("CEC_BUNDLE_MAX", "3")
+    monkeypatch.delenv("CEC_NO_BUNDLE")
+    ctx3 = gpu_ctx(m.aig, engine=capi.CEC_ENGINE_JIT, merge=capi.CEC_MERGE_COST)
+    got = ctx3.sim_exhaustive(m.lit_a, m.lit_b)
+    for a, b in zip((gv, gc, gk), got):
+        assert np.array_equal(a, b)
