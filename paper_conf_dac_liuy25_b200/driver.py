@@ -251,7 +251,10 @@ def check_miter(aig: Aig, lit_a, lit_b, params: Optional[CecParams] = None) -> C
         # equivalence classes on the GPU: random patterns plus the CEX patterns
         # of disproved pairs, which split their classes
         words = pack_patterns(cex_patterns, cur.aig.num_pis) if cex_patterns else None
+        tk = {"classes": 0.0, "global": 0.0, "cuts": 0.0, "local": 0.0}
+        t1 = time.perf_counter()
         cr, cm, cf = ctx.sim_classes(p.sim_words, p.seed + phase_no, words)
+        tk["classes"] += time.perf_counter() - t1
         cand = [(int(r), int(m_), int(f)) for r, m_, f in zip(cr, cm, cf)]
         versions.append(cur.aig)
         # G phase once per miter version: pairs with support <= k_g
@@ -261,7 +264,9 @@ def check_miter(aig: Aig, lit_a, lit_b, params: Optional[CecParams] = None) -> C
         subst = {}
         proved_g = 0
         if gl:
+            t1 = time.perf_counter()
             v, _, k = ctx.sim_exhaustive(la, lb)
+            tk["global"] += time.perf_counter() - t1
             for i in np.nonzero(v == capi.CEC_NOT_EQUIVALENT)[0][:p.max_cex_patterns]:
                 if len(cex_patterns) >= p.max_cex_patterns:
                     break
@@ -289,6 +294,7 @@ def check_miter(aig: Aig, lit_a, lit_b, params: Optional[CecParams] = None) -> C
             todo = [x for x in remaining if x[1] not in subst]
             ql, qm, off, leaves, who = [], [], [0], [], []
             if p.native_cuts and todo:
+                t1 = time.perf_counter()
                 pco, co, lvs = capi.cec_common_cuts(lctx.handle, [x[0] for x in todo], [x[1] for x in todo],
                                                      p.k_l, p.C, pass_id, p.max_cuts_per_pair)
                 for i, (r, m_, f) in enumerate(todo):
@@ -298,6 +304,7 @@ def check_miter(aig: Aig, lit_a, lit_b, params: Optional[CecParams] = None) -> C
                         leaves += [int(x) for x in lvs[co[ct]:co[ct + 1]]]
                         off.append(len(leaves))
                         who.append((r, m_, f))
+                tk["cuts"] += time.perf_counter() - t1
             elif todo:
                 repr_of = {m_: r for r, m_, f in todo}
                 cuts = enumerate_cuts(cur.aig, p.k_l, p.C, pass_id, repr_of)
@@ -316,7 +323,9 @@ def check_miter(aig: Aig, lit_a, lit_b, params: Optional[CecParams] = None) -> C
                         who.append((r, m_, f))
             if not ql:
                 continue
+            t1 = time.perf_counter()
             lv = lctx.check_local_cuts(ql, qm, off, leaves)
+            tk["local"] += time.perf_counter() - t1
             for q, vv in enumerate(lv):
                 checks.append({"version": len(versions) - 1, "phase": phase_no, "pass": pass_id,
                                "lit_a": ql[q], "lit_b": qm[q], "leaves": leaves[off[q]:off[q + 1]], "verdict": int(vv)})
@@ -327,11 +336,15 @@ def check_miter(aig: Aig, lit_a, lit_b, params: Optional[CecParams] = None) -> C
             remaining = [x for x in remaining if x[1] not in subst]
         ctx.close()
         lctx.close()
-        log.append({"phase": f"G+L{phase_no}", "candidates": len(cand), "proved_global": proved_g,
-                    "proved_local": proved_l, "ands": cur.aig.num_ands, "s": time.perf_counter() - t})
+        entry = {"phase": f"G+L{phase_no}", "candidates": len(cand), "proved_global": proved_g,
+                 "proved_local": proved_l, "ands": cur.aig.num_ands, "s": time.perf_counter() - t,
+                 "s_parts": {k_: round(v_, 4) for k_, v_ in tk.items()}}
+        log.append(entry)
         if not subst:
             break  # no progress: undecided remainder
+        t1 = time.perf_counter()
         cur, _ = cur.reduce(subst, p.device)
+        entry["s_parts"]["reduce"] = round(time.perf_counter() - t1, 4)
     st = po_status(cur)
     po_v = np.where(st == capi.CEC_EQUIVALENT, capi.CEC_EQUIVALENT, po_v)
     cex_vec, cex_pair = None, -1

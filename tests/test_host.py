@@ -168,16 +168,22 @@ def test_pext():
         assert capi.cec_pext64(v, m) == want
 
 
-def test_jit_codegen_compiles_for_sm100a_host_only():
+def test_jit_codegen_compiles_for_sm100a_host_only(monkeypatch):
     """The JIT engine's NVRTC path runs on the host (no GPU needed): one kernel per distinct window
-    structure; C5's 256 copies share 3 random + 1 mul12 + bug-variant structures."""
-    from workloads import circuits
+    structure; C5's 256 copies share 3 random + 1 mul12 + bug-variant structures. Structures too
+    small to fill the GPU alone are compiled together into one bundle kernel."""
     m = c5_big(copies=12, n_random=8, n_bugs=2, rand_pis=12, rand_ands=300, mul_n=6)
+    n_struct = len(set(m.meta["types"]))
+    monkeypatch.setenv("CEC_NO_BUNDLE", "1")
     ctx = host_ctx(m.aig, engine=capi.CEC_ENGINE_JIT, k_s=12)  # merge inside a copy, never across
     plan = capi.cec_plan_exhaustive(ctx.handle, m.lit_a, m.lit_b)
     st = ctx.stats()
-    n_struct = len(set(m.meta["types"]))
     assert st["jit_windows"] == 12 and st["jit_kernels"] == n_struct
+    capi.cec_plan_free(plan)
+    monkeypatch.delenv("CEC_NO_BUNDLE")
+    plan = capi.cec_plan_exhaustive(ctx.handle, m.lit_a, m.lit_b)
+    st = ctx.stats()
+    assert st["jit_windows"] == 12 and st["jit_kernels"] == 1  # every structure in one bundle
     capi.cec_plan_free(plan)
     # interpreter only: no JIT
     ctx2 = host_ctx(m.aig, engine=capi.CEC_ENGINE_INTERP)
