@@ -273,6 +273,12 @@ def main():
     # e2e: the public blocking call with host arrays (plan + H2D + kernels + reduce + D2H)
     e2e_ms = []
     la_h, lb_h = np.ascontiguousarray(m.lit_a), np.ascontiguousarray(m.lit_b)
+    # one untimed call first: the pipelined call plans windows in chunks whose JIT bundles are
+    # compiled (and cached) on first use; compile time is reported separately, never timed
+    t = time.perf_counter()
+    ctx.sim_exhaustive(la_h, lb_h)
+    e2e_warm_ms = 1e3 * (time.perf_counter() - t)
+    e2e_jit_ms = ctx.stats()["jit_ms"]
     for _ in range(max(1, args.e2e_steps)):
         if world > 1:
             dist.barrier()
@@ -337,7 +343,8 @@ def main():
             "gpu_launches": int(launches_per_step * args.steps),
             "e2e": {"value": W_all / (e2e / 1e3), "unit": UNIT, "ms_per_miter": e2e,
                     "h2d_bytes_per_step": int(st_e2e["h2d_bytes"]), "d2h_bytes_per_step": int(st_e2e["d2h_bytes"]),
-                    "host_prep_ms": st_e2e["host_prep_ms"], "aig_load_ms": load_ms},
+                    "host_prep_ms": st_e2e["host_prep_ms"], "aig_load_ms": load_ms,
+                    "warmup_call_ms": round(e2e_warm_ms, 2), "warmup_jit_compile_ms": round(e2e_jit_ms, 2)},
             "roofline": ({"bound": "hbm", "achieved": simt_gbs, "peak": hbm_peak, "unit": "GB/s",
                           "frac": simt_gbs / hbm_peak, "traffic": None,
                           "peak_basis": "MEASURED_PEAKS.json hbm_gbs (copy bandwidth)",

@@ -576,7 +576,7 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         }
     }
     // AUTO engine: a window is compiled when its sweep is at least this many node-words
-    uint64_t jit_min_node_words = 1ull << 23;
+    uint64_t jit_min_node_words = 1ull << 20;
     if (const char *e = getenv("CEC_JIT_MIN_NODE_WORDS")) jit_min_node_words = strtoull(e, nullptr, 10);
     // (2) parallel over windows: node order, schedule, engine choice, JIT program
     struct WinRes {
@@ -858,7 +858,9 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
             cur_nodes = 0;
         };
         for (uint32_t i = 0; i < jit_progs.size(); ++i) {
-            if (!can_bundle || work[i] >= fill) {
+            // large bodies (> 4096 ANDs, ~64 KB of SASS each) keep their own kernel: a bundle of
+            // them would share one register allocation and spread SMs over several big bodies
+            if (!can_bundle || work[i] >= fill || nodes_of[i] > 4096) {
                 unit_of[i] = (uint32_t)units.size();
                 sid_of[i] = 0;
                 units.push_back({i});
