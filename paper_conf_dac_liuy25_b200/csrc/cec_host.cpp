@@ -647,7 +647,12 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         if (k >= 10 && !nodes.empty()) {
             if (c->opts.engine == CEC_ENGINE_JIT) R.jit = true;
             else if (c->opts.engine == CEC_ENGINE_SIMT && !local) R.jit = false;
-            else if (c->opts.engine == CEC_ENGINE_AUTO) R.jit = node_words >= jit_min_node_words || R.sc.nslots > max_slot_cap;
+            else if (c->opts.engine == CEC_ENGINE_AUTO)
+                // k <= 16 windows (local checks, G-phase pairs, the sweeping flow's re-planned
+                // miters) finish in microseconds on the interpreter: compiling them pays only in
+                // repeated runs of one plan, so they need 8x the work of larger-k windows
+                R.jit = node_words >= (k <= 16 ? jit_min_node_words << 3 : jit_min_node_words) ||
+                        R.sc.nslots > max_slot_cap;
         }
         if (!R.jit && !(c->opts.engine == CEC_ENGINE_SIMT && !local)) {  // interpreter program
             if (!build_schedule(c, X, W.inputs, nodes, cmps2, wc, R.sc, why)) {

@@ -2,6 +2,8 @@
 
   NEXT-2  cec_sim_classes : partial simulation (random words) + exact equivalence classes + pairs
   NEXT-3  cec_reduce      : miter reduction (merge + strash rebuild)
+  a12     cec_check_local_cuts on the local checks the C4 flow issues in its first L phase
+          (config "c4"): node-patterns/s and the LOP3-pipe fraction of the interpreter kernel
 
 Each row reports the median wall time of the blocking C-ABI call (host schedule, H2D of the merge
 list / D2H of the results included) and the median device time of its kernels (CUDA events on the
@@ -78,6 +80,9 @@ def main():
 
     peak, peak_src = hbm_peak()
     for name in a.configs.split(","):
+        if name == "c4":
+            local_row(a)
+            continue
         m, _, _ = bench.make_workload(name)
         N = m.aig.num_nodes
         ctx = capi.Context.from_aig(m.aig, device=0)
@@ -125,6 +130,46 @@ def main():
                              np.array_equal(out["r"][2], np.array(olits, dtype=np.uint32)))
         print(json.dumps(rec), flush=True)
         ctx.close()
+
+
+def local_row(a):
+    """a12 on C4: the (pair, cut) checks of the flow's first G+L phase, replayed through the C-ABI."""
+    import oracle
+    from paper_conf_dac_liuy25_b200 import driver
+    from workloads import c4_dp
+    m = c4_dp(64)
+    r = driver.check_miter(m.aig, m.lit_a, m.lit_b, driver.CecParams(k_l=16, C=16))
+    v0 = [ch for ch in r.checks if ch["version"] == 0]
+    aig = r.versions[0]
+    la = np.array([ch["lit_a"] for ch in v0], dtype=np.uint32)
+    lb = np.array([ch["lit_b"] for ch in v0], dtype=np.uint32)
+    off, leaves = [0], []
+    for ch in v0:
+        leaves += ch["leaves"]
+        off.append(len(leaves))
+    ctx = capi.Context.from_aig(aig, device=0, k_max=16)
+    out = {}
+    t, tk = timed(lambda: out.__setitem__("v", ctx.check_local_cuts(la, lb, off, leaves)), ctx, a.reps)
+    st = ctx.stats()
+    W = st["node_patterns"]
+    lop3 = st["lop3_words"]
+    sm_mhz = 1965.0
+    lop_peak = 148 * 64 * sm_mhz * 1e6
+    rec = {"row": "a12 cec_check_local_cuts", "config": "c4 first L phase", "checks": int(la.size),
+           "max_leaves": int(max(len(ch["leaves"]) for ch in v0)), "node_patterns": int(W),
+           "call_ms": round(1e3 * t, 3), "kernel_ms": round(1e3 * tk, 3), "host_prep_ms": round(st["host_prep_ms"], 3),
+           "node_patterns_per_s_kernel": W / tk, "node_patterns_per_s_call": W / t,
+           "roofline": {"bound": "alu", "achieved_tlop3": lop3 / tk / 1e12, "peak_tlop3": lop_peak / 1e12,
+                        "frac": lop3 / tk / lop_peak, "peak_basis": "148 SMs x 64 LOP3/clk x 1965 MHz"}}
+    if not a.no_oracle:
+        orc = oracle.Oracle.from_aig(aig)
+        t0 = time.perf_counter()
+        want = orc.check_local(la, lb, off, leaves)
+        rec["oracle"] = {"seconds": round(time.perf_counter() - t0, 3), "cores": 1, "kind": "oracle.check_local",
+                         "node_patterns_per_s": W / max(1e-9, time.perf_counter() - t0)}
+        rec["parity"] = bool(np.array_equal(np.asarray(out["v"]), np.asarray(want)))
+    print(json.dumps(rec), flush=True)
+    ctx.close()
 
 
 if __name__ == "__main__":
