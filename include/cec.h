@@ -193,6 +193,24 @@ cec_status cec_common_cuts(cec_ctx *ctx, uint32_t npairs, const uint32_t *repr, 
                            uint32_t k_l, uint32_t C, int32_t pass_id, uint32_t max_cuts, uint32_t *pair_cut_off,
                            uint32_t *cut_off, uint32_t *leaves);
 
+/* One cut generation + local checking pass, Alg. 2:
+ * the priority cuts of cec_common_cuts (same definition, same cuts) are enumerated level by level
+ * in the enumeration levels of Eq. (2) (the nodes of a level in parallel), and as soon as a
+ * member's cuts exist, the common cuts of its pair (member[q] with repr[q], relative phase
+ * phase[q]: the pair is the literals 2*repr and 2*member ^ phase) enter a buffer that is flushed to
+ * the local-check kernels (cec_check_local_cuts semantics) whenever it holds
+ * buffer_checks checks; the GPU checks one buffer while the host enumerates the next levels.
+ * verdict_out[q] = EQUIVALENT if any common cut of pair q proves it, else UNDECIDED.
+ * *num_checks_out = checks issued. Optional check log (NULL allowed), in issue order, with caller
+ * capacities npairs*max_cuts (+1 for check_cut_off) and npairs*max_cuts*k_l leaves:
+ * check_pair[i], leaves check_leaves[check_cut_off[i] .. check_cut_off[i+1]), check_verdict[i].
+ * Results do not depend on buffer_checks. CEC_E_CUDA without a device. */
+cec_status cec_local_pass(cec_ctx *ctx, uint32_t npairs, const uint32_t *repr, const uint32_t *member,
+                          const uint8_t *phase, uint32_t k_l, uint32_t C, int32_t pass_id, uint32_t max_cuts,
+                          uint32_t buffer_checks, int32_t *verdict_out, uint32_t *num_checks_out,
+                          uint32_t *check_pair, uint32_t *check_cut_off, uint32_t *check_leaves,
+                          int32_t *check_verdict);
+
 /* Miter reduction on the GPU ("reduces the miter by merging the proved equivalent
  * pairs", :185, :187). Merge q redirects every fanout of AND node member[q]
  * to the literal repr_lit[q] (a proved equivalence; repr_lit[q] >> 1 < member[q], representative =

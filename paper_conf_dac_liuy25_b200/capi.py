@@ -28,7 +28,7 @@ EXPORTS = ["cec_default_opts", "cec_load_aig", "cec_sim_exhaustive", "cec_check_
            "cec_pair_support", "cec_plan_exhaustive", "cec_plan_run", "cec_plan_results", "cec_plan_info",
            "cec_plan_window", "cec_plan_free", "cec_stream", "cec_get_stats", "cec_shard_range", "cec_pext64",
            "cec_free", "cec_last_error", "cec_abi_version", "cec_nccl_unique_id", "cec_sim_random",
-           "cec_common_cuts", "cec_sim_patterns", "cec_reduce", "cec_sim_classes"]
+           "cec_common_cuts", "cec_sim_patterns", "cec_reduce", "cec_sim_classes", "cec_local_pass"]
 
 
 class CecOpts(ctypes.Structure):
@@ -92,6 +92,7 @@ def _load() -> ctypes.CDLL:
         "cec_sim_patterns": (ctypes.c_int, [P, u32, P, P, P]),
         "cec_reduce": (ctypes.c_int, [P, u32, P, P, P, P, P, u32, P]),
         "cec_sim_classes": (ctypes.c_int, [P, u32, u64, u32, P, u32, P, P, P, P]),
+        "cec_local_pass": (ctypes.c_int, [P, u32, P, P, P, u32, u32, i32, u32, u32, P, P, P, P, P, P]),
     }
     for name, (res, args) in sig.items():
         fn = getattr(L, name)
@@ -227,6 +228,27 @@ def cec_reduce(ctx, num_pis: int, num_ands: int, member_ids, repr_lits, lits=())
     _check(lib.cec_reduce(ctx, m.size, _p(m), _p(r), ctypes.byref(na), _p(fan), _p(img), lv.size,
                           _p(lv) if lv.size else None), ctx)
     return fan[:2 * na.value].reshape(-1, 2), img, lv
+
+
+def cec_local_pass(ctx, repr_ids, member_ids, phases, k_l: int, C: int, pass_id: int, max_cuts: int,
+                   buffer_checks: int = 4096, log: bool = True):
+    """Alg. 2 pass: (verdict int32[npairs], checks) where checks = (pair uint32[n], cut_off uint32[n+1],
+    leaves uint32[...], verdict int32[n]) in issue order (None when log=False)."""
+    r, m = _u32(repr_ids), _u32(member_ids)
+    ph = np.ascontiguousarray(np.asarray(phases, dtype=np.uint8).reshape(-1))
+    n = r.size
+    v = np.zeros(max(n, 1), np.int32)
+    nc = ctypes.c_uint32()
+    cap = max(1, n * max_cuts)
+    cp = np.zeros(cap, np.uint32) if log else None
+    co = np.zeros(cap + 1, np.uint32) if log else None
+    cl = np.zeros(max(1, cap * k_l), np.uint32) if log else None
+    cv = np.zeros(cap, np.int32) if log else None
+    _check(lib.cec_local_pass(ctx, n, _p(r), _p(m), _p(ph), k_l, C, pass_id, max_cuts, buffer_checks, _p(v),
+                              ctypes.byref(nc), _p(cp), _p(co), _p(cl), _p(cv)), ctx)
+    k = int(nc.value)
+    checks = (cp[:k], co[:k + 1], cl[:int(co[k])], cv[:k]) if log else None
+    return v[:n], checks
 
 
 def cec_get_cex(ctx, pair_idx: int, num_pis: int) -> np.ndarray:

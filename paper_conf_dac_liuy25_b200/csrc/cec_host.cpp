@@ -1682,6 +1682,24 @@ cec_status cec_check_local_cuts(cec_ctx *c, uint32_t n, const uint32_t *la, cons
                                 const uint32_t *cut_off, const uint32_t *leaves, int32_t *verdict) {
     if (!c || (n && (!la || !lb || !cut_off || !verdict))) return fail(c, CEC_E_ARG, "null argument");
     if (c->host_only) return fail(c, CEC_E_CUDA, "host-only context: no CUDA device (no CPU fallback)");
+    std::unique_ptr<cec_plan> P;
+    uint32_t bad = 0, first_bad = 0;
+    cec_status st = local_checks_launch(c, n, la, lb, cut_off, leaves, P, &bad, &first_bad);
+    if (st != CEC_OK) return st;
+    st = local_checks_collect(c, P.get(), verdict);
+    if (st != CEC_OK) return st;
+    if (bad) return fail(c, CEC_E_CUT, "check %u: leaves are not a cut of the pair (%u bad checks)", first_bad, bad);
+    return CEC_OK;
+}
+
+}  // extern "C"
+
+// a12 split in two so a caller can overlap host work with the checks on the GPU (the Alg. 2 pass
+// of cuts.cpp flushes its common-cut buffer through these): validate + plan + upload + launch
+// (asynchronous on the context stream), then collect (wait, read back, free the device block).
+cec_status local_checks_launch(cec_ctx *c, uint32_t n, const uint32_t *la, const uint32_t *lb, const uint32_t *cut_off,
+                               const uint32_t *leaves, std::unique_ptr<cec_plan> &out, uint32_t *bad_out,
+                               uint32_t *first_bad_out) {
     auto t0 = std::chrono::steady_clock::now();
     std::unique_ptr<cec_plan> P(new (std::nothrow) cec_plan());
     if (!P) return CEC_E_NOMEM;
@@ -1745,11 +1763,18 @@ cec_status cec_check_local_cuts(cec_ctx *c, uint32_t n, const uint32_t *la, cons
     c->stats.host_prep_ms = P->host_ms;
     st = upload(c, P.get());
     if (st == CEC_OK && !P->cmps.empty()) st = cec_plan_run(c, P.get());
-    if (st == CEC_OK) st = cec_plan_results(c, P.get(), verdict, nullptr, nullptr);
-    free_dev(P.get());
-    if (st != CEC_OK) return st;
-    if (bad) return fail(c, CEC_E_CUT, "check %u: leaves are not a cut of the pair (%u bad checks)", first_bad, bad);
+    if (st != CEC_OK) {
+        free_dev(P.get());
+        return st;
+    }
+    if (bad_out) *bad_out = bad;
+    if (first_bad_out) *first_bad_out = first_bad;
+    out = std::move(P);
     return CEC_OK;
 }
 
-}  // extern "C"
+cec_status local_checks_collect(cec_ctx *c, cec_plan *P, int32_t *verdict) {
+    cec_status st = cec_plan_results(c, P, verdict, nullptr, nullptr);
+    free_dev(P);
+    return st;
+}

@@ -17,6 +17,10 @@
 // This is the host-minimal stand-in for the paper's GPU cut generator;
 // the checks themselves run on the GPU through cec_check_local_cuts.
 #include <algorithm>
+#include <atomic>
+#include <functional>
+#include <memory>
+#include <thread>
 #include <cstdint>
 #include <cstdlib>
 #include <cstring>
@@ -127,6 +131,129 @@ bool table1_less(const Cut &a, const Cut &b, int pass) {
     return std::lexicographical_compare(a.leaf, a.leaf + a.n, b.leaf, b.leaf + b.n);
 }
 
+Cut trivial_cut(uint32_t id) {  // the constant needs no leaf: its cut is empty
+    Cut t;
+    if (id == 0) return t;
+    t.n = 1;
+    t.leaf[0] = id;
+    t.sig = bit_of(id);
+    return t;
+}
+
+struct CutJob {  // shared, read-only inputs of the per-node enumeration
+    const cec_ctx *c;
+    const std::vector<uint32_t> *fanout, *repr_of;
+    uint32_t k_l, C;
+    int pass;
+};
+
+// P(id) from P(fanins) (and P(repr) for a member): Eq. (1), dominance, Table I / similarity order.
+void node_cuts(const CutJob &J, uint32_t id, std::vector<std::vector<Cut>> &P) {
+    const cec_ctx *c = J.c;
+    const uint32_t a = c->f0[id] >> 1, b = c->f1[id] >> 1;
+    std::vector<Cut> ua(P[a]), vb(P[b]);
+    ua.push_back(trivial_cut(a));
+    vb.push_back(trivial_cut(b));
+    std::vector<Cut> E;
+    Cut m;
+    for (const Cut &u : ua)
+        for (const Cut &v : vb)
+            if (merge(u.leaf, u.n, v.leaf, v.n, (int)J.k_l, m)) {
+                if (m.n == 0 || (m.n == 1 && m.leaf[0] == id)) continue;
+                E.push_back(m);
+            }
+    // dedupe + drop dominated: process by size, keep a cut unless a kept cut is its subset
+    std::sort(E.begin(), E.end(), [](const Cut &x, const Cut &y) {
+        if (x.n != y.n) return x.n < y.n;
+        return std::lexicographical_compare(x.leaf, x.leaf + x.n, y.leaf, y.leaf + y.n);
+    });
+    std::vector<Cut> kept;
+    for (const Cut &x : E) {
+        bool dom = false;
+        for (const Cut &k : kept)
+            if (same(k, x) || subset(k, x)) {
+                dom = true;
+                break;
+            }
+        if (!dom) kept.push_back(x);
+    }
+    for (Cut &x : kept) {
+        x.sum_fanout = x.sum_level = 0;
+        for (int t = 0; t < x.n; ++t) {
+            x.sum_fanout += (*J.fanout)[x.leaf[t]];
+            x.sum_level += c->level[x.leaf[t]];
+        }
+        x.sim = 0;
+    }
+    const uint32_t r = (*J.repr_of)[id];
+    if (r != 0xFFFFFFFFu && !P[r].empty()) {
+        static const unsigned __int128 L = lcm_upto(2 * KMAX);
+        for (Cut &x : kept) {
+            unsigned __int128 sv = 0;
+            for (const Cut &y : P[r]) {
+                const int in = inter(x, y);
+                sv += (unsigned __int128)in * (L / (unsigned __int128)(x.n + y.n - in));
+            }
+            x.sim = sv;
+        }
+        std::sort(kept.begin(), kept.end(), [&](const Cut &x, const Cut &y) {
+            if (x.sim != y.sim) return x.sim > y.sim;
+            return table1_less(x, y, J.pass);
+        });
+    } else {
+        std::sort(kept.begin(), kept.end(), [&](const Cut &x, const Cut &y) { return table1_less(x, y, J.pass); });
+    }
+    if (kept.size() > J.C) kept.resize(J.C);
+    P[id].swap(kept);
+}
+
+// common cuts u|v of a pair (no trivial cuts, <= k_l leaves), smallest first, at most max_cuts
+void common_cuts_of(const std::vector<std::vector<Cut>> &P, uint32_t r, uint32_t mbr, uint32_t k_l, uint32_t max_cuts,
+                    std::vector<Cut> &common) {
+    common.clear();
+    Cut m;
+    for (const Cut &u : P[r])
+        for (const Cut &v : P[mbr])
+            if (merge(u.leaf, u.n, v.leaf, v.n, (int)k_l, m) && m.n > 0) common.push_back(m);
+    std::sort(common.begin(), common.end(), [](const Cut &x, const Cut &y) {
+        if (x.n != y.n) return x.n < y.n;
+        return std::lexicographical_compare(x.leaf, x.leaf + x.n, y.leaf, y.leaf + y.n);
+    });
+    common.erase(std::unique(common.begin(), common.end(), same), common.end());
+    if (common.size() > max_cuts) common.resize(max_cuts);
+}
+
+// fanouts over the whole AIG (Table I metric), the TFI of the pair nodes (need), repr_of[member]
+void cut_inputs(const cec_ctx *c, uint32_t npairs, const uint32_t *repr, const uint32_t *member,
+                std::vector<uint32_t> &fanout, std::vector<uint8_t> &need, std::vector<uint32_t> &repr_of) {
+    const uint32_t N = c->N();
+    fanout.assign(N, 0);
+    for (uint32_t id = c->I + 1; id < N; ++id) {
+        ++fanout[c->f0[id] >> 1];
+        ++fanout[c->f1[id] >> 1];
+    }
+    need.assign(N, 0);
+    std::vector<uint32_t> st;
+    for (uint32_t q = 0; q < npairs; ++q)
+        for (uint32_t r : {repr[q], member[q]})
+            if (!need[r]) {
+                need[r] = 1;
+                st.push_back(r);
+            }
+    while (!st.empty()) {
+        const uint32_t v = st.back();
+        st.pop_back();
+        if (v <= c->I) continue;
+        for (uint32_t f : {c->f0[v] >> 1, c->f1[v] >> 1})
+            if (!need[f]) {
+                need[f] = 1;
+                st.push_back(f);
+            }
+    }
+    repr_of.assign(N, 0xFFFFFFFFu);
+    for (uint32_t q = 0; q < npairs; ++q) repr_of[member[q]] = repr[q];
+}
+
 }  // namespace
 
 extern "C" cec_status cec_common_cuts(cec_ctx *c, uint32_t npairs, const uint32_t *repr, const uint32_t *member,
@@ -138,35 +265,9 @@ extern "C" cec_status cec_common_cuts(cec_ctx *c, uint32_t npairs, const uint32_
     const uint32_t N = c->N();
     for (uint32_t q = 0; q < npairs; ++q)
         if (repr[q] >= N || member[q] >= N || repr[q] >= member[q]) return CEC_E_ARG;
-    // levels and fanouts over the whole AIG (Table I metrics)
-    std::vector<uint32_t> fanout(N, 0);
-    for (uint32_t id = c->I + 1; id < N; ++id) {
-        ++fanout[c->f0[id] >> 1];
-        ++fanout[c->f1[id] >> 1];
-    }
-    // nodes that need cuts: the TFI of every pair node
-    std::vector<uint8_t> need(N, 0);
-    {
-        std::vector<uint32_t> st;
-        for (uint32_t q = 0; q < npairs; ++q)
-            for (uint32_t r : {repr[q], member[q]})
-                if (!need[r]) {
-                    need[r] = 1;
-                    st.push_back(r);
-                }
-        while (!st.empty()) {
-            const uint32_t v = st.back();
-            st.pop_back();
-            if (v <= c->I) continue;
-            for (uint32_t f : {c->f0[v] >> 1, c->f1[v] >> 1})
-                if (!need[f]) {
-                    need[f] = 1;
-                    st.push_back(f);
-                }
-        }
-    }
-    std::vector<uint32_t> repr_of(N, 0xFFFFFFFFu);
-    for (uint32_t q = 0; q < npairs; ++q) repr_of[member[q]] = repr[q];
+    std::vector<uint32_t> fanout, repr_of;
+    std::vector<uint8_t> need;
+    cut_inputs(c, npairs, repr, member, fanout, need, repr_of);
     size_t n_need = 0;
     for (uint32_t id = c->I + 1; id < N; ++id) n_need += need[id];
     // GPU generator for large cones (one launch per enumeration level pays off only at scale);
@@ -211,96 +312,207 @@ extern "C" cec_status cec_common_cuts(cec_ctx *c, uint32_t npairs, const uint32_
         return CEC_OK;
     }
     std::vector<std::vector<Cut>> P(N);
-    auto trivial = [&](uint32_t id) {  // the constant needs no leaf: its cut is empty
-        Cut t;
-        if (id == 0) return t;
-        t.n = 1;
-        t.leaf[0] = id;
-        t.sig = bit_of(id);
-        return t;
-    };
     for (uint32_t id = 1; id <= c->I; ++id)
-        if (need[id]) P[id].push_back(trivial(id));
-    if (need[0]) P[0].push_back(trivial(0));
-    std::vector<Cut> E;
-    for (uint32_t id = c->I + 1; id < N; ++id) {
-        if (!need[id]) continue;
-        const uint32_t a = c->f0[id] >> 1, b = c->f1[id] >> 1;
-        std::vector<Cut> ua(P[a]), vb(P[b]);
-        ua.push_back(trivial(a));
-        vb.push_back(trivial(b));
-        E.clear();
-        Cut m;
-        for (const Cut &u : ua)
-            for (const Cut &v : vb)
-                if (merge(u.leaf, u.n, v.leaf, v.n, (int)k_l, m)) {
-                    if (m.n == 0 || (m.n == 1 && m.leaf[0] == id)) continue;
-                    E.push_back(m);
-                }
-        // dedupe + drop dominated: process by size, keep a cut unless a kept cut is its subset
-        std::sort(E.begin(), E.end(), [](const Cut &x, const Cut &y) {
-            if (x.n != y.n) return x.n < y.n;
-            return std::lexicographical_compare(x.leaf, x.leaf + x.n, y.leaf, y.leaf + y.n);
-        });
-        std::vector<Cut> kept;
-        for (const Cut &x : E) {
-            bool dom = false;
-            for (const Cut &k : kept)
-                if (same(k, x) || subset(k, x)) {
-                    dom = true;
-                    break;
-                }
-            if (!dom) kept.push_back(x);
-        }
-        for (Cut &x : kept) {
-            x.sum_fanout = x.sum_level = 0;
-            for (int t = 0; t < x.n; ++t) {
-                x.sum_fanout += fanout[x.leaf[t]];
-                x.sum_level += c->level[x.leaf[t]];
-            }
-            x.sim = 0;
-        }
-        const uint32_t r = repr_of[id];
-        if (r != 0xFFFFFFFFu && !P[r].empty()) {
-            static const unsigned __int128 L = lcm_upto(2 * KMAX);
-            for (Cut &x : kept) {
-                unsigned __int128 s = 0;
-                for (const Cut &y : P[r]) {
-                    const int in = inter(x, y);
-                    s += (unsigned __int128)in * (L / (unsigned __int128)(x.n + y.n - in));
-                }
-                x.sim = s;
-            }
-            std::sort(kept.begin(), kept.end(), [&](const Cut &x, const Cut &y) {
-                if (x.sim != y.sim) return x.sim > y.sim;
-                return table1_less(x, y, pass_id);
-            });
-        } else {
-            std::sort(kept.begin(), kept.end(), [&](const Cut &x, const Cut &y) { return table1_less(x, y, pass_id); });
-        }
-        if (kept.size() > C) kept.resize(C);
-        P[id].swap(kept);
-    }
+        if (need[id]) P[id].push_back(trivial_cut(id));
+    if (need[0]) P[0].push_back(trivial_cut(0));
+    const CutJob J{c, &fanout, &repr_of, k_l, C, pass_id};
+    for (uint32_t id = c->I + 1; id < N; ++id)
+        if (need[id]) node_cuts(J, id, P);
     // common cuts per pair
     uint32_t ncut = 0, nleaf = 0;
     cut_off[0] = 0;
+    std::vector<Cut> common;
     for (uint32_t q = 0; q < npairs; ++q) {
         pair_cut_off[q] = ncut;
-        std::vector<Cut> common;
-        Cut m;
-        for (const Cut &u : P[repr[q]])
-            for (const Cut &v : P[member[q]])
-                if (merge(u.leaf, u.n, v.leaf, v.n, (int)k_l, m) && m.n > 0) common.push_back(m);
-        std::sort(common.begin(), common.end(), [](const Cut &x, const Cut &y) {
-            if (x.n != y.n) return x.n < y.n;
-            return std::lexicographical_compare(x.leaf, x.leaf + x.n, y.leaf, y.leaf + y.n);
-        });
-        common.erase(std::unique(common.begin(), common.end(), same), common.end());
-        for (size_t i = 0; i < common.size() && i < max_cuts; ++i) {
-            for (int t = 0; t < common[i].n; ++t) leaves[nleaf++] = common[i].leaf[t];
+        common_cuts_of(P, repr[q], member[q], k_l, max_cuts, common);
+        for (const Cut &x : common) {
+            for (int t = 0; t < x.n; ++t) leaves[nleaf++] = x.leaf[t];
             cut_off[++ncut] = nleaf;
         }
     }
     pair_cut_off[npairs] = ncut;
+    return CEC_OK;
+}
+
+// ------------------------------------------------------------------------------------------------
+// Alg. 2: one cut generation + checking pass with a common-cut buffer.
+// Nodes are processed by enumeration level el (Eq. 2: el(PI) = 0, el(n) = 1 + max over the
+// fanins, and above el(repr) for a non-representative), the nodes of one level in parallel on the
+// host threads (they depend only on lower levels). When a member's priority cuts are ready, the
+// common cuts of its pair go into the buffer (Alg. 2 l.11-12); a full buffer is flushed to the
+// local-check kernels (Alg. 2 l.13-18, l.15 "Alg. 1 in local mode"), asynchronously: the GPU checks
+// one buffer while the host enumerates the next levels. Per-pair results equal cec_common_cuts
+// followed by cec_check_local_cuts on the same cuts (the cuts do not depend on the buffering).
+// ------------------------------------------------------------------------------------------------
+namespace {
+
+// persistent worker pool for level-parallel loops (one generation per level, spin + yield)
+struct LevelPool {
+    std::vector<std::thread> th;
+    std::atomic<uint64_t> gen{0};
+    std::atomic<uint32_t> next{0}, busy{0};
+    std::atomic<bool> quit{false};
+    const std::vector<uint32_t> *items = nullptr;
+    std::function<void(uint32_t)> fn;
+    explicit LevelPool(unsigned n) {
+        for (unsigned t = 0; t < n; ++t)
+            th.emplace_back([this]() {
+                uint64_t seen = 0;
+                for (;;) {
+                    uint64_t g;
+                    while ((g = gen.load(std::memory_order_acquire)) == seen) {
+                        if (quit.load(std::memory_order_acquire)) return;
+                        std::this_thread::yield();
+                    }
+                    seen = g;
+                    work();
+                    busy.fetch_sub(1, std::memory_order_acq_rel);
+                }
+            });
+    }
+    void work() {
+        for (uint32_t i; (i = next.fetch_add(1, std::memory_order_relaxed)) < items->size();) fn((*items)[i]);
+    }
+    void run(const std::vector<uint32_t> &v, std::function<void(uint32_t)> f) {
+        if (th.empty() || v.size() < 8) {  // small levels: no hand-off
+            for (uint32_t x : v) f(x);
+            return;
+        }
+        items = &v;
+        fn = std::move(f);
+        next.store(0, std::memory_order_relaxed);
+        busy.store((uint32_t)th.size(), std::memory_order_relaxed);
+        gen.fetch_add(1, std::memory_order_acq_rel);
+        work();
+        while (busy.load(std::memory_order_acquire) != 0) std::this_thread::yield();
+    }
+    ~LevelPool() {
+        quit.store(true, std::memory_order_release);
+        for (auto &t : th) t.join();
+    }
+};
+
+}  // namespace
+
+extern "C" cec_status cec_local_pass(cec_ctx *c, uint32_t npairs, const uint32_t *repr, const uint32_t *member,
+                                     const uint8_t *phase, uint32_t k_l, uint32_t C, int32_t pass_id,
+                                     uint32_t max_cuts, uint32_t buffer_checks, int32_t *verdict_out,
+                                     uint32_t *num_checks_out, uint32_t *check_pair, uint32_t *check_cut_off,
+                                     uint32_t *check_leaves, int32_t *check_verdict) {
+    if (!c || (npairs && (!repr || !member || !phase || !verdict_out)) || !num_checks_out || k_l == 0 || k_l > KMAX ||
+        C == 0 || max_cuts == 0 || pass_id < 0 || pass_id > 2)
+        return CEC_E_ARG;
+    const uint32_t N = c->N();
+    for (uint32_t q = 0; q < npairs; ++q)
+        if (repr[q] >= N || member[q] >= N || repr[q] >= member[q] || member[q] <= c->I) {
+            c->err = "pair " + std::to_string(q) + ": need repr < member and member an AND node";
+            return CEC_E_ARG;
+        }
+    if (c->host_only) {
+        c->err = "host-only context: no CUDA device (no CPU fallback)";
+        return CEC_E_CUDA;
+    }
+    std::vector<uint32_t> fanout, repr_of;
+    std::vector<uint8_t> need;
+    cut_inputs(c, npairs, repr, member, fanout, need, repr_of);
+    // enumeration levels (Eq. 2) of the needed AND nodes
+    std::vector<uint32_t> el(N, 0);
+    std::vector<std::vector<uint32_t>> lists;
+    for (uint32_t id = c->I + 1; id < N; ++id) {
+        if (!need[id]) continue;
+        uint32_t e = 1 + std::max(el[c->f0[id] >> 1], el[c->f1[id] >> 1]);
+        if (repr_of[id] != 0xFFFFFFFFu) e = std::max(e, 1 + el[repr_of[id]]);
+        el[id] = e;
+        if (lists.size() <= e) lists.resize(e + 1);
+        lists[e].push_back(id);
+    }
+    std::vector<std::vector<uint32_t>> pairs_at(lists.size());
+    for (uint32_t q = 0; q < npairs; ++q) pairs_at[el[member[q]]].push_back(q);
+    std::vector<std::vector<Cut>> P(N);
+    for (uint32_t id = 1; id <= c->I; ++id)
+        if (need[id]) P[id].push_back(trivial_cut(id));
+    if (need[0]) P[0].push_back(trivial_cut(0));
+    const CutJob J{c, &fanout, &repr_of, k_l, C, pass_id};
+    const unsigned hw = std::max(1u, std::min(16u, std::thread::hardware_concurrency()));
+    LevelPool pool(hw > 1 ? hw - 1 : 0);
+    for (uint32_t q = 0; q < npairs; ++q) verdict_out[q] = CEC_UNDECIDED;
+    // the buffer: checks (pair, leaves) waiting for a flush; in-flight: one launched flush
+    struct Flush {
+        std::vector<uint32_t> pair, off{0}, leaves, la, lb;
+        std::unique_ptr<cec_plan> plan;
+        std::vector<int32_t> v;
+    };
+    Flush buf, inflight;
+    uint32_t nchecks = 0;
+    std::vector<uint32_t> log_pair, log_off{0}, log_leaves;  // every issued check, in issue order
+    auto collect = [&](Flush &F) -> cec_status {
+        if (!F.plan) return CEC_OK;
+        F.v.assign(F.pair.size(), CEC_UNDECIDED);
+        cec_status st = local_checks_collect(c, F.plan.get(), F.v.data());
+        F.plan.reset();
+        if (st != CEC_OK) return st;
+        for (size_t t = 0; t < F.pair.size(); ++t)
+            if (F.v[t] == CEC_EQUIVALENT) verdict_out[F.pair[t]] = CEC_EQUIVALENT;  // any cut proves the pair
+        return CEC_OK;
+    };
+    std::vector<int32_t> all_v;  // verdicts of every issued check, in issue order
+    auto launch = [&](Flush &F) -> cec_status {
+        if (F.pair.empty()) return CEC_OK;
+        uint32_t bad = 0, first_bad = 0;
+        cec_status st = local_checks_launch(c, (uint32_t)F.pair.size(), F.la.data(), F.lb.data(), F.off.data(),
+                                            F.leaves.data(), F.plan, &bad, &first_bad);
+        if (st != CEC_OK) return st;
+        if (bad) {
+            c->err = "common cut is not a cut (internal error)";
+            return CEC_E_CUT;
+        }
+        return CEC_OK;
+    };
+    auto finish_inflight = [&]() -> cec_status {
+        cec_status st = collect(inflight);
+        if (st != CEC_OK) return st;
+        all_v.insert(all_v.end(), inflight.v.begin(), inflight.v.end());
+        inflight = Flush();
+        return CEC_OK;
+    };
+    auto flush = [&]() -> cec_status {
+        cec_status st = finish_inflight();  // at most one flush in flight
+        if (st != CEC_OK) return st;
+        std::swap(inflight, buf);
+        buf = Flush();
+        return launch(inflight);
+    };
+    std::vector<Cut> common;
+    for (size_t e = 1; e < lists.size(); ++e) {
+        pool.run(lists[e], [&](uint32_t id) { node_cuts(J, id, P); });
+        for (uint32_t q : pairs_at[e]) {  // Alg. 2 l.11-12: common cuts of the new pairs
+            common_cuts_of(P, repr[q], member[q], k_l, max_cuts, common);
+            const uint32_t la = 2u * repr[q], lb = 2u * member[q] ^ (phase[q] & 1u);
+            for (const Cut &x : common) {
+                buf.pair.push_back(q);
+                buf.la.push_back(la);
+                buf.lb.push_back(lb);
+                buf.leaves.insert(buf.leaves.end(), x.leaf, x.leaf + x.n);
+                buf.off.push_back((uint32_t)buf.leaves.size());
+                log_pair.push_back(q);
+                log_leaves.insert(log_leaves.end(), x.leaf, x.leaf + x.n);
+                log_off.push_back((uint32_t)log_leaves.size());
+                ++nchecks;
+            }
+        }
+        if (buf.pair.size() >= std::max<uint32_t>(1, buffer_checks)) {  // Alg. 2 l.13-14: flush
+            cec_status st = flush();
+            if (st != CEC_OK) return st;
+        }
+    }
+    cec_status st = flush();  // Alg. 2 l.18: the remainder
+    if (st == CEC_OK) st = finish_inflight();
+    if (st != CEC_OK) return st;
+    *num_checks_out = nchecks;
+    // optional check log (caller capacities: npairs*max_cuts checks, npairs*max_cuts*k_l leaves)
+    if (check_pair) std::memcpy(check_pair, log_pair.data(), 4 * log_pair.size());
+    if (check_cut_off) std::memcpy(check_cut_off, log_off.data(), 4 * log_off.size());
+    if (check_leaves && !log_leaves.empty()) std::memcpy(check_leaves, log_leaves.data(), 4 * log_leaves.size());
+    if (check_verdict && !all_v.empty()) std::memcpy(check_verdict, all_v.data(), 4 * all_v.size());
     return CEC_OK;
 }

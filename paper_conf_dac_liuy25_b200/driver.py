@@ -40,6 +40,7 @@ class CecParams:
     final_po_check: bool = True  # after the L phases: exhaustive check of undecided POs with k <= k_P
     native_cuts: bool = True     # C++ cut generator (cec_common_cuts); False = the Python reference
     max_cex_patterns: int = 1024  # CEX patterns kept for class refinement
+    buffer_checks: int = 4096     # Alg. 2 common-cut buffer (local checks per flush)
     distance1: bool = True        # also simulate every distance-1 neighbour of each CEX
     device: int = 0
     engine: int = capi.CEC_ENGINE_AUTO
@@ -69,17 +70,22 @@ class Miter:
         self.lit_a = np.asarray(lit_a, dtype=np.uint32).copy()
         self.lit_b = np.asarray(lit_b, dtype=np.uint32).copy()
 
-    def reduce(self, subst: Dict[int, int], device: int = 0) -> Tuple["Miter", np.ndarray]:
+    def reduce(self, subst: Dict[int, int], device: int = 0,
+               ctx: Optional[capi.Context] = None) -> Tuple["Miter", np.ndarray]:
         """Merge proved pairs: node id -> literal of its (lower-id) representative,
-        rebuilt with structural hashing so merged fanouts collapse — on the GPU (cec_reduce).
+        rebuilt with structural hashing so merged fanouts collapse — on the GPU (cec_reduce), with
+        `ctx` (a device context of this miter's AIG) or a temporary one.
         Returns the reduced miter and the image (new literal) of every old node id."""
-        ctx = capi.Context.from_aig(self.aig, device=device)
+        own = ctx is None
+        if own:
+            ctx = capi.Context.from_aig(self.aig, device=device)
         try:
             mem = np.fromiter(subst.keys(), dtype=np.uint32, count=len(subst))
             rep = np.fromiter(subst.values(), dtype=np.uint32, count=len(subst))
             fan, image, lits = ctx.reduce(mem, rep, np.concatenate([self.lit_a, self.lit_b]))
         finally:
-            ctx.close()
+            if own:
+                ctx.close()
         P = self.lit_a.size
         aig = Aig(self.aig.num_pis, np.ascontiguousarray(fan, dtype=np.uint32), lits.astype(np.uint32))
         return Miter(aig, lits[:P], lits[P:]), image
@@ -171,14 +177,6 @@ def enumerate_cuts(aig: Aig, k_l: int, C: int, pass_id: int, repr_of: Optional[D
 # the flow
 # ---------------------------------------------------------------------------------------------
 
-def hctx_support(aig: Aig, la: int, lb: int) -> List[int]:
-    h = capi.Context.from_aig(aig, device=-1, k_max=63)
-    try:
-        return capi.cec_pair_support(h.handle, int(la), int(lb))
-    finally:
-        h.close()
-
-
 def pack_patterns(patterns: List[np.ndarray], num_pis: int) -> np.ndarray:
     """Pack PI assignments (uint8[num_pis] each) into u32 words: pattern j is bit j%32 of word j//32."""
     W = max(1, (len(patterns) + 31) // 32)
@@ -247,7 +245,8 @@ def check_miter(aig: Aig, lit_a, lit_b, params: Optional[CecParams] = None) -> C
             break
         t = time.perf_counter()
         ctx = _ctx(cur.aig, p, p.k_g)
-        lctx = _ctx(cur.aig, p, max(p.k_l, 1))  # local checks: up to k_l leaves
+        # local checks need k_max >= k_l (cut leaves); one context serves both when k_l <= k_g
+        lctx = ctx if p.k_l <= p.k_g else _ctx(cur.aig, p, max(p.k_l, 1))
         # equivalence classes on the GPU: random patterns plus the CEX patterns
         # of disproved pairs, which split their classes
         words = pack_patterns(cex_patterns, cur.aig.num_pis) if cex_patterns else None
@@ -273,7 +272,7 @@ def check_miter(aig: Aig, lit_a, lit_b, params: Optional[CecParams] = None) -> C
                 cx = ctx.get_cex(int(i))
                 cex_patterns.append(cx)
                 if p.distance1:  # distance-1 simulation of the CEX over the pair's support
-                    for pi in hctx_support(cur.aig, la[i], lb[i]):
+                    for pi in capi.cec_pair_support(ctx.handle, la[i], lb[i]):
                         if len(cex_patterns) >= p.max_cex_patterns:
                             break
                         nb = cx.copy()
@@ -294,17 +293,25 @@ def check_miter(aig: Aig, lit_a, lit_b, params: Optional[CecParams] = None) -> C
             todo = [x for x in remaining if x[1] not in subst]
             ql, qm, off, leaves, who = [], [], [0], [], []
             if p.native_cuts and todo:
+                # Alg. 2: level-wise cut enumeration, common-cut buffer flushed
+                # to the local-check kernels while the host enumerates the next levels
                 t1 = time.perf_counter()
-                pco, co, lvs = capi.cec_common_cuts(lctx.handle, [x[0] for x in todo], [x[1] for x in todo],
-                                                     p.k_l, p.C, pass_id, p.max_cuts_per_pair)
+                pv, (cp, cof, cl, cv) = capi.cec_local_pass(
+                    lctx.handle, [x[0] for x in todo], [x[1] for x in todo], [x[2] for x in todo], p.k_l, p.C,
+                    pass_id, p.max_cuts_per_pair, p.buffer_checks)
+                tk["local"] += time.perf_counter() - t1
+                ver = len(versions) - 1
+                for i in range(cp.size):
+                    r, m_, f = todo[int(cp[i])]
+                    checks.append({"version": ver, "phase": phase_no, "pass": pass_id, "lit_a": 2 * r,
+                                   "lit_b": 2 * m_ ^ f, "leaves": cl[cof[i]:cof[i + 1]].tolist(),
+                                   "verdict": int(cv[i])})
                 for i, (r, m_, f) in enumerate(todo):
-                    for ct in range(int(pco[i]), int(pco[i + 1])):
-                        ql.append(2 * r)
-                        qm.append(2 * m_ ^ f)
-                        leaves += [int(x) for x in lvs[co[ct]:co[ct + 1]]]
-                        off.append(len(leaves))
-                        who.append((r, m_, f))
-                tk["cuts"] += time.perf_counter() - t1
+                    if pv[i] == capi.CEC_EQUIVALENT and m_ not in subst:
+                        subst[m_] = 2 * r ^ f
+                        proved_l += 1
+                remaining = [x for x in remaining if x[1] not in subst]
+                continue
             elif todo:
                 repr_of = {m_: r for r, m_, f in todo}
                 cuts = enumerate_cuts(cur.aig, p.k_l, p.C, pass_id, repr_of)
@@ -334,17 +341,21 @@ def check_miter(aig: Aig, lit_a, lit_b, params: Optional[CecParams] = None) -> C
                     subst[m_] = 2 * r ^ f
                     proved_l += 1
             remaining = [x for x in remaining if x[1] not in subst]
-        ctx.close()
-        lctx.close()
         entry = {"phase": f"G+L{phase_no}", "candidates": len(cand), "proved_global": proved_g,
-                 "proved_local": proved_l, "ands": cur.aig.num_ands, "s": time.perf_counter() - t,
+                 "proved_local": proved_l, "ands": cur.aig.num_ands,
                  "s_parts": {k_: round(v_, 4) for k_, v_ in tk.items()}}
         log.append(entry)
+        if subst:
+            t1 = time.perf_counter()
+            nxt, _ = cur.reduce(subst, p.device, ctx=ctx)
+            entry["s_parts"]["reduce"] = round(time.perf_counter() - t1, 4)
+        ctx.close()
+        if lctx is not ctx:
+            lctx.close()
+        entry["s"] = time.perf_counter() - t
         if not subst:
             break  # no progress: undecided remainder
-        t1 = time.perf_counter()
-        cur, _ = cur.reduce(subst, p.device)
-        entry["s_parts"]["reduce"] = round(time.perf_counter() - t1, 4)
+        cur = nxt
     st = po_status(cur)
     po_v = np.where(st == capi.CEC_EQUIVALENT, capi.CEC_EQUIVALENT, po_v)
     cex_vec, cex_pair = None, -1
