@@ -327,6 +327,21 @@ def main():
         cpu = {"value": evals / dt, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": what,
                "seconds": round(dt, 2)}
 
+    # parity against stored oracle results of the same generated miter (tests/golden, written by
+    # scripts/make_golden*.py, which call only oracle/): every pair's verdict, k and canonical CEX
+    parity = None
+    gold_name = {"c5": "c5_big", "c2": "c2_mul12", "c2bug": "c2_mul12_bug1"}.get(args.config)
+    gpath = os.path.join(ROOT, "tests", "golden", f"{gold_name}.json") if gold_name else None
+    if rank == 0 and gpath and os.path.exists(gpath):
+        g = json.load(open(gpath))
+        if g["lit_a"] == [int(x) for x in m.lit_a] and g["lit_b"] == [int(x) for x in m.lit_b]:
+            gv, gk = np.array(g["verdict"]), np.array(g["k"])
+            gc = np.array([int(x) for x in g["cex"]], dtype=np.uint64)
+            neq = gv == capi.CEC_NOT_EQUIVALENT
+            diffs = int((gv != v).sum() + (gk != k).sum() + (neq & (gc != cex)).sum())
+            parity = {"vs": f"tests/golden/{gold_name}.json (oracle/, every pair)", "pairs": int(gv.size),
+                      "diffs": diffs, "ok": diffs == 0}
+
     if rank == 0:
         line = {
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
@@ -340,6 +355,7 @@ def main():
                        "merge": ["off", "paper", "cost-aware"][merge], "engine": engine_name, "jit_kernels": st0["jit_kernels"], "jit_compile_ms": st0["jit_ms"],
                        "verdicts": verdicts},
             "clocks": clocks,
+            "parity": parity,
             "gpu_launches": int(launches_per_step * args.steps),
             "e2e": {"value": W_all / (e2e / 1e3), "unit": UNIT, "ms_per_miter": e2e,
                     "h2d_bytes_per_step": int(st_e2e["h2d_bytes"]), "d2h_bytes_per_step": int(st_e2e["d2h_bytes"]),

@@ -442,3 +442,23 @@ def test_jit_bundles_vs_oracle_and_unbundled(monkeypatch):
     got = ctx3.sim_exhaustive(m.lit_a, m.lit_b)
     for a, b in zip((gv, gc, gk), got):
         assert np.array_equal(a, b)
+
+
+def test_c5_full_vs_stored_oracle():
+    """Full-size C5 (2.1M ANDs, 6320 pairs, 256 windows x 2^24 patterns) in the launch
+    configuration bench.py times, against the oracle's result for EVERY pair
+    (tests/golden/c5_big.json, scripts/make_golden_c5.py: one single-threaded oracle task per copy)."""
+    g = _golden("c5_big")
+    m = c5_big()
+    assert [int(x) for x in m.lit_a] == g["lit_a"] and [int(x) for x in m.lit_b] == g["lit_b"]
+    ctx = gpu_ctx(m.aig)
+    plan = capi.cec_plan_exhaustive(ctx.handle, m.lit_a, m.lit_b)
+    capi.cec_plan_run(ctx.handle, plan)
+    gv, gc, gk = capi.cec_plan_results(ctx.handle, plan, m.num_pairs)
+    capi.cec_plan_free(plan)
+    assert_same(gv, gc, gk, np.array(g["verdict"]), np.array([int(x) for x in g["cex"]], dtype=np.uint64),
+                np.array(g["k"]), "c5 full")
+    orc = Oracle.from_aig(m.aig)
+    for p in np.nonzero(gv == capi.CEC_NOT_EQUIVALENT)[0]:  # each CEX really separates the pair
+        want = orc.cex_vector(int(m.lit_a[p]), int(m.lit_b[p]), int(gc[p]))
+        assert orc.eval_lit(int(m.lit_a[p]), want) != orc.eval_lit(int(m.lit_b[p]), want)
