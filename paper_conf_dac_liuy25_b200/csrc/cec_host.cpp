@@ -711,6 +711,45 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
             for (auto &th : pool) th.join();
         }
     }
+    // Multi-GPU split: a window with at least `world` slices is cut into
+    // contiguous slice ranges, one per rank; a smaller window goes WHOLE to one rank, chosen by
+    // longest-processing-time-first over the node-words of the small windows on top of each rank's
+    // share of the big ones (deterministic: every rank plans the same assignment). The min-reduce
+    // of the results is unchanged: a rank that does not simulate a window reports no mismatch.
+    std::vector<int32_t> owner(wins.size(), -1);
+    if (world > 1) {
+        std::vector<uint64_t> load(world, 0);
+        std::vector<std::pair<uint64_t, uint32_t>> small;
+        for (uint32_t w = 0; w < wins.size(); ++w) {
+            const uint32_t k = (uint32_t)wins[w].inputs.size();
+            const uint64_t ttw = tt_words_of(k), wps = res[w].jit ? 32 : 32 * IV;
+            const uint64_t slices = (ttw + wps - 1) / wps, cost = (uint64_t)res[w].nodes.size() * ttw + 1;
+            if (slices >= (uint64_t)world) {
+                for (int32_t r = 0; r < world; ++r) load[r] += cost / world;
+            } else {
+                small.push_back({cost, w});
+            }
+        }
+        std::stable_sort(small.begin(), small.end(),
+                         [](const std::pair<uint64_t, uint32_t> &a, const std::pair<uint64_t, uint32_t> &b) {
+                             return a.first > b.first;
+                         });
+        for (const auto &sw : small) {
+            int32_t best = 0;
+            for (int32_t r = 1; r < world; ++r)
+                if (load[r] < load[best]) best = r;
+            owner[sw.second] = best;
+            load[best] += sw.first;
+        }
+    }
+    auto win_range = [&](uint32_t w, uint64_t slices, uint64_t *sb, uint64_t *se) {
+        if (owner[w] < 0) {
+            cec_shard_range(slices, rank, world, sb, se);
+        } else {
+            *sb = 0;
+            *se = owner[w] == rank ? slices : 0;
+        }
+    };
     // (3) serial assembly in window order
     for (size_t w = 0; w < wins.size(); ++w) {
         WinHost &W = wins[w];
@@ -755,7 +794,7 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         const uint64_t pats_all = dw.k < 5 ? (1ull << dw.k) : ttw * 32;
         P->W_all += (uint64_t)nodes.size() * pats_all;
         uint64_t sb, se;
-        cec_shard_range(slices, rank, world, &sb, &se);
+        win_range((uint32_t)w, slices, &sb, &se);
         uint64_t wb = sb * wps, we = std::min<uint64_t>(se * wps, ttw);
         uint64_t pats_rank = we > wb ? (dw.k < 5 ? (1ull << dw.k) : (we - wb) * 32) : 0;
         P->W_rank += (uint64_t)nodes.size() * pats_rank;
@@ -951,7 +990,7 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         uint64_t group_slices = 0;
         for (uint32_t w : ws) {
             uint64_t ttw = tt_words_of(P->dwin[w].k), sb, se;
-            cec_shard_range((ttw + wps_of[w] - 1) / wps_of[w], rank, world, &sb, &se);
+            win_range(w, (ttw + wps_of[w] - 1) / wps_of[w], &sb, &se);
             group_slices += se - sb;
         }
         const uint64_t target = (uint64_t)std::max(c->num_sms, 148) * 16 /*resident warps*/ * 8;
@@ -960,7 +999,7 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
             item_slices = std::max<uint64_t>(jit_pass, (item_slices * 16 + jit_pass - 1) / jit_pass * jit_pass);
         for (uint32_t w : ws) {
             uint64_t ttw = tt_words_of(P->dwin[w].k), sb, se;
-            cec_shard_range((ttw + wps_of[w] - 1) / wps_of[w], rank, world, &sb, &se);
+            win_range(w, (ttw + wps_of[w] - 1) / wps_of[w], &sb, &se);
             for (uint64_t s = sb; s < se; s += item_slices) {
                 const uint32_t e = (uint32_t)std::min<uint64_t>(se, s + item_slices);
                 if (jit)

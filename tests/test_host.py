@@ -190,3 +190,24 @@ def test_jit_codegen_compiles_for_sm100a_host_only(monkeypatch):
     plan = capi.cec_plan_exhaustive(ctx2.handle, m.lit_a, m.lit_b)
     assert ctx2.stats()["jit_windows"] == 0
     capi.cec_plan_free(plan)
+
+
+@pytest.mark.parametrize("world", [2, 4, 8])
+def test_small_windows_go_whole_to_one_rank_lpt(world):
+    """SURVEY.md §8(e) "tiny windows": windows with fewer slices than ranks are not split but given
+    whole to one rank by LPT over their node-words, so per-rank work stays balanced; every window's
+    patterns are still covered exactly once (per-rank W adds up to the whole)."""
+    from workloads import circuits
+    m = circuits.c3_rand(n_blocks=40, block_ands=200, num_pis=256, n_internal=300, n_near=8,
+                         k_dist=((40, 10, 14),))
+    Ws = []
+    for r in range(world):
+        ctx = host_ctx(m.aig, rank=r, world=world, engine=capi.CEC_ENGINE_INTERP, merge=capi.CEC_MERGE_OFF)
+        plan = capi.cec_plan_exhaustive(ctx.handle, m.lit_a, m.lit_b)
+        st = ctx.stats()
+        Ws.append(st["node_patterns"])
+        W_all = st["node_patterns_all"]
+        capi.cec_plan_free(plan)
+        ctx.close()
+    assert sum(Ws) == W_all
+    assert max(Ws) <= 1.6 * W_all / world  # balanced (one-rank-takes-all would be `world` x)
