@@ -243,7 +243,10 @@ def combine_shards(results):
 @pytest.mark.parametrize("engine", SHARD_ENGINES)
 def test_shard_emulation_matches_single_gpu(world, engine):
     """rank g of G simulates its slices; min over ranks == the 1-GPU result."""
-    for m in (c2_mul12_bug(seed=1, n=10), c5_big(copies=8, n_random=5, n_bugs=3, rand_pis=16, rand_ands=1500, mul_n=8)):
+    small = circuits.c3_rand(n_blocks=40, block_ands=200, num_pis=256, n_internal=300, n_near=8,
+                             k_dist=((40, 10, 14),))  # windows with fewer slices than ranks: LPT owners
+    for m in (c2_mul12_bug(seed=1, n=10), c5_big(copies=8, n_random=5, n_bugs=3, rand_pis=16, rand_ands=1500, mul_n=8),
+              small):
         ref = gpu_ctx(m.aig, engine=engine).sim_exhaustive(m.lit_a, m.lit_b)
         parts = [gpu_ctx(m.aig, engine=engine, rank=g, world=world).sim_exhaustive(m.lit_a, m.lit_b)
                  for g in range(world)]
