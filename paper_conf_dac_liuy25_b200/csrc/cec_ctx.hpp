@@ -4,8 +4,13 @@
 #include <nccl.h>
 
 #include <algorithm>
+#include <atomic>
+#include <condition_variable>
 #include <cstdint>
+#include <functional>
 #include <memory>
+#include <mutex>
+#include <thread>
 #include <string>
 #include <vector>
 
@@ -52,6 +57,70 @@ struct Scratch {
     }
 };
 
+// Persistent host worker pool of a context (planning, supports, JIT compiles, cut enumeration):
+// threads are created once and sleep on a condition variable between jobs, so a call that plans
+// many small batches (pipelined chunks, Alg. 2 buffer flushes) pays no thread start-up per batch.
+// run(n, fn) calls fn(item, tid) for items 0..n-1; tid in [0, size()] (the caller is the last tid).
+struct WorkPool {
+    std::vector<std::thread> th;
+    std::mutex mu;
+    std::condition_variable cv, done_cv;
+    uint64_t gen = 0;
+    bool quit = false;
+    std::atomic<uint32_t> next{0}, busy{0};
+    uint32_t n = 0;
+    const std::function<void(uint32_t, unsigned)> *fn = nullptr;
+    explicit WorkPool(unsigned workers) {
+        for (unsigned t = 0; t < workers; ++t) th.emplace_back([this, t]() { loop(t); });
+    }
+    unsigned size() const { return (unsigned)th.size(); }
+    void loop(unsigned tid) {
+        uint64_t seen = 0;
+        for (;;) {
+            {
+                std::unique_lock<std::mutex> l(mu);
+                cv.wait(l, [&]() { return quit || gen != seen; });
+                if (quit) return;
+                seen = gen;
+            }
+            work(tid);
+            if (busy.fetch_sub(1, std::memory_order_acq_rel) == 1) {
+                std::lock_guard<std::mutex> l(mu);
+                done_cv.notify_all();
+            }
+        }
+    }
+    void work(unsigned tid) {
+        for (uint32_t i; (i = next.fetch_add(1, std::memory_order_relaxed)) < n;) (*fn)(i, tid);
+    }
+    void run(uint32_t items, const std::function<void(uint32_t, unsigned)> &f) {
+        if (th.empty() || items < 2) {
+            for (uint32_t i = 0; i < items; ++i) f(i, size());
+            return;
+        }
+        {
+            std::lock_guard<std::mutex> l(mu);
+            fn = &f;
+            n = items;
+            next.store(0, std::memory_order_relaxed);
+            busy.store(size(), std::memory_order_relaxed);
+            ++gen;
+        }
+        cv.notify_all();
+        work(size());
+        std::unique_lock<std::mutex> l(mu);
+        done_cv.wait(l, [&]() { return busy.load(std::memory_order_acquire) == 0; });
+    }
+    ~WorkPool() {
+        {
+            std::lock_guard<std::mutex> l(mu);
+            quit = true;
+        }
+        cv.notify_all();
+        for (auto &t : th) t.join();
+    }
+};
+
 struct cec_ctx {
     uint32_t I = 0, A = 0, O = 0;
     std::vector<uint32_t> f0, f1;  // fanin literals indexed by node id (valid for AND ids)
@@ -75,6 +144,15 @@ struct cec_ctx {
     std::shared_ptr<DevPool> devpool;  // plan device blocks + pinned staging (device contexts)
     Scratch scratch;  // for serial host work (supports of single pairs, cut validation)
     std::vector<Scratch> pool;  // one per planning thread, kept across calls (allocated once)
+    std::unique_ptr<WorkPool> wpool;  // persistent host workers (lazy)
+    WorkPool &workers() {
+        if (!wpool) {
+            const unsigned hw = std::max(1u, std::min(32u, std::thread::hardware_concurrency()));
+            wpool.reset(new WorkPool(hw - 1));
+            if (pool.size() < hw) pool.resize(hw);
+        }
+        return *wpool;
+    }
 
     uint32_t N() const { return 1 + I + A; }
     bool is_and(uint32_t id) const { return id > I; }

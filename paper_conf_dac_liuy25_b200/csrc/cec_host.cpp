@@ -694,22 +694,11 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
             R.key = jit_key(jp);
         }
     };
-    {
-        const unsigned hw = std::max(1u, std::min(32u, std::thread::hardware_concurrency()));
-        const unsigned nt = (unsigned)std::min<size_t>(hw, std::max<size_t>(1, wins.size() / 2));
-        if (nt <= 1) {
-            for (size_t w = 0; w < wins.size(); ++w) plan_one(w, c->scratch);
-        } else {
-            std::atomic<size_t> next{0};
-            std::vector<std::thread> pool;
-            if (c->pool.size() < nt) c->pool.resize(nt);
-            for (unsigned t = 0; t < nt; ++t)
-                pool.emplace_back([&, t]() {
-                    Scratch &X = c->pool[t];  // persistent per-thread scratch (no per-call allocation)
-                    for (size_t w; (w = next.fetch_add(1)) < wins.size();) plan_one(w, X);
-                });
-            for (auto &th : pool) th.join();
-        }
+    if (wins.size() < 2) {
+        for (size_t w = 0; w < wins.size(); ++w) plan_one(w, c->scratch);
+    } else {  // persistent per-thread scratch (no per-call allocation), persistent workers
+        WorkPool &wp = c->workers();
+        wp.run((uint32_t)wins.size(), [&](uint32_t w, unsigned tid) { plan_one(w, c->pool[tid]); });
     }
     // Multi-GPU split: a window with at least `world` slices is cut into
     // contiguous slice ranges, one per rank; a smaller window goes WHOLE to one rank, chosen by
@@ -926,18 +915,10 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         for (size_t u = 0; u < units.size(); ++u)
             for (uint32_t i : units[u]) uprogs[u].push_back(&jit_progs[i]);
         // compile (CPU-heavy, thread-safe) in parallel without loading, then load serially
-        const unsigned hw = std::max(1u, std::min(16u, std::thread::hardware_concurrency()));
-        std::vector<std::thread> pool;
-        std::atomic<size_t> next{0};
-        for (unsigned t = 0; t < std::min<size_t>(hw, units.size()); ++t)
-            pool.emplace_back([&]() {
-                for (size_t i; (i = next.fetch_add(1)) < units.size();)
-                {
-                    const char *e = jit_get_unit(uprogs[i], jcfg, false, &kernels[i]);
-                    if (e) errs[i] = e;
-                }
-            });
-        for (auto &th : pool) th.join();
+        c->workers().run((uint32_t)units.size(), [&](uint32_t i, unsigned) {
+            const char *e = jit_get_unit(uprogs[i], jcfg, false, &kernels[i]);
+            if (e) errs[i] = e;
+        });
         for (size_t i = 0; i < units.size(); ++i) {
             if (!errs[i].empty()) return fail(c, CEC_E_CUDA, "JIT: %s", errs[i].c_str());
             if (load) {
@@ -1184,10 +1165,9 @@ static cec_status plan_route(cec_ctx *c, uint32_t n, const uint32_t *la, const u
         tm.lap("supports (gpu)");
     }
     if (std::find(need_walk.begin(), need_walk.end(), (uint8_t)1) != need_walk.end()) {
-        const unsigned hw = std::max(1u, std::min(16u, std::thread::hardware_concurrency()));
-        const unsigned nt = (unsigned)std::min<uint64_t>(hw, (n + 63) / 64);
+        WorkPool &wp = c->workers();
+        const unsigned nt = (unsigned)std::min<uint64_t>(wp.size() + 1, (n + 63) / 64);
         std::atomic<uint32_t> next{0};
-        if (c->pool.size() < nt + 1) c->pool.resize(nt + 1);
         auto work = [&](unsigned tid) {
             Scratch &X = c->pool[tid];
             X.init(c->N());
@@ -1227,11 +1207,9 @@ static cec_status plan_route(cec_ctx *c, uint32_t n, const uint32_t *la, const u
             }
         };
         if (nt <= 1) {
-            work(0);
+            work(wp.size());
         } else {
-            std::vector<std::thread> pool;
-            for (unsigned t = 0; t < nt; ++t) pool.emplace_back(work, t);
-            for (auto &th : pool) th.join();
+            wp.run(nt, [&](uint32_t, unsigned tid) { work(tid); });
         }
     }
     tm.lap("supports");
@@ -1525,13 +1503,19 @@ cec_status cec_sim_exhaustive(cec_ctx *c, uint32_t n, const uint32_t *la, const 
         wcost[w] = std::ldexp(1.0, (int)k) * (double)(1 + std::max<uint64_t>(wins[w].est_nodes, wins[w].cmps.size()));
         total += wcost[w];
     }
-    std::vector<size_t> cut{0};  // contiguous window ranges of about equal cost; the first chunk is
-    {                            // half-size so the GPU starts early
-        double acc = 0;
-        const double unit = total / (K - 0.5);
+    // contiguous window ranges growing geometrically (4%, 8%, 16%, ... of the cost): the GPU starts
+    // after planning a small first chunk, and each chunk's kernels (~2x the host time to plan the
+    // same windows) cover the planning of the next, twice as large, chunk
+    std::vector<size_t> cut{0};
+    {
+        double acc = 0, chunk = K > 1 ? 0.04 * total : total, target = chunk;
         for (size_t w = 0; w < wins.size(); ++w) {
             acc += wcost[w];
-            if ((int)cut.size() < K && acc >= unit * ((double)cut.size() - 0.5) && w + 1 < wins.size()) cut.push_back(w + 1);
+            if (K > 1 && acc >= target && w + 1 < wins.size()) {
+                cut.push_back(w + 1);
+                chunk *= 2.0;
+                target = acc + chunk;
+            }
         }
         cut.push_back(wins.size());
     }

@@ -344,56 +344,6 @@ extern "C" cec_status cec_common_cuts(cec_ctx *c, uint32_t npairs, const uint32_
 // one buffer while the host enumerates the next levels. Per-pair results equal cec_common_cuts
 // followed by cec_check_local_cuts on the same cuts (the cuts do not depend on the buffering).
 // ------------------------------------------------------------------------------------------------
-namespace {
-
-// persistent worker pool for level-parallel loops (one generation per level, spin + yield)
-struct LevelPool {
-    std::vector<std::thread> th;
-    std::atomic<uint64_t> gen{0};
-    std::atomic<uint32_t> next{0}, busy{0};
-    std::atomic<bool> quit{false};
-    const std::vector<uint32_t> *items = nullptr;
-    std::function<void(uint32_t)> fn;
-    explicit LevelPool(unsigned n) {
-        for (unsigned t = 0; t < n; ++t)
-            th.emplace_back([this]() {
-                uint64_t seen = 0;
-                for (;;) {
-                    uint64_t g;
-                    while ((g = gen.load(std::memory_order_acquire)) == seen) {
-                        if (quit.load(std::memory_order_acquire)) return;
-                        std::this_thread::yield();
-                    }
-                    seen = g;
-                    work();
-                    busy.fetch_sub(1, std::memory_order_acq_rel);
-                }
-            });
-    }
-    void work() {
-        for (uint32_t i; (i = next.fetch_add(1, std::memory_order_relaxed)) < items->size();) fn((*items)[i]);
-    }
-    void run(const std::vector<uint32_t> &v, std::function<void(uint32_t)> f) {
-        if (th.empty() || v.size() < 8) {  // small levels: no hand-off
-            for (uint32_t x : v) f(x);
-            return;
-        }
-        items = &v;
-        fn = std::move(f);
-        next.store(0, std::memory_order_relaxed);
-        busy.store((uint32_t)th.size(), std::memory_order_relaxed);
-        gen.fetch_add(1, std::memory_order_acq_rel);
-        work();
-        while (busy.load(std::memory_order_acquire) != 0) std::this_thread::yield();
-    }
-    ~LevelPool() {
-        quit.store(true, std::memory_order_release);
-        for (auto &t : th) t.join();
-    }
-};
-
-}  // namespace
-
 extern "C" cec_status cec_local_pass(cec_ctx *c, uint32_t npairs, const uint32_t *repr, const uint32_t *member,
                                      const uint8_t *phase, uint32_t k_l, uint32_t C, int32_t pass_id,
                                      uint32_t max_cuts, uint32_t buffer_checks, int32_t *verdict_out,
@@ -433,8 +383,7 @@ extern "C" cec_status cec_local_pass(cec_ctx *c, uint32_t npairs, const uint32_t
         if (need[id]) P[id].push_back(trivial_cut(id));
     if (need[0]) P[0].push_back(trivial_cut(0));
     const CutJob J{c, &fanout, &repr_of, k_l, C, pass_id};
-    const unsigned hw = std::max(1u, std::min(16u, std::thread::hardware_concurrency()));
-    LevelPool pool(hw > 1 ? hw - 1 : 0);
+    WorkPool &pool = c->workers();
     for (uint32_t q = 0; q < npairs; ++q) verdict_out[q] = CEC_UNDECIDED;
     // the buffer: checks (pair, leaves) waiting for a flush; in-flight: one launched flush
     struct Flush {
@@ -484,7 +433,12 @@ extern "C" cec_status cec_local_pass(cec_ctx *c, uint32_t npairs, const uint32_t
     };
     std::vector<Cut> common;
     for (size_t e = 1; e < lists.size(); ++e) {
-        pool.run(lists[e], [&](uint32_t id) { node_cuts(J, id, P); });
+        const std::vector<uint32_t> &L = lists[e];
+        if (L.size() < 8) {  // small levels: no hand-off
+            for (uint32_t id : L) node_cuts(J, id, P);
+        } else {
+            pool.run((uint32_t)L.size(), [&](uint32_t i, unsigned) { node_cuts(J, L[i], P); });
+        }
         for (uint32_t q : pairs_at[e]) {  // Alg. 2 l.11-12: common cuts of the new pairs
             common_cuts_of(P, repr[q], member[q], k_l, max_cuts, common);
             const uint32_t la = 2u * repr[q], lb = 2u * member[q] ^ (phase[q] & 1u);
