@@ -46,12 +46,30 @@ def main():
     V, X, K = [None] * P, [None] * P, [None] * P
     evals, cpu_s = 0, 0.0
     t0 = time.time()
-    with mp.Pool(procs, initializer=_init) as pool:
-        for i, (c, off, v, cex, k, ev, dt) in enumerate(pool.imap_unordered(_copy, range(ncopy))):
+    # per-copy checkpoint (resumable: a restarted run skips the copies already in it)
+    part = os.path.join(ROOT, "tests", "golden", "c5_big.partial.jsonl")
+    done = set()
+    if os.path.exists(part):
+        with open(part) as fh:
+            for line in fh:
+                if not line.strip():
+                    continue
+                r = json.loads(line)
+                c, off, v, cex, k = r["copy"], r["off"], r["v"], r["cex"], r["k"]
+                V[off:off + len(v)], X[off:off + len(v)], K[off:off + len(v)] = v, cex, k
+                evals += r["ev"]
+                cpu_s += r["dt"]
+                done.add(c)
+    todo = [c for c in range(ncopy) if c not in done]
+    with mp.Pool(procs, initializer=_init) as pool, open(part, "a") as pf:
+        for i, (c, off, v, cex, k, ev, dt) in enumerate(pool.imap_unordered(_copy, todo)):
             V[off:off + len(v)], X[off:off + len(v)], K[off:off + len(v)] = v, cex, k
             evals += ev
             cpu_s += dt
-            print(f"copy {c} done ({i + 1}/{ncopy}) {dt:.1f}s", file=sys.stderr, flush=True)
+            pf.write(json.dumps({"copy": c, "off": off, "v": v, "cex": cex, "k": k,
+                                 "ev": ev, "dt": round(dt, 2)}) + "\n")
+            pf.flush()
+            print(f"copy {c} done ({len(done) + i + 1}/{ncopy}) {dt:.1f}s", file=sys.stderr, flush=True)
     out = {
         "_about": "oracle/ results for every pair of workloads.c5_big() (defaults); written by "
                   "scripts/make_golden_c5.py (one single-threaded oracle task per copy)",
@@ -64,6 +82,7 @@ def main():
     }
     with open(os.path.join(ROOT, "tests", "golden", "c5_big.json"), "w") as fh:
         json.dump(out, fh)
+    os.remove(part)
 
 
 if __name__ == "__main__":
