@@ -196,6 +196,8 @@ def main():
     ap.add_argument("--cpu-log2-patterns", type=int, default=19)
     ap.add_argument("--ref-log2-patterns", type=int, default=17)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--reduce", default="peer", choices=["peer", "nccl"],
+                    help="N > 1: a10 over NVLink peer memory fused into the compare path (default) or ncclAllReduce")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
@@ -228,6 +230,31 @@ def main():
     ctx = capi.Context.from_aig(m.aig, device=local, rank=rank, world=world, stream=stream.cuda_stream,
                                 engine=args.engine, merge=merge, nccl_unique_id=uid)
     load_ms = 1e3 * (time.perf_counter() - t_load)
+    reduce_mode = "nccl all-reduce (min)" if world > 1 else "none (1 GPU)"
+    if world > 1 and args.reduce == "peer":
+        # a10 over peer memory (include/cec.h cec_peer_export/import): IPC blobs all-gathered here
+        def all_gather(blob):
+            out = [None] * world
+            dist.all_gather_object(out, blob)
+            return out
+
+        try:
+            ctx.peer_connect(all_gather)
+            ok = 1
+        except capi.CecError as e:
+            ok, why = 0, str(e)
+        t = torch.tensor([ok], device="cuda", dtype=torch.int32)
+        dist.all_reduce(t, op=dist.ReduceOp.MIN)  # all ranks take the same path
+        if int(t.item()) == 1:
+            reduce_mode = "peer memory (NVLink, fused atomicMin into rank 0's home arrays + device barriers)"
+        else:  # a context that imported keeps peer mode: rebuild every rank's context on NCCL
+            ctx.close()
+            obj = [capi.cec_nccl_unique_id() if rank == 0 else None]  # a fresh communicator id
+            dist.broadcast_object_list(obj, src=0)
+            uid = obj[0]
+            ctx = capi.Context.from_aig(m.aig, device=local, rank=rank, world=world, stream=stream.cuda_stream,
+                                        engine=args.engine, merge=merge, nccl_unique_id=uid)
+            reduce_mode = "nccl all-reduce (min); peer setup failed" + (f": {why}" if not ok else " on a peer rank")
     plan = capi.cec_plan_exhaustive(ctx.handle, m.lit_a, m.lit_b)
     info = capi.cec_plan_info(plan)
     st0 = ctx.stats()
@@ -350,7 +377,7 @@ def main():
             "config": {"workload": args.config, "description": desc, "ands": int(m.aig.num_ands),
                        "pairs": int(m.num_pairs), "windows": info["num_windows"], "max_k": info["max_k"],
                        "max_slots": info["max_slots"], "node_patterns_per_step": W_all,
-                       "parallelism": f"pattern-space shards x{world}" + (" + NCCL min all-reduce" if world > 1 else ""),
+                       "parallelism": f"pattern-space shards x{world}", "cross_gpu_reduce": reduce_mode,
                        "l2": "flushed between timed steps (256 MiB write, outside the events)",
                        "merge": ["off", "paper", "cost-aware"][merge], "engine": engine_name, "jit_kernels": st0["jit_kernels"], "jit_compile_ms": st0["jit_ms"],
                        "verdicts": verdicts},

@@ -268,6 +268,29 @@ cec_status cec_get_stats(cec_ctx *ctx, cec_stats *stats);
  * unavailable. */
 cec_status cec_nccl_unique_id(void *out128);
 
+/* Cross-GPU reduction over NVLink peer memory instead of NCCL (SURVEY.md §8(e) "B200-native
+ * option", §8(f) NEXT-4): the a10 min-reduction of first_idx fused into the compare path, with
+ * cross-GPU bounded early exit (Q9).
+ * Setup is collective over the `world` ranks of contexts loaded with the same opts.world (2..8):
+ *   1. every rank calls cec_peer_export: allocates its exchange block (~11 MB of device memory:
+ *      arrival slots, and home arrays for up to 2^20 compares and 2^18 windows per run) and writes a
+ *      CEC_PEER_BLOB_BYTES blob (CUDA IPC handle, pid, device, rank) into blob_out;
+ *   2. the caller all-gathers the blobs in rank order (e.g. torch.distributed.all_gather_object);
+ *   3. every rank calls cec_peer_import with the world blobs (world x 128 bytes, rank order): peer
+ *      blocks of other processes are mapped with CUDA IPC, blocks of the same process used directly.
+ * From then on every cec_plan_run / cec_sim_exhaustive / cec_check_local_cuts of this context runs
+ * in peer mode: rank 0's block is the home of the run's first-mismatch indices, bounds and counters;
+ * every rank's window kernels update it with system-scope atomics on the (rare) mismatch path and
+ * read its bounds for early exit; device-side barriers (one-warp kernels, no host round trip; CUDA
+ * graph safe) order reset -> kernels -> gather -> next run. Results are identical to the NCCL path
+ * (the same per-pair minimum index) and identical on every rank. Every rank must issue the same
+ * sequence of runs (SPMD, as for NCCL). A barrier that waits more than 10 s for a peer sets an error
+ * flag instead of hanging: the call returns CEC_E_NCCL. The paper's SIMT engine keeps NCCL.
+ * Errors: CEC_E_ARG (world outside 2..8, blob mismatch), CEC_E_CUDA (allocation / IPC failure). */
+#define CEC_PEER_BLOB_BYTES 128
+cec_status cec_peer_export(cec_ctx *ctx, void *blob_out);
+cec_status cec_peer_import(cec_ctx *ctx, const void *blobs);
+
 /* Host utility exported for tests: the contiguous slice range [*begin, *end) of `n` slices that
  * rank `rank` of `world` simulates (pattern-space sharding). */
 void cec_shard_range(uint64_t n, int32_t rank, int32_t world, uint64_t *begin, uint64_t *end);

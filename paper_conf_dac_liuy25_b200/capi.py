@@ -28,7 +28,8 @@ EXPORTS = ["cec_default_opts", "cec_load_aig", "cec_sim_exhaustive", "cec_check_
            "cec_pair_support", "cec_plan_exhaustive", "cec_plan_run", "cec_plan_results", "cec_plan_info",
            "cec_plan_window", "cec_plan_free", "cec_stream", "cec_get_stats", "cec_shard_range", "cec_pext64",
            "cec_free", "cec_last_error", "cec_abi_version", "cec_nccl_unique_id", "cec_sim_random",
-           "cec_common_cuts", "cec_sim_patterns", "cec_reduce", "cec_sim_classes", "cec_local_pass"]
+           "cec_common_cuts", "cec_sim_patterns", "cec_reduce", "cec_sim_classes", "cec_local_pass",
+           "cec_peer_export", "cec_peer_import"]
 
 
 class CecOpts(ctypes.Structure):
@@ -87,6 +88,8 @@ def _load() -> ctypes.CDLL:
         "cec_last_error": (ctypes.c_char_p, [P]),
         "cec_abi_version": (ctypes.c_int, []),
         "cec_nccl_unique_id": (ctypes.c_int, [P]),
+        "cec_peer_export": (ctypes.c_int, [P, P]),
+        "cec_peer_import": (ctypes.c_int, [P, P]),
         "cec_sim_random": (ctypes.c_int, [P, u32, u64, P, P]),
         "cec_common_cuts": (ctypes.c_int, [P, u32, P, P, u32, u32, i32, u32, P, P, P]),
         "cec_sim_patterns": (ctypes.c_int, [P, u32, P, P, P]),
@@ -337,6 +340,24 @@ def cec_nccl_unique_id() -> bytes:
     return buf.raw
 
 
+PEER_BLOB_BYTES = 128
+
+
+def cec_peer_export(ctx) -> bytes:
+    """This rank's exchange-block blob (CUDA IPC handle + pid/device/rank), include/cec.h."""
+    buf = ctypes.create_string_buffer(PEER_BLOB_BYTES)
+    _check(lib.cec_peer_export(ctx, buf), ctx)
+    return buf.raw
+
+
+def cec_peer_import(ctx, blobs) -> None:
+    """Map every rank's exchange block (blobs in rank order) and switch the context to peer mode."""
+    raw = b"".join(bytes(b) for b in blobs)
+    if len(raw) != PEER_BLOB_BYTES * len(blobs):
+        raise ValueError("peer blobs must be 128 bytes each")
+    _check(lib.cec_peer_import(ctx, ctypes.create_string_buffer(raw, len(raw))), ctx)
+
+
 def cec_abi_version() -> int:
     return int(lib.cec_abi_version())
 
@@ -373,6 +394,12 @@ class Context:
 
     def reduce(self, member_ids, repr_lits, lits=()):
         return cec_reduce(self._ctx, self.num_pis, self.num_ands, member_ids, repr_lits, lits)
+
+    def peer_connect(self, all_gather) -> None:
+        """Peer-memory a10 (include/cec.h cec_peer_export/import): `all_gather(blob) -> [blob of
+        rank 0, ..., rank world-1]` is the caller's collective (e.g. torch.distributed
+        all_gather_object); every rank calls this once, collectively."""
+        cec_peer_import(self._ctx, all_gather(cec_peer_export(self._ctx)))
 
     def pair_k(self, lit_a: int, lit_b: int) -> int:
         return cec_pair_k(self._ctx, lit_a, lit_b)

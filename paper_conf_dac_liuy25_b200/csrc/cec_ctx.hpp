@@ -131,6 +131,7 @@ struct cec_ctx {
     AuxStreams aux;  // side streams for concurrent launch groups
     int num_sms = 0;
     ncclComm_t comm = nullptr;
+    PeerState peer;  // a10 over NVLink peer memory (peer.cu), set up by cec_peer_export/import
     std::string err;
     cec_stats stats{};
     // last global check (for cec_get_cex)
@@ -207,6 +208,7 @@ struct cec_plan {
     uint32_t runs = 0;                     // completed cec_plan_run calls
     void *graph = nullptr, *graph_stream = nullptr;  // captured run (replayed from the 2nd run on)
     uint32_t graph_launches = 0;
+    uint32_t graph_peer_gen = 0;  // PeerState::gen the graph was captured with
 };
 
 

@@ -93,6 +93,13 @@ cec_status fail(cec_ctx *c, cec_status s, const char *fmt, ...) {
         if (e_) return fail((ctx), CEC_E_CUDA, "CUDA: %s (%s)", e_, #expr);          \
     } while (0)
 
+// peer mode: did one of this rank's barriers time out (peer.cu)? Called after a stream sync.
+static bool peer_failed(cec_ctx *c) {
+    if (!c->peer.on) return false;
+    bool t = false;
+    return peer_error(c->peer, c->stream, &t) != nullptr || t;
+}
+
 // Structural TFI of the roots, stopping at nodes with stop_stamp == stop_epoch
 // (cut leaves) and at PIs/const. Visits every reached node once; calls f(id) for each.
 template <class F>
@@ -391,6 +398,21 @@ cec_status cec_nccl_unique_id(void *out128) {
     return CEC_OK;
 }
 
+cec_status cec_peer_export(cec_ctx *c, void *blob_out) {
+    if (!c || !blob_out) return CEC_E_ARG;
+    if (c->host_only) return fail(c, CEC_E_CUDA, "host-only context: no CUDA device");
+    if (c->opts.world < 2 || c->opts.world > PEER_MAX) return fail(c, CEC_E_ARG, "peer mode needs 2 <= world <= 8");
+    const char *e = peer_export(c->peer, c->opts.device, c->opts.rank, c->opts.world, blob_out);
+    return e ? fail(c, CEC_E_CUDA, "CUDA: %s (peer export)", e) : CEC_OK;
+}
+
+cec_status cec_peer_import(cec_ctx *c, const void *blobs) {
+    if (!c || !blobs) return CEC_E_ARG;
+    if (c->host_only) return fail(c, CEC_E_CUDA, "host-only context: no CUDA device");
+    const char *e = peer_import(c->peer, c->opts.device, c->opts.rank, c->opts.world, blobs);
+    return e ? fail(c, CEC_E_CUDA, "peer import: %s", e) : CEC_OK;
+}
+
 uint64_t cec_pext64(uint64_t value, uint64_t mask) {
     uint64_t r = 0;
     int j = 0;
@@ -471,6 +493,10 @@ void cec_free(cec_ctx *ctx) {
     dev_free(ctx->d_f1);
     dev_free(ctx->d_level_ids);
     if (ctx->comm && g_nccl.destroy) g_nccl.destroy(ctx->comm);
+    if (ctx->peer.own) {
+        stream_sync(ctx->stream);
+        peer_close(ctx->peer);
+    }
     aux_destroy(ctx->aux);
     ctx->devpool.reset();  // freed here unless a live plan still holds it
     if (ctx->own_stream) stream_destroy(ctx->own_stream);
@@ -1332,14 +1358,24 @@ cec_status cec_plan_run(cec_ctx *c, cec_plan *P) {
     // a plan that is run again is replayed as a CUDA graph (captured on its second run)
     const bool use_graph = !P->simt.E && P->runs >= 1 && getenv("CEC_NO_GRAPH") == nullptr &&
                            getenv("CEC_PROFILE_GROUPS") == nullptr;
-    if (use_graph && P->graph && P->graph_stream != c->stream) {
+    // a10 over peer memory (peer.cu) when cec_peer_import connected this rank; else NCCL below
+    const bool peer = c->peer.on && !P->simt.E;
+    PeerRun pr;
+    if (peer) {
+        if (P->cmps.size() > c->peer.cap_cmp || P->dwin.size() > c->peer.cap_win)
+            return fail(c, CEC_E_ARG, "plan exceeds the peer exchange capacity (%u compares, %u windows)",
+                        c->peer.cap_cmp, c->peer.cap_win);
+        pr = peer_run_of(c->peer, P->d.first);
+    }
+    if (use_graph && P->graph && (P->graph_stream != c->stream || P->graph_peer_gen != c->peer.gen)) {
         graph_destroy(P->graph);
         P->graph = nullptr;
     }
     if (use_graph && !P->graph) {
         e = graph_capture_run(P->d, P->groups, (uint32_t)P->dwin.size(), (uint32_t)P->cmps.size(), c->stream,
-                              c->num_sms, &P->graph_launches, &c->aux, &P->graph);
+                              c->num_sms, &P->graph_launches, &c->aux, &P->graph, peer ? &pr : nullptr);
         P->graph_stream = c->stream;
+        P->graph_peer_gen = c->peer.gen;
         if (e) return fail(c, CEC_E_CUDA, "CUDA: %s (graph capture)", e);
     }
     CUDA_TRY(c, event_record(P->ev0, c->stream));
@@ -1349,10 +1385,10 @@ cec_status cec_plan_run(cec_ctx *c, cec_plan *P) {
     } else {
         e = P->simt.E ? launch_simt(P->simt, P->d.first, (uint32_t)P->cmps.size(), c->stream, c->num_sms, &nl)
                       : launch_run(P->d, P->groups, (uint32_t)P->dwin.size(), (uint32_t)P->cmps.size(), c->stream,
-                                   c->num_sms, &nl, &c->aux);
+                                   c->num_sms, &nl, &c->aux, peer ? &pr : nullptr);
     }
     if (e) return fail(c, CEC_E_CUDA, "CUDA: %s (kernel launch)", e);
-    if (c->comm && !P->cmps.empty()) {  // a10: one NCCL min all-reduce of first_idx
+    if (c->comm && !peer && !P->cmps.empty()) {  // a10: one NCCL min all-reduce of first_idx
         ncclResult_t r = g_nccl.all_reduce(P->d.first, P->d.first, P->cmps.size(), ncclUint64, ncclMin, c->comm,
                                            (cudaStream_t)c->stream);
         if (r != ncclSuccess) return fail(c, CEC_E_NCCL, "NCCL: %s", g_nccl.err(r));
@@ -1384,6 +1420,7 @@ cec_status cec_plan_results(cec_ctx *c, cec_plan *P, int32_t *verdict, uint64_t 
     c->stats.d2h_bytes = sizeof(unsigned long long) * first.size();
     if (P->ran) {
         CUDA_TRY(c, stream_sync(c->stream));
+        if (peer_failed(c)) return fail(c, CEC_E_NCCL, "peer barrier timed out (a peer rank never arrived)");
         float ms = 0.f;
         CUDA_TRY(c, event_elapsed(&ms, P->ev0, P->ev1));
         c->stats.kernel_ms = ms;
@@ -1585,6 +1622,10 @@ cec_status cec_sim_exhaustive(cec_ctx *c, uint32_t n, const uint32_t *la, const 
         }
     }
     const char *se = stream_sync(c->stream);
+    if (!se && peer_failed(c)) {
+        for (auto &x : subs) free_dev(x.p.get());
+        return fail(c, CEC_E_NCCL, "peer barrier timed out (a peer rank never arrived)");
+    }
     float kms = 0.f;
     if (!se && !subs.empty() && subs.front().p->ran && subs.back().p->ran)
         se = event_elapsed(&kms, subs.front().p->ev0, subs.back().p->ev1);

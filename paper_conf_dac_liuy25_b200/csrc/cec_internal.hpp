@@ -182,10 +182,52 @@ struct AuxStreams {
 };
 const char *aux_create(AuxStreams &a);
 void aux_destroy(AuxStreams &a);
+
+// peer.cu — a10 over NVLink peer memory: rank 0's exchange block is the
+// home of first[] / bound[] / neq_cnt[]; every rank's kernels update it directly.
+constexpr int PEER_MAX = 8;
+constexpr int PEER_EPOCH = PEER_MAX;      // own-block word: this rank's barrier epoch
+constexpr int PEER_ERR = PEER_MAX + 1;    // own-block word: 1 = a barrier timed out
+constexpr size_t PEER_HDR_BYTES = 256;    // slots + epoch + error flag, padded
+struct PeerPtrs {
+    uint32_t *slots[PEER_MAX];            // peer r's block (its arrival slots first), mapped here
+};
+struct PeerState {                        // per context
+    bool on = false;
+    int rank = 0, world = 1;
+    uint32_t cap_cmp = 1u << 20, cap_win = 1u << 18;  // per-run capacity of the home arrays
+    void *own = nullptr;                  // this rank's block (cudaMalloc, IPC-exported)
+    size_t bytes = 0;
+    void *peer[PEER_MAX] = {};            // every rank's block as mapped in this process
+    void *opened[PEER_MAX] = {};          // IPC mappings to close
+    uint32_t gen = 0;                     // bumped per import (invalidates captured graphs)
+};
+struct PeerRun {                          // what one run needs (passed into launch_run)
+    bool on = false;
+    int rank = 0, world = 1;
+    PeerPtrs slots{};
+    uint32_t *own = nullptr;
+    unsigned long long *home_first = nullptr, *home_bound = nullptr;
+    uint32_t *home_neq = nullptr;
+    unsigned long long *local_first = nullptr;  // the plan's first[]: receives the gathered result
+};
+size_t peer_block_bytes(uint32_t cap_cmp, uint32_t cap_win);
+const char *peer_export(PeerState &ps, int device, int rank, int world, void *blob128);
+const char *peer_import(PeerState &ps, int device, int rank, int world, const void *blobs);
+void peer_close(PeerState &ps);
+PeerRun peer_run_of(const PeerState &ps, unsigned long long *local_first);
+const char *peer_barrier_launch(const PeerRun &pr, void *stream);
+const char *peer_gather_launch(const PeerRun &pr, uint32_t n, void *stream);
+const char *peer_error(const PeerState &ps, void *stream, bool *timed_out);
+
+// One run of a plan: reset, every launch group (side streams forked/joined). With pr->on the window
+// kernels take rank 0's home arrays (d's first/bound/neq_cnt are replaced), wrapped in the peer
+// barriers and followed by the gather into d.first.
 const char *launch_run(const DevPlan &d, const std::vector<LaunchGroup> &groups, uint32_t nwin, uint32_t ncmp,
-                       void *stream, int num_sms, uint32_t *launches, AuxStreams *aux);
+                       void *stream, int num_sms, uint32_t *launches, AuxStreams *aux, const PeerRun *pr = nullptr);
 const char *graph_capture_run(const DevPlan &d, const std::vector<LaunchGroup> &groups, uint32_t nwin, uint32_t ncmp,
-                              void *stream, int num_sms, uint32_t *launches, AuxStreams *aux, void **exec_out);
+                              void *stream, int num_sms, uint32_t *launches, AuxStreams *aux, void **exec_out,
+                              const PeerRun *pr = nullptr);
 const char *graph_launch(void *exec, void *stream);
 void graph_destroy(void *exec);
 const char *dev_alloc(void **p, size_t bytes);

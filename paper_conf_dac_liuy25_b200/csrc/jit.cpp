@@ -436,14 +436,14 @@ std::string jit_source(const JitProgram &p, const JitConfig &cfg) {
          "  const u32 dl = __shfl_sync(0xFFFFFFFFu, d, l);\n"
          "  if (lane != 0u) return;\n"
          "  const u64 idx = ((((u64)s << 5) + l) << 5) + (u32)(__ffs(dl) - 1);\n"
-         "  const u64 old = atomicMin(&first[cmp_off + c], idx);\n"
+         "  const u64 old = atomicMin_system(&first[cmp_off + c], idx);  /* system scope: peer mode */\n"
          "  if (old != ~0ull) return;\n"
-         "  __threadfence();\n"
-         "  if (atomicAdd(&neq_cnt[win], 1u) + 1u != ncmp) return;\n"
-         "  __threadfence();\n"
+         "  __threadfence_system();\n"
+         "  if (atomicAdd_system(&neq_cnt[win], 1u) + 1u != ncmp) return;\n"
+         "  __threadfence_system();\n"
          "  u64 mx = 0;\n"
-         "  for (u32 t = 0; t < ncmp; ++t) { u64 v = atomicAdd(&first[cmp_off + t], 0ull); mx = v > mx ? v : mx; }\n"
-         "  atomicMin(&bound[win], mx);\n"
+         "  for (u32 t = 0; t < ncmp; ++t) { u64 v = atomicAdd_system(&first[cmp_off + t], 0ull); mx = v > mx ? v : mx; }\n"
+         "  atomicMin_system(&bound[win], mx);\n"
          "}\n";
     snprintf(buf, sizeof buf,
              "extern \"C\" __global__ void __launch_bounds__(%d, %d) cecjit(const JItem *__restrict__ items, u32 nitems,\n"
@@ -596,14 +596,14 @@ std::string jit_source_bundle(const std::vector<const JitProgram *> &ps, const J
          "  const u32 dl = __shfl_sync(0xFFFFFFFFu, d, l);\n"
          "  if (lane != 0u) return;\n"
          "  const u64 idx = ((((u64)s << 5) + l) << 5) + (u32)(__ffs(dl) - 1);\n"
-         "  const u64 old = atomicMin(&first[cmp_off + c], idx);\n"
+         "  const u64 old = atomicMin_system(&first[cmp_off + c], idx);  /* system scope: peer mode */\n"
          "  if (old != ~0ull) return;\n"
-         "  __threadfence();\n"
-         "  if (atomicAdd(&neq_cnt[win], 1u) + 1u != ncmp) return;\n"
-         "  __threadfence();\n"
+         "  __threadfence_system();\n"
+         "  if (atomicAdd_system(&neq_cnt[win], 1u) + 1u != ncmp) return;\n"
+         "  __threadfence_system();\n"
          "  u64 mx = 0;\n"
-         "  for (u32 t = 0; t < ncmp; ++t) { u64 v = atomicAdd(&first[cmp_off + t], 0ull); mx = v > mx ? v : mx; }\n"
-         "  atomicMin(&bound[win], mx);\n"
+         "  for (u32 t = 0; t < ncmp; ++t) { u64 v = atomicAdd_system(&first[cmp_off + t], 0ull); mx = v > mx ? v : mx; }\n"
+         "  atomicMin_system(&bound[win], mx);\n"
          "}\n";
     snprintf(buf, sizeof buf,
              "extern \"C\" __global__ void __launch_bounds__(%d, %d) cecjit(const JItem *__restrict__ items, u32 nitems,\n"

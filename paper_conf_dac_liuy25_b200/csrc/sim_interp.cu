@@ -57,18 +57,19 @@ __device__ __forceinline__ uint32_t lop3_60(uint32_t t, uint32_t b, uint32_t m) 
 __device__ __noinline__ void record_mismatch(uint32_t c, uint64_t idx, uint32_t win, const DevWin &W,
                                              unsigned long long *first, unsigned long long *bound,
                                              uint32_t *neq_cnt) {
-    unsigned long long old = atomicMin(&first[c], (unsigned long long)idx);
+    // system scope: in peer mode (peer.cu) these arrays are rank 0's, written by every GPU
+    unsigned long long old = atomicMin_system(&first[c], (unsigned long long)idx);
     if (old == ~0ull) {
-        __threadfence();
-        uint32_t n = atomicAdd(&neq_cnt[win], 1u) + 1u;
+        __threadfence_system();
+        uint32_t n = atomicAdd_system(&neq_cnt[win], 1u) + 1u;
         if (n == W.ncmp) {  // every pair of the window is refuted: publish an early-exit bound
-            __threadfence();
+            __threadfence_system();
             unsigned long long mx = 0;
             for (uint32_t t = 0; t < W.ncmp; ++t) {
-                unsigned long long v = atomicAdd(&first[W.cmp_off + t], 0ull);
+                unsigned long long v = atomicAdd_system(&first[W.cmp_off + t], 0ull);
                 mx = v > mx ? v : mx;
             }
-            atomicMin(&bound[win], mx);
+            atomicMin_system(&bound[win], mx);
         }
     }
 }
@@ -192,16 +193,30 @@ void aux_destroy(AuxStreams &a) {
     a = AuxStreams{};
 }
 
-const char *launch_run(const DevPlan &d, const std::vector<LaunchGroup> &groups, uint32_t nwin, uint32_t ncmp,
-                       void *stream, int num_sms, uint32_t *launches, AuxStreams *aux) {
+const char *launch_run(const DevPlan &d0, const std::vector<LaunchGroup> &groups, uint32_t nwin, uint32_t ncmp,
+                       void *stream, int num_sms, uint32_t *launches, AuxStreams *aux, const PeerRun *pr) {
     cudaStream_t main_st = (cudaStream_t)stream;
     cudaStream_t st = main_st;
     const char *e;
-    {  // one launch resets the run state (first-mismatch indices, bounds, counters)
+    const bool peer = pr && pr->on;
+    DevPlan d = d0;
+    if (peer) {  // the window kernels update rank 0's home arrays directly (peer.cu)
+        d.first = pr->home_first;
+        d.bound = pr->home_bound;
+        d.neq_cnt = pr->home_neq;
+    }
+    {  // one launch resets the run state (first-mismatch indices, bounds, counters); in peer mode
+       // only rank 0 resets the home arrays, every rank its own item counters
         const uint32_t ng = (uint32_t)(groups.size() ? groups.size() : 1);
-        const uint32_t n = std::max(std::max(ncmp, nwin), ng);
-        reset_run<<<(n + 255) / 256, 256, 0, st>>>(d.first, ncmp, d.bound, d.neq_cnt, nwin, d.item_ctr, ng);
+        const uint32_t rc = peer && pr->rank != 0 ? 0u : ncmp, rw = peer && pr->rank != 0 ? 0u : nwin;
+        const uint32_t n = std::max(std::max(rc, rw), ng);
+        reset_run<<<(n + 255) / 256, 256, 0, st>>>(d.first, rc, d.bound, d.neq_cnt, rw, d.item_ctr, ng);
         if ((e = ck(cudaGetLastError()))) return e;
+    }
+    uint32_t nl = 0;
+    if (peer) {  // home reset on rank 0 before any rank's kernels touch it
+        if ((e = peer_barrier_launch(*pr, main_st))) return e;
+        ++nl;
     }
     const bool multi = aux && aux->ok && groups.size() > 1 && getenv("CEC_PROFILE_GROUPS") == nullptr;
     if (multi) {
@@ -209,7 +224,6 @@ const char *launch_run(const DevPlan &d, const std::vector<LaunchGroup> &groups,
         for (int i = 0; i < aux->n; ++i)
             if ((e = ck(cudaStreamWaitEvent((cudaStream_t)aux->s[i], (cudaEvent_t)aux->fork, 0)))) return e;
     }
-    uint32_t nl = 0;
     // CEC_PROFILE_GROUPS=1: serial launches, each group timed with events, one line per group on stderr
     static const bool prof = getenv("CEC_PROFILE_GROUPS") != nullptr;
     std::vector<cudaEvent_t> pev;
@@ -278,6 +292,12 @@ const char *launch_run(const DevPlan &d, const std::vector<LaunchGroup> &groups,
             if ((e = ck(cudaStreamWaitEvent(main_st, (cudaEvent_t)aux->join[i], 0)))) return e;
         }
     }
+    if (peer) {  // every rank's kernels done -> gather the minimum -> nobody resets before all gathered
+        if ((e = peer_barrier_launch(*pr, main_st))) return e;
+        if ((e = peer_gather_launch(*pr, ncmp, main_st))) return e;
+        if ((e = peer_barrier_launch(*pr, main_st))) return e;
+        nl += ncmp ? 3 : 2;
+    }
     if (launches) *launches = nl;
     return nullptr;
 }
@@ -286,12 +306,13 @@ const char *launch_run(const DevPlan &d, const std::vector<LaunchGroup> &groups,
 // fork/join): captured once per (plan, stream) and replayed, so a re-run costs one graph launch
 // instead of one host launch per group (C3: ~1.6k launches per run).
 const char *graph_capture_run(const DevPlan &d, const std::vector<LaunchGroup> &groups, uint32_t nwin, uint32_t ncmp,
-                              void *stream, int num_sms, uint32_t *launches, AuxStreams *aux, void **exec_out) {
+                              void *stream, int num_sms, uint32_t *launches, AuxStreams *aux, void **exec_out,
+                              const PeerRun *pr) {
     cudaStream_t st = (cudaStream_t)stream;
     const char *e;
     *exec_out = nullptr;
     if ((e = ck(cudaStreamBeginCapture(st, cudaStreamCaptureModeRelaxed)))) return e;
-    const char *le = launch_run(d, groups, nwin, ncmp, stream, num_sms, launches, aux);
+    const char *le = launch_run(d, groups, nwin, ncmp, stream, num_sms, launches, aux, pr);
     cudaGraph_t g = nullptr;
     const char *ee = ck(cudaStreamEndCapture(st, &g));
     if (le || ee) {

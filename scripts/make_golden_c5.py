@@ -39,6 +39,10 @@ def _copy(c):
 
 def main():
     procs = int(sys.argv[1]) if len(sys.argv) > 1 else max(1, os.cpu_count() - 1)
+    # optional copy range [lo, hi) (several hosts can work on disjoint ranges; their partial files
+    # are concatenated afterwards) and partial-file path (GOLDEN_PARTIAL)
+    lo = int(sys.argv[2]) if len(sys.argv) > 2 else 0
+    hi = int(sys.argv[3]) if len(sys.argv) > 3 else 1 << 30
     from workloads import c5_big
     m = c5_big()
     P = m.num_pairs
@@ -47,7 +51,7 @@ def main():
     evals, cpu_s = 0, 0.0
     t0 = time.time()
     # per-copy checkpoint (resumable: a restarted run skips the copies already in it)
-    part = os.path.join(ROOT, "tests", "golden", "c5_big.partial.jsonl")
+    part = os.environ.get("GOLDEN_PARTIAL", os.path.join(ROOT, "tests", "golden", "c5_big.partial.jsonl"))
     done = set()
     if os.path.exists(part):
         with open(part) as fh:
@@ -60,7 +64,7 @@ def main():
                 evals += r["ev"]
                 cpu_s += r["dt"]
                 done.add(c)
-    todo = [c for c in range(ncopy) if c not in done]
+    todo = [c for c in range(max(0, lo), min(ncopy, hi)) if c not in done]
     with mp.Pool(procs, initializer=_init) as pool, open(part, "a") as pf:
         for i, (c, off, v, cex, k, ev, dt) in enumerate(pool.imap_unordered(_copy, todo)):
             V[off:off + len(v)], X[off:off + len(v)], K[off:off + len(v)] = v, cex, k
@@ -70,6 +74,9 @@ def main():
                                  "ev": ev, "dt": round(dt, 2)}) + "\n")
             pf.flush()
             print(f"copy {c} done ({len(done) + i + 1}/{ncopy}) {dt:.1f}s", file=sys.stderr, flush=True)
+    if any(v is None for v in V):
+        print(f"partial: copies [{lo}, {hi}) done into {part}", file=sys.stderr)
+        return
     out = {
         "_about": "oracle/ results for every pair of workloads.c5_big() (defaults); written by "
                   "scripts/make_golden_c5.py (one single-threaded oracle task per copy)",

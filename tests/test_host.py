@@ -211,3 +211,15 @@ def test_small_windows_go_whole_to_one_rank_lpt(world):
         ctx.close()
     assert sum(Ws) == W_all
     assert max(Ws) <= 1.6 * W_all / world  # balanced (one-rank-takes-all would be `world` x)
+
+
+def test_peer_mode_needs_a_device_and_world():
+    """cec_peer_export (include/cec.h): a host-only context has no device memory to share."""
+    m = c1_add8()
+    ctx = capi.Context.from_aig(m.aig, device=-1, rank=0, world=2)
+    with pytest.raises(capi.CecError) as e:
+        capi.cec_peer_export(ctx.handle)
+    assert e.value.status == capi.CEC_E_CUDA
+    with pytest.raises(capi.CecError) as e:
+        capi.cec_peer_import(ctx.handle, [bytes(128), bytes(128)])
+    assert e.value.status == capi.CEC_E_CUDA
