@@ -579,7 +579,8 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
     std::vector<uint64_t> wps_of;                    // words per slice per window
     std::vector<uint64_t> words_rank_of;             // u32 words this rank simulates per window
     std::vector<JitProgram> jit_progs;
-    std::unordered_map<std::string, uint32_t> jit_index;
+    std::unordered_map<uint64_t, uint32_t> jit_hindex;  // structure hash -> program index
+    std::vector<uint32_t> jit_rep;                      // program index -> window it was taken from
     // (1) serial: lay out compares window by window (contiguous per window) and own-support masks
     std::vector<std::vector<uint32_t>> wcs(wins.size());
     for (size_t w = 0; w < wins.size(); ++w) {
@@ -611,6 +612,7 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         bool jit = false;
         JitProgram jp;
         std::string key, err;
+        uint64_t hkey = 0;  // 64-bit hash of key (computed in parallel; exact compare verifies)
     };
     std::vector<WinRes> res(wins.size());
     auto plan_one = [&](size_t w, Scratch &X) {
@@ -718,6 +720,15 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
                 jp.cmps.push_back(ref(cmps2[ci].lb >> 1) << 1 | (cmps2[ci].lb & 1u));
             }
             R.key = jit_key(jp);
+            uint64_t h = 0x9E3779B97F4A7C15ull ^ R.key.size();  // word-wise multiply-xorshift hash
+            const uint64_t *q = reinterpret_cast<const uint64_t *>(R.key.data());
+            const size_t nq = R.key.size() / 8;
+            for (size_t i = 0; i < nq; ++i) {
+                uint64_t v = q[i] * 0xBF58476D1CE4E5B9ull;
+                h = (h ^ (v ^ (v >> 31))) * 0x94D049BB133111EBull;
+            }
+            for (size_t i = nq * 8; i < R.key.size(); ++i) h = (h ^ (uint8_t)R.key[i]) * 0x100000001B3ull;
+            R.hkey = h ^ (h >> 29);
         }
     };
     if (wins.size() < 2) {
@@ -726,6 +737,7 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         WorkPool &wp = c->workers();
         wp.run((uint32_t)wins.size(), [&](uint32_t w, unsigned tid) { plan_one(w, c->pool[tid]); });
     }
+    tm.lap("per-window plans (parallel)");
     // Multi-GPU split: a window with at least `world` slices is cut into
     // contiguous slice ranges, one per rank; a smaller window goes WHOLE to one rank, chosen by
     // longest-processing-time-first over the node-words of the small windows on top of each rank's
@@ -790,11 +802,12 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         P->win_cmps.push_back(wc);
         nslots_of.push_back(sc.nslots);
         const bool jit = R.jit;
-        if (jit) {
-            auto it = jit_index.find(R.key);
-            if (it == jit_index.end()) {
-                it = jit_index.emplace(R.key, (uint32_t)jit_progs.size()).first;
+        if (jit) {  // windows of identical structure share one program (by hash; verified below)
+            auto it = jit_hindex.find(R.hkey);
+            if (it == jit_hindex.end()) {
+                it = jit_hindex.emplace(R.hkey, (uint32_t)jit_progs.size()).first;
                 jit_progs.push_back(std::move(R.jp));
+                jit_rep.push_back((uint32_t)w);
             }
             win_jit.push_back((int32_t)it->second);
         } else {
@@ -816,6 +829,31 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         words_rank_of.push_back(we > wb ? (we - wb) : 0);
         cost_of.push_back((uint64_t)(sc.ops.size() + 1) * (se - sb));
     }
+    {  // exactness of the hash dedupe: every window's structure key equals its program's (parallel
+       // memcmp); a 64-bit collision (never seen) gets its own program through an exact-key map
+        std::vector<uint8_t> bad(wins.size(), 0);
+        auto verify = [&](uint32_t w, unsigned) {
+            const int32_t pi = win_jit[w];
+            if (pi >= 0 && jit_rep[pi] != w && res[w].key != res[jit_rep[pi]].key) bad[w] = 1;
+        };
+        if (wins.size() < 2) {
+            for (uint32_t w = 0; w < wins.size(); ++w) verify(w, 0);
+        } else {
+            c->workers().run((uint32_t)wins.size(), verify);
+        }
+        std::unordered_map<std::string, uint32_t> exact;
+        for (uint32_t w = 0; w < wins.size(); ++w) {
+            if (!bad[w]) continue;
+            auto it = exact.find(res[w].key);
+            if (it == exact.end()) {
+                it = exact.emplace(res[w].key, (uint32_t)jit_progs.size()).first;
+                jit_progs.push_back(std::move(res[w].jp));
+                jit_rep.push_back(w);
+            }
+            win_jit[w] = (int32_t)it->second;
+        }
+    }
+    tm.lap("structure dedupe (hash)");
     if (c->opts.engine == CEC_ENGINE_SIMT && !local) {  // the paper's Alg. 1 layout (sim_simt.cu)
         if (world != 1) return fail(c, CEC_E_ARG, "CEC_ENGINE_SIMT runs on one GPU (world = 1)");
         SimtPlan &S = P->simt;
@@ -947,7 +985,7 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         });
         for (size_t i = 0; i < units.size(); ++i) {
             if (!errs[i].empty()) return fail(c, CEC_E_CUDA, "JIT: %s", errs[i].c_str());
-            if (load) {
+            if (load && !jit_kernel_loaded(kernels[i])) {  // cache hits of the first pass are loaded
                 const char *e = jit_get_unit(uprogs[i], jcfg, true, &kernels[i]);
                 if (e) return fail(c, CEC_E_CUDA, "JIT load: %s", e);
             }
@@ -1545,12 +1583,15 @@ cec_status cec_sim_exhaustive(cec_ctx *c, uint32_t n, const uint32_t *la, const 
     // same windows) cover the planning of the next, twice as large, chunk
     std::vector<size_t> cut{0};
     {
-        double acc = 0, chunk = K > 1 ? 0.04 * total : total, target = chunk;
+        double first = 0.04, growth = 2.0;  // tunable: CEC_PIPE_FIRST (fraction), CEC_PIPE_GROWTH
+        if (const char *e = getenv("CEC_PIPE_FIRST")) first = std::max(1e-4, atof(e));
+        if (const char *e = getenv("CEC_PIPE_GROWTH")) growth = std::max(1.0, atof(e));
+        double acc = 0, chunk = K > 1 ? first * total : total, target = chunk;
         for (size_t w = 0; w < wins.size(); ++w) {
             acc += wcost[w];
             if (K > 1 && acc >= target && w + 1 < wins.size()) {
                 cut.push_back(w + 1);
-                chunk *= 2.0;
+                chunk *= growth;
                 target = acc + chunk;
             }
         }

@@ -115,6 +115,7 @@ const char *jit_get_kernel(const JitProgram &p, const JitConfig &cfg, bool load,
 // several structures in one kernel (items carry window | sid << 20), see jit_source_bundle
 const char *jit_get_unit(const std::vector<const JitProgram *> &ps, const JitConfig &cfg, bool load, JitKernel **out);
 uint32_t jit_kernel_lop3_sid(const JitKernel *k, uint32_t sid);
+bool jit_kernel_loaded(const JitKernel *k);  // true once the cubin is loaded (kernel handle set)
 double jit_compile_ms(const JitKernel *k);
 int jit_slices_per_pass(const JitKernel *k);
 uint32_t jit_kernel_lop3(const JitKernel *k);

@@ -954,6 +954,7 @@ const char *jit_get_kernel(const JitProgram &p, const JitConfig &cfg, bool load,
 double jit_compile_ms(const JitKernel *k) { return k ? k->compile_ms : 0.0; }
 int jit_slices_per_pass(const JitKernel *k) { return k ? k->slices_per_pass : 1; }
 uint32_t jit_kernel_lop3(const JitKernel *k) { return k ? k->lop3 : 0; }
+bool jit_kernel_loaded(const JitKernel *k) { return k && k->kern; }
 uint32_t jit_kernel_lop3_sid(const JitKernel *k, uint32_t sid) {
     return k && sid < k->lop3s.size() ? k->lop3s[sid] : 0;
 }
