@@ -213,49 +213,79 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    # BENCH_SAME_GPU=1 (testing only): every rank on device 0, gloo process group, peer reduction only
+    # (NCCL refuses two ranks on one GPU). Times are meaningless there (ranks time-slice one GPU).
+    same_gpu = os.environ.get("BENCH_SAME_GPU") == "1"
+    if same_gpu:
+        local = 0
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if same_gpu:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    red_dev = "cpu" if same_gpu else "cuda"
+
+    def allreduce(x, op):
+        t = torch.tensor([x], device=red_dev, dtype=torch.float64)
+        dist.all_reduce(t, op=op)
+        return float(t.item())
+
     stream = torch.cuda.Stream()  # the library launches on this stream; events are recorded on it
     torch.cuda.set_stream(stream)
 
     m, desc, copy_idx = make_workload(args.config)
-    uid = None
-    if world > 1:
+    merge = args.merge if args.merge >= 0 else (capi.CEC_MERGE_COST if args.config == "c3" else capi.CEC_MERGE_PAPER)
+
+    def new_uid():
+        if world == 1 or same_gpu:
+            return None
         obj = [capi.cec_nccl_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(obj, src=0)
-        uid = obj[0]
-    t_load = time.perf_counter()
-    merge = args.merge if args.merge >= 0 else (capi.CEC_MERGE_COST if args.config == "c3" else capi.CEC_MERGE_PAPER)
-    ctx = capi.Context.from_aig(m.aig, device=local, rank=rank, world=world, stream=stream.cuda_stream,
-                                engine=args.engine, merge=merge, nccl_unique_id=uid)
-    load_ms = 1e3 * (time.perf_counter() - t_load)
-    reduce_mode = "nccl all-reduce (min)" if world > 1 else "none (1 GPU)"
-    if world > 1 and args.reduce == "peer":
-        # a10 over peer memory (include/cec.h cec_peer_export/import): IPC blobs all-gathered here
-        def all_gather(blob):
-            out = [None] * world
-            dist.all_gather_object(out, blob)
-            return out
+        return obj[0]
 
+    def all_gather(blob):
+        out = [None] * world
+        dist.all_gather_object(out, blob)
+        return out
+
+    def open_ctx(peer):
+        """Context + plan + one checked run; peer=True: a10 over peer memory (include/cec.h
+        cec_peer_export/import, IPC blobs all-gathered here), else ncclAllReduce."""
+        c = capi.Context.from_aig(m.aig, device=local, rank=rank, world=world, stream=stream.cuda_stream,
+                                  engine=args.engine, merge=merge, nccl_unique_id=new_uid())
+        err = None
         try:
-            ctx.peer_connect(all_gather)
-            ok = 1
+            if peer:
+                c.peer_connect(all_gather)
+            pl = capi.cec_plan_exhaustive(c.handle, m.lit_a, m.lit_b)
+            capi.cec_plan_run(c.handle, pl)
+            capi.cec_plan_results(c.handle, pl, m.num_pairs)  # syncs; raises on a barrier timeout
         except capi.CecError as e:
-            ok, why = 0, str(e)
-        t = torch.tensor([ok], device="cuda", dtype=torch.int32)
-        dist.all_reduce(t, op=dist.ReduceOp.MIN)  # all ranks take the same path
-        if int(t.item()) == 1:
+            err, pl = str(e), None
+        return c, pl, err
+
+    t_load = time.perf_counter()
+    peer = world > 1 and (args.reduce == "peer" or same_gpu)
+    ctx, plan, err = open_ctx(peer)
+    load_ms = 1e3 * (time.perf_counter() - t_load)
+    reduce_mode = "none (1 GPU)"
+    if world > 1:
+        ok = allreduce(0.0 if err else 1.0, dist.ReduceOp.MIN)  # every rank takes the same path
+        if peer and ok == 1.0:
             reduce_mode = "peer memory (NVLink, fused atomicMin into rank 0's home arrays + device barriers)"
-        else:  # a context that imported keeps peer mode: rebuild every rank's context on NCCL
+        elif peer and not same_gpu:  # fall back to the collective on every rank
             ctx.close()
-            obj = [capi.cec_nccl_unique_id() if rank == 0 else None]  # a fresh communicator id
-            dist.broadcast_object_list(obj, src=0)
-            uid = obj[0]
-            ctx = capi.Context.from_aig(m.aig, device=local, rank=rank, world=world, stream=stream.cuda_stream,
-                                        engine=args.engine, merge=merge, nccl_unique_id=uid)
-            reduce_mode = "nccl all-reduce (min); peer setup failed" + (f": {why}" if not ok else " on a peer rank")
-    plan = capi.cec_plan_exhaustive(ctx.handle, m.lit_a, m.lit_b)
+            ctx, plan, err2 = open_ctx(False)
+            if err2:
+                raise SystemExit(f"rank {rank}: {err2}")
+            reduce_mode = "nccl all-reduce (min); peer mode failed" + (f": {err}" if err else " on a peer rank")
+        elif ok != 1.0:
+            raise SystemExit(f"rank {rank}: {err or 'a peer rank failed'}")
+        else:
+            reduce_mode = "nccl all-reduce (min)"
+    elif err:
+        raise SystemExit(err)
     info = capi.cec_plan_info(plan)
     st0 = ctx.stats()
     engine_name = ("simt (paper Alg. 1)" if args.engine == capi.CEC_ENGINE_SIMT else
@@ -292,9 +322,7 @@ def main():
     step_ms = [s.elapsed_time(e) for s, e in zip(starts, ends)]
     ms = sum(step_ms) / len(step_ms)
     if world > 1:
-        t = torch.tensor([ms], device="cuda", dtype=torch.float64)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        ms = float(t.item())
+        ms = allreduce(ms, dist.ReduceOp.MAX)
     value = W_all / (ms / 1e3)
 
     # e2e: the public blocking call with host arrays (plan + H2D + kernels + reduce + D2H)
@@ -317,9 +345,7 @@ def main():
     st_e2e = ctx.stats()
     e2e = statistics.median(e2e_ms)
     if world > 1:
-        t = torch.tensor([e2e], device="cuda", dtype=torch.float64)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        e2e = float(t.item())
+        e2e = allreduce(e2e, dist.ReduceOp.MAX)
 
     clocks = clk.summary()
     sm_clock = clocks.get("sm_mhz") or clocks.get("sm_max_mhz") or 1965.0  # median SM clock seen under load
@@ -357,7 +383,7 @@ def main():
     # parity against stored oracle results of the same generated miter (tests/golden, written by
     # scripts/make_golden*.py, which call only oracle/): every pair's verdict, k and canonical CEX
     parity = None
-    gold_name = {"c5": "c5_big", "c2": "c2_mul12", "c2bug": "c2_mul12_bug1"}.get(args.config)
+    gold_name = {"c5": "c5_big", "c3": "c3_rand", "c2": "c2_mul12", "c2bug": "c2_mul12_bug1"}.get(args.config)
     gpath = os.path.join(ROOT, "tests", "golden", f"{gold_name}.json") if gold_name else None
     if rank == 0 and gpath and os.path.exists(gpath):
         g = json.load(open(gpath))

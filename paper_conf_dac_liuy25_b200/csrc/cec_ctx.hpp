@@ -141,6 +141,7 @@ struct cec_ctx {
     std::vector<std::vector<uint32_t>> last_support;
     // device copy of the AIG for random simulation (lazy)
     uint32_t *d_f0 = nullptr, *d_f1 = nullptr, *d_level_ids = nullptr;
+    NodeSupports supp_table;  // a2 per-node support lists on the device (AIG-only, built once)
     std::vector<uint32_t> level_off;
     std::shared_ptr<DevPool> devpool;  // plan device blocks + pinned staging (device contexts)
     Scratch scratch;  // for serial host work (supports of single pairs, cut validation)

@@ -492,6 +492,7 @@ void cec_free(cec_ctx *ctx) {
     dev_free(ctx->d_f0);
     dev_free(ctx->d_f1);
     dev_free(ctx->d_level_ids);
+    dev_free(ctx->supp_table.lists);
     if (ctx->comm && g_nccl.destroy) g_nccl.destroy(ctx->comm);
     if (ctx->peer.own) {
         stream_sync(ctx->stream);
@@ -1220,7 +1221,7 @@ static cec_status plan_route(cec_ctx *c, uint32_t n, const uint32_t *la, const u
         std::vector<uint32_t> lists, cnt;
         uint32_t nl = 0;
         CUDA_TRY(c, gpu_supports(*c->devpool, c->d_f0, c->d_f1, c->d_level_ids, c->level_off, c->I, c->N(), cap, roots,
-                                 lists, cnt, c->stream, &nl));
+                                 lists, cnt, c->stream, &nl, &c->supp_table));
         for (uint32_t p = 0; p < n; ++p)
             if (cnt[p] < cap) {
                 supp[p].assign(lists.begin() + (size_t)p * cap, lists.begin() + (size_t)p * cap + cnt[p]);

@@ -101,11 +101,16 @@ struct DevPool {
     ~DevPool();
 };
 
-// supp_gpu.cu: a2 supports of all pairs (sorted PI lists saturating at cap = k_max + 1)
+// supp_gpu.cu: a2 supports of all pairs (sorted PI lists saturating at cap = k_max + 1). The per-node
+// table (AIG-only) is computed into *table on first use and reused while table->cap == cap.
+struct NodeSupports {
+    uint32_t *lists = nullptr, *cnt = nullptr;  // one cudaMalloc block, N x cap + N
+    uint32_t cap = 0, launches = 0;
+};
 const char *gpu_supports(DevPool &pool, const uint32_t *d_f0, const uint32_t *d_f1, const uint32_t *d_level_ids,
                          const std::vector<uint32_t> &level_off, uint32_t I, uint32_t N, uint32_t cap,
                          const std::vector<uint2> &roots, std::vector<uint32_t> &lists_out,
-                         std::vector<uint32_t> &cnt_out, void *stream, uint32_t *launches);
+                         std::vector<uint32_t> &cnt_out, void *stream, uint32_t *launches, NodeSupports *table);
 
 // jit.cpp
 std::string jit_key(const JitProgram &p);

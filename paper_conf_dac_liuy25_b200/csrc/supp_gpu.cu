@@ -4,8 +4,9 @@
 // saturating at `cap` = min(k_max, 41) + 1 <= 42 entries (a list of cap entries means "more than
 // k_max": the pair is routed away from exhaustive simulation, and the host recomputes its exact k
 // by a cone walk). One launch per topological level (cec_ensure_device_aig's CSR), one warp per
-// node; then one warp per pair merges the two root lists (C5: 247 levels, 1.8 ms in total). Lists live in one
-// device block of N x cap u32 (C5: 2M nodes x 33 = 270 MB, written once and read twice per call).
+// node; then one warp per pair merges the two root lists (C5: 247 levels, 1.8 ms in total). The node lists live in one
+// device block of N x cap u32 (C5: 2M nodes x 33 = 270 MB) that is a property of the AIG: it is built
+// on a context's first call and kept; every call runs only the per-pair merge.
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -119,22 +120,21 @@ inline const char *ck(cudaError_t e) { return e == cudaSuccess ? nullptr : cudaG
 const char *gpu_supports(DevPool &pool, const uint32_t *d_f0, const uint32_t *d_f1, const uint32_t *d_level_ids,
                          const std::vector<uint32_t> &level_off, uint32_t I, uint32_t N, uint32_t cap,
                          const std::vector<uint2> &roots, std::vector<uint32_t> &lists_out,
-                         std::vector<uint32_t> &cnt_out, void *stream, uint32_t *launches) {
+                         std::vector<uint32_t> &cnt_out, void *stream, uint32_t *launches, NodeSupports *table) {
     cudaStream_t st = (cudaStream_t)stream;
     const uint32_t n = (uint32_t)roots.size();
     auto al = [](size_t x) { return (x + 255) / 256 * 256; };
-    const size_t b_lists = al(sizeof(uint32_t) * (size_t)N * cap), b_cnt = al(sizeof(uint32_t) * N),
-                 b_roots = al(sizeof(uint2) * std::max<uint32_t>(n, 1)),
+    const size_t b_roots = al(sizeof(uint2) * std::max<uint32_t>(n, 1)),
                  b_out = al(sizeof(uint32_t) * (size_t)std::max<uint32_t>(n, 1) * cap),
                  b_ocnt = al(sizeof(uint32_t) * std::max<uint32_t>(n, 1));
     void *blk = nullptr;
     size_t blk_cap = 0;
     const char *e;
-    if ((e = pool.get(b_lists + b_cnt + b_roots + b_out + b_ocnt, &blk, &blk_cap))) return e;
+    if (cap > 64) return "support cap above 64";
+    if ((e = pool.get(b_roots + b_out + b_ocnt, &blk, &blk_cap))) return e;
     char *base = (char *)blk;
-    uint32_t *lists = (uint32_t *)base, *cnt = (uint32_t *)(base + b_lists);
-    uint2 *d_roots = (uint2 *)(base + b_lists + b_cnt);
-    uint32_t *out = (uint32_t *)(base + b_lists + b_cnt + b_roots), *ocnt = (uint32_t *)(base + b_lists + b_cnt + b_roots + b_out);
+    uint2 *d_roots = (uint2 *)base;
+    uint32_t *out = (uint32_t *)(base + b_roots), *ocnt = (uint32_t *)(base + b_roots + b_out);
     uint32_t nl = 0;
     const int T = 256;
     auto fail = [&](const char *m) {
@@ -143,16 +143,30 @@ const char *gpu_supports(DevPool &pool, const uint32_t *d_f0, const uint32_t *d_
         return m;
     };
     if ((e = ck(cudaMemcpyAsync(d_roots, roots.data(), sizeof(uint2) * n, cudaMemcpyHostToDevice, st)))) return fail(e);
-    if (cap > 64) return fail("support cap above 64");
-    supp_init<<<(I + 1 + T - 1) / T, T, 0, st>>>(lists, cnt, I, cap);
-    ++nl;
     auto wgrid = [&](uint32_t m) { return (unsigned)std::min<uint64_t>(148ull * 16, ((uint64_t)m * 32 + T - 1) / T); };
-    for (size_t l = 1; l + 1 < level_off.size(); ++l) {  // one launch per topological level
-        const uint32_t b = level_off[l], m = level_off[l + 1] - b;
-        if (!m) continue;
-        supp_level_smem<<<wgrid(m), T, 0, st>>>(d_level_ids + b, m, d_f0, d_f1, lists, cnt, cap);
+    // The per-node table depends on the AIG only (like its levels, a1): built on the context's first
+    // call, kept in device memory and reused by every later call with the same cap.
+    if (!table->lists || table->cap != cap) {
+        if (table->lists) cudaFree(table->lists);
+        table->lists = nullptr;
+        table->cnt = nullptr;
+        void *tb = nullptr;
+        const size_t b_lists = al(sizeof(uint32_t) * (size_t)N * cap), b_cnt = al(sizeof(uint32_t) * N);
+        if ((e = ck(cudaMalloc(&tb, b_lists + b_cnt)))) return fail(e);
+        table->lists = (uint32_t *)tb;
+        table->cnt = (uint32_t *)((char *)tb + b_lists);
+        table->cap = cap;
+        supp_init<<<(I + 1 + T - 1) / T, T, 0, st>>>(table->lists, table->cnt, I, cap);
         ++nl;
+        for (size_t l = 1; l + 1 < level_off.size(); ++l) {  // one launch per topological level
+            const uint32_t b = level_off[l], m = level_off[l + 1] - b;
+            if (!m) continue;
+            supp_level_smem<<<wgrid(m), T, 0, st>>>(d_level_ids + b, m, d_f0, d_f1, table->lists, table->cnt, cap);
+            ++nl;
+        }
+        table->launches = nl;
     }
+    uint32_t *lists = table->lists, *cnt = table->cnt;
     if (n) {
         supp_pairs<<<wgrid(n), T, 0, st>>>(d_roots, n, lists, cnt, cap, out, ocnt);
         ++nl;

@@ -465,3 +465,26 @@ def test_c5_full_vs_stored_oracle():
     for p in np.nonzero(gv == capi.CEC_NOT_EQUIVALENT)[0]:  # each CEX really separates the pair
         want = orc.cex_vector(int(m.lit_a[p]), int(m.lit_b[p]), int(gc[p]))
         assert orc.eval_lit(int(m.lit_a[p]), want) != orc.eval_lit(int(m.lit_b[p]), want)
+
+
+def test_c3_full_vs_stored_oracle():
+    """Full-size C3 (234k ANDs, 6664 pairs incl. 64 near-miss NEQ pairs, supports up to 29) in the
+    launch configuration bench.py times (cost-aware merge, AUTO engine: JIT bundles + interpreter),
+    against the oracle's result for EVERY pair (tests/golden/c3_rand.json, scripts/make_golden_c3.py:
+    support groups x pattern ranges, min-reduced)."""
+    from workloads import c3_rand
+
+    g = _golden("c3_rand")
+    m = c3_rand()
+    assert [int(x) for x in m.lit_a] == g["lit_a"] and [int(x) for x in m.lit_b] == g["lit_b"]
+    ctx = gpu_ctx(m.aig, merge=capi.CEC_MERGE_COST)
+    plan = capi.cec_plan_exhaustive(ctx.handle, m.lit_a, m.lit_b)
+    capi.cec_plan_run(ctx.handle, plan)
+    gv, gc, gk = capi.cec_plan_results(ctx.handle, plan, m.num_pairs)
+    capi.cec_plan_free(plan)
+    assert_same(gv, gc, gk, np.array(g["verdict"]), np.array([int(x) for x in g["cex"]], dtype=np.uint64),
+                np.array(g["k"]), "c3 full")
+    assert (gv == capi.CEC_NOT_EQUIVALENT).sum() >= 1
+    ve, ce, ke = ctx.sim_exhaustive(m.lit_a, m.lit_b)  # the pipelined public call agrees
+    assert np.array_equal(ve, gv) and np.array_equal(ke, gk)
+    assert np.array_equal(ce[gv == capi.CEC_NOT_EQUIVALENT], gc[gv == capi.CEC_NOT_EQUIVALENT])
