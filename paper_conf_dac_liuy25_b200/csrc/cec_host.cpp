@@ -1196,8 +1196,14 @@ static cec_status plan_route(cec_ctx *c, uint32_t n, const uint32_t *la, const u
     P->pair_cmp.assign(n, -1);
     const uint32_t kmax = c->opts.k_max;
     // a2/a3: supports, trivial pairs, routing by k; identical (unordered) pairs share one compare
-    std::map<std::pair<uint32_t, uint32_t>, uint32_t> seen;
-    std::map<std::vector<uint32_t>, uint32_t> by_support;  // identical supports share a window
+    std::unordered_map<uint64_t, uint32_t> seen;  // unordered literal pair -> compare
+    // identical supports share a window: hash of S -> windows with that hash (exact compare below)
+    std::unordered_map<uint64_t, std::vector<uint32_t>> by_support;
+    auto supp_hash = [](const std::vector<uint32_t> &S) {
+        uint64_t h = 0x9E3779B97F4A7C15ull ^ S.size();
+        for (uint32_t x : S) h = (h ^ x) * 0x100000001B3ull, h ^= h >> 29;
+        return h;
+    };
     std::vector<WinHost> wins0;
     for (uint32_t p = 0; p < n; ++p)
         if ((la[p] >> 1) >= c->N() || (lb[p] >> 1) >= c->N())
@@ -1296,7 +1302,7 @@ static cec_status plan_route(cec_ctx *c, uint32_t n, const uint32_t *la, const u
             continue;
         }
         P->pre_verdict[p] = DECIDED_BY_SIM;
-        auto key = std::make_pair(std::min(la[p], lb[p]), std::max(la[p], lb[p]));
+        const uint64_t key = (uint64_t)std::min(la[p], lb[p]) << 32 | std::max(la[p], lb[p]);
         auto it = seen.find(key);
         if (it != seen.end()) {
             P->pair_cmp[p] = (int32_t)it->second;
@@ -1310,22 +1316,24 @@ static cec_status plan_route(cec_ctx *c, uint32_t n, const uint32_t *la, const u
         P->cmps.push_back(std::move(cm));
         seen[key] = ci;
         P->pair_cmp[p] = (int32_t)ci;
-        auto bs = by_support.find(S);
-        if (bs == by_support.end()) {
-            by_support[S] = (uint32_t)wins0.size();
+        std::vector<uint32_t> &cand = by_support[supp_hash(S)];
+        uint32_t wi = UINT32_MAX;
+        for (uint32_t x : cand)
+            if (wins0[x].inputs == S) wi = x;
+        if (wi == UINT32_MAX) {
+            cand.push_back((uint32_t)wins0.size());
             WinHost w;
             w.inputs = S;
             w.cmps.push_back(ci);
             w.est_nodes = cone;
             wins0.push_back(std::move(w));
         } else {
-            WinHost &w = wins0[bs->second];
+            WinHost &w = wins0[wi];
             w.cmps.push_back(ci);
             w.est_nodes = std::max<uint64_t>(w.est_nodes, cone);
         }
     }
-    // a5: window merging. by_support iterates in lexicographic order already;
-    // sort explicitly to make the paper's rule visible.
+    // a5: window merging: windows sorted lexicographically by input list.
     std::vector<uint32_t> order(wins0.size());
     for (uint32_t i = 0; i < order.size(); ++i) order[i] = i;
     std::stable_sort(order.begin(), order.end(),
