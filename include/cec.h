@@ -286,7 +286,9 @@ cec_status cec_nccl_unique_id(void *out128);
  * (the same per-pair minimum index) and identical on every rank. Every rank must issue the same
  * sequence of runs (SPMD, as for NCCL). A barrier that waits more than 10 s for a peer sets an error
  * flag instead of hanging: the call returns CEC_E_NCCL. The paper's SIMT engine keeps NCCL.
- * Errors: CEC_E_ARG (world outside 2..8, blob mismatch), CEC_E_CUDA (allocation / IPC failure). */
+ * Errors: CEC_E_ARG (world outside 2..8, blob mismatch), CEC_E_CUDA (allocation / IPC failure, a
+ * peer device not visible, or no native P2P atomics between this device and a peer: the caller then
+ * keeps the NCCL path). */
 #define CEC_PEER_BLOB_BYTES 128
 cec_status cec_peer_export(cec_ctx *ctx, void *blob_out);
 cec_status cec_peer_import(cec_ctx *ctx, const void *blobs);

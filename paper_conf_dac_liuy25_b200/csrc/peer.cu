@@ -78,6 +78,7 @@ struct PeerBlob {  // CEC_PEER_BLOB_BYTES (128) on the wire
     int32_t device, rank, world, pad;
     uint64_t ptr, bytes;
     cudaIpcMemHandle_t h;  // 64 B
+    char bus[16];          // PCI bus id of the exporting device (process-independent device identity)
 };
 static_assert(sizeof(PeerBlob) <= 128, "peer blob");
 constexpr uint32_t PEER_MAGIC = 0xCEC0BEEFu;
@@ -107,6 +108,7 @@ const char *peer_export(PeerState &ps, int device, int rank, int world, void *bl
     b.ptr = (uint64_t)(uintptr_t)ps.own;
     b.bytes = ps.bytes;
     if ((e = ck(cudaIpcGetMemHandle(&b.h, ps.own)))) return e;
+    if ((e = ck(cudaDeviceGetPCIBusId(b.bus, (int)sizeof b.bus, device)))) return e;
     memset(blob128, 0, 128);
     memcpy(blob128, &b, sizeof b);
     return nullptr;
@@ -122,6 +124,26 @@ const char *peer_import(PeerState &ps, int device, int rank, int world, const vo
         if (b.magic != PEER_MAGIC || b.rank != r || b.world != world || b.bytes != ps.bytes)
             return "peer blob mismatch (rank order, world or block size)";
         void *p = nullptr;
+        if (r != rank) {
+            // the home arrays take system-scope atomics from every rank: a peer on ANOTHER device
+            // must be reachable with native P2P atomics (NVLink), else the import fails (the caller
+            // then uses the NCCL all-reduce)
+            char bus[17];
+            memcpy(bus, b.bus, 16);
+            bus[16] = 0;
+            int pdev = -1;
+            if (cudaDeviceGetByPCIBusId(&pdev, bus) != cudaSuccess) {
+                cudaGetLastError();
+                return "peer device not visible in this process (PCI bus id lookup failed)";
+            }
+            if (pdev != device) {
+                int atom = 0, access = 0;
+                if ((e = ck(cudaDeviceGetP2PAttribute(&access, cudaDevP2PAttrAccessSupported, device, pdev)))) return e;
+                if ((e = ck(cudaDeviceGetP2PAttribute(&atom, cudaDevP2PAttrNativeAtomicSupported, device, pdev))))
+                    return e;
+                if (!access || !atom) return "no native P2P atomics between this device and a peer";
+            }
+        }
         if (r == rank) {
             p = ps.own;
         } else if (b.pid == (uint32_t)getpid()) {  // same process: the raw pointer (IPC refuses it)
