@@ -251,18 +251,36 @@ def main():
 
     def open_ctx(peer):
         """Context + plan + one checked run; peer=True: a10 over peer memory (include/cec.h
-        cec_peer_export/import, IPC blobs all-gathered here), else ncclAllReduce."""
+        cec_peer_export/import, IPC blobs all-gathered here), else ncclAllReduce. Every collective
+        step is taken by every rank even after a local failure, so no rank waits for a failed one."""
         c = capi.Context.from_aig(m.aig, device=local, rank=rank, world=world, stream=stream.cuda_stream,
                                   engine=args.engine, merge=merge, nccl_unique_id=new_uid())
-        err = None
+        err, pl = None, None
+        if peer:
+            blob = None
+            try:
+                blob = capi.cec_peer_export(c.handle)
+            except capi.CecError as e:
+                err = str(e)
+            blobs = all_gather(blob)
+            if all(b is not None for b in blobs):
+                try:
+                    capi.cec_peer_import(c.handle, blobs)
+                except capi.CecError as e:
+                    err = str(e)
+            else:
+                err = err or "peer export failed on a peer rank"
         try:
-            if peer:
-                c.peer_connect(all_gather)
-            pl = capi.cec_plan_exhaustive(c.handle, m.lit_a, m.lit_b)
+            pl = capi.cec_plan_exhaustive(c.handle, m.lit_a, m.lit_b)  # JIT compiles: ranks skew here
+        except capi.CecError as e:
+            err = err or str(e)
+        if world > 1 and allreduce(0.0 if err else 1.0, dist.ReduceOp.MIN) != 1.0:
+            return c, pl, err or "a peer rank failed"
+        try:
             capi.cec_plan_run(c.handle, pl)
             capi.cec_plan_results(c.handle, pl, m.num_pairs)  # syncs; raises on a barrier timeout
         except capi.CecError as e:
-            err, pl = str(e), None
+            err = str(e)
         return c, pl, err
 
     t_load = time.perf_counter()

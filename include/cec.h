@@ -284,8 +284,9 @@ cec_status cec_nccl_unique_id(void *out128);
  * read its bounds for early exit; device-side barriers (one-warp kernels, no host round trip; CUDA
  * graph safe) order reset -> kernels -> gather -> next run. Results are identical to the NCCL path
  * (the same per-pair minimum index) and identical on every rank. Every rank must issue the same
- * sequence of runs (SPMD, as for NCCL). A barrier that waits more than 10 s for a peer sets an error
- * flag instead of hanging: the call returns CEC_E_NCCL. The paper's SIMT engine keeps NCCL.
+ * sequence of runs (SPMD, as for NCCL). A barrier that waits longer than CEC_PEER_TIMEOUT_S
+ * (environment, default 60 s) for a peer sets an error flag instead of hanging: the call returns
+ * CEC_E_NCCL and the context stays in that state. The paper's SIMT engine keeps NCCL.
  * Errors: CEC_E_ARG (world outside 2..8, blob mismatch), CEC_E_CUDA (allocation / IPC failure, a
  * peer device not visible, or no native P2P atomics between this device and a peer: the caller then
  * keeps the NCCL path). */

@@ -207,6 +207,7 @@ struct PeerState {                        // per context
     void *peer[PEER_MAX] = {};            // every rank's block as mapped in this process
     void *opened[PEER_MAX] = {};          // IPC mappings to close
     uint32_t gen = 0;                     // bumped per import (invalidates captured graphs)
+    uint64_t timeout_ns = 60000000000ull; // barrier wait before the error flag (CEC_PEER_TIMEOUT_S)
 };
 struct PeerRun {                          // what one run needs (passed into launch_run)
     bool on = false;
@@ -216,6 +217,7 @@ struct PeerRun {                          // what one run needs (passed into lau
     unsigned long long *home_first = nullptr, *home_bound = nullptr;
     uint32_t *home_neq = nullptr;
     unsigned long long *local_first = nullptr;  // the plan's first[]: receives the gathered result
+    uint64_t timeout_ns = 60000000000ull;
 };
 size_t peer_block_bytes(uint32_t cap_cmp, uint32_t cap_win);
 const char *peer_export(PeerState &ps, int device, int rank, int world, void *blob128);

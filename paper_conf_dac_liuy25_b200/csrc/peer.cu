@@ -13,12 +13,13 @@
 //                          -> gather (home first[] -> the plan's own first[]) -> barrier
 // Barriers are one-warp kernels over per-source arrival slots: rank r stores its epoch into slot r of
 // every peer (st.release.sys) and waits until every slot of its own block reaches the epoch
-// (ld.acquire.sys), bounded by a 10 s %globaltimer timeout that raises an error flag instead of
+// (ld.acquire.sys), bounded by a %globaltimer timeout (60 s) that raises an error flag instead of
 // hanging the GPU. The epoch lives in device memory and is advanced by the barrier kernel itself, so
 // a run captured in a CUDA graph replays correctly.
 #include <cuda_runtime.h>
 #include <stdint.h>
 #include <string.h>
+#include <stdlib.h>
 #include <unistd.h>
 
 #include "cec_internal.hpp"
@@ -49,7 +50,7 @@ __device__ __forceinline__ uint64_t globaltimer() {
 
 // own[0..PEER_MAX) = arrival slots (slot s = last epoch signalled by rank s), own[PEER_EPOCH] = this
 // rank's epoch, own[PEER_ERR] = error flag (1 = a barrier timed out)
-__global__ void peer_barrier(PeerPtrs pp, uint32_t *own, int rank, int world) {
+__global__ void peer_barrier(PeerPtrs pp, uint32_t *own, int rank, int world, uint64_t timeout_ns) {
     const int l = threadIdx.x;
     const uint32_t e = own[PEER_EPOCH] + 1u;  // written only by this kernel, stream-ordered
     if (l < world) {
@@ -57,7 +58,7 @@ __global__ void peer_barrier(PeerPtrs pp, uint32_t *own, int rank, int world) {
         st_release_sys(pp.slots[l] + rank, e);
         const uint64_t t0 = globaltimer();
         while ((int32_t)(ld_acquire_sys(own + l) - e) < 0) {
-            if (globaltimer() - t0 > 10000000000ull) {  // 10 s: a peer never arrived
+            if (globaltimer() - t0 > timeout_ns) {  // a peer never arrived (default 60 s)
                 atomicExch(own + PEER_ERR, 1u);
                 break;
             }
@@ -161,6 +162,10 @@ const char *peer_import(PeerState &ps, int device, int rank, int world, const vo
     }
     ps.rank = rank;
     ps.world = world;
+    // a rank may still be planning / JIT-compiling while its peers wait at a barrier; only a peer
+    // that is gone should trip the flag (CEC_PEER_TIMEOUT_S, default 60 s)
+    ps.timeout_ns = 60000000000ull;
+    if (const char *t = getenv("CEC_PEER_TIMEOUT_S")) ps.timeout_ns = (uint64_t)(atof(t) * 1e9);
     ps.on = true;
     ++ps.gen;
     return nullptr;
@@ -185,11 +190,12 @@ PeerRun peer_run_of(const PeerState &ps, unsigned long long *local_first) {
     pr.home_bound = pr.home_first + ps.cap_cmp;
     pr.home_neq = (uint32_t *)(pr.home_bound + ps.cap_win);
     pr.local_first = local_first;
+    pr.timeout_ns = ps.timeout_ns;
     return pr;
 }
 
 const char *peer_barrier_launch(const PeerRun &pr, void *stream) {
-    peer_barrier<<<1, 32, 0, (cudaStream_t)stream>>>(pr.slots, pr.own, pr.rank, pr.world);
+    peer_barrier<<<1, 32, 0, (cudaStream_t)stream>>>(pr.slots, pr.own, pr.rank, pr.world, pr.timeout_ns);
     return ck(cudaGetLastError());
 }
 
