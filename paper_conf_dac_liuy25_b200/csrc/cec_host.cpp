@@ -739,6 +739,7 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         wp.run((uint32_t)wins.size(), [&](uint32_t w, unsigned tid) { plan_one(w, c->pool[tid]); });
     }
     tm.lap("per-window plans (parallel)");
+    size_t prog_total = 0;
     // Multi-GPU split: a window with at least `world` slices is cut into
     // contiguous slice ranges, one per rank; a smaller window goes WHOLE to one rank, chosen by
     // longest-processing-time-first over the node-words of the small windows on top of each rank's
@@ -789,14 +790,14 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         DevWin dw{};
         dw.cmp_off = wc.empty() ? (uint32_t)cmps2.size() : wc[0];
         dw.ncmp = (uint32_t)wc.size();
-        dw.prog_off = (uint32_t)P->prog.size();
+        dw.prog_off = (uint32_t)prog_total;
         dw.prog_len = R.jit ? 0u : (uint32_t)sc.ops.size();  // JIT windows need no interpreter ops
+        prog_total += dw.prog_len;
         dw.k = (uint32_t)W.inputs.size();
         dw.const_slot = sc.const_slot;
         const uint64_t ttw = tt_words_of(dw.k);
         dw.tt_words_lo = (uint32_t)ttw;
         dw.tt_words_hi = (uint32_t)(ttw >> 32);
-        if (!R.jit) P->prog.insert(P->prog.end(), sc.ops.begin(), sc.ops.end());
         P->dwin.push_back(dw);
         P->win_inputs.push_back(W.inputs);
         P->win_nodes.push_back((uint32_t)nodes.size());
@@ -830,6 +831,19 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         words_rank_of.push_back(we > wb ? (we - wb) : 0);
         cost_of.push_back((uint64_t)(sc.ops.size() + 1) * (se - sb));
     }
+    {  // interpreter programs copied into their slots of one array in parallel
+        P->prog.resize(prog_total);
+        auto copy = [&](uint32_t w, unsigned) {
+            if (!res[w].jit && !res[w].sc.ops.empty())
+                std::copy(res[w].sc.ops.begin(), res[w].sc.ops.end(), P->prog.begin() + P->dwin[w].prog_off);
+        };
+        if (wins.size() < 2) {
+            for (uint32_t w = 0; w < wins.size(); ++w) copy(w, 0);
+        } else {
+            c->workers().run((uint32_t)wins.size(), copy);
+        }
+    }
+    tm.lap("per-window serial layout");
     {  // exactness of the hash dedupe: every window's structure key equals its program's (parallel
        // memcmp); a 64-bit collision (never seen) gets its own program through an exact-key map
         std::vector<uint8_t> bad(wins.size(), 0);
