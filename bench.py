@@ -2,11 +2,14 @@
 """bench.py — AIG node-pattern evals/s of the exhaustive-simulation hot path on B200.
 
 One "step" = one full cec_plan_run of the workload: every window's whole 2^k pattern space
-simulated and every candidate pair compared, plus the NCCL min
-all-reduce when N > 1. Default workload = C5 (BASELINE.json configs[4], the config the metric is
+simulated and every candidate pair compared, plus the cross-GPU min of
+the first-mismatch indices when N > 1 (default: fused over NVLink peer memory, include/cec.h
+cec_peer_export/import; --reduce nccl: one ncclAllReduce; the line's config.cross_gpu_reduce says
+which ran). Default workload = C5 (BASELINE.json configs[4], the config the metric is
 quoted on at 1/2/4/8 GPUs): 256 disjoint copies, ~2.1M ANDs, 6320 PO pairs, k = 24 per copy.
 
-  python bench.py [--gpus N] [--steps K] [--warmup W] [--config c5|c2|c2bug|c1] [--impl ours|reference]
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config c5|c3|c2|c2bug|c1] [--impl ours|reference]
+                  [--reduce peer|nccl]
 
 value      = W (node-patterns of one step, all ranks) / device time per step (CUDA events on the
              launch stream, max over ranks), schedules resident in HBM, L2 flushed between steps
