@@ -1477,6 +1477,9 @@ cec_status cec_plan_run(cec_ctx *c, cec_plan *P) {
     c->stats.num_windows = (uint32_t)P->dwin.size();
     c->stats.max_k = P->max_k;
     c->stats.max_slots = P->max_slots;
+    c->stats.lop3_words = P->lop3_words;  // this run's algorithmic LOP3 words (local checks included)
+    c->stats.jit_windows = P->jit_windows;
+    c->stats.jit_kernels = P->jit_kernels;
     P->ran = true;
     ++P->runs;
     return CEC_OK;
