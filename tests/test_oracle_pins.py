@@ -251,3 +251,22 @@ def test_aiger_reader_renumbers_non_topological(tmp_path):
     assert orc.num_pis == 3 and orc.num_ands == 2
     v, cex, k, _ = orc.check_pairs([2 * 5], [2 * 5])
     assert v[0] == EQ and k[0] == 3
+
+
+def test_own_index_mapping_V4():
+    """SURVEY.md §8(c) V4 (P:33 index convention, P:81 increasing-id support order): C1 PO s3 has
+    support {a0..a3, b0..b3}; the pattern a = 11, b = 6 is own index 11 + 16*6 = 107, and every
+    index i of that support maps to a = i mod 16, b = i div 16 (closed form, not the oracle's
+    own evaluator)."""
+    m = c1_add8()
+    orc = Oracle.from_aig(m.aig)
+    s3a, s3b = int(m.lit_a[3]), int(m.lit_b[3])
+    for i in (107, 0, 255, 16, 15):
+        pis = np.asarray(orc.cex_vector(s3a, s3b, i))
+        a = sum(int(pis[j]) << j for j in range(8))
+        b = sum(int(pis[8 + j]) << j for j in range(8))
+        assert (a & 15, b & 15) == (i % 16, i // 16)
+        assert a >> 4 == 0 and b >> 4 == 0          # PIs outside the support stay 0
+        assert orc.eval_lit(s3a, pis) == ((a + b) >> 3) & 1
+    pis = np.asarray(orc.cex_vector(s3a, s3b, 107))
+    assert [int(pis[j]) for j in range(4)] == [1, 1, 0, 1] and [int(pis[8 + j]) for j in range(4)] == [0, 1, 1, 0]
