@@ -6,7 +6,7 @@ import pytest
 
 import oracle
 from paper_conf_dac_liuy25_b200 import capi
-from workloads import Builder
+from workloads import Builder, circuits
 
 pytestmark = pytest.mark.gpu
 EQ, NEQ, UND = capi.CEC_EQUIVALENT, capi.CEC_NOT_EQUIVALENT, capi.CEC_UNDECIDED
@@ -81,4 +81,38 @@ def test_k32_window_closed_form(engine):
     assert int(c[2]) == 0  # chain vs !bal: they differ on every pattern
     vec = ctx.get_cex(1)
     assert list(vec) == [1] * 31 + [0]
+    ctx.close()
+
+
+def _minterm(bd, lits, value):
+    """AND of the literals of `lits` set to the bits of `value` (bit j <-> lits[j])."""
+    m = 1
+    for j, l in enumerate(lits):
+        m = bd.AND(m, l if (value >> j) & 1 else l ^ 1)
+    return m
+
+
+def test_own_index_closed_form_V4_merged_windows():
+    """SURVEY.md §8(c) V4 / Q8 (P:33 index convention, P:81 support order, a11 pext): an 8-bit
+    ripple adder; s3 is compared with s3 XOR [a=11, b=6] (one differing pattern) and s1 with
+    s1 XOR [a=3, b=2]. The closed-form own indices are 11 + 16*6 = 107 and 3 + 4*2 = 11. The two
+    pairs share one merged window (supp(s1) is inside supp(s3)), so the second result must come
+    back through the pext of the merged index. Also checked against the oracle."""
+    bd = Builder(16)
+    a = [bd.pi(i) for i in range(8)]
+    b = [bd.pi(8 + i) for i in range(8)]
+    s, _ = circuits.ripple_adder(bd, a, b)
+    g3 = bd.XOR(s[3], _minterm(bd, a[:4] + b[:4], 11 | 6 << 4))
+    g1 = bd.XOR(s[1], _minterm(bd, a[:2] + b[:2], 3 | 2 << 2))
+    aig = bd.finish([s[3], g3, s[1], g1])
+    la, lb = [s[3], s[1], s[3]], [g3, g1, s[3]]
+    ctx = capi.Context.from_aig(aig, device=0)
+    v, c, k = ctx.sim_exhaustive(la, lb)
+    assert list(v) == [NEQ, NEQ, EQ]
+    assert list(k) == [8, 4, 8]
+    assert int(c[0]) == 107 and int(c[1]) == 11
+    orc = oracle.Oracle.from_aig(aig)
+    ov, oc, ok, _ = orc.check_pairs(la, lb)
+    assert list(ov) == list(v) and list(ok) == list(k)
+    assert [int(x) for x in oc[:2]] == [107, 11]
     ctx.close()
