@@ -58,6 +58,18 @@ def make_workload(name: str):
     raise SystemExit(f"unknown config {name}")
 
 
+L2_NOTE = ("ours: L2 flushed between timed steps (256 MiB write, outside the events); "
+           "reference arm: the CPU oracle, no GPU")
+
+
+def workload_config(name, m, desc):
+    """The `config` object of BOTH arms' JSON lines: it names the workload only (generator-derived
+    facts, identical for --impl ours and --impl reference); run-specific facts (plan, engine, reduce
+    mode) go to the line's `plan` object."""
+    return {"workload": name, "description": desc, "pis": int(m.aig.num_pis), "ands": int(m.aig.num_ands),
+            "pairs": int(m.num_pairs), "l2": L2_NOTE}
+
+
 def sample_pairs(m, copy_idx):
     """Pairs of one copy (C5) or all pairs."""
     import numpy as np
@@ -178,7 +190,7 @@ def run_reference(args):
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * secs / args.steps,
         "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u8",
         "data": "synthetic",
-        "config": {"workload": args.config, "description": desc, "sample": what},
+        "config": workload_config(args.config, m, desc),
         "cpu_baseline": {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": what},
         "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
@@ -421,11 +433,10 @@ def main():
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "strong",
             "vs_baseline": None, "dtype": "u32", "data": "synthetic",
-            "config": {"workload": args.config, "description": desc, "ands": int(m.aig.num_ands),
-                       "pairs": int(m.num_pairs), "windows": info["num_windows"], "max_k": info["max_k"],
+            "config": workload_config(args.config, m, desc),
+            "plan": {"windows": info["num_windows"], "max_k": info["max_k"],
                        "max_slots": info["max_slots"], "node_patterns_per_step": W_all,
                        "parallelism": f"pattern-space shards x{world}", "cross_gpu_reduce": reduce_mode,
-                       "l2": "flushed between timed steps (256 MiB write, outside the events)",
                        "merge": ["off", "paper", "cost-aware"][merge], "engine": engine_name, "jit_kernels": st0["jit_kernels"], "jit_compile_ms": st0["jit_ms"],
                        "verdicts": verdicts},
             "clocks": clocks,

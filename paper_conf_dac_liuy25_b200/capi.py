@@ -154,8 +154,24 @@ def cec_free(ctx) -> None:
     lib.cec_free(ctx)
 
 
-def cec_sim_exhaustive(ctx, lit_a, lit_b) -> Tuple[np.ndarray, np.ndarray, np.ndarray]:
+def _pair_arrays(lit_a, lit_b) -> Tuple[np.ndarray, np.ndarray]:
+    """Both sides of a pair list as uint32 arrays of ONE length: the C side reads num_pairs entries
+    of each, so a shorter buffer would be read past its end."""
     la, lb = _u32(lit_a), _u32(lit_b)
+    if la.size != lb.size:
+        raise ValueError(f"lit_a has {la.size} entries, lit_b {lb.size}")
+    return la, lb
+
+
+def _ids_arrays(*arrs) -> Tuple[np.ndarray, ...]:
+    out = tuple(_u32(a) for a in arrs)
+    if len({a.size for a in out}) > 1:
+        raise ValueError(f"per-pair arrays differ in length: {[a.size for a in out]}")
+    return out
+
+
+def cec_sim_exhaustive(ctx, lit_a, lit_b) -> Tuple[np.ndarray, np.ndarray, np.ndarray]:
+    la, lb = _pair_arrays(lit_a, lit_b)
     n = la.size
     v = np.zeros(max(n, 1), np.int32)
     cex = np.zeros(max(n, 1), np.uint64)
@@ -165,9 +181,14 @@ def cec_sim_exhaustive(ctx, lit_a, lit_b) -> Tuple[np.ndarray, np.ndarray, np.nd
 
 
 def cec_check_local_cuts(ctx, lit_a, lit_b, cut_off, cut_leaves, raise_on_bad_cut: bool = False) -> np.ndarray:
-    la, lb, off = _u32(lit_a), _u32(lit_b), _u32(cut_off)
-    lv = _u32(cut_leaves) if len(cut_leaves) else np.zeros(1, np.uint32)
+    la, lb = _pair_arrays(lit_a, lit_b)
+    off = _u32(cut_off)
     n = la.size
+    nl = len(cut_leaves)
+    # CSR cut_off[n+1] (include/cec.h): the C side reads cut_leaves[cut_off[i] .. cut_off[i+1])
+    if off.size != n + 1 or int(off[0]) != 0 or int(off[-1]) != nl or (n and np.any(np.diff(off.astype(np.int64)) < 0)):
+        raise ValueError(f"cut_off must be a non-decreasing CSR offset array of {n + 1} entries from 0 to {nl}")
+    lv = _u32(cut_leaves) if nl else np.zeros(1, np.uint32)
     v = np.zeros(max(n, 1), np.int32)
     st = lib.cec_check_local_cuts(ctx, n, _p(la), _p(lb), _p(off), _p(lv), _p(v))
     if st == CEC_E_CUT and not raise_on_bad_cut:
@@ -195,7 +216,7 @@ def cec_sim_patterns(ctx, num_nodes: int, pi_words: np.ndarray):
 
 def cec_common_cuts(ctx, repr_ids, member_ids, k_l: int, C: int, pass_id: int, max_cuts: int):
     """Common cuts per candidate pair: (pair_cut_off[n+1], cut_off[ncut+1], leaves[...])."""
-    r, m = _u32(repr_ids), _u32(member_ids)
+    r, m = _ids_arrays(repr_ids, member_ids)
     n = r.size
     pco = np.zeros(n + 1, np.uint32)
     co = np.zeros(n * max_cuts + 1, np.uint32)
@@ -224,7 +245,8 @@ def cec_sim_classes(ctx, num_words: int, seed: int, pi_words: Optional[np.ndarra
 
 def cec_reduce(ctx, num_pis: int, num_ands: int, member_ids, repr_lits, lits=()):
     """GPU miter reduction: returns (new_fanins uint32 [A', 2], image uint32 [N], mapped lits)."""
-    m, r, lv = _u32(member_ids), _u32(repr_lits), _u32(lits).copy()
+    m, r = _ids_arrays(member_ids, repr_lits)
+    lv = _u32(lits).copy()
     fan = np.zeros(max(2 * num_ands, 2), np.uint32)
     img = np.zeros(1 + num_pis + num_ands, np.uint32)
     na = ctypes.c_uint32()
@@ -237,8 +259,10 @@ def cec_local_pass(ctx, repr_ids, member_ids, phases, k_l: int, C: int, pass_id:
                    buffer_checks: int = 4096, log: bool = True):
     """Alg. 2 pass: (verdict int32[npairs], checks) where checks = (pair uint32[n], cut_off uint32[n+1],
     leaves uint32[...], verdict int32[n]) in issue order (None when log=False)."""
-    r, m = _u32(repr_ids), _u32(member_ids)
+    r, m = _ids_arrays(repr_ids, member_ids)
     ph = np.ascontiguousarray(np.asarray(phases, dtype=np.uint8).reshape(-1))
+    if ph.size != r.size:
+        raise ValueError(f"phases has {ph.size} entries, expected {r.size}")
     n = r.size
     v = np.zeros(max(n, 1), np.int32)
     nc = ctypes.c_uint32()
@@ -276,7 +300,7 @@ def cec_pair_k(ctx, lit_a: int, lit_b: int) -> int:
 
 
 def cec_plan_exhaustive(ctx, lit_a, lit_b):
-    la, lb = _u32(lit_a), _u32(lit_b)
+    la, lb = _pair_arrays(lit_a, lit_b)
     plan = ctypes.c_void_p()
     _check(lib.cec_plan_exhaustive(ctx, la.size, _p(la), _p(lb), ctypes.byref(plan)), ctx)
     return plan

@@ -821,6 +821,8 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         wps_of.push_back(wps);
         // W accounting: nodes x patterns, per rank and all ranks
         const uint64_t slices = (ttw + wps - 1) / wps;
+        if (dw.k > MAX_K_ENUM || slices > UINT32_MAX)  // work items carry u32 slice bounds
+            return fail(c, CEC_E_ARG, "window %zu: k = %u exceeds the enumeration limit %zu", w, dw.k, MAX_K_ENUM);
         const uint64_t pats_all = dw.k < 5 ? (1ull << dw.k) : ttw * 32;
         P->W_all += (uint64_t)nodes.size() * pats_all;
         uint64_t sb, se;
@@ -1368,7 +1370,9 @@ static cec_status plan_route(cec_ctx *c, uint32_t n, const uint32_t *la, const u
     for (uint32_t i = 0; i < order.size(); ++i) order[i] = i;
     std::stable_sort(order.begin(), order.end(),
                      [&](uint32_t a, uint32_t b) { return lex_less(wins0[a].inputs, wins0[b].inputs); });
-    const uint32_t ks = std::min(c->opts.k_s, kmax);
+    // a merged window is enumerated like a single pair's: never more than MAX_K_ENUM inputs
+    // (its slice indices are u32), whatever k_s / k_max the caller passed
+    const uint32_t ks = std::min({c->opts.k_s, kmax, (uint32_t)MAX_K_ENUM});
     for (uint32_t oi : order) {
         WinHost &w = wins0[oi];
         if (!wins.empty() && c->opts.merge != CEC_MERGE_OFF) {

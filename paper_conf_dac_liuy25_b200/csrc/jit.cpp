@@ -466,7 +466,9 @@ std::string jit_source(const JitProgram &p, const JitConfig &cfg) {
              "    if (it >= nitems) return;\n"
              "    const JItem I = items[it];\n"
              "    for (u32 s = I.s_begin; s < I.s_end; ++s) {\n"
-             "      if (((u64)s << 10) >= *((volatile u64 *)&bound[I.win])) break;\n"
+             "      u64 bw = 0ull;\n"
+             "      if (lane == 0u) bw = *((volatile u64 *)&bound[I.win]);\n"
+             "      if (((u64)s << 10) >= __shfl_sync(0xFFFFFFFFu, bw, 0)) break;  /* warp-uniform exit */\n"
              "      const bool live = true;\n";
     } else {
         // block-synchronous: the block pulls an item and its warps take consecutive slices; a
@@ -572,7 +574,7 @@ std::string jit_source(const JitProgram &p, const JitConfig &cfg) {
                 s += "      __syncthreads();\n";
         }
     }
-    s += block_sync ? "      bnd = bnd_next;\n    }\n" ITEM_WAIT "    __syncthreads();\n  }\n}\n" : "    }\n  }\n}\n";
+    s += block_sync ? "      bnd = __shfl_sync(0xFFFFFFFFu, bnd_next, 0);\n    }\n" ITEM_WAIT "    __syncthreads();\n  }\n}\n" : "    }\n  }\n}\n";
     return s;
 }
 
@@ -674,7 +676,7 @@ std::string jit_source_bundle(const std::vector<const JitProgram *> &ps, const J
         }
         s += "      } break;\n";
     }
-    s += "      default: break;\n      }\n      bnd = bnd_next;\n    }\n" ITEM_WAIT "    __syncthreads();\n  }\n}\n";
+    s += "      default: break;\n      }\n      bnd = __shfl_sync(0xFFFFFFFFu, bnd_next, 0);\n    }\n" ITEM_WAIT "    __syncthreads();\n  }\n}\n";
     return s;
 }
 

@@ -107,7 +107,11 @@ interp_kernel(const Item *__restrict__ items, uint32_t nitems, uint32_t *__restr
         const uint64_t tt_words = ((uint64_t)W.tt_words_hi << 32) | W.tt_words_lo;
         for (uint32_t s = item.s_begin; s < item.s_end; ++s) {
             const uint64_t base = (uint64_t)s * (32u * IV);  // first word of the slice
-            if ((base << 5) >= *((volatile unsigned long long *)&bound[item.win])) break;
+            // bounded early exit (Q9): lane 0 reads the window bound and the warp takes ITS value,
+            // so the break and the full-mask votes below stay warp-uniform
+            unsigned long long bw = 0ull;
+            if (lane == 0) bw = *((volatile unsigned long long *)&bound[item.win]);
+            if ((base << 5) >= __shfl_sync(FULL, bw, 0)) break;
             const uint64_t w0 = base + lane, w1 = base + 32u + lane;
             const bool act0 = w0 < tt_words, act1 = w1 < tt_words;
             for (uint32_t j = 0; j < W.k; ++j) SLOT(j * SLOT_BYTES) = make_uint2(proj_word(j, w0), proj_word(j, w1));

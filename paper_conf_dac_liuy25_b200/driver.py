@@ -91,6 +91,20 @@ class Miter:
         return Miter(aig, lits[:P], lits[P:]), image
 
 
+def _remap_tried(tried, image: np.ndarray):
+    """(repr, member, phase) tuples of one miter version -> the same functional pairs in the reduced
+    version, whose node ids are renumbered (cec_reduce). `image[id]` = new literal of old node id.
+    A pair whose two sides collapsed into one node is dropped (nothing left to decide)."""
+    out = set()
+    for r, m_, f in tried:
+        a, b = int(image[r]), int(image[m_]) ^ f
+        if a >> 1 == b >> 1:
+            continue
+        lo, hi = (a, b) if (a >> 1) < (b >> 1) else (b, a)
+        out.add((lo >> 1, hi >> 1, (a ^ b) & 1))
+    return out
+
+
 def _ctx(aig: Aig, p: CecParams, k_max: int, k_s: Optional[int] = None) -> capi.Context:
     return capi.Context.from_aig(aig, device=p.device, k_max=k_max, k_s=k_s or k_max, engine=p.engine)
 
@@ -347,7 +361,7 @@ def check_miter(aig: Aig, lit_a, lit_b, params: Optional[CecParams] = None) -> C
         log.append(entry)
         if subst:
             t1 = time.perf_counter()
-            nxt, _ = cur.reduce(subst, p.device, ctx=ctx)
+            nxt, image = cur.reduce(subst, p.device, ctx=ctx)
             entry["s_parts"]["reduce"] = round(time.perf_counter() - t1, 4)
         ctx.close()
         if lctx is not ctx:
@@ -356,6 +370,10 @@ def check_miter(aig: Aig, lit_a, lit_b, params: Optional[CecParams] = None) -> C
         if not subst:
             break  # no progress: undecided remainder
         cur = nxt
+        # tried_global holds node ids of the old version: carry each decided pair over to its image
+        # in the new one (the reduction preserves every node's function), so a refuted pair is not
+        # re-simulated and a new pair that reuses old ids is not skipped
+        tried_global = _remap_tried(tried_global, image)
     st = po_status(cur)
     po_v = np.where(st == capi.CEC_EQUIVALENT, capi.CEC_EQUIVALENT, po_v)
     cex_vec, cex_pair = None, -1

@@ -137,3 +137,19 @@ def test_native_common_cuts_match_cut_oracle(case):
     for i in range(len(P)):
         got = [tuple(int(v) for v in lv[co[t]:co[t + 1]]) for t in range(int(pco[i]), int(pco[i + 1]))]
         assert got == want[i], (i, P[i], got, want[i])
+
+
+def test_tried_pairs_follow_the_reduction():
+    """ADVICE r1: the G phase's record of decided pairs is keyed by node ids of one miter version;
+    after cec_reduce renumbers the ANDs each entry must denote the same functional pair (the image
+    literals), and pairs whose sides collapsed are dropped."""
+    from paper_conf_dac_liuy25_b200.driver import _remap_tried
+    import numpy as np
+    # old ids 0..9; image = new literal of each old id
+    image = np.array([0, 2, 4, 6, 8, 10, 8, 13, 14, 9], np.uint32)
+    tried = {(4, 5, 0),   # images 8, 10 -> (4, 5, 0)
+             (4, 6, 0),   # 6 collapsed onto 4 (both image 8): dropped
+             (5, 7, 1),   # 10 vs 13 ^ 1 = 12 -> (5, 6, 0)
+             (3, 9, 0),   # 6 vs 9 -> (3, 4, 1)
+             (8, 2, 1)}   # 14 vs 4 ^ 1 = 5 -> lower id first: (2, 7, 1)
+    assert _remap_tried(tried, image) == {(4, 5, 0), (5, 6, 0), (3, 4, 1), (2, 7, 1)}

@@ -223,3 +223,57 @@ def test_peer_mode_needs_a_device_and_world():
     with pytest.raises(capi.CecError) as e:
         capi.cec_peer_import(ctx.handle, [bytes(128), bytes(128)])
     assert e.value.status == capi.CEC_E_CUDA
+
+
+def test_merge_never_exceeds_enumeration_limit():
+    """merging was bounded by min(k_s, k_max) only, so with k_max = 63 two
+    30-input windows could merge into a 45-input window whose 2^40 slices do not fit the u32 work
+    items (the tail was never simulated: a false EQ). The merge threshold is now also capped at the
+    enumeration limit (41 inputs, cec_host.cpp MAX_K_ENUM) that single pairs already obey."""
+    bd = Builder(60, strash=False)
+
+    def chain(lo, hi):
+        x = bd.pi(lo)
+        for i in range(lo + 1, hi):
+            x = bd.raw_and(x, bd.pi(i))
+        return x
+
+    f1, f2 = chain(0, 30), chain(15, 45)  # supports {1..30}, {16..45}: union of 45 PIs
+    aig = bd.finish([f1, f2])
+    for k_s in (0, 45, 63):
+        ctx = host_ctx(aig, k_max=63, k_s=k_s, engine=capi.CEC_ENGINE_INTERP)
+        plan = capi.cec_plan_exhaustive(ctx.handle, [f1, f2], [0, 0])
+        info = capi.cec_plan_info(plan)
+        assert info["num_windows"] == 2 and info["max_k"] == 30, (k_s, info)
+        capi.cec_plan_free(plan)
+        ctx.close()
+    # a pair whose own support exceeds the limit stays UNDECIDED (never enumerated)
+    f3 = chain(0, 42)
+    aig = bd.finish([f3])
+    ctx = host_ctx(aig, k_max=63, engine=capi.CEC_ENGINE_INTERP)
+    plan = capi.cec_plan_exhaustive(ctx.handle, [f3], [0])
+    assert capi.cec_plan_info(plan)["num_windows"] == 0
+    capi.cec_plan_free(plan)
+    ctx.close()
+
+
+def test_binding_rejects_mismatched_pair_arrays():
+    """the binding passes n = len(lit_a) to the C side, which reads n entries of every
+    per-pair array; mismatched lengths (or a cut_off that is not the CSR of the leaves) must be
+    refused before the call instead of reading past a numpy buffer."""
+    m = c1_add8()
+    ctx = host_ctx(m.aig)
+    with pytest.raises(ValueError):
+        ctx.sim_exhaustive(m.lit_a, m.lit_b[:-1])
+    with pytest.raises(ValueError):
+        capi.cec_plan_exhaustive(ctx.handle, m.lit_a[:3], m.lit_b)
+    for off, leaves in (([0], [1, 9]), ([0, 2, 2], [1, 9]), ([0, 3], [1, 9]), ([1, 2], [1, 9])):
+        with pytest.raises(ValueError):
+            ctx.check_local_cuts(m.lit_a[:1], m.lit_b[:1], off, leaves)
+    with pytest.raises(ValueError):
+        ctx.check_local_cuts(m.lit_a[:2], m.lit_b[:2], [0, 2, 1], [1, 9])
+    with pytest.raises(ValueError):
+        capi.cec_local_pass(ctx.handle, [1, 2], [3], [0, 0], 4, 4, 0, 4)
+    # well-formed arguments still reach the C side (which refuses: no device, no CPU fallback)
+    with pytest.raises(capi.CecError):
+        ctx.check_local_cuts(m.lit_a[:1], m.lit_b[:1], [0, 2], [1, 9])
