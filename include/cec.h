@@ -33,7 +33,7 @@
 extern "C" {
 #endif
 
-#define CEC_ABI_VERSION 1
+#define CEC_ABI_VERSION 2  /* 2: cec_stats.imad_words */
 #define CEC_NO_CEX UINT64_MAX
 
 typedef struct cec_ctx cec_ctx;
@@ -120,6 +120,9 @@ typedef struct {
     uint64_t lop3_words;       /* LOP3 instructions x u32 words this rank executes per run for the AND
                                   nodes: mapped 3-input LUTs for JIT windows (a LUT may evaluate
                                   two ANDs), one per AND for interpreter windows */
+    uint64_t imad_words;       /* IMAD cells x u32 words this rank executes per run: AND nodes of JIT
+                                  windows evaluated on the FMA pipe (mad.lo.u32 with a word-uniform
+                                  input word, 0 or ~0; jit.cpp "Dual-pipe cells") */
 } cec_stats;
 
 /* Fill *opts with the defaults above. */

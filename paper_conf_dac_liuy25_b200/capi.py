@@ -49,7 +49,8 @@ class CecStats(ctypes.Structure):
                 ("num_windows", ctypes.c_uint32), ("max_k", ctypes.c_uint32), ("max_slots", ctypes.c_uint32),
                 ("num_launches", ctypes.c_uint32), ("kernel_ms", ctypes.c_float), ("host_prep_ms", ctypes.c_float),
                 ("h2d_bytes", ctypes.c_uint64), ("d2h_bytes", ctypes.c_uint64), ("jit_ms", ctypes.c_float),
-                ("jit_kernels", ctypes.c_uint32), ("jit_windows", ctypes.c_uint32), ("lop3_words", ctypes.c_uint64)]
+                ("jit_kernels", ctypes.c_uint32), ("jit_windows", ctypes.c_uint32), ("lop3_words", ctypes.c_uint64),
+                ("imad_words", ctypes.c_uint64)]
 
     def as_dict(self):
         return {f: getattr(self, f) for f, _ in self._fields_}

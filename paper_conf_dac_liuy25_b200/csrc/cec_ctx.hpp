@@ -194,6 +194,7 @@ struct cec_plan {
     uint32_t jit_windows = 0, jit_kernels = 0;
     float jit_ms = 0.f;
     uint64_t lop3_words = 0;
+    uint64_t imad_words = 0;  // IMAD cells x words (JIT mode 3)
     SimtPlan simt;  // CEC_ENGINE_SIMT plans
     uint64_t W_rank = 0, W_all = 0;
     uint32_t max_k = 0, max_slots = 0;

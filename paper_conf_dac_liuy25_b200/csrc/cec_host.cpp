@@ -1028,6 +1028,10 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         const int32_t pi = win_jit[w];
         return pi >= 0 ? jit_kernel_lop3_sid(kernels[unit_of[pi]], sid_of[pi]) : P->win_nodes[w];
     };
+    auto imad_of = [&](uint32_t w) -> uint64_t {
+        const int32_t pi = win_jit[w];
+        return pi >= 0 ? jit_kernel_imad_sid(kernels[unit_of[pi]], sid_of[pi]) : 0;
+    };
     auto jwin = [&](uint32_t w) -> uint32_t {  // item window field: window | sid << 20 in bundles
         const int32_t pi = win_jit[w];
         return units[unit_of[pi]].size() > 1 ? (w | sid_of[pi] << 20) : w;
@@ -1037,9 +1041,11 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
     P->jit_kernels = (uint32_t)units.size();
     P->jit_windows = 0;
     P->lop3_words = 0;
+    P->imad_words = 0;
     for (uint32_t w = 0; w < win_jit.size(); ++w) {
         P->jit_windows += win_jit[w] >= 0;
         P->lop3_words += lop3_of(w) * words_rank_of[w];
+        P->imad_words += imad_of(w) * words_rank_of[w];
     }
     // work items: slices of each window split into chunks; interpreter windows grouped by slot
     // budget, JIT windows by structure; largest windows first inside a group
@@ -1420,6 +1426,7 @@ cec_status cec_plan_exhaustive(cec_ctx *c, uint32_t n, const uint32_t *la, const
     c->stats.jit_kernels = P->jit_kernels;
     c->stats.jit_windows = P->jit_windows;
     c->stats.lop3_words = P->lop3_words;
+    c->stats.imad_words = P->imad_words;
     st = upload(c, P.get());
     if (st != CEC_OK) {
         free_dev(P.get());
@@ -1481,6 +1488,7 @@ cec_status cec_plan_run(cec_ctx *c, cec_plan *P) {
     c->stats.num_windows = (uint32_t)P->dwin.size();
     c->stats.max_k = P->max_k;
     c->stats.max_slots = P->max_slots;
+    c->stats.imad_words = P->imad_words;
     c->stats.lop3_words = P->lop3_words;  // this run's algorithmic LOP3 words (local checks included)
     c->stats.jit_windows = P->jit_windows;
     c->stats.jit_kernels = P->jit_kernels;
@@ -1687,6 +1695,7 @@ cec_status cec_sim_exhaustive(cec_ctx *c, uint32_t n, const uint32_t *la, const 
         agg.jit_kernels += S.p->jit_kernels;
         agg.jit_windows += S.p->jit_windows;
         agg.lop3_words += S.p->lop3_words;
+        agg.imad_words += S.p->imad_words;
         agg.h2d_bytes += c->stats.h2d_bytes;
         jit_ms += S.p->jit_ms;
         subs.push_back(std::move(S));
@@ -1737,6 +1746,7 @@ cec_status cec_sim_exhaustive(cec_ctx *c, uint32_t n, const uint32_t *la, const 
     c->stats.jit_kernels = agg.jit_kernels;
     c->stats.jit_windows = agg.jit_windows;
     c->stats.lop3_words = agg.lop3_words;
+    c->stats.imad_words = agg.imad_words;
     c->stats.h2d_bytes = agg.h2d_bytes;
     c->stats.d2h_bytes = sizeof(unsigned long long) * first.size();
     c->stats.jit_ms = jit_ms;

@@ -60,8 +60,9 @@ struct JitConfig {
     int threads = 512;      // threads per block
     int min_blocks = 1;     // __launch_bounds__ min blocks per SM (registers <= 64K / (threads*min_blocks))
     int sync_every = 512;   // block-synchronous: __syncthreads() every this many LOP3s; 0 = warp-independent
-    int fuse = 2;           // 3-input LUT mapping: 0 none, 1 greedy (absorb single-fanout ANDs into the
-                            // reader's LOP3), 2 area-flow mapping over 3-feasible cuts
+    int fuse = 3;           // 3-input LUT mapping: 0 none, 1 greedy (absorb single-fanout ANDs into the
+                            // reader's LOP3), 2 area-flow mapping over 3-feasible cuts, 3 = 2 plus
+                            // IMAD cells on the FMA pipe (jit.cpp, "Dual-pipe cells")
     bool splice = true;     // body as generated PTX spliced into an NVRTC skeleton (skips NVVM on it)
 };
 struct LaunchGroup {       // windows sharing one kernel launch
@@ -124,7 +125,9 @@ bool jit_kernel_loaded(const JitKernel *k);  // true once the cubin is loaded (k
 double jit_compile_ms(const JitKernel *k);
 int jit_slices_per_pass(const JitKernel *k);
 uint32_t jit_kernel_lop3(const JitKernel *k);
-uint32_t jit_lop3_count(const JitProgram &p, int mode);
+uint32_t jit_lop3_count(const JitProgram &p, int mode, uint32_t *imads = nullptr);
+uint32_t jit_kernel_imad_sid(const JitKernel *k, uint32_t sid);
+int jit_eff_mode(const JitConfig &cfg);
 const char *jit_launch(JitKernel *K, const JItem *items, uint32_t nitems, uint32_t *ctr, unsigned long long *first,
                        unsigned long long *bound, uint32_t *neq_cnt, void *stream, int num_sms);
 

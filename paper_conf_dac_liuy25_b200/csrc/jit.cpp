@@ -20,6 +20,7 @@
 
 #include <algorithm>
 #include <chrono>
+#include <cmath>
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
@@ -100,6 +101,7 @@ struct JitKernel {
     int slices_per_pass = 1;  // block-synchronous kernels: warps per block
     uint32_t lop3 = 0;        // LOP3 instructions per word of the mapped window (structure 0)
     std::vector<uint32_t> lop3s;  // per structure of a bundle (sid order)
+    std::vector<uint32_t> imads;  // IMAD cells per word, per structure (mode 3)
     double compile_ms = 0;
     size_t src_bytes = 0, cubin_bytes = 0;
 };
@@ -127,8 +129,11 @@ std::string jit_key(const JitProgram &p) {
 struct MappedNode {
     bool absorbed = false;
     uint8_t nleaves = 0;
-    uint32_t leaf[3] = {0, 0, 0};  // operand refs
-    uint8_t tt = 0;
+    uint32_t leaf[3] = {0, 0, 0};  // operand refs (IMAD: leaf[0] = y, leaf[1] = the word-uniform input m)
+    uint8_t tt = 0;                // LOP3 table over the STORED leaf values
+    bool imad = false;             // cell on the FMA pipe: mad.lo.u32 (see imad_cell below)
+    uint8_t imad_c = 0;            // addend of the mad: 0 = m, 1 = y, 2 = -1
+    bool pol = false;              // the register holds the complement of the node's function
 };
 
 std::vector<MappedNode> jit_map(const JitProgram &p, bool fuse) {
@@ -214,12 +219,86 @@ std::vector<MappedNode> jit_map(const JitProgram &p, bool fuse) {
 // then walks from the compare roots down: a node is materialised (one LOP3) iff it is a root or a
 // leaf of a chosen cut; every other AND is evaluated inside the LUT of the node that covers it
 // (possibly inside several LUTs — duplication is what lets multi-fanout logic be absorbed too).
-std::vector<MappedNode> jit_map_area(const JitProgram &p) {
+//
+// Dual-pipe cells (mode 3). The ALU pipe that runs LOP3 is the bound (64 LOP3/clk/SM); the FMA pipe
+// beside it (IMAD, same rate, B300_MICROARCH.md "Pipe rates") is idle. A window input j >= 5 is
+// word-uniform: every u32 word of it is 0 or ~0 (PAPER.md:33 projection words; j = 5..9 depend on
+// the lane, j >= 10 on the slice). For such an m and ANY word y, mad.lo.u32 computes exact bitwise
+// logic: y*m + m = ~y & m, y*m + y = y & ~m, y*m - 1 = ~(y & m) (m = 0 -> the addend; m = ~0 = -1
+// -> addend - y). So a node whose function over a 2-leaf cut {y, m} is an AND of the two with any
+// edge complements except ~y & ~m can be evaluated by ONE IMAD on the FMA pipe (the register then
+// holds the function or its complement; readers fold that polarity into their LOP3 tables, just as
+// they fold edge complements). Every AND node is still evaluated on every pattern — on the other
+// pipe. The mapper prices an IMAD cell at `imad_cost` LUTs, so it takes them where they relieve the
+// ALU pipe; ~y & ~m (no single-IMAD form with operands y, m, -1) and XOR-type cuts stay LOP3s.
+namespace {
+constexpr uint8_t kLeafTT[3] = {0xF0, 0xCC, 0xAA};
+// g = the 2-input function of (y, m) as a 4-bit table, bit (2*y + m). Returns the IMAD form
+// (addend: 0 = m, 1 = y, 2 = -1; *pol: register holds the complement) or -1 if none exists.
+int imad_cell(uint8_t g, bool *pol) {
+    switch (g) {
+        case 0x2: *pol = false; return 0;  // ~y & m   = y*m + m
+        case 0x4: *pol = false; return 1;  // y & ~m   = y*m + y
+        case 0x7: *pol = false; return 2;  // ~(y & m) = y*m - 1
+        case 0x8: *pol = true; return 2;   // y & m    = ~(y*m - 1)
+        case 0xB: *pol = true; return 1;   // y | ~m   = ~(y*m + y)
+        case 0xD: *pol = true; return 0;   // ~y | m   = ~(y*m + m)
+        default: return -1;
+    }
+}
+// 4-bit (y, m) table of an 8-bit LOP3-style table whose leaf ypos / mpos carry y / m
+uint8_t g_of(uint8_t tt, int ypos, int mpos) {
+    uint8_t g = 0;
+    for (int yv = 0; yv < 2; ++yv)
+        for (int mv = 0; mv < 2; ++mv) {
+            int idx = 0;
+            idx |= yv << (2 - ypos);
+            idx |= mv << (2 - mpos);
+            g |= (uint8_t)(((tt >> idx) & 1) << (2 * yv + mv));
+        }
+    return g;
+}
+}  // namespace
+
+std::vector<MappedNode> jit_map_area(const JitProgram &p, double imad_cost) {
     const uint32_t n = (uint32_t)(p.nodes.size() / 2), ncmp = (uint32_t)(p.cmps.size() / 2);
     const uint32_t R = p.k + 1 + n;
     struct C3 {
         uint8_t m;
+        uint8_t tt;  // the node's function over l[0..m-1] at (0xF0, 0xCC, 0xAA); const-0 leaves read 0
         uint32_t l[3];
+    };
+    const bool dual = imad_cost >= 0.0;
+    auto word_uniform = [&](uint32_t r) { return r >= 6 && r <= p.k; };  // input index r-1 >= 5
+    // an IMAD form for cut c: returns the m leaf position (y = the other) or -1
+    auto imad_pos = [&](const C3 &c) -> int {
+        if (!dual || c.m != 2) return -1;
+        for (int mp = 1; mp >= 0; --mp) {
+            const int yp = 1 - mp;
+            if (!word_uniform(c.l[mp]) || c.l[yp] == 0) continue;
+            bool pl;
+            const uint8_t g = g_of(c.tt, yp, mp);
+            if (imad_cell(g, &pl) >= 0) return mp;
+            // ~y & ~m and y | m have a form once y is held complemented: fine when y is a LOP3
+            // output (its polarity is free), decided by the readers' votes below
+            if ((g == 0x1 || g == 0xE) && c.l[yp] > p.k) return mp;
+        }
+        return -1;
+    };
+    // truth table of cut u re-expressed over the (sorted) leaf list L[0..m)
+    auto tt_on = [&](const C3 &u, const uint32_t *L, int m) -> uint8_t {
+        uint8_t v[3] = {0, 0, 0};
+        for (int i = 0; i < u.m; ++i) {
+            if (u.l[i] == 0) continue;
+            for (int j = 0; j < m; ++j)
+                if (L[j] == u.l[i]) v[i] = kLeafTT[j];
+        }
+        uint8_t out = 0;
+        for (int bit = 0; bit < 8; ++bit) {
+            const int idx = (((v[0] >> bit) & 1) << 2) | (((v[1] >> bit) & 1) << 1) | ((v[2] >> bit) & 1);
+            out |= (uint8_t)(((u.tt >> idx) & 1) << bit);
+        }
+        return out;
     };
     std::vector<uint32_t> fanout(R, 0);
     for (uint32_t i = 0; i < 2 * n; ++i) ++fanout[p.nodes[i] >> 1];
@@ -230,6 +309,7 @@ std::vector<MappedNode> jit_map_area(const JitProgram &p) {
     std::vector<std::vector<C3>> cuts(R);
     std::vector<double> af(R, 0.0);
     std::vector<C3> best(R);
+    std::vector<uint8_t> bim(R, 0);  // best implementation is an IMAD cell
     std::vector<bool> req(R, false);
     std::vector<double> est(fanout.begin(), fanout.end());  // fanout estimate used by area flow
     static const size_t CAP = getenv("CEC_MAP_CAP") ? (size_t)atoi(getenv("CEC_MAP_CAP")) : 16;
@@ -237,8 +317,9 @@ std::vector<MappedNode> jit_map_area(const JitProgram &p) {
     for (int iter = 0; iter < ITER; ++iter) {
         for (uint32_t r = 0; r < R; ++r) cuts[r].clear();
         for (uint32_t r = 0; r <= p.k; ++r) {
-            cuts[r].push_back(C3{1, {r, 0, 0}});
+            cuts[r].push_back(C3{1, 0xF0, {r, 0, 0}});
             best[r] = cuts[r][0];
+            bim[r] = 0;
             af[r] = 0.0;
         }
         auto cost = [&](const C3 &c) {
@@ -248,7 +329,8 @@ std::vector<MappedNode> jit_map_area(const JitProgram &p) {
         };
         for (uint32_t t = 0; t < n; ++t) {
             const uint32_t me = p.k + 1 + t;
-            const uint32_t a = p.nodes[2 * t] >> 1, b = p.nodes[2 * t + 1] >> 1;
+            const uint32_t oa = p.nodes[2 * t], ob = p.nodes[2 * t + 1];
+            const uint32_t a = oa >> 1, b = ob >> 1;
             std::vector<C3> cand;
             for (const C3 &u : cuts[a])
                 for (const C3 &v : cuts[b]) {
@@ -259,8 +341,9 @@ std::vector<MappedNode> jit_map_area(const JitProgram &p) {
                     std::sort(L, L + m);
                     m = (int)(std::unique(L, L + m) - L);
                     if (m > 3) continue;
-                    C3 c{(uint8_t)m, {0, 0, 0}};
+                    C3 c{(uint8_t)m, 0, {0, 0, 0}};
                     for (int i = 0; i < m; ++i) c.l[i] = L[i];
+                    c.tt = (uint8_t)((tt_on(u, L, m) ^ ((oa & 1u) ? 0xFF : 0)) & (tt_on(v, L, m) ^ ((ob & 1u) ? 0xFF : 0)));
                     bool dup = false;
                     for (const C3 &d : cand)
                         if (d.m == c.m && std::equal(d.l, d.l + d.m, c.l)) dup = true;
@@ -272,11 +355,22 @@ std::vector<MappedNode> jit_map_area(const JitProgram &p) {
                 if (x.m != y.m) return x.m < y.m;
                 return std::lexicographical_compare(x.l, x.l + x.m, y.l, y.l + y.m);
             });
-            if (cand.size() > CAP) cand.resize(CAP);
             best[me] = cand[0];  // the trivial {a, b} merge always exists
             af[me] = cost(cand[0]);
+            bim[me] = 0;
+            for (const C3 &c : cand)  // an IMAD cell over a 2-leaf cut: same flow, cheaper cell
+                if (imad_pos(c) >= 0 && cost(c) - 1.0 + imad_cost < af[me]) {
+                    best[me] = c;
+                    af[me] = cost(c) - 1.0 + imad_cost;
+                    bim[me] = 1;
+                }
+            if (cand.size() > CAP) cand.resize(CAP);
             cuts[me] = cand;
-            cuts[me].push_back(C3{1, {me, 0, 0}});  // the trivial cut, for readers
+            if (bim[me] && std::find_if(cand.begin(), cand.end(), [&](const C3 &c) {
+                    return c.m == best[me].m && std::equal(c.l, c.l + c.m, best[me].l);
+                }) == cand.end())
+                cuts[me].push_back(best[me]);  // keep the chosen IMAD cut among the node's cuts
+            cuts[me].push_back(C3{1, 0xF0, {me, 0, 0}});  // the trivial cut, for readers
         }
         // cover from the roots
         std::fill(req.begin(), req.end(), false);
@@ -299,6 +393,8 @@ std::vector<MappedNode> jit_map_area(const JitProgram &p) {
     // exact local area recovery: with the cover's reference counts, each node in topological order
     // takes the cut whose LUTs NOT already shared with the rest of the cover are fewest (the area
     // it adds if referenced = LUTs that become live; dereferencing gives it back). Two passes.
+    // areas in quarter-LUTs: a LOP3 cell = 4, an IMAD cell = round(4 * imad_cost)
+    const uint32_t WL = 4, WI = dual ? (uint32_t)std::lround(4.0 * std::max(0.0, imad_cost)) : 4;
     std::vector<int32_t> nref(R, 0);
     for (uint32_t r = 0; r < R; ++r)
         if (root[r]) ++nref[r];
@@ -308,7 +404,7 @@ std::vector<MappedNode> jit_map_area(const JitProgram &p) {
             for (int i = 0; i < best[me].m; ++i) ++nref[best[me].l[i]];
     }
     std::function<uint32_t(uint32_t)> ref_cut = [&](uint32_t r) -> uint32_t {
-        uint32_t a = 1;
+        uint32_t a = bim[r] ? WI : WL;
         for (int i = 0; i < best[r].m; ++i) {
             const uint32_t l = best[r].l[i];
             if (l > p.k && nref[l]++ == 0) a += ref_cut(l);
@@ -316,7 +412,7 @@ std::vector<MappedNode> jit_map_area(const JitProgram &p) {
         return a;
     };
     std::function<uint32_t(uint32_t)> deref_cut = [&](uint32_t r) -> uint32_t {
-        uint32_t a = 1;
+        uint32_t a = bim[r] ? WI : WL;
         for (int i = 0; i < best[r].m; ++i) {
             const uint32_t l = best[r].l[i];
             if (l > p.k && --nref[l] == 0) a += deref_cut(l);
@@ -330,18 +426,25 @@ std::vector<MappedNode> jit_map_area(const JitProgram &p) {
             const bool mapped = nref[me] > 0;
             if (mapped) deref_cut(me);
             C3 keep = best[me];
+            uint8_t keep_im = bim[me];
             uint32_t best_a = UINT32_MAX;
             for (const C3 &c : cuts[me]) {
                 if (c.m == 1 && c.l[0] == me) continue;  // the trivial cut
-                best[me] = c;
-                const uint32_t a = ref_cut(me);
-                deref_cut(me);
-                if (a < best_a) {
-                    best_a = a;
-                    keep = c;
+                for (uint8_t im = 0; im < 2; ++im) {
+                    if (im && imad_pos(c) < 0) continue;
+                    best[me] = c;
+                    bim[me] = im;
+                    const uint32_t a = ref_cut(me);
+                    deref_cut(me);
+                    if (a < best_a) {
+                        best_a = a;
+                        keep = c;
+                        keep_im = im;
+                    }
                 }
             }
             best[me] = keep;
+            bim[me] = keep_im;
             if (mapped) ref_cut(me);
         }
     for (uint32_t r = 0; r < R; ++r) req[r] = nref[r] > 0;
@@ -368,6 +471,23 @@ std::vector<MappedNode> jit_map_area(const JitProgram &p) {
         val[r] = v;
         return v;
     };
+    // polarity of every materialised signal: the register holds function ^ pol (inputs: 0). A LOP3
+    // cell may hold either polarity for free: it takes the one most of its IMAD readers need (an
+    // IMAD whose (y, m) table is y & ~m or ~y | m needs y as is, ~y & ~m or y | m needs ~y).
+    std::vector<int32_t> vote(R, 0);
+    for (uint32_t t = 0; t < n; ++t) {
+        const uint32_t me = p.k + 1 + t;
+        if (!req[me] || !bim[me]) continue;
+        const C3 &c = best[me];
+        const int mp = imad_pos(c);
+        if (mp < 0) continue;
+        const uint32_t y = c.l[1 - mp];
+        if (y <= p.k || bim[y]) continue;
+        const uint8_t g = g_of(c.tt, 1 - mp, mp);
+        if (g == 0x4 || g == 0xD) --vote[y];
+        if (g == 0x1 || g == 0xE) ++vote[y];
+    }
+    std::vector<uint8_t> pol(R, 0);
     for (uint32_t t = 0; t < n; ++t) {
         const uint32_t me = p.k + 1 + t;
         MappedNode &x = out[t];
@@ -375,9 +495,9 @@ std::vector<MappedNode> jit_map_area(const JitProgram &p) {
         if (x.absorbed) continue;
         const C3 &c = best[me];
         ++ep;
-        for (int i = 0; i < c.m; ++i) {
+        for (int i = 0; i < c.m; ++i) {  // leaf i is read as its STORED value (polarity folded in)
             stamp[c.l[i]] = ep;
-            val[c.l[i]] = c.l[i] == 0 ? 0 : K[i];
+            val[c.l[i]] = c.l[i] == 0 ? 0 : (uint8_t)(K[i] ^ (pol[c.l[i]] ? 0xFF : 0));
         }
         // evaluate node me itself over its cut (its own value is not a leaf)
         const uint32_t oa = p.nodes[2 * t], ob = p.nodes[2 * t + 1];
@@ -385,17 +505,122 @@ std::vector<MappedNode> jit_map_area(const JitProgram &p) {
         x.tt = va & vb;
         x.nleaves = c.m;
         for (int i = 0; i < 3; ++i) x.leaf[i] = i < c.m ? c.l[i] : 0;
+        if (!bim[me] && vote[me] > 0) {  // LOP3 cell holding the complement
+            x.tt = (uint8_t)~x.tt;
+            x.pol = true;
+        }
+        if (bim[me]) {  // IMAD cell, if the stored polarity of y still admits a form (else a LOP3)
+            for (int mp = 1; mp >= 0 && !x.imad; --mp) {
+                const int yp = 1 - mp;
+                if (!word_uniform(c.l[mp]) || c.l[yp] == 0) continue;
+                bool pl = false;
+                const int form = imad_cell(g_of(x.tt, yp, mp), &pl);
+                if (form < 0) continue;
+                x.imad = true;
+                x.imad_c = (uint8_t)form;
+                x.pol = pl;
+                x.leaf[0] = c.l[yp];
+                x.leaf[1] = c.l[mp];
+                x.leaf[2] = 0;
+            }
+        }
+        pol[me] = x.pol;
     }
     return out;
 }
 
-std::vector<MappedNode> jit_map_mode(const JitProgram &p, int mode) {
-    return mode == 2 ? jit_map_area(p) : jit_map(p, mode != 0);
+// IMAD cells (mode 3) are emitted by the PTX-splice body only; other code paths map with mode 2
+int jit_eff_mode(const JitConfig &cfg) {
+    return cfg.fuse == 3 && !(cfg.splice && cfg.sync_every > 0) ? 2 : cfg.fuse;
 }
 
-uint32_t jit_lop3_count(const JitProgram &p, int mode) {
-    uint32_t c = 0;
-    for (const MappedNode &x : jit_map_mode(p, mode)) c += !x.absorbed;
+double jit_imad_cost() {  // CEC_MAP_IMAD: price of an IMAD cell in LUTs (mode 3)
+    static const double v = getenv("CEC_MAP_IMAD") ? atof(getenv("CEC_MAP_IMAD")) : 0.25;
+    return v;
+}
+
+std::vector<MappedNode> jit_map_mode(const JitProgram &p, int mode) {
+    if (mode == 3) return jit_map_area(p, jit_imad_cost());
+    return mode == 2 ? jit_map_area(p, -1.0) : jit_map(p, mode != 0);
+}
+
+// Host-side check of a mapping (CEC_JIT_VERIFY=1, and the CPU tests): evaluate the mapped cell
+// network exactly as the body executes it (lop3.b32 tables over stored leaf values, mad.lo.u32 with
+// 32-bit wrap-around, %cz for missing leaves) on `words` u32 words — inputs 0..4 the P:33 masks,
+// inputs >= 5 random 0 / ~0 words (word-uniform, as in the kernels) — and compare every
+// materialised cell with the AIG's own AND evaluation, polarity included, and every compare's diff.
+const char *jit_verify_map(const JitProgram &p, int mode, uint32_t words, uint64_t seed) {
+    static const uint32_t masks[5] = {0xAAAAAAAAu, 0xCCCCCCCCu, 0xF0F0F0F0u, 0xFF00FF00u, 0xFFFF0000u};
+    const uint32_t n = (uint32_t)(p.nodes.size() / 2), ncmp = (uint32_t)(p.cmps.size() / 2);
+    const std::vector<MappedNode> map = jit_map_mode(p, mode);
+    std::vector<uint32_t> v(p.k + 1 + n), st(p.k + 1 + n);
+    uint64_t x = seed * 0x9E3779B97F4A7C15ull + 1;
+    auto rnd = [&]() {  // splitmix64
+        uint64_t z = (x += 0x9E3779B97F4A7C15ull);
+        z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+        z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+        return z ^ (z >> 31);
+    };
+    static thread_local std::string msg;
+    // test hook (tests/test_jit_map.py): emulate the first IMAD cell with a wrong addend, so the
+    // check itself is shown to catch a wrong cell
+    const bool break_imad = getenv("CEC_JIT_BREAK_IMAD") != nullptr;
+    uint32_t first_imad = UINT32_MAX;
+    for (uint32_t t = 0; t < n && first_imad == UINT32_MAX; ++t)
+        if (map[t].imad) first_imad = t;
+    for (uint32_t w = 0; w < words; ++w) {
+        v[0] = st[0] = 0;
+        for (uint32_t j = 0; j < p.k; ++j) v[j + 1] = st[j + 1] = j < 5 ? masks[j] : ((rnd() & 1) ? ~0u : 0u);
+        for (uint32_t t = 0; t < n; ++t) {
+            const uint32_t oa = p.nodes[2 * t], ob = p.nodes[2 * t + 1], me = p.k + 1 + t;
+            v[me] = (v[oa >> 1] ^ ((oa & 1u) ? ~0u : 0u)) & (v[ob >> 1] ^ ((ob & 1u) ? ~0u : 0u));
+            const MappedNode &c = map[t];
+            if (c.absorbed) continue;
+            uint32_t r;
+            if (c.imad) {
+                const uint32_t y = st[c.leaf[0]], m = st[c.leaf[1]];
+                const uint8_t form = (break_imad && t == first_imad) ? (uint8_t)((c.imad_c + 1) % 3) : c.imad_c;
+                r = y * m + (form == 0 ? m : form == 1 ? y : ~0u);
+            } else {
+                const uint32_t a = c.nleaves > 0 ? st[c.leaf[0]] : 0u, b = c.nleaves > 1 ? st[c.leaf[1]] : 0u,
+                               d = c.nleaves > 2 ? st[c.leaf[2]] : 0u;
+                r = 0;
+                for (int bit = 0; bit < 32; ++bit) {
+                    const int idx = (((a >> bit) & 1) << 2) | (((b >> bit) & 1) << 1) | ((d >> bit) & 1);
+                    r |= (uint32_t)((c.tt >> idx) & 1) << bit;
+                }
+            }
+            st[me] = r;
+            if (r != (v[me] ^ (c.pol ? ~0u : 0u))) {
+                char b[200];
+                snprintf(b, sizeof b, "mapped cell of node %u (%s, pol %d) = %08x, AIG gives %08x", t,
+                         c.imad ? "imad" : "lop3", (int)c.pol, r, v[me]);
+                msg = b;
+                return msg.c_str();
+            }
+        }
+        for (uint32_t q = 0; q < ncmp; ++q) {  // the body's diff: stored a ^ stored b ^ folded polarity
+            const uint32_t a = p.cmps[2 * q], b = p.cmps[2 * q + 1];
+            auto pl = [&](uint32_t r) { return r > p.k ? map[r - p.k - 1].pol : false; };
+            const bool inv = (((a ^ b) & 1u) != 0) != (pl(a >> 1) != pl(b >> 1));
+            const uint32_t d = st[a >> 1] ^ st[b >> 1] ^ (inv ? ~0u : 0u);
+            const uint32_t want = (v[a >> 1] ^ ((a & 1u) ? ~0u : 0u)) ^ (v[b >> 1] ^ ((b & 1u) ? ~0u : 0u));
+            if (d != want) {
+                msg = "compare " + std::to_string(q) + ": mapped diff differs from the AIG's";
+                return msg.c_str();
+            }
+        }
+    }
+    return nullptr;
+}
+
+uint32_t jit_lop3_count(const JitProgram &p, int mode, uint32_t *imads) {
+    uint32_t c = 0, im = 0;
+    for (const MappedNode &x : jit_map_mode(p, mode)) {
+        c += !x.absorbed && !x.imad;
+        im += x.imad;
+    }
+    if (imads) *imads = im;
     return c;
 }
 
@@ -550,7 +775,7 @@ std::string jit_source(const JitProgram &p, const JitConfig &cfg) {
             s += buf;
         }
     } else {
-        const std::vector<MappedNode> map = jit_map_mode(p, cfg.fuse);
+        const std::vector<MappedNode> map = jit_map_mode(p, jit_eff_mode(cfg));
         uint32_t lut_total = 0;
         for (const MappedNode &x : map) lut_total += !x.absorbed;
         for (uint32_t c : after[0]) emit_cmp(c);
@@ -686,9 +911,11 @@ std::string jit_source_bundle(const std::vector<const JitProgram *> &ps, const J
 std::string jit_body_ptx(const JitProgram &p, const JitConfig &cfg, const std::vector<std::string> &masks,
                          const std::vector<std::string> &in_regs, const std::string &dbuf) {
     const uint32_t n = (uint32_t)(p.nodes.size() / 2), ncmp = (uint32_t)(p.cmps.size() / 2);
-    const std::vector<MappedNode> map = jit_map_mode(p, cfg.fuse);
+    const std::vector<MappedNode> map = jit_map_mode(p, jit_eff_mode(cfg));
     uint32_t lut_total = 0;
     for (const MappedNode &x : map) lut_total += !x.absorbed;
+    std::vector<uint8_t> pol(p.k + 1 + n, 0);  // stored polarity per ref (IMAD cells may hold ~f)
+    for (uint32_t t = 0; t < n; ++t) pol[p.k + 1 + t] = map[t].pol;
     std::string s;
     s.reserve(64 * (size_t)n + 160 * (size_t)ncmp + 4096);
     char buf[320];
@@ -709,7 +936,8 @@ std::string jit_body_ptx(const JitProgram &p, const JitConfig &cfg, const std::v
     }
     auto emit_cmp = [&](uint32_t c) {
         const uint32_t a = p.cmps[2 * c], b = p.cmps[2 * c + 1];
-        const unsigned lut = ((a ^ b) & 1u) ? 0xC3u : 0x3Cu;  // ~(a ^ b) : a ^ b on (0xF0, 0xCC)
+        const bool inv = (((a ^ b) & 1u) != 0) != (pol[a >> 1] != pol[b >> 1]);
+        const unsigned lut = inv ? 0xC3u : 0x3Cu;  // ~(a ^ b) : a ^ b on (0xF0, 0xCC)
         snprintf(buf, sizeof buf,
                  "lop3.b32 %%cd, %s, %s, %%cz, 0x%02X;\nsetp.ne.b32 %%cp, %%cd, 0;\nvote.sync.any.pred %%cq, %%cp, 0xffffffff;\n"
                  "@%%cq st.u32 [%s+%u], %%cd;\n@%%cq or.b32 %s, %s, %u;\n",
@@ -721,7 +949,13 @@ std::string jit_body_ptx(const JitProgram &p, const JitConfig &cfg, const std::v
     uint32_t emitted = 0;
     for (uint32_t t = 0; t < n; ++t) {
         const MappedNode &x = map[t];
-        if (!x.absorbed) {
+        if (x.imad) {  // FMA-pipe cell: y * m + {m, y, -1} (imad_cell)
+            const std::string y = reg(x.leaf[0]), m = reg(x.leaf[1]);
+            snprintf(buf, sizeof buf, "mad.lo.u32 %%cn%u, %s, %s, %s;\n", t, y.c_str(), m.c_str(),
+                     x.imad_c == 0 ? m.c_str() : x.imad_c == 1 ? y.c_str() : "-1");
+            s += buf;
+            ++emitted;
+        } else if (!x.absorbed) {
             snprintf(buf, sizeof buf, "lop3.b32 %%cn%u, %s, %s, %s, 0x%02X;\n", t,
                      x.nleaves > 0 ? reg(x.leaf[0]).c_str() : "%cz", x.nleaves > 1 ? reg(x.leaf[1]).c_str() : "%cz",
                      x.nleaves > 2 ? reg(x.leaf[2]).c_str() : "%cz", x.tt);
@@ -900,6 +1134,9 @@ const char *jit_get_unit(const std::vector<const JitProgram *> &ps, const JitCon
         }
     }
     auto t0 = std::chrono::steady_clock::now();
+    if (getenv("CEC_JIT_VERIFY"))  // host emulation of every mapped body against the AIG
+        for (const JitProgram *p : ps)
+            if (const char *e = jit_verify_map(*p, jit_eff_mode(cfg), 64, p->nodes.size())) return e;
     const std::string src = bundle ? jit_source_bundle(ps, cfg) : jit_source(*ps[0], cfg);
     std::vector<char> cubin;
     std::string log;
@@ -926,7 +1163,11 @@ const char *jit_get_unit(const std::vector<const JitProgram *> &ps, const JitCon
     }
     std::unique_ptr<JitKernel> K(new JitKernel());
     K->block = cfg.threads;
-    for (const JitProgram *p : ps) K->lop3s.push_back(jit_lop3_count(*p, cfg.fuse));
+    for (const JitProgram *p : ps) {
+        uint32_t im = 0;
+        K->lop3s.push_back(jit_lop3_count(*p, jit_eff_mode(cfg), &im));
+        K->imads.push_back(im);
+    }
     K->lop3 = K->lop3s[0];
     K->slices_per_pass = cfg.sync_every > 0 ? cfg.threads / 32 : 1;
     K->src_bytes = src.size();
@@ -959,6 +1200,9 @@ uint32_t jit_kernel_lop3(const JitKernel *k) { return k ? k->lop3 : 0; }
 bool jit_kernel_loaded(const JitKernel *k) { return k && k->kern; }
 uint32_t jit_kernel_lop3_sid(const JitKernel *k, uint32_t sid) {
     return k && sid < k->lop3s.size() ? k->lop3s[sid] : 0;
+}
+uint32_t jit_kernel_imad_sid(const JitKernel *k, uint32_t sid) {
+    return k && sid < k->imads.size() ? k->imads[sid] : 0;
 }
 
 const char *jit_launch(JitKernel *K, const JItem *items, uint32_t nitems, uint32_t *ctr, unsigned long long *first,

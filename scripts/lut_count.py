@@ -20,5 +20,6 @@ info = capi.cec_plan_info(plan)
 st = ctx.stats()
 print(st)
 W = info["node_patterns"]
-print(f"{name}: W={W:.4g} lop3_words={st['lop3_words']} lop3/and={st['lop3_words'] * 32 / W:.4f} plan {dt:.1f}s")
+print(f"{name}: W={W:.4g} lop3_words={st['lop3_words']} lop3/and={st['lop3_words'] * 32 / W:.4f} "
+      f"imad/and={st['imad_words'] * 32 / W:.4f} plan {dt:.1f}s")
 capi.cec_plan_free(plan)

@@ -116,3 +116,37 @@ def test_own_index_closed_form_V4_merged_windows():
     assert list(ov) == list(v) and list(ok) == list(k)
     assert [int(x) for x in oc[:2]] == [107, 11]
     ctx.close()
+
+
+def test_k41_maximum_window_closed_form():
+    """The largest enumerated window (k = 41 = the enumeration limit, 2^41 patterns = 2^31 JIT
+    slices: the top of the u32 slice range; input 40 is bit 30 of the slice index). A 41-input AND
+    chain vs a balanced tree is EQ over the whole cube; vs constant 0 it differs ONLY at the very
+    last pattern, own index 2^41 - 1, so the last slice must be simulated; vs the AND of the first
+    40 inputs it first differs at 2^40 - 1 (x1..x40 = 1, x41 = 0). k = 42 exceeds the limit and is
+    routed to UNDECIDED even with k_max = 63. Closed forms (P:33 index convention)."""
+    bd = Builder(42)
+    x = [bd.pi(i) for i in range(42)]
+
+    def chain(v):
+        c = v[0]
+        for t in v[1:]:
+            c = bd.AND(c, t)
+        return c
+
+    def tree(v):
+        while len(v) > 1:
+            v = [bd.AND(v[i], v[i + 1]) if i + 1 < len(v) else v[i] for i in range(0, len(v), 2)]
+        return v[0]
+
+    c41, t41, c40, c42 = chain(x[:41]), tree(list(reversed(x[:41]))), tree(x[:40]), chain(x)
+    aig = bd.finish([c41, t41, c40, c42])
+    ctx = capi.Context.from_aig(aig, device=0, k_max=63, engine=capi.CEC_ENGINE_JIT)
+    v, c, k = ctx.sim_exhaustive([c41, c41, c40, c42], [t41, 0, c41, 0])
+    assert list(k) == [41, 41, 41, 42]
+    assert list(v) == [EQ, NEQ, NEQ, UND]
+    assert int(c[1]) == (1 << 41) - 1
+    assert int(c[2]) == (1 << 40) - 1
+    assert list(ctx.get_cex(1)) == [1] * 41 + [0]
+    assert list(ctx.get_cex(2)) == [1] * 40 + [0, 0]
+    ctx.close()

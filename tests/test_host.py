@@ -26,7 +26,7 @@ def test_exports_match_header():
     assert declared == set(capi.EXPORTS), declared ^ set(capi.EXPORTS)
     for name in declared:
         assert hasattr(capi.lib, name)  # dlsym succeeds
-    assert capi.cec_abi_version() == 1
+    assert capi.cec_abi_version() == 2
 
 
 def test_opts_layout_and_defaults():
