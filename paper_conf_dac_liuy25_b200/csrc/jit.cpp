@@ -269,8 +269,21 @@ std::vector<MappedNode> jit_map_area(const JitProgram &p, double imad_cost) {
         uint32_t l[3];
     };
     const bool dual = imad_cost >= 0.0;
-    auto word_uniform = [&](uint32_t r) { return r >= 6 && r <= p.k; };  // input index r-1 >= 5
-    // an IMAD form for cut c: returns the m leaf position (y = the other) or -1
+    // word-uniform signals: inputs j >= 5 and every node whose support lies inside them (its words
+    // are then 0 or ~0 too); CEC_MAP_WU_NODES=0 keeps the inputs only
+    static const bool wu_nodes = !getenv("CEC_MAP_WU_NODES") || atoi(getenv("CEC_MAP_WU_NODES")) != 0;
+    std::vector<uint8_t> wu(R, 0);
+    for (uint32_t r = 6; r <= p.k; ++r) wu[r] = 1;
+    if (wu_nodes)
+        for (uint32_t t = 0; t < n; ++t) {
+            const uint32_t a = p.nodes[2 * t] >> 1, b = p.nodes[2 * t + 1] >> 1;
+            wu[p.k + 1 + t] = (a == 0 || wu[a]) && (b == 0 || wu[b]);
+        }
+    auto word_uniform = [&](uint32_t r) { return r != 0 && wu[r] != 0; };
+    // an IMAD form for cut c: returns the m leaf position (y = the other) or -1. The form depends
+    // on the stored polarities of y and m (see imad_cell); the mapper accepts any AND-type table
+    // that has a form now, or could get one by flipping a leaf that is a node (whose polarity is
+    // chosen below); the final pass falls back to a LOP3 where no form remains.
     auto imad_pos = [&](const C3 &c) -> int {
         if (!dual || c.m != 2) return -1;
         for (int mp = 1; mp >= 0; --mp) {
@@ -279,9 +292,7 @@ std::vector<MappedNode> jit_map_area(const JitProgram &p, double imad_cost) {
             bool pl;
             const uint8_t g = g_of(c.tt, yp, mp);
             if (imad_cell(g, &pl) >= 0) return mp;
-            // ~y & ~m and y | m have a form once y is held complemented: fine when y is a LOP3
-            // output (its polarity is free), decided by the readers' votes below
-            if ((g == 0x1 || g == 0xE) && c.l[yp] > p.k) return mp;
+            if ((g == 0x1 || g == 0xE) && (c.l[yp] > p.k || c.l[mp] > p.k)) return mp;
         }
         return -1;
     };
@@ -472,22 +483,34 @@ std::vector<MappedNode> jit_map_area(const JitProgram &p, double imad_cost) {
         return v;
     };
     // polarity of every materialised signal: the register holds function ^ pol (inputs: 0). A LOP3
-    // cell may hold either polarity for free: it takes the one most of its IMAD readers need (an
-    // IMAD whose (y, m) table is y & ~m or ~y | m needs y as is, ~y & ~m or y | m needs ~y).
-    std::vector<int32_t> vote(R, 0);
+    // cell may hold either polarity for free: in topological order it takes the one under which
+    // more of its IMAD readers have a form (each reader's other leaf at its polarity if already
+    // decided, else as is). An IMAD cell's polarity is fixed by its form.
+    std::vector<std::vector<uint32_t>> readers(R);
     for (uint32_t t = 0; t < n; ++t) {
         const uint32_t me = p.k + 1 + t;
-        if (!req[me] || !bim[me]) continue;
-        const C3 &c = best[me];
-        const int mp = imad_pos(c);
-        if (mp < 0) continue;
-        const uint32_t y = c.l[1 - mp];
-        if (y <= p.k || bim[y]) continue;
-        const uint8_t g = g_of(c.tt, 1 - mp, mp);
-        if (g == 0x4 || g == 0xD) --vote[y];
-        if (g == 0x1 || g == 0xE) ++vote[y];
+        if (req[me] && bim[me] && best[me].m == 2)
+            for (int i = 0; i < 2; ++i) readers[best[me].l[i]].push_back(me);
     }
-    std::vector<uint8_t> pol(R, 0);
+    std::vector<uint8_t> pol(R, 0), decided(R, 0);
+    auto flip = [](uint8_t g, bool fy, bool fm) {  // (y, m) table with y and/or m complemented
+        uint8_t o = 0;
+        for (int yv = 0; yv < 2; ++yv)
+            for (int mv = 0; mv < 2; ++mv)
+                o |= (uint8_t)(((g >> (2 * yv + mv)) & 1) << (2 * (yv ^ (int)fy) + (mv ^ (int)fm)));
+        return o;
+    };
+    auto reader_fits = [&](uint32_t q, uint32_t who, bool who_pol) {
+        const C3 &c = best[q];
+        for (int mp = 1; mp >= 0; --mp) {
+            const int yp = 1 - mp;
+            if (!word_uniform(c.l[mp]) || c.l[yp] == 0) continue;
+            auto pl = [&](uint32_t r) { return r == who ? who_pol : (decided[r] ? pol[r] != 0 : false); };
+            bool f;
+            if (imad_cell(flip(g_of(c.tt, yp, mp), pl(c.l[yp]), pl(c.l[mp])), &f) >= 0) return true;
+        }
+        return false;
+    };
     for (uint32_t t = 0; t < n; ++t) {
         const uint32_t me = p.k + 1 + t;
         MappedNode &x = out[t];
@@ -505,9 +528,13 @@ std::vector<MappedNode> jit_map_area(const JitProgram &p, double imad_cost) {
         x.tt = va & vb;
         x.nleaves = c.m;
         for (int i = 0; i < 3; ++i) x.leaf[i] = i < c.m ? c.l[i] : 0;
-        if (!bim[me] && vote[me] > 0) {  // LOP3 cell holding the complement
-            x.tt = (uint8_t)~x.tt;
-            x.pol = true;
+        if (!bim[me] && !readers[me].empty()) {
+            int score = 0;
+            for (uint32_t q : readers[me]) score += (int)reader_fits(q, me, true) - (int)reader_fits(q, me, false);
+            if (score > 0) {  // LOP3 cell holding the complement
+                x.tt = (uint8_t)~x.tt;
+                x.pol = true;
+            }
         }
         if (bim[me]) {  // IMAD cell, if the stored polarity of y still admits a form (else a LOP3)
             for (int mp = 1; mp >= 0 && !x.imad; --mp) {
@@ -525,6 +552,7 @@ std::vector<MappedNode> jit_map_area(const JitProgram &p, double imad_cost) {
             }
         }
         pol[me] = x.pol;
+        decided[me] = 1;
     }
     return out;
 }

@@ -19,6 +19,10 @@ KEYS = [
     ("gpu__time_duration.sum", "duration"),
     ("sm__throughput.avg.pct_of_peak_sustained_elapsed", "SM throughput % of peak"),
     ("sm__pipe_alu_cycles_active.avg.pct_of_peak_sustained_active", "ALU pipe active % of peak"),
+    ("sm__pipe_fma_cycles_active.avg.pct_of_peak_sustained_active", "FMA pipe active % of peak"),
+    ("sm__inst_executed_pipe_alu.sum", "warp instructions on the ALU pipe"),
+    ("sm__inst_executed_pipe_fma.sum", "warp instructions on the FMA pipe"),
+    ("smsp__issue_active.avg.pct_of_peak_sustained_active", "issue slots busy %"),
     ("sm__inst_executed.avg.per_cycle_active", "IPC (per SM, active)"),
     ("smsp__inst_executed.sum", "warp instructions executed"),
     ("sm__warps_active.avg.pct_of_peak_sustained_active", "achieved occupancy %"),
