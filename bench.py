@@ -15,8 +15,9 @@ value      = W (node-patterns of one step, all ranks) / device time per step (CU
              launch stream, max over ranks), schedules resident in HBM, L2 flushed between steps
 e2e        = same metric through the public blocking C call cec_sim_exhaustive with host arrays
              (planning + H2D of schedules + kernels + all-reduce + D2H of results per step)
-roofline   = ALU (LOP3) bound: 1 LOP3 per node per 32 patterns (u32 word) is the algorithmic work;
-             peak = 148 SMs x 64 LOP3/clk/SM x SM clock
+roofline   = ALU (LOP3) bound: the mapped window's lop3.b32 cells per u32 word (32 patterns) are the
+             work of the binding pipe; peak = 148 SMs x 64 LOP3/clk/SM x SM clock.
+             IMAD cells (AND nodes with a word-uniform operand, FMA pipe) are reported beside it.
 cpu_baseline / --impl reference = the oracle (oracle/, plain single-threaded C) timed on a bounded
              sample of the same workload on this host.
 """
@@ -455,6 +456,10 @@ def main():
                          "frac": achieved / peak, "traffic": traffic,
                          "peak_basis": f"{props.multi_processor_count} SMs x {LOP3_PER_CLK_PER_SM} LOP3/clk x {sm_clock:.0f} MHz (guide unit counts, SM clock; microbenchmark scripts/peaks.cu measured 64.00 LOP3/clk/SM = 18.53 TLOP3/s at 1957 MHz, profiles/round1_peaks.json)",
                          "lop3_per_word_per_and": stats["lop3_words"] / max(1.0, W_rank / 32.0),
+                         "imad_per_word_per_and": stats.get("imad_words", 0) / max(1.0, W_rank / 32.0),
+                         "fma_pipe_timad_s": stats.get("imad_words", 0) / (ms / 1e3) / 1e12,
+                         "cells": "3-input LUTs = lop3.b32 on the ALU pipe (the bound); AND nodes with a "
+                                  "word-uniform operand = mad.lo.u32 on the FMA pipe (DESIGN.md §4.1)",
                          "and_evals_tops": (W_rank / 32.0) / (ms / 1e3) / 1e12}),
             "step_ms": step_ms, "wall_s": wall,
         }

@@ -1,0 +1,128 @@
+// pipes.cu — does work on the FMA pipe (mad.lo.u32) come for free beside a saturated ALU pipe
+// (lop3.b32)? Measurement tooling for the dual-pipe cells of jit.cpp (not part of libcec).
+//
+// Each thread runs 8 independent LOP3 chains and J independent IMAD chains per unrolled step
+// (J = 0, 1, 2, 4, 8: 0 .. 1 IMAD per LOP3), 16 warps per SM like the window kernels. Reported
+// per mix: LOP3/clk/SM and IMAD/clk/SM from the SM's own clock64. A second set interleaves the
+// two kinds in ONE dependency chain (lop3 -> mad -> lop3 ...) to expose the cross-pipe latency.
+// Build: nvcc -O3 -gencode arch=compute_100a,code=sm_100a -o pipes scripts/pipes.cu
+#include <cuda_runtime.h>
+
+#include <cstdint>
+#include <cstdio>
+#include <vector>
+
+#define CK(x)                                                                         \
+    do {                                                                              \
+        cudaError_t e_ = (x);                                                         \
+        if (e_ != cudaSuccess) {                                                      \
+            fprintf(stderr, "%s:%d %s\n", __FILE__, __LINE__, cudaGetErrorString(e_)); \
+            return 1;                                                                 \
+        }                                                                             \
+    } while (0)
+
+__device__ __forceinline__ uint32_t lop3(uint32_t a, uint32_t b, uint32_t c) {
+    uint32_t r;
+    asm volatile("lop3.b32 %0, %1, %2, %3, 0x96;" : "=r"(r) : "r"(a), "r"(b), "r"(c));
+    return r;
+}
+__device__ __forceinline__ uint32_t imad(uint32_t a, uint32_t b, uint32_t c) {
+    uint32_t r;
+    asm volatile("mad.lo.u32 %0, %1, %2, %3;" : "=r"(r) : "r"(a), "r"(b), "r"(c));
+    return r;
+}
+__device__ __forceinline__ unsigned smid() {
+    unsigned r;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(r));
+    return r;
+}
+
+constexpr int CHAINS = 8, UNROLL = 32;
+
+template <int J, bool MIXED>
+__global__ void __launch_bounds__(256) mix(uint32_t *out, int iters, unsigned long long *sm_t0, unsigned long long *sm_t1) {
+    uint32_t x[CHAINS], w[J > 0 ? J : 1];
+    const uint32_t y = threadIdx.x * 0x9E3779B9u, z = blockIdx.x * 0x85EBCA6Bu;
+    const uint32_t m = (threadIdx.x & 32u) ? ~0u : 0u;  // word-uniform mask, as in the kernels
+    for (int c = 0; c < CHAINS; ++c) x[c] = threadIdx.x + c;
+    for (int j = 0; j < J; ++j) w[j] = threadIdx.x * 7u + j;
+    __syncthreads();
+    const unsigned long long t0 = clock64();
+    for (int i = 0; i < iters; ++i) {
+#pragma unroll
+        for (int u = 0; u < UNROLL; ++u) {
+#pragma unroll
+            for (int c = 0; c < CHAINS; ++c) x[c] = lop3(x[c], y, z);
+            if (MIXED) {  // IMADs fed by the LOP3 chains and feeding them back
+#pragma unroll
+                for (int j = 0; j < J; ++j) x[j] = imad(x[j], m, m);
+            } else {
+#pragma unroll
+                for (int j = 0; j < J; ++j) w[j] = imad(w[j], m, y);
+            }
+        }
+    }
+    __syncthreads();
+    const unsigned long long t1 = clock64();
+    uint32_t acc = 0;
+    for (int c = 0; c < CHAINS; ++c) acc ^= x[c];
+    for (int j = 0; j < J; ++j) acc ^= w[j];
+    if (acc == 0x12345678u) out[0] = acc;
+    if (threadIdx.x == 0) {
+        const unsigned s = smid();
+        atomicMin(&sm_t0[s], t0);
+        atomicMax(&sm_t1[s], t1);
+    }
+}
+
+template <int J, bool MIXED>
+int run(int sms, uint32_t *out, unsigned long long *t0, unsigned long long *t1, bool last) {
+    const int blocks = sms * 2, threads = 256, iters = 1000;
+    mix<J, MIXED><<<blocks, threads>>>(out, 20, t0, t1);
+    CK(cudaDeviceSynchronize());
+    double best = 0;
+    for (int rep = 0; rep < 3; ++rep) {
+        CK(cudaMemset(t0, 0xFF, 8 * 1024));
+        CK(cudaMemset(t1, 0, 8 * 1024));
+        mix<J, MIXED><<<blocks, threads>>>(out, iters, t0, t1);
+        CK(cudaDeviceSynchronize());
+        std::vector<unsigned long long> h0(1024), h1(1024);
+        CK(cudaMemcpy(h0.data(), t0, 8 * 1024, cudaMemcpyDeviceToHost));
+        CK(cudaMemcpy(h1.data(), t1, 8 * 1024, cudaMemcpyDeviceToHost));
+        double cyc = 0;
+        int n = 0;
+        for (int s = 0; s < 1024; ++s)
+            if (h1[s] > 0 && h0[s] != ~0ull) {
+                cyc += (double)(h1[s] - h0[s]);
+                ++n;
+            }
+        cyc /= n;
+        const double lop = (double)blocks * threads * iters * UNROLL * CHAINS / n / cyc;
+        if (lop > best) best = lop;
+    }
+    printf("{\"imad_per_lop3\": %.3f, \"mixed_chain\": %s, \"lop3_per_clk_per_sm\": %.2f, \"imad_per_clk_per_sm\": %.2f}%s\n",
+           (double)J / CHAINS, MIXED ? "true" : "false", best, best * J / CHAINS, last ? "" : ",");
+    return 0;
+}
+
+int main() {
+    cudaDeviceProp prop;
+    CK(cudaGetDeviceProperties(&prop, 0));
+    const int sms = prop.multiProcessorCount;
+    uint32_t *out;
+    unsigned long long *t0, *t1;
+    CK(cudaMalloc(&out, 4));
+    CK(cudaMalloc(&t0, 8 * 1024));
+    CK(cudaMalloc(&t1, 8 * 1024));
+    printf("[\n");
+    run<0, false>(sms, out, t0, t1, false);
+    run<1, false>(sms, out, t0, t1, false);
+    run<2, false>(sms, out, t0, t1, false);
+    run<4, false>(sms, out, t0, t1, false);
+    run<8, false>(sms, out, t0, t1, false);
+    run<1, true>(sms, out, t0, t1, false);
+    run<2, true>(sms, out, t0, t1, false);
+    run<4, true>(sms, out, t0, t1, true);
+    printf("]\n");
+    return 0;
+}

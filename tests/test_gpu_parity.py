@@ -488,3 +488,19 @@ def test_c3_full_vs_stored_oracle():
     ve, ce, ke = ctx.sim_exhaustive(m.lit_a, m.lit_b)  # the pipelined public call agrees
     assert np.array_equal(ve, gv) and np.array_equal(ke, gk)
     assert np.array_equal(ce[gv == capi.CEC_NOT_EQUIVALENT], gc[gv == capi.CEC_NOT_EQUIVALENT])
+
+
+@pytest.mark.parametrize("mode", ["0", "1", "2", "3"])
+def test_jit_cell_mappings_vs_oracle(mode, monkeypatch):
+    """Every cell mapping of the JIT body (0: one LOP3 per AND, 1: greedy fusion, 2: area-flow
+    3-LUTs, 3: 3-LUTs + IMAD cells on the FMA pipe, the default) gives the oracle's verdicts, k and
+    canonical CEX indices bit for bit: a multiplier with an injected bug (NEQ, early exit), a
+    reduced C5 (word-uniform masks from inputs and nodes) and C3-style random windows."""
+    monkeypatch.setenv("CEC_JIT_FUSE", mode)
+    for m in (c2_mul12_bug(seed=1, n=10), c5_big(copies=6, n_random=4, n_bugs=2, rand_pis=18, rand_ands=1200, mul_n=9),
+              circuits.random_miter(20, 900, 12, seed=77, window=40)):
+        ctx, gv, gc, gk = check_vs_oracle(m, engine=capi.CEC_ENGINE_JIT)
+        st = ctx.stats()
+        assert st["jit_windows"] >= 1
+        assert (st["imad_words"] > 0) == (mode == "3") or m.name.startswith("rand")
+        ctx.close()
