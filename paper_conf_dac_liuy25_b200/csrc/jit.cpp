@@ -563,7 +563,7 @@ int jit_eff_mode(const JitConfig &cfg) {
 }
 
 double jit_imad_cost() {  // CEC_MAP_IMAD: price of an IMAD cell in LUTs (mode 3)
-    static const double v = getenv("CEC_MAP_IMAD") ? atof(getenv("CEC_MAP_IMAD")) : 0.25;
+    static const double v = getenv("CEC_MAP_IMAD") ? atof(getenv("CEC_MAP_IMAD")) : 0.5;
     return v;
 }
 
