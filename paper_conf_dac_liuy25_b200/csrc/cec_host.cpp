@@ -634,27 +634,39 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         std::vector<uint32_t> &nodes = R.nodes;
         {
             const uint32_t ep = X.next_epoch();
-            std::vector<std::pair<uint32_t, uint8_t>> st;
+            // raw pointers: the loop is latency-bound on these lookups (no vector reloads)
+            const uint32_t *f0 = c->f0.data(), *f1 = c->f1.data(), *lvl = c->level.data();
+            uint32_t *stamp = X.stamp.data();
+            const uint32_t *stop = X.stop.data();
+            const uint32_t I = c->I;
+            std::vector<uint32_t> st;  // node << 1 | (second fanin done)
+            st.reserve(256);
+            nodes.reserve(1024);
+            auto enter = [&](uint32_t x) { return stamp[x] != ep && x > I && stop[x] != sep; };
             for (uint32_t r : roots) {
-                if (X.stamp[r] == ep || !c->is_and(r) || X.stop[r] == sep) continue;
-                st.push_back({r, 0});
-                X.stamp[r] = ep;
+                if (!enter(r)) continue;
+                stamp[r] = ep;
+                st.push_back(r << 1);
                 while (!st.empty()) {
-                    auto &top = st.back();
-                    const uint32_t v = top.first;
-                    if (top.second < 2) {
-                        uint32_t a = c->f0[v] >> 1, b = c->f1[v] >> 1;
-                        if (c->level[b] > c->level[a]) std::swap(a, b);  // deeper first
-                        const uint32_t nxt = top.second == 0 ? a : b;
-                        ++top.second;
-                        if (X.stamp[nxt] != ep && c->is_and(nxt) && X.stop[nxt] != sep) {
-                            X.stamp[nxt] = ep;
-                            st.push_back({nxt, 0});
+                    const uint32_t top = st.back(), v = top >> 1;
+                    uint32_t a = f0[v] >> 1, b = f1[v] >> 1;
+                    if (lvl[b] > lvl[a]) std::swap(a, b);  // deeper fanin first
+                    if (!(top & 1u)) {  // first visit: descend into a (then b)
+                        st.back() = top | 1u;
+                        if (enter(a)) {
+                            stamp[a] = ep;
+                            st.push_back(a << 1);
+                            continue;
                         }
-                    } else {
-                        nodes.push_back(v);
-                        st.pop_back();
                     }
+                    // a done: descend into b unless done, else emit v
+                    if (enter(b)) {
+                        stamp[b] = ep;
+                        st.push_back(b << 1);
+                        continue;
+                    }
+                    nodes.push_back(v);
+                    st.pop_back();
                 }
             }
         }
@@ -662,8 +674,21 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         // order with the smaller live set (counted without building the schedule)
         std::string why;
         {
-            std::vector<uint32_t> by_id(nodes);
-            std::sort(by_id.begin(), by_id.end());
+            // ascending ids: a flag scan over the window's id range (ids of a window are dense
+            // in practice: one copy / one block), else a sort
+            std::vector<uint32_t> by_id;
+            by_id.reserve(nodes.size());
+            uint32_t lo = UINT32_MAX, hi = 0;
+            for (uint32_t v : nodes) lo = std::min(lo, v), hi = std::max(hi, v);
+            if (!nodes.empty() && (uint64_t)(hi - lo) + 1 <= 8 * (uint64_t)nodes.size() + 64) {
+                std::vector<uint8_t> flag(hi - lo + 1, 0);
+                for (uint32_t v : nodes) flag[v - lo] = 1;
+                for (uint32_t i = 0; i <= hi - lo; ++i)
+                    if (flag[i]) by_id.push_back(lo + i);
+            } else {
+                by_id = nodes;
+                std::sort(by_id.begin(), by_id.end());
+            }
             const uint32_t l_id = live_peak(c, X, W.inputs, by_id, cmps2, wc);
             const uint32_t l_dfs = live_peak(c, X, W.inputs, nodes, cmps2, wc);
             if (l_id < l_dfs) nodes.swap(by_id);
@@ -1322,8 +1347,9 @@ static cec_status plan_route(cec_ctx *c, uint32_t n, const uint32_t *la, const u
         }
     }
     tm.lap("supports");
+    seen.reserve(2 * (size_t)n);
     for (uint32_t p = 0; p < n; ++p) {
-        const std::vector<uint32_t> &S = supp[p];
+        std::vector<uint32_t> &S = supp[p];
         const uint64_t cone = cones[p];
         P->k[p] = (uint32_t)S.size();
         if (la[p] == lb[p]) {
@@ -1346,13 +1372,8 @@ static cec_status plan_route(cec_ctx *c, uint32_t n, const uint32_t *la, const u
             P->pair_cmp[p] = (int32_t)it->second;
             continue;
         }
-        Cmp cm;
-        cm.la = la[p];
-        cm.lb = lb[p];
-        cm.S = S;
         const uint32_t ci = (uint32_t)P->cmps.size();
-        P->cmps.push_back(std::move(cm));
-        seen[key] = ci;
+        seen.emplace(key, ci);
         P->pair_cmp[p] = (int32_t)ci;
         std::vector<uint32_t> &cand = by_support[supp_hash(S)];
         uint32_t wi = UINT32_MAX;
@@ -1370,6 +1391,11 @@ static cec_status plan_route(cec_ctx *c, uint32_t n, const uint32_t *la, const u
             w.cmps.push_back(ci);
             w.est_nodes = std::max<uint64_t>(w.est_nodes, cone);
         }
+        Cmp cm;  // the pair's support moves into its compare (no copy)
+        cm.la = la[p];
+        cm.lb = lb[p];
+        cm.S = std::move(S);
+        P->cmps.push_back(std::move(cm));
     }
     // a5: window merging: windows sorted lexicographically by input list.
     std::vector<uint32_t> order(wins0.size());

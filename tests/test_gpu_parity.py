@@ -504,3 +504,16 @@ def test_jit_cell_mappings_vs_oracle(mode, monkeypatch):
         assert st["jit_windows"] >= 1
         assert (st["imad_words"] > 0) == (mode == "3") or m.name.startswith("rand")
         ctx.close()
+
+
+@pytest.mark.parametrize("seed", range(24))
+def test_fuzz_jit_windows_word_uniform_inputs(seed):
+    """JIT windows at the input positions where the dual-pipe cells change: k = 10..14 (inputs 0..4
+    per-bit masks, 5..9 lane-uniform, >= 10 slice-uniform words), random AIGs whose ANDs read PIs
+    often (many IMAD candidates: AND of a PI or of a node over PIs >= 5 with anything), random
+    pair literals including complemented and constant ones; JIT engine vs the oracle, bit for bit."""
+    rng = np.random.default_rng(500 + seed)
+    I = int(rng.integers(10, 15))
+    m = tiny_random(I, int(rng.integers(40, 260)), 20, 9000 + seed)
+    ctx, gv, gc, gk = check_vs_oracle(m, k_max=14, merge=int(rng.integers(0, 3)), engine=capi.CEC_ENGINE_JIT)
+    ctx.close()
