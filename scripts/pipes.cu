@@ -39,6 +39,38 @@ __device__ __forceinline__ unsigned smid() {
 
 constexpr int CHAINS = 8, UNROLL = 32;
 
+// register-read pressure variant: every LOP3 reads three DIFFERENT live chain registers (no operand
+// reuse across instructions), every IMAD reads its own chain register, a mask and another chain
+template <int J>
+__global__ void __launch_bounds__(256) mixrf(uint32_t *out, int iters, unsigned long long *sm_t0, unsigned long long *sm_t1) {
+    uint32_t x[CHAINS], w[J > 0 ? J : 1];
+    const uint32_t m = (threadIdx.x & 32u) ? ~0u : 0u;
+    for (int c = 0; c < CHAINS; ++c) x[c] = threadIdx.x * (c + 3);
+    for (int j = 0; j < J; ++j) w[j] = threadIdx.x * 7u + j;
+    __syncthreads();
+    const unsigned long long t0 = clock64();
+    for (int i = 0; i < iters; ++i) {
+#pragma unroll
+        for (int u = 0; u < UNROLL; ++u) {
+#pragma unroll
+            for (int c = 0; c < CHAINS; ++c) x[c] = lop3(x[c], x[(c + 3) % CHAINS], x[(c + 5) % CHAINS]);
+#pragma unroll
+            for (int j = 0; j < J; ++j) w[j] = imad(w[j], m, x[(j + 1) % CHAINS]);
+        }
+    }
+    __syncthreads();
+    const unsigned long long t1 = clock64();
+    uint32_t acc = 0;
+    for (int c = 0; c < CHAINS; ++c) acc ^= x[c];
+    for (int j = 0; j < J; ++j) acc ^= w[j];
+    if (acc == 0x12345678u) out[0] = acc;
+    if (threadIdx.x == 0) {
+        const unsigned s = smid();
+        atomicMin(&sm_t0[s], t0);
+        atomicMax(&sm_t1[s], t1);
+    }
+}
+
 template <int J, bool MIXED>
 __global__ void __launch_bounds__(256) mix(uint32_t *out, int iters, unsigned long long *sm_t0, unsigned long long *sm_t1) {
     uint32_t x[CHAINS], w[J > 0 ? J : 1];
@@ -75,16 +107,20 @@ __global__ void __launch_bounds__(256) mix(uint32_t *out, int iters, unsigned lo
     }
 }
 
-template <int J, bool MIXED>
+template <int J, bool MIXED, bool RF = false>
 int run(int sms, uint32_t *out, unsigned long long *t0, unsigned long long *t1, bool last) {
     const int blocks = sms * 2, threads = 256, iters = 1000;
-    mix<J, MIXED><<<blocks, threads>>>(out, 20, t0, t1);
+    auto launch = [&](int it) {
+        if (RF) mixrf<J><<<blocks, threads>>>(out, it, t0, t1);
+        else mix<J, MIXED><<<blocks, threads>>>(out, it, t0, t1);
+    };
+    launch(20);
     CK(cudaDeviceSynchronize());
     double best = 0;
     for (int rep = 0; rep < 3; ++rep) {
         CK(cudaMemset(t0, 0xFF, 8 * 1024));
         CK(cudaMemset(t1, 0, 8 * 1024));
-        mix<J, MIXED><<<blocks, threads>>>(out, iters, t0, t1);
+        launch(iters);
         CK(cudaDeviceSynchronize());
         std::vector<unsigned long long> h0(1024), h1(1024);
         CK(cudaMemcpy(h0.data(), t0, 8 * 1024, cudaMemcpyDeviceToHost));
@@ -100,8 +136,8 @@ int run(int sms, uint32_t *out, unsigned long long *t0, unsigned long long *t1, 
         const double lop = (double)blocks * threads * iters * UNROLL * CHAINS / n / cyc;
         if (lop > best) best = lop;
     }
-    printf("{\"imad_per_lop3\": %.3f, \"mixed_chain\": %s, \"lop3_per_clk_per_sm\": %.2f, \"imad_per_clk_per_sm\": %.2f}%s\n",
-           (double)J / CHAINS, MIXED ? "true" : "false", best, best * J / CHAINS, last ? "" : ",");
+    printf("{\"imad_per_lop3\": %.3f, \"mixed_chain\": %s, \"distinct_operands\": %s, \"lop3_per_clk_per_sm\": %.2f, \"imad_per_clk_per_sm\": %.2f}%s\n",
+           (double)J / CHAINS, MIXED ? "true" : "false", RF ? "true" : "false", best, best * J / CHAINS, last ? "" : ",");
     return 0;
 }
 
@@ -122,7 +158,11 @@ int main() {
     run<8, false>(sms, out, t0, t1, false);
     run<1, true>(sms, out, t0, t1, false);
     run<2, true>(sms, out, t0, t1, false);
-    run<4, true>(sms, out, t0, t1, true);
+    run<4, true>(sms, out, t0, t1, false);
+    run<0, false, true>(sms, out, t0, t1, false);
+    run<1, false, true>(sms, out, t0, t1, false);
+    run<2, false, true>(sms, out, t0, t1, false);
+    run<4, false, true>(sms, out, t0, t1, true);
     printf("]\n");
     return 0;
 }
