@@ -207,6 +207,7 @@ struct cec_plan {
     size_t arena_cap = 0;
     void *ev0 = nullptr, *ev1 = nullptr;
     bool ran = false;
+    bool no_join = false;  // pipelined call, not its last chunk: skip the side-stream join (launch_run)
     uint32_t runs = 0;                     // completed cec_plan_run calls
     void *graph = nullptr, *graph_stream = nullptr;  // captured run (replayed from the 2nd run on)
     uint32_t graph_launches = 0;

@@ -1499,7 +1499,8 @@ cec_status cec_plan_run(cec_ctx *c, cec_plan *P) {
     } else {
         e = P->simt.E ? launch_simt(P->simt, P->d.first, (uint32_t)P->cmps.size(), c->stream, c->num_sms, &nl)
                       : launch_run(P->d, P->groups, (uint32_t)P->dwin.size(), (uint32_t)P->cmps.size(), c->stream,
-                                   c->num_sms, &nl, &c->aux, peer ? &pr : nullptr);
+                                   c->num_sms, &nl, &c->aux, peer ? &pr : nullptr,
+                                   P->no_join && !c->comm && !peer);
     }
     if (e) return fail(c, CEC_E_CUDA, "CUDA: %s (kernel launch)", e);
     if (c->comm && !peer && !P->cmps.empty()) {  // a10: one NCCL min all-reduce of first_idx
@@ -1704,6 +1705,9 @@ cec_status cec_sim_exhaustive(cec_ctx *c, uint32_t n, const uint32_t *la, const 
         S.p->pair_cmp.resize(S.gcmp.size());
         for (uint32_t j = 0; j < S.gcmp.size(); ++j) S.p->pair_cmp[j] = (int32_t)j;
         if ((st = finish_plan(c, S.p.get(), cw, nullptr, false)) != CEC_OK) return st;
+        // chunks before the last do not join the side streams: the next chunk's kernels start while
+        // this chunk's tails drain (the last chunk's join, in stream order, covers them all)
+        S.p->no_join = ch + 2 < cut.size() && getenv("CEC_PIPE_JOIN") == nullptr;
         if ((st = upload(c, S.p.get())) != CEC_OK) {
             free_dev(S.p.get());
             return st;

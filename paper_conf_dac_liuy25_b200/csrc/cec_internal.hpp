@@ -233,9 +233,13 @@ const char *peer_error(const PeerState &ps, void *stream, bool *timed_out);
 
 // One run of a plan: reset, every launch group (side streams forked/joined). With pr->on the window
 // kernels take rank 0's home arrays (d's first/bound/neq_cnt are replaced), wrapped in the peer
-// barriers and followed by the gather into d.first.
+// barriers and followed by the gather into d.first. no_join: the caller's stream does NOT wait for
+// the side streams at the end (the pipelined call's earlier chunks: the next chunk's kernels touch
+// only their own arrays, so they may start while this chunk's side-stream kernels finish; the last
+// chunk joins, and side streams run in order, so its join covers every chunk).
 const char *launch_run(const DevPlan &d, const std::vector<LaunchGroup> &groups, uint32_t nwin, uint32_t ncmp,
-                       void *stream, int num_sms, uint32_t *launches, AuxStreams *aux, const PeerRun *pr = nullptr);
+                       void *stream, int num_sms, uint32_t *launches, AuxStreams *aux, const PeerRun *pr = nullptr,
+                       bool no_join = false);
 const char *graph_capture_run(const DevPlan &d, const std::vector<LaunchGroup> &groups, uint32_t nwin, uint32_t ncmp,
                               void *stream, int num_sms, uint32_t *launches, AuxStreams *aux, void **exec_out,
                               const PeerRun *pr = nullptr);

@@ -198,7 +198,8 @@ void aux_destroy(AuxStreams &a) {
 }
 
 const char *launch_run(const DevPlan &d0, const std::vector<LaunchGroup> &groups, uint32_t nwin, uint32_t ncmp,
-                       void *stream, int num_sms, uint32_t *launches, AuxStreams *aux, const PeerRun *pr) {
+                       void *stream, int num_sms, uint32_t *launches, AuxStreams *aux, const PeerRun *pr,
+                       bool no_join) {
     cudaStream_t main_st = (cudaStream_t)stream;
     cudaStream_t st = main_st;
     const char *e;
@@ -290,7 +291,7 @@ const char *launch_run(const DevPlan &d0, const std::vector<LaunchGroup> &groups
         }
         for (auto &x : pev) cudaEventDestroy(x);
     }
-    if (multi) {  // join: the caller's stream waits for every side stream
+    if (multi && !(no_join && !peer)) {  // join: the caller's stream waits for every side stream
         for (int i = 0; i < aux->n; ++i) {
             if ((e = ck(cudaEventRecord((cudaEvent_t)aux->join[i], (cudaStream_t)aux->s[i])))) return e;
             if ((e = ck(cudaStreamWaitEvent(main_st, (cudaEvent_t)aux->join[i], 0)))) return e;
