@@ -190,6 +190,7 @@ struct cec_plan {
     std::vector<uint4> prog;
     std::vector<Item> items;
     std::vector<JItem> jitems;
+    std::vector<uint32_t> joff;  // free-warp groups' per-warp item offsets (relative to the group)
     std::vector<LaunchGroup> groups;
     uint32_t jit_windows = 0, jit_kernels = 0;
     float jit_ms = 0.f;

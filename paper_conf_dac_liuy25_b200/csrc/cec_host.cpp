@@ -565,6 +565,7 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
     P->prog.clear();
     P->items.clear();
     P->jitems.clear();
+    P->joff.clear();
     P->groups.clear();
     P->win_inputs.clear();
     P->win_nodes.clear();
@@ -1025,6 +1026,10 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
             if (mx <= 4096) {
                 ucfg[u].threads = 256;
                 ucfg[u].min_blocks = 2;
+                // one small structure: static per-warp partition of its slices (no barriers, no
+                // work-queue atomics); bundles keep the block-synchronous item loop
+                ucfg[u].free_warps = units[u].size() == 1 && jcfg.splice &&
+                                     !(getenv("CEC_JIT_FREE") && atoi(getenv("CEC_JIT_FREE")) == 0);
             }
         }
     P->jit_ms = 0.f;
@@ -1087,6 +1092,7 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
     }
     // Each launch is a persistent grid pulling items; size items per GROUP so even a one-window
     // group (e.g. a bug-variant structure) splits into enough items to fill every SM.
+    int cur_min_blocks = 1;  // the unit's configured blocks per SM (host-only plans: no occupancy query)
     auto add_items = [&](std::vector<uint32_t> ws, bool jit, LaunchGroup &g) {
         std::stable_sort(ws.begin(), ws.end(), [&](uint32_t a, uint32_t b) { return cost_of[a] > cost_of[b]; });
         g.nwin = (uint32_t)ws.size();
@@ -1103,6 +1109,42 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         }
         const uint64_t target = (uint64_t)std::max(c->num_sms, 148) * 16 /*resident warps*/ * 8;
         uint64_t item_slices = std::min<uint64_t>(4096, std::max<uint64_t>(1, group_slices / target));
+        if (jit && g.jit && jit_kernel_free(g.jit)) {
+            // free warps: warp gw of the launch takes the contiguous slices [gw T / GW, (gw+1) T / GW)
+            // of the group's concatenated (window, slice) space, cut into items at window ends
+            const uint64_t wpb = (uint64_t)std::max(1, jit_kernel_block(g.jit) / 32);
+            uint64_t blocks = (uint64_t)jit_kernel_blocks(g.jit, c->num_sms > 0 ? c->num_sms : 148, std::max(1, cur_min_blocks));
+            blocks = std::max<uint64_t>(1, std::min(blocks, (group_slices + wpb - 1) / wpb));
+            const uint64_t GW = blocks * wpb;
+            g.free_blocks = (uint32_t)blocks;
+            g.joff_off = (uint32_t)P->joff.size();
+            std::vector<std::pair<uint32_t, uint64_t>> wl;  // (window, first slice) in group order
+            std::vector<uint64_t> wstart{0};
+            for (uint32_t w : ws) {
+                uint64_t ttw = tt_words_of(P->dwin[w].k), sb, se;
+                win_range(w, (ttw + wps_of[w] - 1) / wps_of[w], &sb, &se);
+                if (se <= sb) continue;
+                wl.push_back({w, sb});
+                wstart.push_back(wstart.back() + (se - sb));
+            }
+            const size_t base = P->jitems.size();
+            size_t wi = 0;
+            for (uint64_t gw = 0; gw < GW; ++gw) {
+                P->joff.push_back((uint32_t)(P->jitems.size() - base));
+                uint64_t lo = gw * group_slices / GW;
+                const uint64_t hi = (gw + 1) * group_slices / GW;
+                while (lo < hi) {
+                    while (wstart[wi + 1] <= lo) ++wi;
+                    const uint64_t e = std::min(hi, wstart[wi + 1]);
+                    const uint32_t w = wl[wi].first;
+                    const uint64_t s0 = wl[wi].second + (lo - wstart[wi]);
+                    P->jitems.push_back(JItem{jwin(w), (uint32_t)s0, (uint32_t)(s0 + (e - lo)), P->dwin[w].cmp_off});
+                    lo = e;
+                }
+            }
+            P->joff.push_back((uint32_t)(P->jitems.size() - base));
+            return;
+        }
         // block-synchronous JIT: an item is whole passes of one slice per warp of the kernel's block
         const uint64_t gpass = jit && g.jit ? (uint64_t)std::max(1, jit_slices_per_pass(g.jit)) : jit_pass;
         if (jit && gpass > 1) item_slices = std::max<uint64_t>(gpass, item_slices * gpass);
@@ -1121,6 +1163,7 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
     for (auto &kv : jgroups) {
         LaunchGroup g{};
         g.jit = kernels[kv.first];
+        cur_min_blocks = ucfg[kv.first].min_blocks;
         g.item_off = (uint32_t)P->jitems.size();
         add_items(kv.second, true, g);
         g.nitems = (uint32_t)(P->jitems.size() - g.item_off);
@@ -1150,12 +1193,14 @@ cec_status upload(cec_ctx *c, cec_plan *P) {
     // then [first | bound | neq_cnt | item_ctr] (initialised on the device by the reset kernel)
     auto al = [](size_t x) { return (x + 255) / 256 * 256; };
     const size_t b_wins = sizeof(DevWin) * P->dwin.size(), b_prog = sizeof(uint4) * P->prog.size(),
-                 b_items = sizeof(Item) * P->items.size(), b_jitems = sizeof(JItem) * P->jitems.size();
+                 b_items = sizeof(Item) * P->items.size(), b_jitems = sizeof(JItem) * P->jitems.size(),
+                 b_joff = sizeof(uint32_t) * P->joff.size();
     size_t off = 0;
     const size_t o_wins = off; off += al(std::max<size_t>(b_wins, 1));
     const size_t o_prog = off; off += al(std::max<size_t>(b_prog, 1));
     const size_t o_items = off; off += al(std::max<size_t>(b_items, 1));
     const size_t o_jitems = off; off += al(std::max<size_t>(b_jitems, 1));
+    const size_t o_joff = off; off += al(std::max<size_t>(b_joff, 1));
     const size_t up_bytes = off;
     const size_t o_first = off; off += al(sizeof(unsigned long long) * ncmp);
     const size_t o_bound = off; off += al(sizeof(unsigned long long) * nwin);
@@ -1169,6 +1214,7 @@ cec_status upload(cec_ctx *c, cec_plan *P) {
     d.prog = (uint4 *)(base + o_prog);
     d.items = (Item *)(base + o_items);
     d.jitems = (JItem *)(base + o_jitems);
+    d.joff = (uint32_t *)(base + o_joff);
     d.first = (unsigned long long *)(base + o_first);
     d.bound = (unsigned long long *)(base + o_bound);
     d.neq_cnt = (uint32_t *)(base + o_neq);
@@ -1181,7 +1227,8 @@ cec_status upload(cec_ctx *c, cec_plan *P) {
         if (b_prog) memcpy(h + o_prog, P->prog.data(), b_prog);
         if (b_items) memcpy(h + o_items, P->items.data(), b_items);
         if (b_jitems) memcpy(h + o_jitems, P->jitems.data(), b_jitems);
-        CUDA_TRY(c, h2d(base, h, o_jitems + b_jitems, c->stream));
+        if (b_joff) memcpy(h + o_joff, P->joff.data(), b_joff);
+        CUDA_TRY(c, h2d(base, h, o_joff + b_joff, c->stream));
         CUDA_TRY(c, P->pool->staged(c->stream));
     }
     if (P->simt.E) {
@@ -1199,7 +1246,8 @@ cec_status upload(cec_ctx *c, cec_plan *P) {
     CUDA_TRY(c, event_create(&P->ev0));
     CUDA_TRY(c, event_create(&P->ev1));
     c->stats.h2d_bytes = sizeof(DevWin) * P->dwin.size() + sizeof(uint4) * P->prog.size() +
-                         sizeof(Item) * P->items.size() + sizeof(JItem) * P->jitems.size();
+                         sizeof(Item) * P->items.size() + sizeof(JItem) * P->jitems.size() +
+                         sizeof(uint32_t) * P->joff.size();
     P->uploaded = true;
     return CEC_OK;
 }

@@ -64,6 +64,7 @@ struct JitConfig {
                             // reader's LOP3), 2 area-flow mapping over 3-feasible cuts, 3 = 2 plus
                             // IMAD cells on the FMA pipe (jit.cpp, "Dual-pipe cells")
     bool splice = true;     // body as generated PTX spliced into an NVRTC skeleton (skips NVVM on it)
+    bool free_warps = false;  // single small structure: static per-warp slice partition, no barriers
 };
 struct LaunchGroup {       // windows sharing one kernel launch
     uint32_t nslots;       // interpreter: slots per warp in this launch
@@ -71,6 +72,8 @@ struct LaunchGroup {       // windows sharing one kernel launch
     JitKernel *jit = nullptr;  // non-null: a JIT structure group (items index DevPlan::jitems)
     uint64_t lop3_words = 0;   // executed LOP3 x u32 words of the group (CEC_PROFILE_GROUPS report)
     uint32_t nwin = 0, max_k = 0, nodes = 0;
+    uint32_t free_blocks = 0;  // free-warp JIT kernel: grid size the slices were partitioned over
+    uint32_t joff_off = 0;     // ... and its per-warp item offsets (DevPlan::joff, free_blocks*warps+1)
 };
 
 // Device buffers of one plan.
@@ -83,6 +86,7 @@ struct DevPlan {
     uint32_t *neq_cnt = nullptr;          // [nwin]
     uint32_t *item_ctr = nullptr;         // [ngroups]
     JItem *jitems = nullptr;
+    uint32_t *joff = nullptr;             // free-warp groups: per-warp CSR offsets into jitems
 };
 
 // Per-context cache of device blocks and one pinned host staging buffer (sim_interp.cu): a plan takes
@@ -129,7 +133,10 @@ uint32_t jit_lop3_count(const JitProgram &p, int mode, uint32_t *imads = nullptr
 uint32_t jit_kernel_imad_sid(const JitKernel *k, uint32_t sid);
 int jit_eff_mode(const JitConfig &cfg);
 const char *jit_launch(JitKernel *K, const JItem *items, uint32_t nitems, uint32_t *ctr, unsigned long long *first,
-                       unsigned long long *bound, uint32_t *neq_cnt, void *stream, int num_sms);
+                       unsigned long long *bound, uint32_t *neq_cnt, void *stream, int num_sms, uint32_t free_blocks = 0);
+bool jit_kernel_free(const JitKernel *k);
+int jit_kernel_blocks(const JitKernel *k, int num_sms, int fallback_per_sm);
+int jit_kernel_block(const JitKernel *k);
 
 // cuts_gpu.cu
 uint32_t gpu_cuts_max_C();

@@ -99,6 +99,7 @@ struct JitKernel {
     int block = 128;
     int blocks_per_sm = 0;
     int slices_per_pass = 1;  // block-synchronous kernels: warps per block
+    bool free_warps = false;  // static per-warp partition: grid fixed at plan time, `ctr` = CSR offsets
     uint32_t lop3 = 0;        // LOP3 instructions per word of the mapped window (structure 0)
     std::vector<uint32_t> lop3s;  // per structure of a bundle (sid order)
     std::vector<uint32_t> imads;  // IMAD cells per word, per structure (mode 3)
@@ -559,7 +560,7 @@ std::vector<MappedNode> jit_map_area(const JitProgram &p, double imad_cost) {
 
 // IMAD cells (mode 3) are emitted by the PTX-splice body only; other code paths map with mode 2
 int jit_eff_mode(const JitConfig &cfg) {
-    return cfg.fuse == 3 && !(cfg.splice && cfg.sync_every > 0) ? 2 : cfg.fuse;
+    return cfg.fuse == 3 && !(cfg.splice && (cfg.sync_every > 0 || cfg.free_warps)) ? 2 : cfg.fuse;
 }
 
 double jit_imad_cost() {  // CEC_MAP_IMAD: price of an IMAD cell in LUTs (mode 3)
@@ -675,7 +676,12 @@ uint32_t jit_lop3_count(const JitProgram &p, int mode, uint32_t *imads) {
 
 std::string jit_source(const JitProgram &p, const JitConfig &cfg) {
     const uint32_t n = (uint32_t)(p.nodes.size() / 2), ncmp = (uint32_t)(p.cmps.size() / 2);
-    const bool block_sync = cfg.sync_every > 0;
+    // free warps (small bodies, splice only): every warp runs its own static, contiguous share of
+    // the group's slices (host-partitioned items, CSR offsets passed in `ctr`): no work-queue
+    // atomics and no block barriers at all; the code path below is the block-synchronous one with
+    // its loop header and tail replaced
+    const bool free_w = cfg.free_warps && cfg.splice;
+    const bool block_sync = cfg.sync_every > 0 || free_w;
     const int nw = cfg.threads / 32;
     std::string s;
     s.reserve(96 * (size_t)n + 160 * (size_t)ncmp + 4096);
@@ -710,7 +716,21 @@ std::string jit_source(const JitProgram &p, const JitConfig &cfg) {
         snprintf(buf, sizeof buf, "  const u32 x%u = 0u - ((lane >> %u) & 1u);\n", j, j - 5);
         s += buf;
     }
-    if (!block_sync) {
+    if (free_w) {
+        snprintf(buf, sizeof buf,
+                 "  const u32 gw = blockIdx.x * %du + (threadIdx.x >> 5);\n"
+                 "  const u32 i1 = ctr[gw + 1u];\n"
+                 "  for (u32 i = ctr[gw]; i < i1; ++i) {\n"
+                 "    const JItem I = items[i];\n"
+                 "    u64 bnd = ~0ull;\n"
+                 "    for (u32 s = I.s_begin; s < I.s_end; ++s) {\n"
+                 "      if (((u64)s << 10) >= bnd) break;  /* warp-uniform (lane 0's bound, shuffled) */\n"
+                 "      const bool live = true;\n"
+                 "      u64 bnd_next = 0ull;\n"
+                 "      if (lane == 0u) bnd_next = *((volatile u64 *)&bound[I.win]);  // used next slice\n",
+                 nw);
+        s += buf;
+    } else if (!block_sync) {
         // every warp independent: pulls items itself, one 32-word slice per pass
         s += "  for (;;) {\n"
              "    u32 it = 0;\n"
@@ -827,7 +847,10 @@ std::string jit_source(const JitProgram &p, const JitConfig &cfg) {
                 s += "      __syncthreads();\n";
         }
     }
-    s += block_sync ? "      bnd = __shfl_sync(0xFFFFFFFFu, bnd_next, 0);\n    }\n" ITEM_WAIT "    __syncthreads();\n  }\n}\n" : "    }\n  }\n}\n";
+    if (free_w)
+        s += "      bnd = __shfl_sync(0xFFFFFFFFu, bnd_next, 0);\n    }\n  }\n}\n";
+    else
+        s += block_sync ? "      bnd = __shfl_sync(0xFFFFFFFFu, bnd_next, 0);\n    }\n" ITEM_WAIT "    __syncthreads();\n  }\n}\n" : "    }\n  }\n}\n";
     return s;
 }
 
@@ -1148,8 +1171,8 @@ const char *jit_get_unit(const std::vector<const JitProgram *> &ps, const JitCon
     const bool bundle = ps.size() > 1;
     if (bundle && !(cfg.splice && cfg.sync_every > 0)) return "JIT bundles need the block-synchronous splice mode";
     char ck[64];
-    snprintf(ck, sizeof ck, "|%d,%d,%d,%d,%d", cfg.threads, cfg.min_blocks, cfg.sync_every, (int)cfg.fuse,
-             (int)cfg.splice);
+    snprintf(ck, sizeof ck, "|%d,%d,%d,%d,%d,%d", cfg.threads, cfg.min_blocks, cfg.sync_every, (int)cfg.fuse,
+             (int)cfg.splice, (int)cfg.free_warps);
     std::string key;
     for (const JitProgram *p : ps) key += jit_key(*p) + "#";
     key += ck;
@@ -1168,8 +1191,8 @@ const char *jit_get_unit(const std::vector<const JitProgram *> &ps, const JitCon
     const std::string src = bundle ? jit_source_bundle(ps, cfg) : jit_source(*ps[0], cfg);
     std::vector<char> cubin;
     std::string log;
-    const char *e = (cfg.splice && cfg.sync_every > 0) ? jit_compile_splice(ps, cfg, src, cubin, log)
-                                                       : jit_compile_cubin(src, cubin, log);
+    const char *e = (cfg.splice && (cfg.sync_every > 0 || cfg.free_warps)) ? jit_compile_splice(ps, cfg, src, cubin, log)
+                                                                          : jit_compile_cubin(src, cubin, log);
     if (e) {
         static thread_local std::string msg;
         msg = std::string(e) + ": " + log.substr(0, 400);
@@ -1197,7 +1220,8 @@ const char *jit_get_unit(const std::vector<const JitProgram *> &ps, const JitCon
         K->imads.push_back(im);
     }
     K->lop3 = K->lop3s[0];
-    K->slices_per_pass = cfg.sync_every > 0 ? cfg.threads / 32 : 1;
+    K->slices_per_pass = cfg.sync_every > 0 && !cfg.free_warps ? cfg.threads / 32 : 1;
+    K->free_warps = cfg.free_warps && cfg.splice && ps.size() == 1;
     K->src_bytes = src.size();
     K->cubin_bytes = cubin.size();
     if (load) {
@@ -1229,17 +1253,27 @@ bool jit_kernel_loaded(const JitKernel *k) { return k && k->kern; }
 uint32_t jit_kernel_lop3_sid(const JitKernel *k, uint32_t sid) {
     return k && sid < k->lop3s.size() ? k->lop3s[sid] : 0;
 }
+bool jit_kernel_free(const JitKernel *k) { return k && k->free_warps; }
+int jit_kernel_blocks(const JitKernel *k, int num_sms, int fallback_per_sm) {  // resident grid of a kernel
+    const int per_sm = k && k->blocks_per_sm > 0 ? k->blocks_per_sm : fallback_per_sm;
+    return std::max(1, num_sms) * std::max(1, per_sm);
+}
+int jit_kernel_block(const JitKernel *k) { return k ? k->block : 32; }
 uint32_t jit_kernel_imad_sid(const JitKernel *k, uint32_t sid) {
     return k && sid < k->imads.size() ? k->imads[sid] : 0;
 }
 
 const char *jit_launch(JitKernel *K, const JItem *items, uint32_t nitems, uint32_t *ctr, unsigned long long *first,
-                       unsigned long long *bound, uint32_t *neq_cnt, void *stream, int num_sms) {
+                       unsigned long long *bound, uint32_t *neq_cnt, void *stream, int num_sms, uint32_t free_blocks) {
     if (!K || !K->kern) return "JIT kernel not loaded";
     if (nitems == 0) return nullptr;
     uint64_t grid = (uint64_t)num_sms * K->blocks_per_sm;
     const uint64_t need = K->slices_per_pass > 1 ? nitems : (nitems + (K->block / 32) - 1) / (K->block / 32);
     if (grid > need) grid = need;
+    if (K->free_warps) {  // the plan partitioned the slices over exactly this many blocks (ctr = offsets)
+        if (!free_blocks) return "free-warp kernel launched without its partition";
+        grid = free_blocks;
+    }
     void *args[] = {(void *)&items, (void *)&nitems, (void *)&ctr, (void *)&first, (void *)&bound, (void *)&neq_cnt};
     cudaError_t e = cudaLaunchKernel((const void *)K->kern, dim3((unsigned)grid), dim3(K->block), args, 0,
                                      (cudaStream_t)stream);

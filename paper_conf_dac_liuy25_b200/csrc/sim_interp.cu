@@ -245,8 +245,10 @@ const char *launch_run(const DevPlan &d0, const std::vector<LaunchGroup> &groups
         st = (multi && g > 0) ? (cudaStream_t)aux->s[(g - 1) % aux->n] : main_st;
         stream = st;
         if (G.jit) {
-            if ((e = jit_launch(G.jit, d.jitems + G.item_off, G.nitems, d.item_ctr + g, d.first, d.bound, d.neq_cnt,
-                                stream, num_sms)))
+            // a free-warp kernel reads its per-warp item offsets where the others take their counter
+            uint32_t *ctr = G.free_blocks ? d.joff + G.joff_off : d.item_ctr + g;
+            if ((e = jit_launch(G.jit, d.jitems + G.item_off, G.nitems, ctr, d.first, d.bound, d.neq_cnt,
+                                stream, num_sms, G.free_blocks)))
                 return e;
             ++nl;
             continue;
