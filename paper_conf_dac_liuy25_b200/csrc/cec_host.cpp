@@ -1026,10 +1026,11 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
             if (mx <= 4096) {
                 ucfg[u].threads = 256;
                 ucfg[u].min_blocks = 2;
-                // one small structure: static per-warp partition of its slices (no barriers, no
-                // work-queue atomics); bundles keep the block-synchronous item loop
-                ucfg[u].free_warps = units[u].size() == 1 && jcfg.splice &&
-                                     !(getenv("CEC_JIT_FREE") && atoi(getenv("CEC_JIT_FREE")) == 0);
+                // small structures (single or bundled): static per-warp partition of the slices (no
+                // barriers, no work-queue atomics); CEC_JIT_FREE=0 keeps the block-synchronous loop,
+                // =1 frees single structures only
+                const int fm = getenv("CEC_JIT_FREE") ? atoi(getenv("CEC_JIT_FREE")) : 2;
+                ucfg[u].free_warps = jcfg.splice && (fm == 2 || (fm == 1 && units[u].size() == 1));
             }
         }
     P->jit_ms = 0.f;

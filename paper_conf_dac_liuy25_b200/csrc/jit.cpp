@@ -888,19 +888,39 @@ std::string jit_source_bundle(const std::vector<const JitProgram *> &ps, const J
              "    u32 *ctr, u64 *first, u64 *bound, u32 *neq_cnt) {\n",
              cfg.threads, cfg.min_blocks);
     s += buf;
-    s += "  const u32 lane = threadIdx.x & 31u;\n"
-         "  const u32 warp = threadIdx.x >> 5;\n" ITEM_PIPELINE "    JItem I = s_item[cur];\n" ITEM_PREFETCH;
-    snprintf(buf, sizeof buf,
-             "    const u32 sid = I.win >> 20;\n"
-             "    I.win &= 0xFFFFFu;\n"
-             "    u64 bnd = ~0ull;  /* first pass of an item: no skip test, so no exposed bound load */\n"
-             "    for (u32 s0 = I.s_begin; s0 < I.s_end; s0 += %du) {\n"
-             "      const u32 s = s0 + warp;\n"
-             "      const bool live = s < I.s_end && ((u64)s << 10) < bnd;\n"
-             "      if (!__syncthreads_or(live)) break;\n"
-             "      const u64 bnd_next = *((volatile u64 *)&bound[I.win]);\n",
-             nw);
-    s += buf;
+    const bool free_w = cfg.free_warps;
+    if (free_w) {  // static per-warp partition (see jit_source): items = (window | sid << 20, slices)
+        snprintf(buf, sizeof buf,
+                 "  const u32 lane = threadIdx.x & 31u;\n"
+                 "  const u32 gw = blockIdx.x * %du + (threadIdx.x >> 5);\n"
+                 "  const u32 i1 = ctr[gw + 1u];\n"
+                 "  for (u32 i = ctr[gw]; i < i1; ++i) {\n"
+                 "    JItem I = items[i];\n"
+                 "    const u32 sid = I.win >> 20;\n"
+                 "    I.win &= 0xFFFFFu;\n"
+                 "    u64 bnd = ~0ull;\n"
+                 "    for (u32 s = I.s_begin; s < I.s_end; ++s) {\n"
+                 "      if (((u64)s << 10) >= bnd) break;\n"
+                 "      const bool live = true;\n"
+                 "      u64 bnd_next = 0ull;\n"
+                 "      if (lane == 0u) bnd_next = *((volatile u64 *)&bound[I.win]);\n",
+                 nw);
+        s += buf;
+    } else {
+        s += "  const u32 lane = threadIdx.x & 31u;\n"
+             "  const u32 warp = threadIdx.x >> 5;\n" ITEM_PIPELINE "    JItem I = s_item[cur];\n" ITEM_PREFETCH;
+        snprintf(buf, sizeof buf,
+                 "    const u32 sid = I.win >> 20;\n"
+                 "    I.win &= 0xFFFFFu;\n"
+                 "    u64 bnd = ~0ull;  /* first pass of an item: no skip test, so no exposed bound load */\n"
+                 "    for (u32 s0 = I.s_begin; s0 < I.s_end; s0 += %du) {\n"
+                 "      const u32 s = s0 + warp;\n"
+                 "      const bool live = s < I.s_end && ((u64)s << 10) < bnd;\n"
+                 "      if (!__syncthreads_or(live)) break;\n"
+                 "      const u64 bnd_next = *((volatile u64 *)&bound[I.win]);\n",
+                 nw);
+        s += buf;
+    }
     for (uint32_t j = 0; j < kmax; ++j) {
         if (j < 5)
             snprintf(buf, sizeof buf, "      const u32 x%u = %s;\n", j, kMask[j]);
@@ -952,7 +972,8 @@ std::string jit_source_bundle(const std::vector<const JitProgram *> &ps, const J
         }
         s += "      } break;\n";
     }
-    s += "      default: break;\n      }\n      bnd = __shfl_sync(0xFFFFFFFFu, bnd_next, 0);\n    }\n" ITEM_WAIT "    __syncthreads();\n  }\n}\n";
+    s += "      default: break;\n      }\n      bnd = __shfl_sync(0xFFFFFFFFu, bnd_next, 0);\n    }\n";
+    s += free_w ? "  }\n}\n" : ITEM_WAIT "    __syncthreads();\n  }\n}\n";
     return s;
 }
 
@@ -1014,7 +1035,10 @@ std::string jit_body_ptx(const JitProgram &p, const JitConfig &cfg, const std::v
             ++emitted;
         }
         for (uint32_t c : after[t + 1]) emit_cmp(c);
-        if (!x.absorbed && lut_total > 2048 && emitted % (uint32_t)cfg.sync_every == 0) s += "bar.sync 0;\n";
+        // (never in free-warp kernels: their warps are not in step)
+        if (!cfg.free_warps && !x.absorbed && lut_total > 2048 && cfg.sync_every > 0 &&
+            emitted % (uint32_t)cfg.sync_every == 0)
+            s += "bar.sync 0;\n";
     }
     s += "}\n";
     return s;
@@ -1169,7 +1193,8 @@ std::map<std::string, std::unique_ptr<JitKernel>> g_cache;  // process-wide, key
 const char *jit_get_unit(const std::vector<const JitProgram *> &ps, const JitConfig &cfg, bool load, JitKernel **out) {
     if (ps.empty()) return "empty JIT unit";
     const bool bundle = ps.size() > 1;
-    if (bundle && !(cfg.splice && cfg.sync_every > 0)) return "JIT bundles need the block-synchronous splice mode";
+    if (bundle && !(cfg.splice && (cfg.sync_every > 0 || cfg.free_warps)))
+        return "JIT bundles need the splice mode (block-synchronous or free warps)";
     char ck[64];
     snprintf(ck, sizeof ck, "|%d,%d,%d,%d,%d,%d", cfg.threads, cfg.min_blocks, cfg.sync_every, (int)cfg.fuse,
              (int)cfg.splice, (int)cfg.free_warps);
@@ -1221,7 +1246,7 @@ const char *jit_get_unit(const std::vector<const JitProgram *> &ps, const JitCon
     }
     K->lop3 = K->lop3s[0];
     K->slices_per_pass = cfg.sync_every > 0 && !cfg.free_warps ? cfg.threads / 32 : 1;
-    K->free_warps = cfg.free_warps && cfg.splice && ps.size() == 1;
+    K->free_warps = cfg.free_warps && cfg.splice;
     K->src_bytes = src.size();
     K->cubin_bytes = cubin.size();
     if (load) {
