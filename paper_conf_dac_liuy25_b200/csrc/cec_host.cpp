@@ -1026,10 +1026,10 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
             if (mx <= 4096) {
                 ucfg[u].threads = 256;
                 ucfg[u].min_blocks = 2;
-                // small structures (single or bundled): static per-warp partition of the slices (no
-                // barriers, no work-queue atomics); CEC_JIT_FREE=0 keeps the block-synchronous loop,
-                // =1 frees single structures only
-                const int fm = getenv("CEC_JIT_FREE") ? atoi(getenv("CEC_JIT_FREE")) : 2;
+                // a single small structure: static per-warp partition of its slices (no barriers, no
+                // work-queue atomics). CEC_JIT_FREE=0 keeps the block-synchronous loop everywhere, =2
+                // frees bundles too (C3 4.07 vs 3.91 ms: warps of one SM then run different bodies)
+                const int fm = getenv("CEC_JIT_FREE") ? atoi(getenv("CEC_JIT_FREE")) : 1;
                 ucfg[u].free_warps = jcfg.splice && (fm == 2 || (fm == 1 && units[u].size() == 1));
             }
         }
