@@ -686,9 +686,16 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
                 for (uint32_t v : nodes) flag[v - lo] = 1;
                 for (uint32_t i = 0; i <= hi - lo; ++i)
                     if (flag[i]) by_id.push_back(lo + i);
-            } else {
+            } else {  // two or more clusters (e.g. a block of A and its image in B): LSD radix sort
                 by_id = nodes;
-                std::sort(by_id.begin(), by_id.end());
+                std::vector<uint32_t> tmp(by_id.size());
+                for (int sh = 0; sh < 32 && (hi >> sh) != 0; sh += 11) {
+                    uint32_t cnt[2049] = {0};
+                    for (uint32_t v : by_id) ++cnt[((v >> sh) & 2047u) + 1];
+                    for (int b = 0; b < 2048; ++b) cnt[b + 1] += cnt[b];
+                    for (uint32_t v : by_id) tmp[cnt[(v >> sh) & 2047u]++] = v;
+                    by_id.swap(tmp);
+                }
             }
             const uint32_t l_id = live_peak(c, X, W.inputs, by_id, cmps2, wc);
             const uint32_t l_dfs = live_peak(c, X, W.inputs, nodes, cmps2, wc);
