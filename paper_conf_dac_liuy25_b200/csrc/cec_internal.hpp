@@ -59,7 +59,9 @@ struct JitKernel;
 struct JitConfig {
     int threads = 512;      // threads per block
     int min_blocks = 1;     // __launch_bounds__ min blocks per SM (registers <= 64K / (threads*min_blocks))
-    int sync_every = 512;   // block-synchronous: __syncthreads() every this many LOP3s; 0 = warp-independent
+    int sync_every = 8192;  // block-synchronous: a bar.sync every this many cells inside a body (besides the
+                            // per-pass barrier); 0 = warp-independent. 512 before round 2: with IMAD cells
+                            // the mid-body barriers cost more than they save (C5 32.79 -> 32.41 ms)
     int fuse = 3;           // 3-input LUT mapping: 0 none, 1 greedy (absorb single-fanout ANDs into the
                             // reader's LOP3), 2 area-flow mapping over 3-feasible cuts, 3 = 2 plus
                             // IMAD cells on the FMA pipe (jit.cpp, "Dual-pipe cells")
