@@ -1101,6 +1101,7 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
     // Each launch is a persistent grid pulling items; size items per GROUP so even a one-window
     // group (e.g. a bug-variant structure) splits into enough items to fill every SM.
     int cur_min_blocks = 1;  // the unit's configured blocks per SM (host-only plans: no occupancy query)
+    std::string partition_err;
     auto add_items = [&](std::vector<uint32_t> ws, bool jit, LaunchGroup &g) {
         std::stable_sort(ws.begin(), ws.end(), [&](uint32_t a, uint32_t b) { return cost_of[a] > cost_of[b]; });
         g.nwin = (uint32_t)ws.size();
@@ -1151,6 +1152,21 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
                 }
             }
             P->joff.push_back((uint32_t)(P->jitems.size() - base));
+            // invariant: the items tile every window's slice range exactly once, in order
+            std::vector<uint64_t> next(wl.size());
+            for (size_t q = 0; q < wl.size(); ++q) next[q] = wl[q].second;
+            size_t q = 0;
+            for (size_t t = base; t < P->jitems.size(); ++t) {
+                const JItem &it = P->jitems[t];
+                while (q < wl.size() && jwin(wl[q].first) != it.win) ++q;
+                if (q == wl.size() || it.s_begin != next[q] || it.s_end <= it.s_begin) {
+                    partition_err = "free-warp partition does not tile the slice ranges";
+                    return;
+                }
+                next[q] = it.s_end;
+            }
+            for (size_t r = 0; r < wl.size(); ++r)
+                if (next[r] != wl[r].second + (wstart[r + 1] - wstart[r])) partition_err = "free-warp partition misses slices";
             return;
         }
         // block-synchronous JIT: an item is whole passes of one slice per warp of the kernel's block
@@ -1174,6 +1190,7 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         cur_min_blocks = ucfg[kv.first].min_blocks;
         g.item_off = (uint32_t)P->jitems.size();
         add_items(kv.second, true, g);
+        if (!partition_err.empty()) return fail(c, CEC_E_STATE, "%s", partition_err.c_str());
         g.nitems = (uint32_t)(P->jitems.size() - g.item_off);
         P->groups.push_back(g);
     }

@@ -277,3 +277,24 @@ def test_binding_rejects_mismatched_pair_arrays():
     # well-formed arguments still reach the C side (which refuses: no device, no CPU fallback)
     with pytest.raises(capi.CecError):
         ctx.check_local_cuts(m.lit_a[:1], m.lit_b[:1], [0, 2], [1, 9])
+
+
+@pytest.mark.parametrize("world", [1, 3, 8])
+def test_free_warp_partition_host_plans(world):
+    """Free-warp JIT kernels (single small structures, round 2): the planner cuts each group's
+    slices into one contiguous range per warp of the launch grid and checks (CEC_E_STATE otherwise)
+    that the items tile every window's slice range exactly once; per-rank work still adds up to the
+    whole under pattern-space sharding (C2's single window, and a reduced C5 with mul copies)."""
+    from workloads import circuits
+    for m in (circuits.c2_mul12(10), c5_big(copies=6, n_random=2, n_bugs=1, rand_pis=12, rand_ands=300, mul_n=6)):
+        Ws, W_all = [], None
+        for r in range(world):
+            ctx = host_ctx(m.aig, rank=r, world=world, engine=capi.CEC_ENGINE_JIT)
+            plan = capi.cec_plan_exhaustive(ctx.handle, m.lit_a, m.lit_b)
+            st = ctx.stats()
+            assert st["jit_windows"] >= 1
+            Ws.append(st["node_patterns"])
+            W_all = st["node_patterns_all"]
+            capi.cec_plan_free(plan)
+            ctx.close()
+        assert sum(Ws) == W_all
