@@ -1333,8 +1333,10 @@ static cec_status plan_route(cec_ctx *c, uint32_t n, const uint32_t *la, const u
     const uint32_t kmax = c->opts.k_max;
     // a2/a3: supports, trivial pairs, routing by k; identical (unordered) pairs share one compare
     std::unordered_map<uint64_t, uint32_t> seen;  // unordered literal pair -> compare
-    // identical supports share a window: hash of S -> windows with that hash (exact compare below)
-    std::unordered_map<uint64_t, std::vector<uint32_t>> by_support;
+    // identical supports share a window: hash of S -> first window with that hash, then a chain
+    // through win_next (exact compare below); no per-window allocation
+    std::unordered_map<uint64_t, uint32_t> by_support;
+    std::vector<uint32_t> win_next;
     auto supp_hash = [](const std::vector<uint32_t> &S) {
         uint64_t h = 0x9E3779B97F4A7C15ull ^ S.size();
         for (uint32_t x : S) h = (h ^ x) * 0x100000001B3ull, h ^= h >> 29;
@@ -1421,6 +1423,10 @@ static cec_status plan_route(cec_ctx *c, uint32_t n, const uint32_t *la, const u
     }
     tm.lap("supports");
     seen.reserve(2 * (size_t)n);
+    by_support.reserve(2 * (size_t)n);
+    P->cmps.reserve(n);
+    wins0.reserve(n);
+    win_next.reserve(n);
     for (uint32_t p = 0; p < n; ++p) {
         std::vector<uint32_t> &S = supp[p];
         const uint64_t cone = cones[p];
@@ -1448,12 +1454,13 @@ static cec_status plan_route(cec_ctx *c, uint32_t n, const uint32_t *la, const u
         const uint32_t ci = (uint32_t)P->cmps.size();
         seen.emplace(key, ci);
         P->pair_cmp[p] = (int32_t)ci;
-        std::vector<uint32_t> &cand = by_support[supp_hash(S)];
+        auto hit = by_support.emplace(supp_hash(S), UINT32_MAX).first;
         uint32_t wi = UINT32_MAX;
-        for (uint32_t x : cand)
+        for (uint32_t x = hit->second; x != UINT32_MAX && wi == UINT32_MAX; x = win_next[x])
             if (wins0[x].inputs == S) wi = x;
         if (wi == UINT32_MAX) {
-            cand.push_back((uint32_t)wins0.size());
+            win_next.push_back(hit->second);
+            hit->second = (uint32_t)wins0.size();
             WinHost w;
             w.inputs = S;
             w.cmps.push_back(ci);
