@@ -19,7 +19,8 @@ roofline   = ALU (LOP3) bound: the mapped window's lop3.b32 cells per u32 word (
              work of the binding pipe; peak = 148 SMs x 64 LOP3/clk/SM x SM clock.
              IMAD cells (AND nodes with a word-uniform operand, FMA pipe) are reported beside it.
 cpu_baseline / --impl reference = the oracle (oracle/, plain single-threaded C) timed on a bounded
-             sample of the same workload on this host.
+             sample of the same workload on this host's cores (one oracle process per core, each on
+             its own pattern range: the sharded oracle of SURVEY.md §8(c)).
 """
 from __future__ import annotations
 
@@ -82,16 +83,52 @@ def sample_pairs(m, copy_idx):
     return m.lit_a[off:off + n], m.lit_b[off:off + n], f"the {n} PO pairs of copy {copy_idx}"
 
 
-def oracle_sample(m, copy_idx, log2_patterns):
-    """Time the oracle (as it stands) on patterns [0, 2^log2_patterns) of one copy's pair group."""
+_SHARD = {}  # the oracle and pairs a forked shard process inherits
+
+
+def _oracle_shard(rng):
+    lo, hi = rng
+    _, _, _, evals = _SHARD["orc"].check_pairs(_SHARD["la"], _SHARD["lb"], k_max=32, lo=lo, hi=hi)
+    return evals
+
+
+def host_cores():
+    try:
+        return len(os.sched_getaffinity(0))
+    except Exception:
+        return os.cpu_count() or 1
+
+
+def oracle_sample(m, copy_idx, log2_patterns, procs=1, reps=1):
+    """Time the oracle (as it stands: single-threaded C) on one copy's pair group. procs > 1: the
+    sharded oracle of SURVEY.md §8(c) — procs forked processes, one per host core, each enumerating
+    its own 2^log2_patterns-pattern range of the window (min over ranges = the full scan); the
+    timed region is the parallel map only (workers are forked and warmed before it)."""
+    import multiprocessing
+
     import oracle
 
     la, lb, what = sample_pairs(m, copy_idx)
     orc = oracle.Oracle.from_aig(m.aig)
-    t = time.perf_counter()
-    _, _, _, evals = orc.check_pairs(la, lb, k_max=32, lo=0, hi=1 << log2_patterns)
-    dt = time.perf_counter() - t
-    return evals, dt, f"{what}, patterns [0, 2^{log2_patterns}) of its 2^24-pattern window, single thread"
+    n = 1 << log2_patterns
+    if procs <= 1:
+        evals, dt = 0, 0.0
+        for _ in range(reps):
+            t = time.perf_counter()
+            _, _, _, e = orc.check_pairs(la, lb, k_max=32, lo=0, hi=n)
+            dt += time.perf_counter() - t
+            evals += e
+        return evals, dt, f"{what}, patterns [0, 2^{log2_patterns}) of its 2^24-pattern window, single thread"
+    _SHARD.update(orc=orc, la=la, lb=lb)
+    with multiprocessing.get_context("fork").Pool(procs) as pool:
+        pool.map(_oracle_shard, [(0, 1)] * procs)  # fork + warm every worker outside the timed region
+        evals, dt = 0, 0.0
+        for _ in range(reps):
+            t = time.perf_counter()
+            evals += sum(pool.map(_oracle_shard, [(r * n, (r + 1) * n) for r in range(procs)], chunksize=1))
+            dt += time.perf_counter() - t
+    return evals, dt, (f"{what}, patterns [0, {procs}*2^{log2_patterns}) of its 2^24-pattern window in {procs} "
+                       f"ranges, one single-threaded oracle process per host core (SURVEY.md §8(c) sharded oracle)")
 
 
 class ClockSampler:
@@ -177,14 +214,9 @@ def run_reference(args):
     oracle.build()
     m, desc, copy_idx = make_workload(args.config)
     log2p = args.ref_log2_patterns
-    for _ in range(args.warmup):
-        oracle_sample(m, copy_idx, log2p)
-    evals = 0
-    secs = 0.0
-    for _ in range(args.steps):
-        e, dt, what = oracle_sample(m, copy_idx, log2p)
-        evals += e
-        secs += dt
+    procs = host_cores() if args.cpu_procs <= 0 else args.cpu_procs
+    oracle_sample(m, copy_idx, log2p - 2, procs, reps=args.warmup)  # warm-up steps (smaller)
+    evals, secs, what = oracle_sample(m, copy_idx, log2p, procs, reps=args.steps)
     v = evals / secs
     line = {
         "impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": args.gpus,
@@ -192,7 +224,7 @@ def run_reference(args):
         "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u8",
         "data": "synthetic",
         "config": workload_config(args.config, m, desc),
-        "cpu_baseline": {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": what},
+        "cpu_baseline": {"value": v, "unit": UNIT, "cores": procs, "kind": "oracle", "sample": what},
         "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
@@ -212,6 +244,7 @@ def main():
     ap.add_argument("--cpu-log2-patterns", type=int, default=19)
     ap.add_argument("--ref-log2-patterns", type=int, default=17)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-procs", type=int, default=0, help="oracle processes for cpu_baseline / reference (0 = host cores)")
     ap.add_argument("--reduce", default="peer", choices=["peer", "nccl"],
                     help="N > 1: a10 over NVLink peer memory fused into the compare path (default) or ncclAllReduce")
     args = ap.parse_args()
@@ -410,8 +443,9 @@ def main():
         import oracle
 
         oracle.build()
-        evals, dt, what = oracle_sample(m, copy_idx, args.cpu_log2_patterns)
-        cpu = {"value": evals / dt, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": what,
+        procs = host_cores() if args.cpu_procs <= 0 else args.cpu_procs
+        evals, dt, what = oracle_sample(m, copy_idx, args.cpu_log2_patterns, procs)
+        cpu = {"value": evals / dt, "unit": UNIT, "cores": procs, "kind": "oracle", "sample": what,
                "seconds": round(dt, 2)}
 
     # parity against stored oracle results of the same generated miter (tests/golden, written by

@@ -517,3 +517,27 @@ def test_fuzz_jit_windows_word_uniform_inputs(seed):
     m = tiny_random(I, int(rng.integers(40, 260)), 20, 9000 + seed)
     ctx, gv, gc, gk = check_vs_oracle(m, k_max=14, merge=int(rng.integers(0, 3)), engine=capi.CEC_ENGINE_JIT)
     ctx.close()
+
+
+@pytest.mark.parametrize("seed", range(8))
+def test_local_checks_jit_engine_vs_oracle(seed):
+    """a12 local checks through the JIT register kernels (engine forced): cut leaves are the window
+    inputs, so leaves 5.. are word-uniform words and feed the IMAD cells exactly like PIs do;
+    random cuts of 10..16 leaves (valid or not: invalid cuts must come back CEC_E_CUT-marked the
+    same way) against the oracle's local check."""
+    rng = np.random.default_rng(900 + seed)
+    I = int(rng.integers(10, 15))
+    m = tiny_random(I, int(rng.integers(60, 200)), 12, 900 + seed)
+    N = m.aig.num_nodes
+    la, lb, off, lv = [], [], [0], []
+    for q in range(m.num_pairs):
+        cand = rng.choice(np.arange(1, N), size=int(rng.integers(4, 12)), replace=False)
+        cand = np.unique(np.concatenate([cand, np.arange(1, I + 1)]))[:16]  # PIs make most cuts valid
+        la.append(int(m.lit_a[q])); lb.append(int(m.lit_b[q]))
+        lv += [int(x) for x in cand]
+        off.append(len(lv))
+    ctx = gpu_ctx(m.aig, engine=capi.CEC_ENGINE_JIT)
+    got = ctx.check_local_cuts(la, lb, off, lv)
+    want = Oracle.from_aig(m.aig).check_local(la, lb, off, lv)
+    assert list(map(int, got)) == list(map(int, want))
+    ctx.close()
