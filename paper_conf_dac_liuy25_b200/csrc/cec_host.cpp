@@ -1038,6 +1038,8 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
                 // frees bundles too (C3 4.07 vs 3.91 ms: warps of one SM then run different bodies)
                 const int fm = getenv("CEC_JIT_FREE") ? atoi(getenv("CEC_JIT_FREE")) : 1;
                 ucfg[u].free_warps = jcfg.splice && (fm == 2 || (fm == 1 && units[u].size() == 1));
+                if (ucfg[u].free_warps && units[u].size() == 1 && getenv("CEC_JIT_ILP"))
+                    ucfg[u].ilp = std::max(1, std::min(2, atoi(getenv("CEC_JIT_ILP"))));
             }
         }
     P->jit_ms = 0.f;

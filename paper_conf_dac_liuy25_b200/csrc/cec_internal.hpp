@@ -67,6 +67,7 @@ struct JitConfig {
                             // IMAD cells on the FMA pipe (jit.cpp, "Dual-pipe cells")
     bool splice = true;     // body as generated PTX spliced into an NVRTC skeleton (skips NVVM on it)
     bool free_warps = false;  // single small structure: static per-warp slice partition, no barriers
+    int ilp = 1;              // free warps: slices evaluated per pass (2 = two interleaved body copies)
 };
 struct LaunchGroup {       // windows sharing one kernel launch
     uint32_t nslots;       // interpreter: slots per warp in this launch

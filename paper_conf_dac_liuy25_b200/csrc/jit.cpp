@@ -681,6 +681,10 @@ std::string jit_source(const JitProgram &p, const JitConfig &cfg) {
     // atomics and no block barriers at all; the code path below is the block-synchronous one with
     // its loop header and tail replaced
     const bool free_w = cfg.free_warps && cfg.splice;
+    // ILP 2 (free warps only): each pass evaluates slices s and s + 1 with two copies of the body
+    // (BODY0, BODY1) in one basic block, so ptxas can interleave two independent dependency chains;
+    // slice s + 1 past the item's end is computed but its compares are masked (liveB)
+    const bool ilp2 = free_w && cfg.ilp == 2;
     const bool block_sync = cfg.sync_every > 0 || free_w;
     const int nw = cfg.threads / 32;
     std::string s;
@@ -723,12 +727,12 @@ std::string jit_source(const JitProgram &p, const JitConfig &cfg) {
                  "  for (u32 i = ctr[gw]; i < i1; ++i) {\n"
                  "    const JItem I = items[i];\n"
                  "    u64 bnd = ~0ull;\n"
-                 "    for (u32 s = I.s_begin; s < I.s_end; ++s) {\n"
+                 "    for (u32 s = I.s_begin; s < I.s_end; s += %du) {\n"
                  "      if (((u64)s << 10) >= bnd) break;  /* warp-uniform (lane 0's bound, shuffled) */\n"
                  "      const bool live = true;\n"
                  "      u64 bnd_next = 0ull;\n"
                  "      if (lane == 0u) bnd_next = *((volatile u64 *)&bound[I.win]);  // used next slice\n",
-                 nw);
+                 nw, ilp2 ? 2 : 1);
         s += buf;
     } else if (!block_sync) {
         // every warp independent: pulls items itself, one 32-word slice per pass
@@ -767,6 +771,16 @@ std::string jit_source(const JitProgram &p, const JitConfig &cfg) {
             snprintf(buf, sizeof buf, "      const u32 x%u = 0u - ((s >> %u) & 1u);\n", j, j - 10);
         s += buf;
     }
+    if (ilp2) {
+        s += "      const u32 sB = s + 1u;\n      const bool liveB = sB < I.s_end;\n";
+        for (uint32_t j = 0; j < p.k; ++j) {
+            if (j < 10)
+                snprintf(buf, sizeof buf, "      const u32 y%u = x%u;\n", j, j);
+            else
+                snprintf(buf, sizeof buf, "      const u32 y%u = 0u - ((sB >> %u) & 1u);\n", j, j - 10);
+            s += buf;
+        }
+    }
     // compares are placed right after their later root so roots die early (fewer live registers)
     std::vector<std::vector<uint32_t>> after(n + 1);
     for (uint32_t c = 0; c < ncmp; ++c) {
@@ -789,39 +803,50 @@ std::string jit_source(const JitProgram &p, const JitConfig &cfg) {
         // per warp; a mismatching compare sets its bit in the warp masks m* and stores the lanes'
         // diff words to dbuf (rare path), so only the masks stay live through the body.
         const uint32_t M = (ncmp + 31) / 32;
-        if (ncmp) {
-            snprintf(buf, sizeof buf, "      u32 dbuf[%u];\n", ncmp);
-            s += buf;
+        // body b: masks m<b>_*, diff buffer dbuf<b>, inputs x* (b = 0) or y* (b = 1, ILP 2)
+        const int nb = ilp2 ? 2 : 1;
+        for (int b = 0; b < nb; ++b) {
+            if (ncmp) {
+                snprintf(buf, sizeof buf, "      u32 dbuf%d[%u];\n", b, ncmp);
+                s += buf;
+            }
+            for (uint32_t w = 0; w < M; ++w) {
+                snprintf(buf, sizeof buf, "      u32 m%d_%u;\n", b, w);
+                s += buf;
+            }
         }
-        for (uint32_t w = 0; w < M; ++w) {
-            snprintf(buf, sizeof buf, "      u32 m%u;\n", w);
+        for (int b = 0; b < nb; ++b) {
+            snprintf(buf, sizeof buf, "      asm volatile(\"//@@BODY%d@@", b);
             s += buf;
+            for (uint32_t i = 0; i < M + p.k + (ncmp ? 1 : 0); ++i) {
+                snprintf(buf, sizeof buf, " %%%u", i);
+                s += buf;
+            }
+            s += "\" :";
+            for (uint32_t w = 0; w < M; ++w) {
+                snprintf(buf, sizeof buf, "%s \"=r\"(m%d_%u)", w ? "," : "", b, w);
+                s += buf;
+            }
+            s += " :";
+            for (uint32_t j = 0; j < p.k; ++j) {
+                snprintf(buf, sizeof buf, "%s \"r\"(%c%u)", j ? "," : "", b ? 'y' : 'x', j);
+                s += buf;
+            }
+            if (ncmp) {
+                snprintf(buf, sizeof buf, ", \"l\"(dbuf%d)", b);
+                s += buf;
+            }
+            s += " : \"memory\");\n";
         }
-        s += "      asm volatile(\"//@@BODY0@@";
-        for (uint32_t i = 0; i < M + p.k + (ncmp ? 1 : 0); ++i) {
-            snprintf(buf, sizeof buf, " %%%u", i);
-            s += buf;
-        }
-        s += "\" :";
-        for (uint32_t w = 0; w < M; ++w) {
-            snprintf(buf, sizeof buf, "%s \"=r\"(m%u)", w ? "," : "", w);
-            s += buf;
-        }
-        s += " :";
-        for (uint32_t j = 0; j < p.k; ++j) {
-            snprintf(buf, sizeof buf, "%s \"r\"(x%u)", j ? "," : "", j);
-            s += buf;
-        }
-        if (ncmp) s += ", \"l\"(dbuf)";
-        s += " : \"memory\");\n";
-        for (uint32_t w = 0; w < M; ++w) {
-            snprintf(buf, sizeof buf,
-                     "      for (u32 mk = m%u; mk; mk &= mk - 1u) { const u32 c = %uu + (u32)__ffs(mk) - 1u;\n"
-                     "        const u32 d = live ? dbuf[c] : 0u;\n"
-                     "        if (__any_sync(0xFFFFFFFFu, d != 0u)) rep(d, c, I.win, s, lane, %uu, I.cmp_off, first, bound, neq_cnt); }\n",
-                     w, 32 * w, ncmp);
-            s += buf;
-        }
+        for (int b = 0; b < nb; ++b)
+            for (uint32_t w = 0; w < M; ++w) {
+                snprintf(buf, sizeof buf,
+                         "      for (u32 mk = m%d_%u; mk; mk &= mk - 1u) { const u32 c = %uu + (u32)__ffs(mk) - 1u;\n"
+                         "        const u32 d = %s ? dbuf%d[c] : 0u;\n"
+                         "        if (__any_sync(0xFFFFFFFFu, d != 0u)) rep(d, c, I.win, %s, lane, %uu, I.cmp_off, first, bound, neq_cnt); }\n",
+                         b, w, 32 * w, b ? "liveB" : "live", b, b ? "sB" : "s", ncmp);
+                s += buf;
+            }
     } else {
         const std::vector<MappedNode> map = jit_map_mode(p, jit_eff_mode(cfg));
         uint32_t lut_total = 0;
@@ -1196,8 +1221,8 @@ const char *jit_get_unit(const std::vector<const JitProgram *> &ps, const JitCon
     if (bundle && !(cfg.splice && (cfg.sync_every > 0 || cfg.free_warps)))
         return "JIT bundles need the splice mode (block-synchronous or free warps)";
     char ck[64];
-    snprintf(ck, sizeof ck, "|%d,%d,%d,%d,%d,%d", cfg.threads, cfg.min_blocks, cfg.sync_every, (int)cfg.fuse,
-             (int)cfg.splice, (int)cfg.free_warps);
+    snprintf(ck, sizeof ck, "|%d,%d,%d,%d,%d,%d,%d", cfg.threads, cfg.min_blocks, cfg.sync_every, (int)cfg.fuse,
+             (int)cfg.splice, (int)cfg.free_warps, cfg.ilp);
     std::string key;
     for (const JitProgram *p : ps) key += jit_key(*p) + "#";
     key += ck;
@@ -1216,7 +1241,10 @@ const char *jit_get_unit(const std::vector<const JitProgram *> &ps, const JitCon
     const std::string src = bundle ? jit_source_bundle(ps, cfg) : jit_source(*ps[0], cfg);
     std::vector<char> cubin;
     std::string log;
-    const char *e = (cfg.splice && (cfg.sync_every > 0 || cfg.free_warps)) ? jit_compile_splice(ps, cfg, src, cubin, log)
+    // ILP 2 (single free-warp structure): the same program is spliced into BODY0 and BODY1
+    const bool ilp2 = !bundle && cfg.free_warps && cfg.splice && cfg.ilp == 2;
+    const std::vector<const JitProgram *> sps = ilp2 ? std::vector<const JitProgram *>{ps[0], ps[0]} : ps;
+    const char *e = (cfg.splice && (cfg.sync_every > 0 || cfg.free_warps)) ? jit_compile_splice(sps, cfg, src, cubin, log)
                                                                           : jit_compile_cubin(src, cubin, log);
     if (e) {
         static thread_local std::string msg;
