@@ -270,3 +270,33 @@ def test_own_index_mapping_V4():
         assert orc.eval_lit(s3a, pis) == ((a + b) >> 3) & 1
     pis = np.asarray(orc.cex_vector(s3a, s3b, 107))
     assert [int(pis[j]) for j in range(4)] == [1, 1, 0, 1] and [int(pis[8 + j]) for j in range(4)] == [0, 1, 1, 0]
+
+
+@pytest.mark.parametrize("n", [8, 64])
+def test_datapath_closed_form_C4(n):
+    """C4: both sides of the n-bit datapath miter compute s = a + b + cin,
+    lt = (a < b) and y = lt ? b : a — checked bit by bit through the oracle's own evaluator at
+    random assignments (arithmetic, not the oracle, is the reference), and the bug variant's B side
+    differs from the closed form at some assignment the oracle finds (it must never be EQ)."""
+    m = circuits.c4_dp(n)
+    orc = Oracle.from_aig(m.aig)
+    rng = np.random.default_rng(n)
+    mask = (1 << n) - 1
+    for _ in range(40):
+        a = int(rng.integers(0, 1 << 62)) & mask if n > 62 else int(rng.integers(0, 1 << n))
+        b = int(rng.integers(0, 1 << 62)) & mask if n > 62 else int(rng.integers(0, 1 << n))
+        if n > 62:
+            a |= int(rng.integers(0, 4)) << 62
+            b |= int(rng.integers(0, 4)) << 62
+        cin = int(rng.integers(0, 2))
+        pis = np.array([(a >> i) & 1 for i in range(n)] + [(b >> i) & 1 for i in range(n)] + [cin], np.uint8)
+        s = a + b + cin
+        want = [(s >> i) & 1 for i in range(n + 1)] + [int(a < b)] + [((b if a < b else a) >> i) & 1 for i in range(n)]
+        for side in (m.lit_a, m.lit_b):
+            got = [orc.eval_lit(int(l), pis) for l in side]
+            assert got == want, (n, a, b, cin)
+    if n == 8:  # small enough for the exhaustive oracle: the bug variant is refuted, never EQ
+        mb = circuits.c4_dp(n, bug=4)
+        ob = Oracle.from_aig(mb.aig)
+        v, _, _, _ = ob.check_pairs(mb.lit_a, mb.lit_b, k_max=17)
+        assert (v == NEQ).any() and not (v == EQ).all()
