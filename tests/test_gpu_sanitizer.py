@@ -16,8 +16,11 @@ import sys
 sys.path.insert(0, %r)
 from paper_conf_dac_liuy25_b200 import capi
 from workloads import c1_add8, circuits
+# JIT: c1 / mul6 run as single-structure free-warp kernels with IMAD cells; the reduced C5 as a
+# block-synchronous bundle kernel (several structures)
+mini = circuits.c5_big(copies=4, n_random=2, n_bugs=1, rand_pis=12, rand_ands=200, mul_n=6)
 for eng in (capi.CEC_ENGINE_INTERP, capi.CEC_ENGINE_JIT):
-    for m in (c1_add8(), circuits.c2_mul12_bug(seed=1, n=6)):
+    for m in (c1_add8(), circuits.c2_mul12_bug(seed=1, n=6), mini):
         ctx = capi.Context.from_aig(m.aig, engine=eng)
         v, c, k = ctx.sim_exhaustive(m.lit_a, m.lit_b)
         ctx.check_local_cuts(m.lit_a[:2], m.lit_b[:2], [0, 2, 4], [1, 2, 3, 4])
