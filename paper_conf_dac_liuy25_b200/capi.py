@@ -415,7 +415,8 @@ class Context:
         return cec_get_cex(self._ctx, pair_idx, self.num_pis)
 
     def sim_classes(self, num_words: int, seed: int, pi_words=None, cap=None):
-        return cec_sim_classes(self._ctx, num_words, seed, pi_words, cap)
+        # every member is an AND node, so num_ands bounds the pair count: one call, no count pass
+        return cec_sim_classes(self._ctx, num_words, seed, pi_words, max(1, self.num_ands) if cap is None else cap)
 
     def reduce(self, member_ids, repr_lits, lits=()):
         return cec_reduce(self._ctx, self.num_pis, self.num_ands, member_ids, repr_lits, lits)
