@@ -261,10 +261,11 @@ def check_miter(aig: Aig, lit_a, lit_b, params: Optional[CecParams] = None) -> C
         ctx = _ctx(cur.aig, p, p.k_g)
         # local checks need k_max >= k_l (cut leaves); one context serves both when k_l <= k_g
         lctx = ctx if p.k_l <= p.k_g else _ctx(cur.aig, p, max(p.k_l, 1))
+        t_ctx = time.perf_counter() - t
         # equivalence classes on the GPU: random patterns plus the CEX patterns
         # of disproved pairs, which split their classes
         words = pack_patterns(cex_patterns, cur.aig.num_pis) if cex_patterns else None
-        tk = {"classes": 0.0, "global": 0.0, "cuts": 0.0, "local": 0.0}
+        tk = {"ctx": t_ctx, "classes": 0.0, "global": 0.0, "cuts": 0.0, "local": 0.0}
         t1 = time.perf_counter()
         cr, cm, cf = ctx.sim_classes(p.sim_words, p.seed + phase_no, words)
         tk["classes"] += time.perf_counter() - t1
@@ -363,9 +364,11 @@ def check_miter(aig: Aig, lit_a, lit_b, params: Optional[CecParams] = None) -> C
             t1 = time.perf_counter()
             nxt, image = cur.reduce(subst, p.device, ctx=ctx)
             entry["s_parts"]["reduce"] = round(time.perf_counter() - t1, 4)
+        t1 = time.perf_counter()
         ctx.close()
         if lctx is not ctx:
             lctx.close()
+        entry["s_parts"]["close"] = round(time.perf_counter() - t1, 4)
         entry["s"] = time.perf_counter() - t
         if not subst:
             break  # no progress: undecided remainder
