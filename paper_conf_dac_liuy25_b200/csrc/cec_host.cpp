@@ -1251,7 +1251,16 @@ cec_status upload(cec_ctx *c, cec_plan *P) {
         CUDA_TRY(c, P->pool->staging(up_bytes, &hst));
         char *h = (char *)hst;
         if (b_wins) memcpy(h + o_wins, P->dwin.data(), b_wins);
-        if (b_prog) memcpy(h + o_prog, P->prog.data(), b_prog);
+        if (b_prog >= (4u << 20)) {  // large interpreter programs (C3: ~9 MB): copied by the worker pool
+            const size_t chunk = 1u << 20, nch = (b_prog + chunk - 1) / chunk;
+            const char *src = reinterpret_cast<const char *>(P->prog.data());
+            c->workers().run((uint32_t)nch, [&](uint32_t i, unsigned) {
+                const size_t o = (size_t)i * chunk;
+                memcpy(h + o_prog + o, src + o, std::min(chunk, b_prog - o));
+            });
+        } else if (b_prog) {
+            memcpy(h + o_prog, P->prog.data(), b_prog);
+        }
         if (b_items) memcpy(h + o_items, P->items.data(), b_items);
         if (b_jitems) memcpy(h + o_jitems, P->jitems.data(), b_jitems);
         if (b_joff) memcpy(h + o_joff, P->joff.data(), b_joff);
