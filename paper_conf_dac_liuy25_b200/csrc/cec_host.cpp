@@ -589,7 +589,7 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         for (uint32_t ci : wins[w].cmps) {
             remap[ci] = (int32_t)cmps2.size();
             wcs[w].push_back((uint32_t)cmps2.size());
-            cmps2.push_back(P->cmps[ci]);
+            cmps2.push_back(std::move(P->cmps[ci]));  // each compare sits in one window
         }
         for (uint32_t ci : wcs[w]) {  // a11 pext masks
             Cmp &cm = cmps2[ci];
@@ -1207,6 +1207,7 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
     // biggest groups first so the small launches fill in behind them
     std::stable_sort(P->groups.begin(), P->groups.end(),
                      [](const LaunchGroup &a, const LaunchGroup &b) { return a.nitems > b.nitems; });
+    tm2.lap("work items + launch groups");
     (void)stop;
     (void)local;
     return CEC_OK;
@@ -1233,9 +1234,11 @@ cec_status upload(cec_ctx *c, cec_plan *P) {
     const size_t o_bound = off; off += al(sizeof(unsigned long long) * nwin);
     const size_t o_neq = off; off += al(sizeof(uint32_t) * nwin);
     const size_t o_ctr = off; off += al(sizeof(uint32_t) * std::max<size_t>(1, P->groups.size()));
+    PhaseTimer tu;
     if (!c->devpool) c->devpool = std::make_shared<DevPool>();
     P->pool = c->devpool;
     CUDA_TRY(c, P->pool->get(off, &P->arena, &P->arena_cap));
+    tu.lap("upload: device block");
     char *base = (char *)P->arena;
     d.wins = (DevWin *)(base + o_wins);
     d.prog = (uint4 *)(base + o_prog);
@@ -1249,6 +1252,7 @@ cec_status upload(cec_ctx *c, cec_plan *P) {
     {
         void *hst = nullptr;
         CUDA_TRY(c, P->pool->staging(up_bytes, &hst));
+        tu.lap("upload: staging wait/alloc");
         char *h = (char *)hst;
         if (b_wins) memcpy(h + o_wins, P->dwin.data(), b_wins);
         if (b_prog >= (4u << 20)) {  // large interpreter programs (C3: ~9 MB): copied by the worker pool
@@ -1264,8 +1268,10 @@ cec_status upload(cec_ctx *c, cec_plan *P) {
         if (b_items) memcpy(h + o_items, P->items.data(), b_items);
         if (b_jitems) memcpy(h + o_jitems, P->jitems.data(), b_jitems);
         if (b_joff) memcpy(h + o_joff, P->joff.data(), b_joff);
+        tu.lap("upload: staging copies");
         CUDA_TRY(c, h2d(base, h, o_joff + b_joff, c->stream));
         CUDA_TRY(c, P->pool->staged(c->stream));
+        tu.lap("upload: h2d issue");
     }
     if (P->simt.E) {
         SimtPlan &S = P->simt;
@@ -1782,14 +1788,16 @@ cec_status cec_sim_exhaustive(cec_ctx *c, uint32_t n, const uint32_t *la, const 
         S.p.reset(new (std::nothrow) cec_plan());
         if (!S.p) return CEC_E_NOMEM;
         std::vector<WinHost> cw;
+        // the chunk takes the windows' inputs and the compares' supports by move (each window /
+        // compare belongs to one chunk); the supports move back at the gather
         for (size_t w = cut[ch]; w < cut[ch + 1]; ++w) {
             WinHost h;
-            h.inputs = wins[w].inputs;
+            h.inputs = std::move(wins[w].inputs);
             h.est_nodes = wins[w].est_nodes;
             for (uint32_t ci : wins[w].cmps) {
                 h.cmps.push_back((uint32_t)S.gcmp.size());
                 S.gcmp.push_back(ci);
-                S.p->cmps.push_back(P->cmps[ci]);
+                S.p->cmps.push_back(std::move(P->cmps[ci]));
             }
             cw.push_back(std::move(h));
         }
@@ -1803,6 +1811,7 @@ cec_status cec_sim_exhaustive(cec_ctx *c, uint32_t n, const uint32_t *la, const 
             free_dev(S.p.get());
             return st;
         }
+        tm.lap("call: chunk upload");
         if (!S.p->cmps.empty() && (st = cec_plan_run(c, S.p.get())) != CEC_OK) {
             free_dev(S.p.get());
             return st;
@@ -1851,6 +1860,7 @@ cec_status cec_sim_exhaustive(cec_ctx *c, uint32_t n, const uint32_t *la, const 
         for (uint32_t j = 0; j < S.gcmp.size(); ++j) {
             const int32_t lj = S.p->pair_cmp[j];  // finish_plan's renumbering of local compare j
             P->cmps[S.gcmp[j]].ownmask = S.p->cmps[lj].ownmask;
+            P->cmps[S.gcmp[j]].S = std::move(S.p->cmps[lj].S);
             first[S.gcmp[j]] = part[i][lj];
         }
         free_dev(S.p.get());
