@@ -120,13 +120,18 @@ def oracle_sample(m, copy_idx, log2_patterns, procs=1, reps=1):
             evals += e
         return evals, dt, f"{what}, patterns [0, 2^{log2_patterns}) of its 2^24-pattern window, single thread"
     _SHARD.update(orc=orc, la=la, lb=lb)
-    with multiprocessing.get_context("fork").Pool(procs) as pool:
-        pool.map(_oracle_shard, [(0, 1)] * procs)  # fork + warm every worker outside the timed region
-        evals, dt = 0, 0.0
-        for _ in range(reps):
-            t = time.perf_counter()
-            evals += sum(pool.map(_oracle_shard, [(r * n, (r + 1) * n) for r in range(procs)], chunksize=1))
-            dt += time.perf_counter() - t
+    try:  # forked after CUDA init: the workers only run the C oracle; bounded wait, else one thread
+        with multiprocessing.get_context("fork").Pool(procs) as pool:
+            pool.map_async(_oracle_shard, [(0, 1)] * procs).get(timeout=120)  # fork + warm, untimed
+            evals, dt = 0, 0.0
+            for _ in range(reps):
+                t = time.perf_counter()
+                evals += sum(pool.map_async(_oracle_shard, [(r * n, (r + 1) * n) for r in range(procs)],
+                                            chunksize=1).get(timeout=600))
+                dt += time.perf_counter() - t
+    except Exception as e:  # pragma: no cover - safety net
+        print(f"bench: sharded oracle failed ({e!r}); single-thread sample instead", file=sys.stderr)
+        return oracle_sample(m, copy_idx, log2_patterns, 1, reps)
     return evals, dt, (f"{what}, patterns [0, {procs}*2^{log2_patterns}) of its 2^24-pattern window in {procs} "
                        f"ranges, one single-threaded oracle process per host core (SURVEY.md §8(c) sharded oracle)")
 
