@@ -230,8 +230,12 @@ std::vector<MappedNode> jit_map(const JitProgram &p, bool fuse) {
 // edge complements except ~y & ~m can be evaluated by ONE IMAD on the FMA pipe (the register then
 // holds the function or its complement; readers fold that polarity into their LOP3 tables, just as
 // they fold edge complements). Every AND node is still evaluated on every pattern — on the other
-// pipe. The mapper prices an IMAD cell at `imad_cost` LUTs, so it takes them where they relieve the
-// ALU pipe; ~y & ~m (no single-IMAD form with operands y, m, -1) and XOR-type cuts stay LOP3s.
+// pipe. m may also be a node whose support lies inside those inputs (its words are 0 or ~0 too).
+// The mapper prices an IMAD cell at `imad_cost` LUTs (the measured ALU cost of its register reads,
+// scripts/pipes.cu), so it takes them where they relieve the ALU pipe. ~y & ~m has no form with
+// operands y, m, -1; it becomes y & ~m when y's register holds the complement (LOP3 outputs take the
+// polarity most of their IMAD readers need), else the cell falls back to a LOP3. XOR-type cuts stay
+// LOP3s. jit_verify_map emulates the result against the AIG (CEC_JIT_VERIFY).
 namespace {
 constexpr uint8_t kLeafTT[3] = {0xF0, 0xCC, 0xAA};
 // g = the 2-input function of (y, m) as a 4-bit table, bit (2*y + m). Returns the IMAD form
