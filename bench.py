@@ -456,7 +456,8 @@ def main():
     # parity against stored oracle results of the same generated miter (tests/golden, written by
     # scripts/make_golden*.py, which call only oracle/): every pair's verdict, k and canonical CEX
     parity = None
-    gold_name = {"c5": "c5_big", "c3": "c3_rand", "c2": "c2_mul12", "c2bug": "c2_mul12_bug1"}.get(args.config)
+    gold_name = {"c5": "c5_big", "c3": "c3_rand", "c2": "c2_mul12", "c2bug": "c2_mul12_bug1",
+                 "c1": "c1_add8"}.get(args.config)
     gpath = os.path.join(ROOT, "tests", "golden", f"{gold_name}.json") if gold_name else None
     if rank == 0 and gpath and os.path.exists(gpath):
         g = json.load(open(gpath))

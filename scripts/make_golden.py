@@ -1,4 +1,4 @@
-"""Write oracle results for the full-size configs whose oracle run takes minutes (C2, C2-bug).
+"""Write oracle results for the full-size configs C1, C2 and C2-bug (C2's oracle run takes minutes).
 
 Calls only oracle/ (and the seeded generators). Output: tests/golden/<name>.json with per-pair
 verdict, k and canonical CEX index, plus the generator parameters, so GPU parity tests on the box
@@ -12,9 +12,10 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
 
 import oracle  # noqa: E402
-from workloads import c2_mul12, c2_mul12_bug  # noqa: E402
+from workloads import c1_add8, c2_mul12, c2_mul12_bug  # noqa: E402
 
 CASES = {
+    "c1_add8": (c1_add8, {}),
     "c2_mul12": (c2_mul12, {}),
     "c2_mul12_bug1": (c2_mul12_bug, {"seed": 1}),
 }

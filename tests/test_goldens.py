@@ -10,10 +10,11 @@ import numpy as np
 import pytest
 
 import oracle
-from workloads import c2_mul12, c2_mul12_bug, c3_rand, c5_big
+from workloads import c1_add8, c2_mul12, c2_mul12_bug, c3_rand, c5_big
 
 GOLD = os.path.join(os.path.dirname(__file__), "golden")
 CASES = {
+    "c1_add8": lambda: c1_add8(),
     "c2_mul12": lambda: c2_mul12(),
     "c2_mul12_bug1": lambda: c2_mul12_bug(seed=1),
     "c3_rand": lambda: c3_rand(),
@@ -40,6 +41,6 @@ def test_golden_matches_generator_and_cex_separates(name):
         vec = orc.cex_vector(la, lb, idx)
         assert orc.eval_lit(la, vec) != orc.eval_lit(lb, vec), (name, p, idx)
     # the bug-free configurations have no NEQ pair; the bugged ones do
-    assert (len(neq) == 0) == (name == "c2_mul12")
+    assert (len(neq) == 0) == (name in ("c1_add8", "c2_mul12"))
     if name == "c5_big":
         assert len(neq) == 8  # one observable bug per bugged copy
