@@ -18,19 +18,29 @@ import numpy as np  # noqa: E402
 
 import oracle  # noqa: E402
 from paper_conf_dac_liuy25_b200 import capi  # noqa: E402
-from workloads import tiny_random  # noqa: E402
+from workloads import circuits, tiny_random  # noqa: E402
 
 
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--seeds", type=int, default=300)
     ap.add_argument("--start", type=int, default=0)
+    ap.add_argument("--miters", action="store_true",
+                    help="random-block miters A vs rewritten A (mostly EQ: full sweeps) instead of random pairs")
     a = ap.parse_args()
     bad, pairs, neq, t0 = [], 0, 0, time.time()
     for seed in range(a.start, a.start + a.seeds):
         rng = np.random.default_rng(70000 + seed)
         I = int(rng.integers(10, 17))
-        m = tiny_random(I, int(rng.integers(30, 400)), 24, 80000 + seed)
+        if a.miters:
+            m = circuits.random_miter(I, int(rng.integers(100, 600)), 12, seed=90000 + seed,
+                                      window=int(rng.integers(16, 64)))
+            if rng.random() < 0.3:  # an injected observable-or-not single-gate bug in B
+                lo, hi = circuits.b_side_ids(m)
+                if hi > lo:
+                    m = circuits.flip_fanin(m, int(rng.integers(lo, hi)), int(rng.integers(0, 2)))
+        else:
+            m = tiny_random(I, int(rng.integers(30, 400)), 24, 80000 + seed)
         merge = int(rng.integers(0, 3))
         ctx = capi.Context.from_aig(m.aig, k_max=16, merge=merge, engine=capi.CEC_ENGINE_JIT)
         gv, gc, gk = ctx.sim_exhaustive(m.lit_a, m.lit_b)
@@ -48,7 +58,7 @@ def main():
         pairs += m.num_pairs
         neq += int((ov == oracle.NOT_EQUIVALENT).sum())
         ctx.close()
-    print(json.dumps({"fuzz": "jit engine vs oracle", "seeds": a.seeds, "start": a.start, "pairs": pairs,
+    print(json.dumps({"fuzz": "jit engine vs oracle" + (" (A vs rewritten A miters)" if a.miters else ""), "seeds": a.seeds, "start": a.start, "pairs": pairs,
                       "neq_pairs": neq, "mismatching_seeds": bad, "ok": not bad,
                       "seconds": round(time.time() - t0, 1)}), flush=True)
     return 1 if bad else 0
