@@ -500,7 +500,10 @@ def main():
                          "fma_pipe_timad_s": stats.get("imad_words", 0) / (ms / 1e3) / 1e12,
                          "cells": "3-input LUTs = lop3.b32 on the ALU pipe (the bound); AND nodes with a "
                                   "word-uniform operand = mad.lo.u32 on the FMA pipe (DESIGN.md §4.1)",
-                         "and_evals_tops": (W_rank / 32.0) / (ms / 1e3) / 1e12}),
+                         "and_evals_tops": (W_rank / 32.0) / (ms / 1e3) / 1e12,
+                         # the SURVEY §8(d) unit (one 2-input op per AND per u32 word) against the same
+                         # peak: > 1 because a mapped LOP3/IMAD cell evaluates ~1.9 ANDs
+                         "and_evals_per_lop3_peak": (W_rank / 32.0) / (ms / 1e3) / 1e12 / peak}),
             "step_ms": step_ms, "wall_s": wall,
         }
         if cpu:
