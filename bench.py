@@ -268,7 +268,8 @@ def main():
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
     # BENCH_SAME_GPU=1 (testing only): every rank on device 0, gloo process group, peer reduction only
-    # (NCCL refuses two ranks on one GPU). Times are meaningless there (ranks time-slice one GPU).
+    # (NCCL refuses two ranks on one GPU) with HOST barriers (cec_peer_host_barrier: kernels that wait
+    # on one another must not share one GPU). Times are meaningless there (ranks time-slice one GPU).
     same_gpu = os.environ.get("BENCH_SAME_GPU") == "1"
     if same_gpu:
         local = 0
@@ -320,6 +321,8 @@ def main():
             if all(b is not None for b in blobs):
                 try:
                     capi.cec_peer_import(c.handle, blobs)
+                    if same_gpu:  # ranks on one device never spin on each other (include/cec.h)
+                        c._host_barrier_cb = capi.cec_peer_host_barrier(c.handle, dist.barrier)
                 except capi.CecError as e:
                     err = str(e)
             else:
@@ -345,7 +348,9 @@ def main():
     if world > 1:
         ok = allreduce(0.0 if err else 1.0, dist.ReduceOp.MIN)  # every rank takes the same path
         if peer and ok == 1.0:
-            reduce_mode = "peer memory (NVLink, fused atomicMin into rank 0's home arrays + device barriers)"
+            reduce_mode = ("peer memory (one-GPU emulation: fused atomicMin into rank 0's home arrays + HOST barriers)"
+                           if same_gpu else
+                           "peer memory (NVLink, fused atomicMin into rank 0's home arrays + device barriers)")
         elif peer and not same_gpu:  # fall back to the collective on every rank
             ctx.close()
             ctx, plan, err2 = open_ctx(False)

@@ -297,6 +297,18 @@ cec_status cec_nccl_unique_id(void *out128);
 cec_status cec_peer_export(cec_ctx *ctx, void *blob_out);
 cec_status cec_peer_import(cec_ctx *ctx, const void *blobs);
 
+/* Emulation of several ranks on ONE device (tests only; a one-GPU box has no second GPU). Kernels
+ * that wait on one another must not run as separate launches on one GPU: nothing makes them
+ * co-resident, and on B200 two or four such processes raised Xid 109 (context-switch timeout,
+ * /opt/skills/guides/B200_PROFILING.md). With `fn` set, every peer barrier of a run becomes
+ * "drain this rank's stream, then call fn(user)", where fn is the caller's host barrier across the
+ * emulated ranks (e.g. a gloo dist.barrier()); no kernel ever waits for another rank, and runs are
+ * not captured in CUDA graphs. Everything else of the peer path is unchanged (IPC mappings,
+ * system-scope atomicMin into rank 0's home arrays, cross-rank bounds, gather). fn = NULL restores
+ * the device barriers. Call after cec_peer_import, on every rank.
+ * Errors: CEC_E_ARG (null ctx), CEC_E_STATE (the context is not in peer mode). */
+cec_status cec_peer_host_barrier(cec_ctx *ctx, void (*fn)(void *user), void *user);
+
 /* Host utility exported for tests: the contiguous slice range [*begin, *end) of `n` slices that
  * rank `rank` of `world` simulates (pattern-space sharding). */
 void cec_shard_range(uint64_t n, int32_t rank, int32_t world, uint64_t *begin, uint64_t *end);

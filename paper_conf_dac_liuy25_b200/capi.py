@@ -29,7 +29,7 @@ EXPORTS = ["cec_default_opts", "cec_load_aig", "cec_sim_exhaustive", "cec_check_
            "cec_plan_window", "cec_plan_free", "cec_stream", "cec_get_stats", "cec_shard_range", "cec_pext64",
            "cec_free", "cec_last_error", "cec_abi_version", "cec_nccl_unique_id", "cec_sim_random",
            "cec_common_cuts", "cec_sim_patterns", "cec_reduce", "cec_sim_classes", "cec_local_pass",
-           "cec_peer_export", "cec_peer_import"]
+           "cec_peer_export", "cec_peer_import", "cec_peer_host_barrier"]
 
 
 class CecOpts(ctypes.Structure):
@@ -91,6 +91,7 @@ def _load() -> ctypes.CDLL:
         "cec_nccl_unique_id": (ctypes.c_int, [P]),
         "cec_peer_export": (ctypes.c_int, [P, P]),
         "cec_peer_import": (ctypes.c_int, [P, P]),
+        "cec_peer_host_barrier": (ctypes.c_int, [P, P, P]),
         "cec_sim_random": (ctypes.c_int, [P, u32, u64, P, P]),
         "cec_common_cuts": (ctypes.c_int, [P, u32, P, P, u32, u32, i32, u32, P, P, P]),
         "cec_sim_patterns": (ctypes.c_int, [P, u32, P, P, P]),
@@ -383,6 +384,18 @@ def cec_peer_import(ctx, blobs) -> None:
     _check(lib.cec_peer_import(ctx, ctypes.create_string_buffer(raw, len(raw))), ctx)
 
 
+HOST_BARRIER_FN = ctypes.CFUNCTYPE(None, ctypes.c_void_p)
+
+
+def cec_peer_host_barrier(ctx, fn) -> object:
+    """Several ranks emulated on ONE device (tests): every peer barrier becomes "drain the stream,
+    then fn()" (include/cec.h cec_peer_host_barrier). Returns the ctypes callback, which the caller
+    keeps alive as long as the context uses it; fn = None restores the device barriers."""
+    cb = HOST_BARRIER_FN(lambda _user: fn()) if fn is not None else None
+    _check(lib.cec_peer_host_barrier(ctx, ctypes.cast(cb, ctypes.c_void_p) if cb else None, None), ctx)
+    return cb
+
+
 def cec_abi_version() -> int:
     return int(lib.cec_abi_version())
 
@@ -421,11 +434,14 @@ class Context:
     def reduce(self, member_ids, repr_lits, lits=()):
         return cec_reduce(self._ctx, self.num_pis, self.num_ands, member_ids, repr_lits, lits)
 
-    def peer_connect(self, all_gather) -> None:
+    def peer_connect(self, all_gather, host_barrier=None) -> None:
         """Peer-memory a10 (include/cec.h cec_peer_export/import): `all_gather(blob) -> [blob of
         rank 0, ..., rank world-1]` is the caller's collective (e.g. torch.distributed
-        all_gather_object); every rank calls this once, collectively."""
+        all_gather_object); every rank calls this once, collectively. `host_barrier` (ranks
+        emulated on one device only): the callable that replaces the device barriers."""
         cec_peer_import(self._ctx, all_gather(cec_peer_export(self._ctx)))
+        if host_barrier is not None:
+            self._host_barrier_cb = cec_peer_host_barrier(self._ctx, host_barrier)
 
     def pair_k(self, lit_a: int, lit_b: int) -> int:
         return cec_pair_k(self._ctx, lit_a, lit_b)

@@ -413,6 +413,15 @@ cec_status cec_peer_import(cec_ctx *c, const void *blobs) {
     return e ? fail(c, CEC_E_CUDA, "peer import: %s", e) : CEC_OK;
 }
 
+cec_status cec_peer_host_barrier(cec_ctx *c, void (*fn)(void *), void *user) {
+    if (!c) return CEC_E_ARG;
+    if (!c->peer.on) return fail(c, CEC_E_STATE, "cec_peer_host_barrier needs a connected peer context");
+    c->peer.host_barrier = fn;
+    c->peer.host_user = user;
+    ++c->peer.gen;  // graphs captured with device barriers are stale
+    return CEC_OK;
+}
+
 uint64_t cec_pext64(uint64_t value, uint64_t mask) {
     uint64_t r = 0;
     int j = 0;
@@ -1567,8 +1576,9 @@ cec_status cec_plan_run(cec_ctx *c, cec_plan *P) {
     uint32_t nl = 0;
     const char *e = nullptr;
     // a plan that is run again is replayed as a CUDA graph (captured on its second run)
+    // (host-barrier emulation synchronises inside the run: no graph capture)
     const bool use_graph = !P->simt.E && P->runs >= 1 && getenv("CEC_NO_GRAPH") == nullptr &&
-                           getenv("CEC_PROFILE_GROUPS") == nullptr;
+                           getenv("CEC_PROFILE_GROUPS") == nullptr && !(c->peer.on && c->peer.host_barrier);
     // a10 over peer memory (peer.cu) when cec_peer_import connected this rank; else NCCL below
     const bool peer = c->peer.on && !P->simt.E;
     PeerRun pr;
@@ -1756,11 +1766,55 @@ cec_status cec_sim_exhaustive(cec_ctx *c, uint32_t n, const uint32_t *la, const 
         wcost[w] = std::ldexp(1.0, (int)k) * (double)(1 + std::max<uint64_t>(wins[w].est_nodes, wins[w].cmps.size()));
         total += wcost[w];
     }
+    // Many small windows (C3: median k < 20, thousands of windows): geometric chunks would only
+    // fragment the bundle kernels, but the sweep is still dominated by a few large windows. Those
+    // (estimated sweep >= 2^26 node-words) form a first chunk that is planned and launched alone;
+    // the GPU runs them while the host plans the rest
+    // (bundles and interpreter windows). CEC_PIPE_SPLIT = the node-word threshold (0 = off); C3:
+    // 154 of 3253 windows carry 95% of the sweep at 2^26, and the call takes 15.6-16.3 ms instead
+    // of 18.4-18.6 (2^24: 16.1, 2^28: 16.5, 2^30: 17.3-18.9; profiles/round2s2_c3_split_sweep.txt).
+    std::vector<size_t> cut{0};
+    double split_nw = std::ldexp(1.0, 26);
+    if (const char *e = getenv("CEC_PIPE_SPLIT")) split_nw = atof(e);
+    size_t split_min = 256;  // windows; CEC_PIPE_SPLIT_MINWIN
+    if (const char *e = getenv("CEC_PIPE_SPLIT_MINWIN")) split_min = strtoull(e, nullptr, 10);
+    bool split = false;
+    if (getenv("CEC_PIPE_SPLIT_DEBUG"))
+        for (int e = 20; e <= 38; e += 2) {
+            size_t nb = 0;
+            double bc = 0;
+            for (size_t w = 0; w < wins.size(); ++w)
+                if (wcost[w] / 32.0 >= std::ldexp(1.0, e)) ++nb, bc += wcost[w];
+            fprintf(stderr, "[cec] split 2^%d: %zu of %zu windows, %.3f of the cost\n", e, nb, wins.size(), bc / total);
+        }
+    if (K == 1 && split_nw > 0 && wins.size() >= split_min && c->opts.engine != CEC_ENGINE_SIMT) {
+        std::vector<uint8_t> big(wins.size(), 0);
+        size_t nbig = 0;
+        double big_cost = 0;
+        for (size_t w = 0; w < wins.size(); ++w)
+            if (wcost[w] / 32.0 >= split_nw) big[w] = 1, ++nbig, big_cost += wcost[w];
+        // worth it only when the first chunk is a small share of the windows and carries most of
+        // the sweep (its kernels then cover the planning of everything else)
+        if (nbig > 0 && nbig * 8 <= wins.size() && big_cost >= 0.5 * total) {
+            std::vector<WinHost> reord;
+            std::vector<double> rc;
+            reord.reserve(wins.size());
+            for (int pass = 0; pass < 2; ++pass)
+                for (size_t w = 0; w < wins.size(); ++w)
+                    if (big[w] == (pass == 0)) reord.push_back(std::move(wins[w])), rc.push_back(wcost[w]);
+            wins.swap(reord);
+            wcost.swap(rc);
+            cut.push_back(nbig);
+            split = true;
+            char what[64];
+            snprintf(what, sizeof what, "call: split %zu big of %zu", nbig, wins.size());
+            tm.lap(what);
+        }
+    }
     // contiguous window ranges growing geometrically (4%, 8%, 16%, ... of the cost): the GPU starts
     // after planning a small first chunk, and each chunk's kernels (~2x the host time to plan the
     // same windows) cover the planning of the next, twice as large, chunk
-    std::vector<size_t> cut{0};
-    {
+    if (!split) {
         double first = 0.04, growth = 2.0;  // tunable: CEC_PIPE_FIRST (fraction), CEC_PIPE_GROWTH
         if (const char *e = getenv("CEC_PIPE_FIRST")) first = std::max(1e-4, atof(e));
         if (const char *e = getenv("CEC_PIPE_GROWTH")) growth = std::max(1.0, atof(e));
@@ -1773,8 +1827,8 @@ cec_status cec_sim_exhaustive(cec_ctx *c, uint32_t n, const uint32_t *la, const 
                 target = acc + chunk;
             }
         }
-        cut.push_back(wins.size());
     }
+    cut.push_back(wins.size());
     struct Sub {
         std::unique_ptr<cec_plan> p;
         std::vector<uint32_t> gcmp;  // local compare j (before finish_plan's renumbering) -> global
@@ -1816,6 +1870,7 @@ cec_status cec_sim_exhaustive(cec_ctx *c, uint32_t n, const uint32_t *la, const 
             free_dev(S.p.get());
             return st;
         }
+        tm.lap("call: chunk launch");
         agg.num_launches += c->stats.num_launches;
         agg.node_patterns += S.p->W_rank;
         agg.node_patterns_all += S.p->W_all;

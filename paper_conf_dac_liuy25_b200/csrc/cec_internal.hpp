@@ -221,6 +221,8 @@ struct PeerState {                        // per context
     void *opened[PEER_MAX] = {};          // IPC mappings to close
     uint32_t gen = 0;                     // bumped per import (invalidates captured graphs)
     uint64_t timeout_ns = 60000000000ull; // barrier wait before the error flag (CEC_PEER_TIMEOUT_S)
+    void (*host_barrier)(void *) = nullptr;  // emulation of several ranks on ONE device (tests):
+    void *host_user = nullptr;               // barriers become stream sync + this host callback
 };
 struct PeerRun {                          // what one run needs (passed into launch_run)
     bool on = false;
@@ -231,6 +233,8 @@ struct PeerRun {                          // what one run needs (passed into lau
     uint32_t *home_neq = nullptr;
     unsigned long long *local_first = nullptr;  // the plan's first[]: receives the gathered result
     uint64_t timeout_ns = 60000000000ull;
+    void (*host_barrier)(void *) = nullptr;
+    void *host_user = nullptr;
 };
 size_t peer_block_bytes(uint32_t cap_cmp, uint32_t cap_win);
 const char *peer_export(PeerState &ps, int device, int rank, int world, void *blob128);

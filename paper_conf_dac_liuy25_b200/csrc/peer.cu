@@ -191,10 +191,21 @@ PeerRun peer_run_of(const PeerState &ps, unsigned long long *local_first) {
     pr.home_neq = (uint32_t *)(pr.home_bound + ps.cap_win);
     pr.local_first = local_first;
     pr.timeout_ns = ps.timeout_ns;
+    pr.host_barrier = ps.host_barrier;
+    pr.host_user = ps.host_user;
     return pr;
 }
 
 const char *peer_barrier_launch(const PeerRun &pr, void *stream) {
+    if (pr.host_barrier) {
+        // several ranks emulated on ONE device (cec_peer_host_barrier): kernels that wait on one
+        // another must not be separate launches on one GPU (nothing makes them co-resident;
+        // B200_PROFILING.md), so the barrier is this rank's work drained + the caller's host barrier
+        const char *e = ck(cudaStreamSynchronize((cudaStream_t)stream));
+        if (e) return e;
+        pr.host_barrier(pr.host_user);
+        return nullptr;
+    }
     peer_barrier<<<1, 32, 0, (cudaStream_t)stream>>>(pr.slots, pr.own, pr.rank, pr.world, pr.timeout_ns);
     return ck(cudaGetLastError());
 }

@@ -447,6 +447,28 @@ def test_jit_bundles_vs_oracle_and_unbundled(monkeypatch):
         assert np.array_equal(a, b)
 
 
+def test_split_pipeline_vs_oracle(monkeypatch, capfd):
+    """Many small windows: the public call plans and launches the large windows (estimated sweep
+    >= CEC_PIPE_SPLIT node-words) as a first chunk and the rest while they run. Any split point
+    gives the oracle's results (verdicts, k, CEX indices); at least one threshold really splits."""
+    m = _c3_small()
+    orc = Oracle.from_aig(m.aig)
+    ov, oc, ok, _ = orc.check_pairs(m.lit_a, m.lit_b, k_max=32)
+    monkeypatch.setenv("CEC_TIMING", "1")
+    monkeypatch.setenv("CEC_PIPE_SPLIT_MINWIN", "8")
+    splits = 0
+    for e in range(6, 20, 2):
+        monkeypatch.setenv("CEC_PIPE_SPLIT", str(float(2 ** e)))
+        ctx = gpu_ctx(m.aig, merge=capi.CEC_MERGE_COST)
+        gv, gc, gk = ctx.sim_exhaustive(m.lit_a, m.lit_b)
+        assert_same(gv, gc, gk, ov, oc, ok, f"split 2^{e}")
+        for p in np.nonzero(gv == capi.CEC_NOT_EQUIVALENT)[0][:8]:
+            vec = ctx.get_cex(int(p))
+            assert orc.eval_lit(int(m.lit_a[p]), vec) != orc.eval_lit(int(m.lit_b[p]), vec)
+        splits += "call: split" in capfd.readouterr().err
+    assert splits >= 1
+
+
 def test_c5_full_vs_stored_oracle():
     """Full-size C5 (2.1M ANDs, 6320 pairs, 256 windows x 2^24 patterns) in the launch
     configuration bench.py times, against the oracle's result for EVERY pair

@@ -3,11 +3,15 @@ csrc/peer.cu; SURVEY.md §8(e) "B200-native option", §8(f) NEXT-4).
 
 The box has one GPU, so `world` ranks are emulated as `world` PROCESSES on device 0, each with its
 own CUDA context (time-sliced by the driver), exchanging CUDA IPC handles over a gloo process group —
-the same cross-process mapping a one-process-per-GPU run uses. (Several ranks as threads of ONE
-process do not work: a synchronous pageable copy in one thread serialises on the shared context
-while another thread's barrier kernel waits for it.) Every rank must return exactly the single-GPU
-result — the same per-pair minimum index the NCCL all-reduce produces (min over a partition of an
-ascending scan) — checked against the oracle (bit-exact verdicts, k, canonical CEX)."""
+the same cross-process mapping a one-process-per-GPU run uses. Kernels that wait on one another must
+not run as separate launches on one GPU (B200_PROFILING.md: such ranks raised Xid 109), so the
+emulated ranks replace the device barriers by host barriers (cec_peer_host_barrier: drain the stream,
+then a gloo dist.barrier()); the rest of the peer path is the real one — IPC mappings, every rank's
+window kernels doing system-scope atomicMin into rank 0's home arrays, cross-rank early-exit
+bounds, the gather. Every rank must return exactly the single-GPU result — the same per-pair minimum
+index the NCCL all-reduce produces (min over a partition of an ascending scan) — checked against the
+oracle (bit-exact verdicts, k, canonical CEX). The device barrier kernel itself runs here only
+alone (its timeout path), never against another rank's kernel."""
 import os
 
 import numpy as np
@@ -71,7 +75,7 @@ def _proc(rank, world, port, q, kind, name, engine):
             dist.all_gather_object(out, blob)
             return out
 
-        ctx.peer_connect(all_gather)
+        ctx.peer_connect(all_gather, host_barrier=dist.barrier)
         if kind == "sim":  # two blocking calls (the second reuses pools and JIT kernels)
             out = [_lists(ctx.sim_exhaustive(m.lit_a, m.lit_b)) for _ in range(2)]
             neq = [int(p) for p in np.nonzero(np.array(out[0][0]) == capi.CEC_NOT_EQUIVALENT)[0][:4]]
@@ -163,6 +167,22 @@ def test_peer_local_checks_match_single():
     for outs in _mp_run("local", "tiny_local", 2):
         for v in outs:
             assert np.array_equal(np.array(v), rv)
+
+
+def test_peer_device_barrier_timeout_alone(monkeypatch):
+    """The device barrier kernel, run ALONE (no other rank's kernel ever waits on it or is waited
+    for): rank 1 of a connected pair never runs, so every barrier of rank 0's run times out after
+    CEC_PEER_TIMEOUT_S, sets the error flag, and the call returns CEC_E_NCCL instead of hanging."""
+    monkeypatch.setenv("CEC_PEER_TIMEOUT_S", "0.2")
+    m = tiny_random(6, 20, 4, 503)
+    a = capi.Context.from_aig(m.aig, device=0, rank=0, world=2)
+    b = capi.Context.from_aig(m.aig, device=0, rank=1, world=2)
+    blobs = [capi.cec_peer_export(a.handle), capi.cec_peer_export(b.handle)]
+    capi.cec_peer_import(a.handle, blobs)
+    capi.cec_peer_import(b.handle, blobs)
+    with pytest.raises(capi.CecError) as ei:
+        a.sim_exhaustive(m.lit_a, m.lit_b)
+    assert ei.value.status == capi.CEC_E_NCCL
 
 
 def test_peer_import_rejects_bad_blobs():

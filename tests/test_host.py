@@ -223,6 +223,9 @@ def test_peer_mode_needs_a_device_and_world():
     with pytest.raises(capi.CecError) as e:
         capi.cec_peer_import(ctx.handle, [bytes(128), bytes(128)])
     assert e.value.status == capi.CEC_E_CUDA
+    with pytest.raises(capi.CecError) as e:  # host barriers only for a connected peer context
+        capi.cec_peer_host_barrier(ctx.handle, lambda: None)
+    assert e.value.status == capi.CEC_E_STATE
 
 
 def test_merge_never_exceeds_enumeration_limit():
