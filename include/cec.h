@@ -133,6 +133,17 @@ void cec_default_opts(cec_opts *opts);
  * (collective: every rank must call it). *ctx is set only on CEC_OK. */
 cec_status cec_load_aig(cec_ctx **ctx, const cec_aig *aig, const cec_opts *opts);
 
+/* Replace the context's AIG by the next version of the miter (the miter is
+ * reduced after each phase and the next phase works on the reduced one), keeping everything that
+ * does not depend on the AIG: device, streams, host workers, device buffer pool, compiled JIT
+ * kernels, NCCL communicator / peer mappings (so a P -> G -> L* flow pays no context creation per
+ * phase). Validation as in cec_load_aig; a rejected AIG (CEC_E_AIG / CEC_E_ARG) leaves the context
+ * unchanged. k_max / k_s: the new limits (0 = keep; k_s = 0 with k_max > 0 means k_s = k_max).
+ * Blocking (waits for the context's stream). Drops what the old AIG produced: the device copy of
+ * the AIG, the per-node support table, the last global check (cec_get_cex -> CEC_E_NOCEX).
+ * Collective when world > 1 in the sense that every rank must reload the same AIG. */
+cec_status cec_reload_aig(cec_ctx *ctx, const cec_aig *aig, uint32_t k_max, uint32_t k_s);
+
 /* Global exhaustive check of num_pairs literal pairs (Alg. 1 :89-108).
  * For a pair with k = |supp(a) U supp(b)| <= k_max the verdict is exact: EQUIVALENT, or
  * NOT_EQUIVALENT with cex_index_out = the minimum mismatching pattern in the pair's own support

@@ -29,7 +29,7 @@ EXPORTS = ["cec_default_opts", "cec_load_aig", "cec_sim_exhaustive", "cec_check_
            "cec_plan_window", "cec_plan_free", "cec_stream", "cec_get_stats", "cec_shard_range", "cec_pext64",
            "cec_free", "cec_last_error", "cec_abi_version", "cec_nccl_unique_id", "cec_sim_random",
            "cec_common_cuts", "cec_sim_patterns", "cec_reduce", "cec_sim_classes", "cec_local_pass",
-           "cec_peer_export", "cec_peer_import", "cec_peer_host_barrier"]
+           "cec_peer_export", "cec_peer_import", "cec_peer_host_barrier", "cec_reload_aig"]
 
 
 class CecOpts(ctypes.Structure):
@@ -71,6 +71,7 @@ def _load() -> ctypes.CDLL:
     sig = {
         "cec_default_opts": (None, [P]),
         "cec_load_aig": (ctypes.c_int, [P, P, P]),
+        "cec_reload_aig": (ctypes.c_int, [P, P, ctypes.c_uint32, ctypes.c_uint32]),
         "cec_sim_exhaustive": (ctypes.c_int, [P, u32, P, P, P, P, P]),
         "cec_check_local_cuts": (ctypes.c_int, [P, u32, P, P, P, P, P]),
         "cec_get_cex": (ctypes.c_int, [P, u32, P]),
@@ -150,6 +151,15 @@ def cec_load_aig(num_pis: int, fanins: np.ndarray, pos: np.ndarray, opts: Option
     st = lib.cec_load_aig(ctypes.byref(ctx), ctypes.byref(aig), ctypes.byref(opts))
     _check(st, None)
     return ctx
+
+
+def cec_reload_aig(ctx, num_pis: int, fanins: np.ndarray, pos: np.ndarray, k_max: int = 0, k_s: int = 0) -> None:
+    """Next miter version into the same context (include/cec.h cec_reload_aig; 0 = keep the limit)."""
+    fan = _u32(fanins)
+    po = _u32(pos)
+    aig = CecAig(num_pis, fan.size // 2, po.size, fan.ctypes.data if fan.size else None,
+                 po.ctypes.data if po.size else None)
+    _check(lib.cec_reload_aig(ctx, ctypes.byref(aig), int(k_max), int(k_s)), ctx)
 
 
 def cec_free(ctx) -> None:
@@ -417,6 +427,13 @@ class Context:
     @property
     def handle(self):
         return self._ctx
+
+    def reload(self, aig, k_max: int = 0, k_s: int = 0) -> "Context":
+        """Replace the AIG (the next miter version), keeping streams, workers, pools and JIT kernels."""
+        cec_reload_aig(self._ctx, aig.num_pis, aig.fanins, aig.pos, k_max, k_s)
+        self.num_pis = aig.num_pis
+        self.num_ands = int(aig.num_ands)
+        return self
 
     def sim_exhaustive(self, lit_a, lit_b):
         return cec_sim_exhaustive(self._ctx, lit_a, lit_b)

@@ -434,6 +434,50 @@ uint64_t cec_pext64(uint64_t value, uint64_t mask) {
     return r;
 }
 
+}  // extern "C"
+
+// a1: validate the AIGER arrays (fanin id < own id, PO literals in range) and
+// compute levels into temporaries; only a valid AIG replaces the context's arrays.
+static cec_status set_aig(cec_ctx *c, const cec_aig *aig, std::string &err) {
+    if (aig->num_ands && !aig->fanin_lits) return CEC_E_ARG;
+    const uint64_t N = 1ull + aig->num_pis + aig->num_ands;
+    if (N >= (1ull << 31)) return CEC_E_ARG;
+    const uint32_t I = aig->num_pis, A = aig->num_ands, O = aig->num_pos;
+    std::vector<uint32_t> f0, f1, level;
+    try {
+        f0.assign(N, 0);
+        f1.assign(N, 0);
+        level.assign(N, 0);
+    } catch (...) {
+        return CEC_E_NOMEM;
+    }
+    for (uint32_t i = 0; i < A; ++i) {
+        const uint32_t id = 1 + I + i;
+        const uint32_t l0 = aig->fanin_lits[2 * i], l1 = aig->fanin_lits[2 * i + 1];
+        if ((l0 >> 1) >= id || (l1 >> 1) >= id) {
+            err = "AIG: fanin id >= own id at AND " + std::to_string(id);
+            return CEC_E_AIG;
+        }
+        f0[id] = l0;
+        f1[id] = l1;
+        level[id] = 1 + std::max(level[l0 >> 1], level[l1 >> 1]);
+    }
+    for (uint32_t i = 0; i < O; ++i)
+        if (aig->po_lits && (aig->po_lits[i] >> 1) >= N) {
+            err = "AIG: PO literal out of range";
+            return CEC_E_AIG;
+        }
+    c->I = I;
+    c->A = A;
+    c->O = O;
+    c->f0.swap(f0);
+    c->f1.swap(f1);
+    c->level.swap(level);
+    return CEC_OK;
+}
+
+extern "C" {
+
 cec_status cec_load_aig(cec_ctx **out, const cec_aig *aig, const cec_opts *opts) {
     if (!out || !aig) return CEC_E_ARG;
     *out = nullptr;
@@ -445,33 +489,9 @@ cec_status cec_load_aig(cec_ctx **out, const cec_aig *aig, const cec_opts *opts)
     if (c->opts.k_s == 0) c->opts.k_s = c->opts.k_max;
     if (c->opts.world < 1) c->opts.world = 1;
     if (c->opts.rank < 0 || c->opts.rank >= c->opts.world) return CEC_E_ARG;
-    if (aig->num_ands && !aig->fanin_lits) return CEC_E_ARG;
-    const uint64_t N = 1ull + aig->num_pis + aig->num_ands;
-    if (N >= (1ull << 31)) return CEC_E_ARG;
-    c->I = aig->num_pis;
-    c->A = aig->num_ands;
-    c->O = aig->num_pos;
-    try {
-        c->f0.assign(N, 0);
-        c->f1.assign(N, 0);
-        c->level.assign(N, 0);
-    } catch (...) {
-        return CEC_E_NOMEM;
-    }
-    for (uint32_t i = 0; i < c->A; ++i) {  // a1: validation and levels
-        const uint32_t id = 1 + c->I + i;
-        const uint32_t l0 = aig->fanin_lits[2 * i], l1 = aig->fanin_lits[2 * i + 1];
-        if ((l0 >> 1) >= id || (l1 >> 1) >= id) {
-            c->err = "AIG: fanin id >= own id at AND " + std::to_string(id);
-            *out = nullptr;
-            return CEC_E_AIG;
-        }
-        c->f0[id] = l0;
-        c->f1[id] = l1;
-        c->level[id] = 1 + std::max(c->level[l0 >> 1], c->level[l1 >> 1]);
-    }
-    for (uint32_t i = 0; i < c->O; ++i)
-        if (aig->po_lits && (aig->po_lits[i] >> 1) >= N) return CEC_E_AIG;
+    std::string err;
+    const cec_status st = set_aig(c.get(), aig, err);  // a1: validation and levels
+    if (st != CEC_OK) return err.empty() ? st : fail(nullptr, st, "%s", err.c_str());
     if (c->opts.device >= 0) {
         c->host_only = false;
         const char *e = dev_init(c->opts.device, &c->own_stream, &c->num_sms);
@@ -511,6 +531,38 @@ void cec_free(cec_ctx *ctx) {
     ctx->devpool.reset();  // freed here unless a live plan still holds it
     if (ctx->own_stream) stream_destroy(ctx->own_stream);
     delete ctx;
+}
+
+cec_status cec_reload_aig(cec_ctx *c, const cec_aig *aig, uint32_t k_max, uint32_t k_s) {
+    if (!c || !aig) return CEC_E_ARG;
+    if (k_max > 63) return fail(c, CEC_E_ARG, "k_max > 63");
+    if (!c->host_only) {  // nothing of the old AIG may still be in flight
+        const char *e = stream_sync(c->stream);
+        if (e) return fail(c, CEC_E_CUDA, "CUDA: %s (reload)", e);
+    }
+    std::string err;
+    const cec_status st = set_aig(c, aig, err);
+    if (st != CEC_OK) return fail(c, st, "%s", err.empty() ? "invalid AIG arrays" : err.c_str());
+    // everything derived from the old AIG: its device copy + level CSR, the per-node support table,
+    // the last global check (cec_get_cex)
+    dev_free(c->d_f0);
+    dev_free(c->d_f1);
+    dev_free(c->d_level_ids);
+    dev_free(c->supp_table.lists);
+    c->d_f0 = c->d_f1 = c->d_level_ids = nullptr;
+    c->supp_table = NodeSupports{};
+    c->level_off.clear();
+    c->have_last = false;
+    c->last_verdict.clear();
+    c->last_cex.clear();
+    c->last_support.clear();
+    if (k_max) {
+        c->opts.k_max = k_max;
+        c->opts.k_s = k_s ? k_s : k_max;
+    } else if (k_s) {
+        c->opts.k_s = k_s;
+    }
+    return CEC_OK;
 }
 
 void *cec_stream(cec_ctx *ctx) { return ctx ? ctx->stream : nullptr; }

@@ -17,6 +17,8 @@
 // This is the host-minimal stand-in for the paper's GPU cut generator;
 // the checks themselves run on the GPU through cec_check_local_cuts.
 #include <algorithm>
+#include <chrono>
+#include <cstdio>
 #include <atomic>
 #include <functional>
 #include <memory>
@@ -151,33 +153,49 @@ struct CutJob {  // shared, read-only inputs of the per-node enumeration
 void node_cuts(const CutJob &J, uint32_t id, std::vector<std::vector<Cut>> &P) {
     const cec_ctx *c = J.c;
     const uint32_t a = c->f0[id] >> 1, b = c->f1[id] >> 1;
-    std::vector<Cut> ua(P[a]), vb(P[b]);
-    ua.push_back(trivial_cut(a));
-    vb.push_back(trivial_cut(b));
-    std::vector<Cut> E;
+    const std::vector<Cut> &Pa = P[a], &Pb = P[b];
+    const Cut ta = trivial_cut(a), tb = trivial_cut(b);
+    // candidates in the order P(n0) + {{n0}} x P(n1) + {{n1}}; ranked through index arrays (a Cut
+    // is ~150 bytes: sorting the objects themselves dominated the enumeration)
+    thread_local std::vector<Cut> E;
+    thread_local std::vector<uint32_t> ord, kept;
+    E.clear();
     Cut m;
-    for (const Cut &u : ua)
-        for (const Cut &v : vb)
+    for (size_t i = 0; i <= Pa.size(); ++i) {
+        const Cut &u = i < Pa.size() ? Pa[i] : ta;
+        for (size_t j = 0; j <= Pb.size(); ++j) {
+            const Cut &v = j < Pb.size() ? Pb[j] : tb;
+            // more distinct signature bits than k_l means more than k_l distinct leaves
+            if (__builtin_popcountll(u.sig | v.sig) > (int)J.k_l) continue;
             if (merge(u.leaf, u.n, v.leaf, v.n, (int)J.k_l, m)) {
                 if (m.n == 0 || (m.n == 1 && m.leaf[0] == id)) continue;
                 E.push_back(m);
             }
+        }
+    }
     // dedupe + drop dominated: process by size, keep a cut unless a kept cut is its subset
-    std::sort(E.begin(), E.end(), [](const Cut &x, const Cut &y) {
+    ord.resize(E.size());
+    for (uint32_t i = 0; i < ord.size(); ++i) ord[i] = i;
+    std::sort(ord.begin(), ord.end(), [](uint32_t xi, uint32_t yi) {
+        const Cut &x = E[xi], &y = E[yi];
         if (x.n != y.n) return x.n < y.n;
         return std::lexicographical_compare(x.leaf, x.leaf + x.n, y.leaf, y.leaf + y.n);
     });
-    std::vector<Cut> kept;
-    for (const Cut &x : E) {
+    kept.clear();
+    for (uint32_t xi : ord) {
+        const Cut &x = E[xi];
         bool dom = false;
-        for (const Cut &k : kept)
+        for (uint32_t ki : kept) {
+            const Cut &k = E[ki];
             if (same(k, x) || subset(k, x)) {
                 dom = true;
                 break;
             }
-        if (!dom) kept.push_back(x);
+        }
+        if (!dom) kept.push_back(xi);
     }
-    for (Cut &x : kept) {
+    for (uint32_t xi : kept) {
+        Cut &x = E[xi];
         x.sum_fanout = x.sum_level = 0;
         for (int t = 0; t < x.n; ++t) {
             x.sum_fanout += (*J.fanout)[x.leaf[t]];
@@ -188,7 +206,8 @@ void node_cuts(const CutJob &J, uint32_t id, std::vector<std::vector<Cut>> &P) {
     const uint32_t r = (*J.repr_of)[id];
     if (r != 0xFFFFFFFFu && !P[r].empty()) {
         static const unsigned __int128 L = lcm_upto(2 * KMAX);
-        for (Cut &x : kept) {
+        for (uint32_t xi : kept) {
+            Cut &x = E[xi];
             unsigned __int128 sv = 0;
             for (const Cut &y : P[r]) {
                 const int in = inter(x, y);
@@ -196,15 +215,18 @@ void node_cuts(const CutJob &J, uint32_t id, std::vector<std::vector<Cut>> &P) {
             }
             x.sim = sv;
         }
-        std::sort(kept.begin(), kept.end(), [&](const Cut &x, const Cut &y) {
+        std::sort(kept.begin(), kept.end(), [&](uint32_t xi, uint32_t yi) {
+            const Cut &x = E[xi], &y = E[yi];
             if (x.sim != y.sim) return x.sim > y.sim;
             return table1_less(x, y, J.pass);
         });
     } else {
-        std::sort(kept.begin(), kept.end(), [&](const Cut &x, const Cut &y) { return table1_less(x, y, J.pass); });
+        std::sort(kept.begin(), kept.end(), [&](uint32_t xi, uint32_t yi) { return table1_less(E[xi], E[yi], J.pass); });
     }
-    if (kept.size() > J.C) kept.resize(J.C);
-    P[id].swap(kept);
+    std::vector<Cut> out;
+    out.reserve(std::min<size_t>(kept.size(), J.C));
+    for (size_t t = 0; t < kept.size() && t < J.C; ++t) out.push_back(E[kept[t]]);
+    P[id].swap(out);
 }
 
 // common cuts u|v of a pair (no trivial cuts, <= k_l leaves), smallest first, at most max_cuts
@@ -214,7 +236,9 @@ void common_cuts_of(const std::vector<std::vector<Cut>> &P, uint32_t r, uint32_t
     Cut m;
     for (const Cut &u : P[r])
         for (const Cut &v : P[mbr])
-            if (merge(u.leaf, u.n, v.leaf, v.n, (int)k_l, m) && m.n > 0) common.push_back(m);
+            if (__builtin_popcountll(u.sig | v.sig) <= (int)k_l && merge(u.leaf, u.n, v.leaf, v.n, (int)k_l, m) &&
+                m.n > 0)
+                common.push_back(m);
     std::sort(common.begin(), common.end(), [](const Cut &x, const Cut &y) {
         if (x.n != y.n) return x.n < y.n;
         return std::lexicographical_compare(x.leaf, x.leaf + x.n, y.leaf, y.leaf + y.n);
@@ -432,17 +456,51 @@ extern "C" cec_status cec_local_pass(cec_ctx *c, uint32_t npairs, const uint32_t
         return launch(inflight);
     };
     std::vector<Cut> common;
+    std::vector<std::vector<Cut>> cmn;  // per-pair common cuts of a level computed in parallel
+    uint32_t par_min = 2;               // CEC_CUT_PAR_MIN: smallest level run on the pool
+    if (const char *e = getenv("CEC_CUT_PAR_MIN")) par_min = std::max(1, atoi(e));
+    // CEC_TIMING_LOCAL=1: where a pass spends its host time (stderr)
+    static const bool lt = getenv("CEC_TIMING_LOCAL") != nullptr;
+    using clk = std::chrono::steady_clock;
+    double t_enum = 0, t_common = 0, t_flush = 0;
+    auto t_begin = clk::now(), tq = t_begin;
+    auto acc = [&](double &a) {
+        if (!lt) return;
+        const auto t = clk::now();
+        a += std::chrono::duration<double, std::milli>(t - tq).count();
+        tq = t;
+    };
+    uint32_t n_par = 0, n_flush = 0, nodes_par = 0, nodes_ser = 0;
+    double t_ser = 0;
     for (size_t e = 1; e < lists.size(); ++e) {
         const std::vector<uint32_t> &L = lists[e];
-        if (L.size() < 8) {  // small levels: no hand-off
+        if (lt) tq = clk::now();
+        // a node's enumeration (~10-25 us at k_l = C = 16) outweighs a pool hand-off, so even
+        // levels of 2 nodes run in parallel (C4's carry chains: 109 of 133 levels have < 8 nodes)
+        if (L.size() < par_min) {
             for (uint32_t id : L) node_cuts(J, id, P);
+            nodes_ser += (uint32_t)L.size();
+            acc(t_ser);
         } else {
-            pool.run((uint32_t)L.size(), [&](uint32_t i, unsigned) { node_cuts(J, L[i], P); });
+            ++n_par;
+            nodes_par += (uint32_t)L.size();
+            pool.run((uint32_t)L.size(), [&](uint32_t i, unsigned) { node_cuts(J, L[i], P); }, true);
+            acc(t_enum);
         }
-        for (uint32_t q : pairs_at[e]) {  // Alg. 2 l.11-12: common cuts of the new pairs
-            common_cuts_of(P, repr[q], member[q], k_l, max_cuts, common);
+        // Alg. 2 l.11-12: common cuts of the new pairs (in parallel, inserted in pair order)
+        const std::vector<uint32_t> &QE = pairs_at[e];
+        if (QE.size() >= par_min) {
+            if (cmn.size() < QE.size()) cmn.resize(QE.size());
+            pool.run((uint32_t)QE.size(), [&](uint32_t i, unsigned) {
+                common_cuts_of(P, repr[QE[i]], member[QE[i]], k_l, max_cuts, cmn[i]);
+            }, true);
+        }
+        for (size_t qi = 0; qi < QE.size(); ++qi) {
+            const uint32_t q = QE[qi];
+            if (QE.size() < par_min) common_cuts_of(P, repr[q], member[q], k_l, max_cuts, common);
+            const std::vector<Cut> &cc = QE.size() < par_min ? common : cmn[qi];
             const uint32_t la = 2u * repr[q], lb = 2u * member[q] ^ (phase[q] & 1u);
-            for (const Cut &x : common) {
+            for (const Cut &x : cc) {
                 buf.pair.push_back(q);
                 buf.la.push_back(la);
                 buf.lb.push_back(lb);
@@ -454,14 +512,24 @@ extern "C" cec_status cec_local_pass(cec_ctx *c, uint32_t npairs, const uint32_t
                 ++nchecks;
             }
         }
+        acc(t_common);
         if (buf.pair.size() >= std::max<uint32_t>(1, buffer_checks)) {  // Alg. 2 l.13-14: flush
+            ++n_flush;
             cec_status st = flush();
             if (st != CEC_OK) return st;
+            acc(t_flush);
         }
     }
+    if (lt) tq = clk::now();
     cec_status st = flush();  // Alg. 2 l.18: the remainder
     if (st == CEC_OK) st = finish_inflight();
     if (st != CEC_OK) return st;
+    acc(t_flush);
+    if (lt)
+        fprintf(stderr, "[cec] local pass %d: %zu levels (%u parallel, %u nodes; serial %u nodes), %u pairs, %u checks, "
+                        "%u+1 flushes: enum par %.2f ser %.2f  common %.2f  flush %.2f  total %.2f ms\n", pass_id,
+                lists.size(), n_par, nodes_par, nodes_ser, npairs, nchecks, n_flush, t_enum, t_ser, t_common, t_flush,
+                std::chrono::duration<double, std::milli>(clk::now() - t_begin).count());
     *num_checks_out = nchecks;
     // optional check log (caller capacities: npairs*max_cuts checks, npairs*max_cuts*k_l leaves)
     if (check_pair) std::memcpy(check_pair, log_pair.data(), 4 * log_pair.size());

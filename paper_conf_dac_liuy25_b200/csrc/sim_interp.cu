@@ -17,6 +17,7 @@
 //    lowest mismatching lane (= lowest word), __ffs the lowest bit; a window whose pairs are all
 //    refuted publishes a bound and later slices above it are skipped (bounded early exit, Q9).
 #include <cuda_runtime.h>
+#include <chrono>
 
 #include <cstdio>
 #include <cstdlib>
@@ -237,8 +238,18 @@ const char *launch_run(const DevPlan &d0, const std::vector<LaunchGroup> &groups
         for (auto &x : pev) cudaEventCreate(&x);
         cudaEventRecord(pev[0], main_st);
     }
+    // CEC_TIMING=2: host time of each launch (stderr)
+    static const bool lt = getenv("CEC_TIMING") && atoi(getenv("CEC_TIMING")) >= 2;
+    auto lnow = []() { return std::chrono::steady_clock::now(); };
+    auto lt0 = lnow();
     for (size_t g = 0; g < groups.size(); ++g) {
         const LaunchGroup &G = groups[g];
+        if (lt && g > 0) {
+            const auto t = lnow();
+            fprintf(stderr, "[cec]   launch group %zu (%s): %.3f ms host\n", g - 1, groups[g - 1].jit ? "jit" : "interp",
+                    std::chrono::duration<double, std::milli>(t - lt0).count());
+            lt0 = t;
+        }
         if (!pev.empty() && g > 0) cudaEventRecord(pev[g], main_st);
         if (G.nitems == 0) continue;
         // the biggest group stays on the caller's stream; the others round-robin on side streams

@@ -17,6 +17,7 @@ then hands the reduced miter to ABC, which is out of scope).
 from __future__ import annotations
 
 import dataclasses
+import gc
 import time
 from typing import Dict, List, Optional, Tuple
 
@@ -213,6 +214,34 @@ def check_miter(aig: Aig, lit_a, lit_b, params: Optional[CecParams] = None) -> C
         return np.array([capi.CEC_EQUIVALENT if a == b else capi.CEC_UNDECIDED for a, b in zip(m.lit_a, m.lit_b)],
                         dtype=np.int32)
 
+    # One device context serves every phase: each new miter version is loaded into it
+    # (cec_reload_aig), keeping streams, workers, device pools and JIT kernels.
+    # A second one (slot 1) holds the local-check limit when k_l > k_g.
+    dev: List[Optional[capi.Context]] = [None, None]
+
+    def dctx(m: Miter, k_max: int, slot: int = 0) -> capi.Context:
+        if dev[slot] is None:
+            dev[slot] = _ctx(m.aig, p, k_max)
+        else:
+            dev[slot].reload(m.aig, k_max=k_max)
+        return dev[slot]
+
+    # The flow allocates only acyclic records (tens of thousands of per-check entries), which
+    # reference counting frees; the cyclic collector's full passes over them cost 0.1-0.3 s spikes
+    # in random phases, so it is paused for the flow and restored afterwards.
+    gc_was_on = gc.isenabled()
+    gc.disable()
+    try:
+        return _flow(p, cur, log, checks, versions, P, po_v, po_status, dctx)
+    finally:
+        for c in dev:
+            if c is not None:
+                c.close()
+        if gc_was_on:
+            gc.enable()
+
+
+def _flow(p, cur, log, checks, versions, P, po_v, po_status, dctx) -> CecResult:
     # ---- P phase -------------------------------------------------------------
     t = time.perf_counter()
     hctx = capi.Context.from_aig(cur.aig, device=-1, k_max=63)
@@ -221,8 +250,9 @@ def check_miter(aig: Aig, lit_a, lit_b, params: Optional[CecParams] = None) -> C
     thr = p.k_P if (ks <= p.k_P).all() else p.k_p
     sel = np.nonzero(ks <= thr)[0]
     subst: Dict[int, int] = {}
+    ctx = None
     if sel.size:
-        ctx = _ctx(cur.aig, p, thr)
+        ctx = dctx(cur, thr)
         v, cex, k = ctx.sim_exhaustive(cur.lit_a[sel], cur.lit_b[sel])
         for i, q in enumerate(sel):
             if v[i] == capi.CEC_NOT_EQUIVALENT:
@@ -243,12 +273,11 @@ def check_miter(aig: Aig, lit_a, lit_b, params: Optional[CecParams] = None) -> C
                 hi, lo = (a, b) if (a >> 1) > (b >> 1) else (b, a)
                 # an identical node pair (a >> 1 == b >> 1) needs no merge (and merging a node
                 # into itself is not a reduction)
-                if (hi >> 1) > aig.num_pis and (hi >> 1) != (lo >> 1):
+                if (hi >> 1) > cur.aig.num_pis and (hi >> 1) != (lo >> 1):
                     subst[hi >> 1] = lo ^ (hi & 1)
-        ctx.close()
     log.append({"phase": "P", "threshold": thr, "simulated": int(sel.size), "s": time.perf_counter() - t})
     if subst:
-        cur, _ = cur.reduce(subst, p.device)
+        cur, _ = cur.reduce(subst, p.device, ctx=ctx)
 
     # ---- G and L phases -----------------------------------------------------------------------
     tried_global = set()
@@ -258,9 +287,9 @@ def check_miter(aig: Aig, lit_a, lit_b, params: Optional[CecParams] = None) -> C
         if (st == capi.CEC_EQUIVALENT).all():
             break
         t = time.perf_counter()
-        ctx = _ctx(cur.aig, p, p.k_g)
         # local checks need k_max >= k_l (cut leaves); one context serves both when k_l <= k_g
-        lctx = ctx if p.k_l <= p.k_g else _ctx(cur.aig, p, max(p.k_l, 1))
+        ctx = dctx(cur, p.k_g)
+        lctx = ctx if p.k_l <= p.k_g else dctx(cur, max(p.k_l, 1), slot=1)
         t_ctx = time.perf_counter() - t
         # equivalence classes on the GPU: random patterns plus the CEX patterns
         # of disproved pairs, which split their classes
@@ -364,11 +393,6 @@ def check_miter(aig: Aig, lit_a, lit_b, params: Optional[CecParams] = None) -> C
             t1 = time.perf_counter()
             nxt, image = cur.reduce(subst, p.device, ctx=ctx)
             entry["s_parts"]["reduce"] = round(time.perf_counter() - t1, 4)
-        t1 = time.perf_counter()
-        ctx.close()
-        if lctx is not ctx:
-            lctx.close()
-        entry["s_parts"]["close"] = round(time.perf_counter() - t1, 4)
         entry["s"] = time.perf_counter() - t
         if not subst:
             break  # no progress: undecided remainder
@@ -390,7 +414,7 @@ def check_miter(aig: Aig, lit_a, lit_b, params: Optional[CecParams] = None) -> C
                hctx.pair_k(int(cur.lit_a[q]), int(cur.lit_b[q])) <= p.k_P]
         hctx.close()
         if und:
-            ctx = _ctx(cur.aig, p, p.k_P)
+            ctx = dctx(cur, p.k_P)
             v, _, _ = ctx.sim_exhaustive(cur.lit_a[und], cur.lit_b[und])
             for i, q in enumerate(und):
                 if v[i] != capi.CEC_UNDECIDED:
@@ -398,7 +422,6 @@ def check_miter(aig: Aig, lit_a, lit_b, params: Optional[CecParams] = None) -> C
             neq = [i for i, q in enumerate(und) if v[i] == capi.CEC_NOT_EQUIVALENT]
             if neq:
                 cex_vec, cex_pair = ctx.get_cex(neq[0]), und[neq[0]]
-            ctx.close()
         log.append({"phase": "final-P", "threshold": p.k_P, "simulated": len(und), "s": time.perf_counter() - t})
     if (po_v == capi.CEC_NOT_EQUIVALENT).any():
         verdict = capi.CEC_NOT_EQUIVALENT

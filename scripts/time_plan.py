@@ -5,7 +5,7 @@ import sys
 import time
 
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
-os.environ["CEC_TIMING"] = "1"
+os.environ.setdefault("CEC_TIMING", "1")
 
 import numpy as np  # noqa: E402
 import torch  # noqa: E402

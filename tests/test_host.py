@@ -301,3 +301,25 @@ def test_free_warp_partition_host_plans(world):
             capi.cec_plan_free(plan)
             ctx.close()
         assert sum(Ws) == W_all
+
+
+def test_reload_aig_replaces_the_miter_and_rejects_bad_arrays():
+    """cec_reload_aig (include/cec.h): the next miter version in the same context gives exactly what
+    a fresh context of that AIG gives; a malformed AIG is rejected and leaves the context unchanged."""
+    a, b = c1_add8(), c2_mul12()
+    ctx = capi.Context.from_aig(a.aig, device=-1)
+    sa = [ctx.pair_k(int(x), int(y)) for x, y in zip(a.lit_a, a.lit_b)]
+    ctx.reload(b.aig, k_max=24)
+    fresh = capi.Context.from_aig(b.aig, device=-1)
+    for x, y in zip(b.lit_a, b.lit_b):
+        assert capi.cec_pair_support(ctx.handle, int(x), int(y)) == capi.cec_pair_support(fresh.handle, int(x), int(y))
+    assert ctx.opts is not None and ctx.num_ands == b.aig.num_ands
+    bad = np.array(b.aig.fanins, dtype=np.uint32).copy()
+    bad[0, 0] = 2 * (1 + b.aig.num_pis + 5)  # fanin id above its own id
+    with pytest.raises(capi.CecError) as e:
+        capi.cec_reload_aig(ctx.handle, b.aig.num_pis, bad, b.aig.pos)
+    assert e.value.status == capi.CEC_E_AIG
+    for x, y in zip(b.lit_a[:4], b.lit_b[:4]):  # unchanged: still the valid C2 AIG
+        assert capi.cec_pair_support(ctx.handle, int(x), int(y)) == capi.cec_pair_support(fresh.handle, int(x), int(y))
+    ctx.reload(a.aig)
+    assert [ctx.pair_k(int(x), int(y)) for x, y in zip(a.lit_a, a.lit_b)] == sa
