@@ -184,6 +184,27 @@ struct cec_ctx {
     bool is_and(uint32_t id) const { return id > I; }
 };
 
+// std::allocator that default-initialises (no zero fill on resize): the interpreter programs of a
+// plan (~9 MB for C3) are resized and then fully overwritten by a parallel copy.
+template <class T>
+struct DefaultInitAlloc : std::allocator<T> {
+    template <class U>
+    struct rebind {
+        using other = DefaultInitAlloc<U>;
+    };
+    DefaultInitAlloc() = default;
+    template <class U>
+    DefaultInitAlloc(const DefaultInitAlloc<U> &) noexcept {}
+    template <class U>
+    void construct(U *p) noexcept {
+        ::new (static_cast<void *>(p)) U;
+    }
+    template <class U, class... A>
+    void construct(U *p, A &&...a) {
+        ::new (static_cast<void *>(p)) U(std::forward<A>(a)...);
+    }
+};
+
 struct WinHost {
     std::vector<uint32_t> inputs;  // node ids, increasing
     std::vector<uint32_t> cmps;    // compare indices of this window
@@ -211,7 +232,7 @@ struct cec_plan {
     std::vector<uint32_t> win_nodes;          // AND-node count per window
     std::vector<std::vector<uint32_t>> win_cmps;
     std::vector<DevWin> dwin;
-    std::vector<uint4> prog;
+    std::vector<uint4, DefaultInitAlloc<uint4>> prog;  // every slot written by finish_plan
     std::vector<Item> items;
     std::vector<JItem> jitems;
     std::vector<uint32_t> joff;  // free-warp groups' per-warp item offsets (relative to the group)

@@ -735,7 +735,18 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         // the id order (the netlist's own construction order) is often the better one: keep the
         // order with the smaller live set (counted without building the schedule)
         std::string why;
-        {
+        // An interpreter window whose depth-first order already fits the smallest slot bucket (32
+        // slots: the launch configuration cannot get better) skips the id-order evaluation.
+        const uint32_t kw = (uint32_t)W.inputs.size();
+        const uint64_t nw_est = (uint64_t)nodes.size() * tt_words_of(kw);
+        const bool interp_bound =
+            c->opts.engine == CEC_ENGINE_INTERP ||
+            (c->opts.engine == CEC_ENGINE_AUTO &&
+             (kw < 10 || nw_est < (kw <= 16 ? jit_min_node_words << 3 : jit_min_node_words)));
+        const uint32_t l_dfs0 = interp_bound ? live_peak(c, X, W.inputs, nodes, cmps2, wc) : UINT32_MAX;
+        if (interp_bound && l_dfs0 <= 32) {
+            R.sc.nslots = l_dfs0;
+        } else {
             // ascending ids: a flag scan over the window's id range (ids of a window are dense
             // in practice: one copy / one block), else a sort
             std::vector<uint32_t> by_id;
@@ -759,7 +770,7 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
                 }
             }
             const uint32_t l_id = live_peak(c, X, W.inputs, by_id, cmps2, wc);
-            const uint32_t l_dfs = live_peak(c, X, W.inputs, nodes, cmps2, wc);
+            const uint32_t l_dfs = l_dfs0 != UINT32_MAX ? l_dfs0 : live_peak(c, X, W.inputs, nodes, cmps2, wc);
             if (l_id < l_dfs) nodes.swap(by_id);
             R.sc.nslots = std::min(l_id, l_dfs);
         }
@@ -927,6 +938,7 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         words_rank_of.push_back(we > wb ? (we - wb) : 0);
         cost_of.push_back((uint64_t)(sc.ops.size() + 1) * (se - sb));
     }
+    tm.lap("layout: serial window loop");
     {  // interpreter programs copied into their slots of one array in parallel
         P->prog.resize(prog_total);
         auto copy = [&](uint32_t w, unsigned) {

@@ -39,6 +39,8 @@ def test_compute_sanitizer(tool):
         pytest.skip("compute-sanitizer not found")
     r = subprocess.run([cs, "--tool", tool, "--error-exitcode", "9", sys.executable, "-c", SCRIPT],
                        capture_output=True, text=True, timeout=1200)
+    if "closed on this pool" in r.stdout + r.stderr:  # the GPU pool's operators disabled the tool
+        pytest.skip("compute-sanitizer is disabled on this GPU pool: " + (r.stdout + r.stderr).strip()[:200])
     assert "SANITIZER-RUN-OK" in r.stdout, r.stdout[-2000:] + r.stderr[-2000:]
     assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-2000:]
     out = r.stdout + r.stderr
