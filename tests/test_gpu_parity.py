@@ -563,3 +563,27 @@ def test_local_checks_jit_engine_vs_oracle(seed):
     want = Oracle.from_aig(m.aig).check_local(la, lb, off, lv)
     assert list(map(int, got)) == list(map(int, want))
     ctx.close()
+
+
+def test_reload_aig_matches_fresh_context_and_oracle():
+    """cec_reload_aig (include/cec.h): a device context reloaded with the next miter gives exactly
+    the oracle's results for it (and a fresh context's), with no state of the previous AIG left:
+    its per-node support table, device AIG copy and last CEX are dropped."""
+    a = circuits.c2_mul12_bug(seed=1, n=8)
+    b = c5_big(copies=6, n_random=4, n_bugs=2, rand_pis=14, rand_ands=800, mul_n=7)
+    ctx = gpu_ctx(a.aig)
+    va, ca, ka = ctx.sim_exhaustive(a.lit_a, a.lit_b)
+    assert (va == capi.CEC_NOT_EQUIVALENT).any()
+    ctx.reload(b.aig, k_max=32)
+    with pytest.raises(capi.CecError) as e:  # the last check belonged to the old AIG
+        ctx.get_cex(int(np.nonzero(va == capi.CEC_NOT_EQUIVALENT)[0][0]))
+    assert e.value.status == capi.CEC_E_NOCEX
+    got = ctx.sim_exhaustive(b.lit_a, b.lit_b)
+    orc = Oracle.from_aig(b.aig)
+    ov, oc, ok, _ = orc.check_pairs(b.lit_a, b.lit_b, k_max=32)
+    assert_same(*got, ov, oc, ok, "reloaded")
+    for x, y in zip(got, gpu_ctx(b.aig).sim_exhaustive(b.lit_a, b.lit_b)):
+        assert np.array_equal(x, y)
+    ctx.reload(a.aig)  # and back: the first AIG's results again
+    for x, y in zip(ctx.sim_exhaustive(a.lit_a, a.lit_b), (va, ca, ka)):
+        assert np.array_equal(x, y)
