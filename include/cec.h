@@ -140,7 +140,7 @@ cec_status cec_load_aig(cec_ctx **ctx, const cec_aig *aig, const cec_opts *opts)
  * phase). Validation as in cec_load_aig; a rejected AIG (CEC_E_AIG / CEC_E_ARG) leaves the context
  * unchanged. k_max / k_s: the new limits (0 = keep; k_s = 0 with k_max > 0 means k_s = k_max).
  * Blocking (waits for the context's stream). Drops what the old AIG produced: the device copy of
- * the AIG, the per-node support table, the last global check (cec_get_cex -> CEC_E_NOCEX).
+ * the AIG, the per-node support table, the last global check (cec_get_cex -> CEC_E_STATE).
  * Collective when world > 1 in the sense that every rank must reload the same AIG. */
 cec_status cec_reload_aig(cec_ctx *ctx, const cec_aig *aig, uint32_t k_max, uint32_t k_s);
 

@@ -577,7 +577,7 @@ def test_reload_aig_matches_fresh_context_and_oracle():
     ctx.reload(b.aig, k_max=32)
     with pytest.raises(capi.CecError) as e:  # the last check belonged to the old AIG
         ctx.get_cex(int(np.nonzero(va == capi.CEC_NOT_EQUIVALENT)[0][0]))
-    assert e.value.status == capi.CEC_E_NOCEX
+    assert e.value.status == capi.CEC_E_STATE
     got = ctx.sim_exhaustive(b.lit_a, b.lit_b)
     orc = Oracle.from_aig(b.aig)
     ov, oc, ok, _ = orc.check_pairs(b.lit_a, b.lit_b, k_max=32)
