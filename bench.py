@@ -394,6 +394,19 @@ def main():
             ends[i].record(stream)
         torch.cuda.synchronize()
         wall = time.perf_counter() - t0
+        # the window kernels' own device time: the same K steps again with CUDA events around the
+        # window kernels (include/cec.h cec_plan_sweep_timing / _ms; off in the steps above, where
+        # the two event nodes would add ~7 us to a small config's captured run)
+        sweep_ms = []
+        if args.engine != capi.CEC_ENGINE_SIMT:
+            capi.cec_plan_sweep_timing(plan, True)
+            capi.cec_plan_run(ctx.handle, plan)  # recapture with the event nodes (untimed)
+            for i in range(args.steps):
+                flush.zero_()
+                capi.cec_plan_run(ctx.handle, plan)
+                torch.cuda.synchronize()
+                sweep_ms.append(capi.cec_plan_sweep_ms(plan))
+            capi.cec_plan_sweep_timing(plan, False)
     if world > 1:
         dist.barrier()
     step_ms = [s.elapsed_time(e) for s, e in zip(starts, ends)]
@@ -429,8 +442,13 @@ def main():
     props = torch.cuda.get_device_properties(local)
     peak = props.multi_processor_count * LOP3_PER_CLK_PER_SM * sm_clock * 1e6 / 1e12  # TLOP3/s
     # algorithmic LOP3s of the path: one 3-input LUT per mapped node group per u32 word (JIT), one
-    # per AND (interpreter) — the AND-node count itself is the metric W
-    achieved = stats["lop3_words"] / (ms / 1e3) / 1e12
+    # per AND (interpreter) — the AND-node count itself is the metric W — over the window kernels'
+    # own device time per launch (CUDA events around them on the launch stream, every timed step;
+    # the step adds the reset kernel and the graph launch); step_frac is the same over the step
+    kern_ms = statistics.mean(sweep_ms) if sweep_ms else ms
+    if world > 1:
+        kern_ms = allreduce(kern_ms, dist.ReduceOp.MAX)
+    achieved = stats["lop3_words"] / (kern_ms / 1e3) / 1e12
     simt = args.engine == capi.CEC_ENGINE_SIMT
     traffic = None
     prof = os.path.join(ROOT, "profiles", "ncu_summary.json")
@@ -500,16 +518,19 @@ def main():
                          if simt else
                          {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "TLOP3/s",
                          "frac": achieved / peak, "traffic": traffic,
+                         "kernel_ms": kern_ms, "kernel_timing": "CUDA events around the window kernels "
+                         "(cec_plan_sweep_ms), mean over the timed steps",
+                         "step_frac": stats["lop3_words"] / (ms / 1e3) / 1e12 / peak,
                          "peak_basis": f"{props.multi_processor_count} SMs x {LOP3_PER_CLK_PER_SM} LOP3/clk x {sm_clock:.0f} MHz (guide unit counts, SM clock; microbenchmark scripts/peaks.cu measured 64.00 LOP3/clk/SM = 18.53 TLOP3/s at 1957 MHz, profiles/round1_peaks.json)",
                          "lop3_per_word_per_and": stats["lop3_words"] / max(1.0, W_rank / 32.0),
                          "imad_per_word_per_and": stats.get("imad_words", 0) / max(1.0, W_rank / 32.0),
-                         "fma_pipe_timad_s": stats.get("imad_words", 0) / (ms / 1e3) / 1e12,
+                         "fma_pipe_timad_s": stats.get("imad_words", 0) / (kern_ms / 1e3) / 1e12,
                          "cells": "3-input LUTs = lop3.b32 on the ALU pipe (the bound); AND nodes with a "
                                   "word-uniform operand = mad.lo.u32 on the FMA pipe (DESIGN.md §4.1)",
-                         "and_evals_tops": (W_rank / 32.0) / (ms / 1e3) / 1e12,
+                         "and_evals_tops": (W_rank / 32.0) / (kern_ms / 1e3) / 1e12,
                          # the SURVEY §8(d) unit (one 2-input op per AND per u32 word) against the same
                          # peak: > 1 because a mapped LOP3/IMAD cell evaluates ~1.9 ANDs
-                         "and_evals_per_lop3_peak": (W_rank / 32.0) / (ms / 1e3) / 1e12 / peak}),
+                         "and_evals_per_lop3_peak": (W_rank / 32.0) / (kern_ms / 1e3) / 1e12 / peak}),
             "step_ms": step_ms, "wall_s": wall,
         }
         if cpu:

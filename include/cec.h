@@ -266,6 +266,15 @@ cec_status cec_plan_results(cec_ctx *ctx, cec_plan *plan, int32_t *verdict_out, 
 /* Plan shape: windows after merging, W for one full run, largest k and live set. */
 cec_status cec_plan_info(const cec_plan *plan, uint32_t *num_windows, uint64_t *node_patterns, uint32_t *max_k,
                          uint32_t *max_slots);
+/* Kernel timing of a plan (the denominator of the kernels' roofline fraction in bench.py). With
+ * cec_plan_sweep_timing(plan, 1), every run records two CUDA events on the context's stream, right
+ * before the first window kernel and right after the side streams joined: the sweep itself,
+ * without the reset kernel, peer barriers / gather or all-reduce and the graph launch latency. Off
+ * by default: the two event nodes add a few microseconds to a captured run (C2: ~7 us of 38).
+ * cec_plan_sweep_ms = that interval for the last completed run (the caller synchronises first).
+ * CEC_E_STATE: the last run was not timed / has not completed, or a plan of the SIMT engine. */
+cec_status cec_plan_sweep_timing(cec_plan *plan, int on);
+cec_status cec_plan_sweep_ms(const cec_plan *plan, float *ms);
 /* Per-window description, for tests of the host logic: window w's inputs (node ids, increasing),
  * its AND-node count and its pair indices. Arrays may be NULL to query sizes only. */
 cec_status cec_plan_window(const cec_plan *plan, uint32_t w, uint32_t *inputs, uint32_t *k, uint32_t *num_nodes,

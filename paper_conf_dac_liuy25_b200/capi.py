@@ -29,7 +29,8 @@ EXPORTS = ["cec_default_opts", "cec_load_aig", "cec_sim_exhaustive", "cec_check_
            "cec_plan_window", "cec_plan_free", "cec_stream", "cec_get_stats", "cec_shard_range", "cec_pext64",
            "cec_free", "cec_last_error", "cec_abi_version", "cec_nccl_unique_id", "cec_sim_random",
            "cec_common_cuts", "cec_sim_patterns", "cec_reduce", "cec_sim_classes", "cec_local_pass",
-           "cec_peer_export", "cec_peer_import", "cec_peer_host_barrier", "cec_reload_aig"]
+           "cec_peer_export", "cec_peer_import", "cec_peer_host_barrier", "cec_reload_aig", "cec_plan_sweep_ms",
+           "cec_plan_sweep_timing"]
 
 
 class CecOpts(ctypes.Structure):
@@ -72,6 +73,8 @@ def _load() -> ctypes.CDLL:
         "cec_default_opts": (None, [P]),
         "cec_load_aig": (ctypes.c_int, [P, P, P]),
         "cec_reload_aig": (ctypes.c_int, [P, P, ctypes.c_uint32, ctypes.c_uint32]),
+        "cec_plan_sweep_ms": (ctypes.c_int, [P, P]),
+        "cec_plan_sweep_timing": (ctypes.c_int, [P, ctypes.c_int]),
         "cec_sim_exhaustive": (ctypes.c_int, [P, u32, P, P, P, P, P]),
         "cec_check_local_cuts": (ctypes.c_int, [P, u32, P, P, P, P, P]),
         "cec_get_cex": (ctypes.c_int, [P, u32, P]),
@@ -328,6 +331,18 @@ def cec_plan_results(ctx, plan, num_pairs: int):
     k = np.zeros(max(num_pairs, 1), np.uint32)
     _check(lib.cec_plan_results(ctx, plan, _p(v), _p(cex), _p(k)), ctx)
     return v[:num_pairs], cex[:num_pairs], k[:num_pairs]
+
+
+def cec_plan_sweep_timing(plan, on: bool) -> None:
+    """Record (or stop recording) the window-kernel events in the plan's runs (include/cec.h)."""
+    _check(lib.cec_plan_sweep_timing(plan, 1 if on else 0), None)
+
+
+def cec_plan_sweep_ms(plan) -> float:
+    """Window-kernel device time of the plan's last completed run (include/cec.h); sync first."""
+    ms = ctypes.c_float()
+    _check(lib.cec_plan_sweep_ms(plan, ctypes.byref(ms)), None)
+    return float(ms.value)
 
 
 def cec_plan_info(plan) -> dict:

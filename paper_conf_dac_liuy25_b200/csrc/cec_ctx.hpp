@@ -252,6 +252,9 @@ struct cec_plan {
     void *arena = nullptr;          // one device block holding every DevPlan buffer
     size_t arena_cap = 0;
     void *ev0 = nullptr, *ev1 = nullptr;
+    void *sev[2] = {nullptr, nullptr};  // around the window kernels only (launch_run sweep_ev)
+    bool sweep_timing = false;           // record sev in runs (cec_plan_sweep_timing; off: no cost)
+    bool sweep_timed_last = false;       // the last run recorded sev
     bool ran = false;
     bool no_join = false;  // pipelined call, not its last chunk: skip the side-stream join (launch_run)
     uint32_t runs = 0;                     // completed cec_plan_run calls

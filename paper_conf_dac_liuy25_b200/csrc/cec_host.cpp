@@ -1360,6 +1360,8 @@ cec_status upload(cec_ctx *c, cec_plan *P) {
     }
     CUDA_TRY(c, event_create(&P->ev0));
     CUDA_TRY(c, event_create(&P->ev1));
+    CUDA_TRY(c, event_create(&P->sev[0]));
+    CUDA_TRY(c, event_create(&P->sev[1]));
     c->stats.h2d_bytes = sizeof(DevWin) * P->dwin.size() + sizeof(uint4) * P->prog.size() +
                          sizeof(Item) * P->items.size() + sizeof(JItem) * P->jitems.size() +
                          sizeof(uint32_t) * P->joff.size();
@@ -1383,7 +1385,9 @@ void free_dev(cec_plan *P) {
     P->simt.d_ttw = nullptr;
     event_destroy(P->ev0);
     event_destroy(P->ev1);
-    P->ev0 = P->ev1 = nullptr;
+    event_destroy(P->sev[0]);
+    event_destroy(P->sev[1]);
+    P->ev0 = P->ev1 = P->sev[0] = P->sev[1] = nullptr;
     graph_destroy(P->graph);
     P->graph = P->graph_stream = nullptr;
 }
@@ -1658,7 +1662,8 @@ cec_status cec_plan_run(cec_ctx *c, cec_plan *P) {
     }
     if (use_graph && !P->graph) {
         e = graph_capture_run(P->d, P->groups, (uint32_t)P->dwin.size(), (uint32_t)P->cmps.size(), c->stream,
-                              c->num_sms, &P->graph_launches, &c->aux, &P->graph, peer ? &pr : nullptr);
+                              c->num_sms, &P->graph_launches, &c->aux, &P->graph, peer ? &pr : nullptr,
+                              P->sweep_timing ? P->sev : nullptr);
         P->graph_stream = c->stream;
         P->graph_peer_gen = c->peer.gen;
         if (e) return fail(c, CEC_E_CUDA, "CUDA: %s (graph capture)", e);
@@ -1671,9 +1676,10 @@ cec_status cec_plan_run(cec_ctx *c, cec_plan *P) {
         e = P->simt.E ? launch_simt(P->simt, P->d.first, (uint32_t)P->cmps.size(), c->stream, c->num_sms, &nl)
                       : launch_run(P->d, P->groups, (uint32_t)P->dwin.size(), (uint32_t)P->cmps.size(), c->stream,
                                    c->num_sms, &nl, &c->aux, peer ? &pr : nullptr,
-                                   P->no_join && !c->comm && !peer);
+                                   P->no_join && !c->comm && !peer, P->sweep_timing ? P->sev : nullptr);
     }
     if (e) return fail(c, CEC_E_CUDA, "CUDA: %s (kernel launch)", e);
+    P->sweep_timed_last = P->sweep_timing && !P->simt.E;
     if (c->comm && !peer && !P->cmps.empty()) {  // a10: one NCCL min all-reduce of first_idx
         ncclResult_t r = g_nccl.all_reduce(P->d.first, P->d.first, P->cmps.size(), ncclUint64, ncclMin, c->comm,
                                            (cudaStream_t)c->stream);
@@ -1759,6 +1765,23 @@ static void resolve_results(cec_ctx *c, cec_plan *P, const std::vector<unsigned 
 }
 
 extern "C" {
+
+cec_status cec_plan_sweep_timing(cec_plan *P, int on) {
+    if (!P) return CEC_E_ARG;
+    if (P->sweep_timing != (on != 0) && P->graph) {  // the captured run has (no) event nodes: recapture
+        graph_destroy(P->graph);
+        P->graph = nullptr;
+    }
+    P->sweep_timing = on != 0;
+    return CEC_OK;
+}
+
+cec_status cec_plan_sweep_ms(const cec_plan *P, float *ms) {
+    if (!P || !ms) return CEC_E_ARG;
+    if (!P->ran || !P->sweep_timed_last || P->simt.E || !P->sev[0] || !P->sev[1] || P->no_join) return CEC_E_STATE;
+    const char *e = event_elapsed(ms, P->sev[0], P->sev[1]);  // fails if the run has not completed
+    return e ? CEC_E_STATE : CEC_OK;
+}
 
 cec_status cec_plan_info(const cec_plan *P, uint32_t *nw, uint64_t *W, uint32_t *mk, uint32_t *ms) {
     if (!P) return CEC_E_ARG;

@@ -251,12 +251,16 @@ const char *peer_error(const PeerState &ps, void *stream, bool *timed_out);
 // the side streams at the end (the pipelined call's earlier chunks: the next chunk's kernels touch
 // only their own arrays, so they may start while this chunk's side-stream kernels finish; the last
 // chunk joins, and side streams run in order, so its join covers every chunk).
+// sweep_ev (optional, two events): recorded on the caller's stream right before the first window
+// kernel (after the reset) and right after the side streams joined, i.e. around the window kernels
+// only (not the reset, peer barriers, gather or all-reduce); inside a graph capture as external
+// event-record nodes, so every replay re-records them.
 const char *launch_run(const DevPlan &d, const std::vector<LaunchGroup> &groups, uint32_t nwin, uint32_t ncmp,
                        void *stream, int num_sms, uint32_t *launches, AuxStreams *aux, const PeerRun *pr = nullptr,
-                       bool no_join = false);
+                       bool no_join = false, void *const *sweep_ev = nullptr);
 const char *graph_capture_run(const DevPlan &d, const std::vector<LaunchGroup> &groups, uint32_t nwin, uint32_t ncmp,
                               void *stream, int num_sms, uint32_t *launches, AuxStreams *aux, void **exec_out,
-                              const PeerRun *pr = nullptr);
+                              const PeerRun *pr = nullptr, void *const *sweep_ev = nullptr);
 const char *graph_launch(void *exec, void *stream);
 void graph_destroy(void *exec);
 const char *dev_alloc(void **p, size_t bytes);

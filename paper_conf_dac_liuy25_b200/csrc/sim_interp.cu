@@ -198,9 +198,19 @@ void aux_destroy(AuxStreams &a) {
     a = AuxStreams{};
 }
 
+// event record that also works inside a stream capture (as an external event-record node)
+static const char *record_span_event(void *ev, cudaStream_t st) {
+    cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+    const char *e = ck(cudaStreamIsCapturing(st, &cs));
+    if (e) return e;
+    return ck(cs == cudaStreamCaptureStatusActive
+                  ? cudaEventRecordWithFlags((cudaEvent_t)ev, st, cudaEventRecordExternal)
+                  : cudaEventRecord((cudaEvent_t)ev, st));
+}
+
 const char *launch_run(const DevPlan &d0, const std::vector<LaunchGroup> &groups, uint32_t nwin, uint32_t ncmp,
                        void *stream, int num_sms, uint32_t *launches, AuxStreams *aux, const PeerRun *pr,
-                       bool no_join) {
+                       bool no_join, void *const *sweep_ev) {
     cudaStream_t main_st = (cudaStream_t)stream;
     cudaStream_t st = main_st;
     const char *e;
@@ -225,6 +235,8 @@ const char *launch_run(const DevPlan &d0, const std::vector<LaunchGroup> &groups
         ++nl;
     }
     const bool multi = aux && aux->ok && groups.size() > 1 && getenv("CEC_PROFILE_GROUPS") == nullptr;
+    const bool span = sweep_ev && sweep_ev[0] && sweep_ev[1] && !(multi && no_join);
+    if (span && (e = record_span_event(sweep_ev[0], main_st))) return e;
     if (multi) {
         if ((e = ck(cudaEventRecord((cudaEvent_t)aux->fork, main_st)))) return e;
         for (int i = 0; i < aux->n; ++i)
@@ -310,6 +322,7 @@ const char *launch_run(const DevPlan &d0, const std::vector<LaunchGroup> &groups
             if ((e = ck(cudaStreamWaitEvent(main_st, (cudaEvent_t)aux->join[i], 0)))) return e;
         }
     }
+    if (span && (e = record_span_event(sweep_ev[1], main_st))) return e;
     if (peer) {  // every rank's kernels done -> gather the minimum -> nobody resets before all gathered
         if ((e = peer_barrier_launch(*pr, main_st))) return e;
         if ((e = peer_gather_launch(*pr, ncmp, main_st))) return e;
@@ -325,12 +338,12 @@ const char *launch_run(const DevPlan &d0, const std::vector<LaunchGroup> &groups
 // instead of one host launch per group (C3: ~1.6k launches per run).
 const char *graph_capture_run(const DevPlan &d, const std::vector<LaunchGroup> &groups, uint32_t nwin, uint32_t ncmp,
                               void *stream, int num_sms, uint32_t *launches, AuxStreams *aux, void **exec_out,
-                              const PeerRun *pr) {
+                              const PeerRun *pr, void *const *sweep_ev) {
     cudaStream_t st = (cudaStream_t)stream;
     const char *e;
     *exec_out = nullptr;
     if ((e = ck(cudaStreamBeginCapture(st, cudaStreamCaptureModeRelaxed)))) return e;
-    const char *le = launch_run(d, groups, nwin, ncmp, stream, num_sms, launches, aux, pr);
+    const char *le = launch_run(d, groups, nwin, ncmp, stream, num_sms, launches, aux, pr, false, sweep_ev);
     cudaGraph_t g = nullptr;
     const char *ee = ck(cudaStreamEndCapture(st, &g));
     if (le || ee) {

@@ -587,3 +587,31 @@ def test_reload_aig_matches_fresh_context_and_oracle():
     ctx.reload(a.aig)  # and back: the first AIG's results again
     for x, y in zip(ctx.sim_exhaustive(a.lit_a, a.lit_b), (va, ca, ka)):
         assert np.array_equal(x, y)
+
+
+def test_plan_sweep_timing_events():
+    """cec_plan_sweep_timing / cec_plan_sweep_ms (include/cec.h): off by default (CEC_E_STATE), on:
+    the window kernels' event interval of the last run, positive and inside the run's own events,
+    also across a CUDA-graph replay; results are unchanged by the extra event nodes."""
+    m = c5_big(copies=6, n_random=4, n_bugs=2, rand_pis=14, rand_ands=800, mul_n=7)
+    ctx = gpu_ctx(m.aig)
+    plan = capi.cec_plan_exhaustive(ctx.handle, m.lit_a, m.lit_b)
+    capi.cec_plan_run(ctx.handle, plan)
+    ref = capi.cec_plan_results(ctx.handle, plan, m.num_pairs)
+    with pytest.raises(capi.CecError) as e:
+        capi.cec_plan_sweep_ms(plan)
+    assert e.value.status == capi.CEC_E_STATE
+    capi.cec_plan_sweep_timing(plan, True)
+    for _ in range(3):  # direct launch, capture, replay
+        capi.cec_plan_run(ctx.handle, plan)
+        got = capi.cec_plan_results(ctx.handle, plan, m.num_pairs)
+        for a, b in zip(ref, got):
+            assert np.array_equal(a, b)
+        sw = capi.cec_plan_sweep_ms(plan)
+        assert 0.0 < sw <= ctx.stats()["kernel_ms"] + 1e-3
+    capi.cec_plan_sweep_timing(plan, False)
+    capi.cec_plan_run(ctx.handle, plan)
+    capi.cec_plan_results(ctx.handle, plan, m.num_pairs)
+    with pytest.raises(capi.CecError):
+        capi.cec_plan_sweep_ms(plan)
+    capi.cec_plan_free(plan)
