@@ -1758,7 +1758,11 @@ static void resolve_results(cec_ctx *c, cec_plan *P, const std::vector<unsigned 
         if (!P->local) {
             c->last_verdict[p] = v;
             c->last_cex[p] = x;
-            if (v == CEC_NOT_EQUIVALENT) support_of(c, P->la[p], P->lb[p], c->last_support[p]);
+            // cec_get_cex maps bit j of the own index to the j-th support PI: a simulated pair's
+            // compare holds exactly that sorted support (no second TFI walk); a pair refuted
+            // without simulation (lit_a == lit_b ^ 1) has index 0, i.e. every PI 0
+            if (v == CEC_NOT_EQUIVALENT && P->pre_verdict[p] == DECIDED_BY_SIM)
+                c->last_support[p] = P->cmps[P->pair_cmp[p]].S;
         }
     }
     if (!P->local) c->have_last = true;
@@ -1990,6 +1994,7 @@ cec_status cec_sim_exhaustive(cec_ctx *c, uint32_t n, const uint32_t *la, const 
         }
     }
     const char *se = stream_sync(c->stream);
+    tm.lap("call: wait for the GPU");
     if (!se && peer_failed(c)) {
         for (auto &x : subs) free_dev(x.p.get());
         return fail(c, CEC_E_NCCL, "peer barrier timed out (a peer rank never arrived)");
@@ -2008,7 +2013,9 @@ cec_status cec_sim_exhaustive(cec_ctx *c, uint32_t n, const uint32_t *la, const 
         free_dev(S.p.get());
     }
     if (se) return fail(c, CEC_E_CUDA, "CUDA: %s", se);
+    tm.lap("call: gather + free chunks");
     resolve_results(c, P.get(), first, verdict, cex, k_out);
+    tm.lap("call: resolve results");
     const float host_ms = P->host_ms;
     c->stats.num_launches = agg.num_launches;
     c->stats.node_patterns = agg.node_patterns;
@@ -2025,7 +2032,7 @@ cec_status cec_sim_exhaustive(cec_ctx *c, uint32_t n, const uint32_t *la, const 
     c->stats.jit_ms = jit_ms;
     c->stats.kernel_ms = kms;
     c->stats.host_prep_ms = host_ms;
-    tm.lap("call: sync+results");
+    tm.lap("call: stats + return");
     return CEC_OK;
 }
 
