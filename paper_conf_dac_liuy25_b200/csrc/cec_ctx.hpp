@@ -165,6 +165,8 @@ struct cec_ctx {
     std::vector<std::vector<uint32_t>> last_support;
     // device copy of the AIG for random simulation (lazy)
     uint32_t *d_f0 = nullptr, *d_f1 = nullptr, *d_level_ids = nullptr;
+    uint64_t d_aig_cap = 0;     // entries allocated in each of d_f0 / d_f1 / d_level_ids
+    bool d_aig_valid = false;   // they hold THIS AIG (cec_reload_aig keeps the buffers, not the data)
     NodeSupports supp_table;  // a2 per-node support lists on the device (AIG-only, built once)
     std::vector<uint32_t> level_off;
     std::shared_ptr<DevPool> devpool;  // plan device blocks + pinned staging (device contexts)

@@ -545,11 +545,10 @@ cec_status cec_reload_aig(cec_ctx *c, const cec_aig *aig, uint32_t k_max, uint32
     if (st != CEC_OK) return fail(c, st, "%s", err.empty() ? "invalid AIG arrays" : err.c_str());
     // everything derived from the old AIG: its device copy + level CSR, the per-node support table,
     // the last global check (cec_get_cex)
-    dev_free(c->d_f0);
-    dev_free(c->d_f1);
-    dev_free(c->d_level_ids);
+    // the device AIG buffers are kept for the next upload (a reduced miter fits: cudaFree /
+    // cudaMalloc here cost up to 0.5 s spikes per phase on the B200 box); only their data is stale
+    c->d_aig_valid = false;
     dev_free(c->supp_table.lists);
-    c->d_f0 = c->d_f1 = c->d_level_ids = nullptr;
     c->supp_table = NodeSupports{};
     c->level_off.clear();
     c->have_last = false;
@@ -2042,7 +2041,7 @@ static cec_status sim_signatures(cec_ctx *c, uint32_t W, uint64_t seed, const ui
 cec_status cec_ensure_device_aig(cec_ctx *c) {
     if (c->host_only) return fail(c, CEC_E_CUDA, "host-only context");
     const uint32_t N = c->N();
-    if (!c->d_f0) {  // AIG and level CSR on the device (a1)
+    if (!c->d_aig_valid) {  // AIG and level CSR on the device (a1)
         uint32_t maxl = 0;
         for (uint32_t id = 0; id < N; ++id) maxl = std::max(maxl, c->level[id]);
         c->level_off.assign(maxl + 2, 0);
@@ -2050,13 +2049,22 @@ cec_status cec_ensure_device_aig(cec_ctx *c) {
         for (size_t l = 1; l < c->level_off.size(); ++l) c->level_off[l] += c->level_off[l - 1];
         std::vector<uint32_t> ids(std::max<uint32_t>(1, c->A)), fill(c->level_off.begin(), c->level_off.end());
         for (uint32_t id = 1 + c->I; id < N; ++id) ids[fill[c->level[id]]++] = id;
-        CUDA_TRY(c, dev_alloc((void **)&c->d_f0, sizeof(uint32_t) * N));
-        CUDA_TRY(c, dev_alloc((void **)&c->d_f1, sizeof(uint32_t) * N));
-        CUDA_TRY(c, dev_alloc((void **)&c->d_level_ids, sizeof(uint32_t) * ids.size()));
+        if (!c->d_f0 || c->d_aig_cap < N) {  // (re)allocate; ids.size() <= N
+            dev_free(c->d_f0);
+            dev_free(c->d_f1);
+            dev_free(c->d_level_ids);
+            c->d_f0 = c->d_f1 = c->d_level_ids = nullptr;
+            c->d_aig_cap = 0;
+            CUDA_TRY(c, dev_alloc((void **)&c->d_f0, sizeof(uint32_t) * N));
+            CUDA_TRY(c, dev_alloc((void **)&c->d_f1, sizeof(uint32_t) * N));
+            CUDA_TRY(c, dev_alloc((void **)&c->d_level_ids, sizeof(uint32_t) * N));
+            c->d_aig_cap = N;
+        }
         CUDA_TRY(c, h2d(c->d_f0, c->f0.data(), sizeof(uint32_t) * N, c->stream));
         CUDA_TRY(c, h2d(c->d_f1, c->f1.data(), sizeof(uint32_t) * N, c->stream));
         CUDA_TRY(c, h2d(c->d_level_ids, ids.data(), sizeof(uint32_t) * ids.size(), c->stream));
         CUDA_TRY(c, stream_sync(c->stream));
+        c->d_aig_valid = true;
     }
     return CEC_OK;
 }

@@ -149,16 +149,164 @@ struct CutJob {  // shared, read-only inputs of the per-node enumeration
     int pass;
 };
 
+// Fast path of node_cuts: the leaves of every candidate cut of n are drawn from the leaves of
+// P(n0) + {{n0}} and P(n1) + {{n1}}; when that dictionary has <= 128 node ids, a cut is a 128-bit
+// mask over it (dictionary sorted by id) and every operation of Eq. (1) and the ranking is exact
+// bit arithmetic: union = OR, |cut| = popcount, subset = (x & ~y) == 0, and for two cuts of EQUAL
+// size the lexicographic order of their sorted leaf lists is decided by the lowest node of their
+// symmetric difference (the list holding it is the smaller one: every smaller node is in both).
+// Same candidates, same order relations, same result as the list path below (pinned by
+// tests/test_driver_host.py against oracle/cuts.py); returns false when the dictionary is larger.
+typedef unsigned __int128 u128;
+inline int pop128(u128 x) { return __builtin_popcountll((uint64_t)x) + __builtin_popcountll((uint64_t)(x >> 64)); }
+inline int ctz128(u128 x) {
+    const uint64_t lo = (uint64_t)x;
+    return lo ? __builtin_ctzll(lo) : 64 + __builtin_ctzll((uint64_t)(x >> 64));
+}
+inline bool lex_less_masks(u128 x, u128 y) {  // equal popcounts; sorted leaf lists x < y
+    const u128 d = x ^ y;
+    return d != 0 && ((x >> ctz128(d)) & 1) != 0;
+}
+
+bool node_cuts_masks(const CutJob &J, uint32_t id, std::vector<std::vector<Cut>> &P) {
+    const cec_ctx *c = J.c;
+    const uint32_t a = c->f0[id] >> 1, b = c->f1[id] >> 1;
+    const std::vector<Cut> &Pa = P[a], &Pb = P[b];
+    const Cut ta = trivial_cut(a), tb = trivial_cut(b);
+    // thread_local scratch bound to plain references once: every access of a thread_local in a
+    // shared library is a __tls_get_addr call, which dominated the sort comparators
+    thread_local std::vector<uint32_t> tD;
+    thread_local std::vector<u128> tma, tmb, tE;
+    thread_local std::vector<uint8_t> tEn;
+    thread_local std::vector<uint32_t> tord, tkept, trk;
+    thread_local std::vector<uint64_t> tdfan, tdlev;
+    thread_local std::vector<Cut> tK;
+    std::vector<uint32_t> &D = tD, &ord = tord, &kept = tkept, &rk = trk;
+    std::vector<u128> &ma = tma, &mb = tmb, &E = tE;
+    std::vector<uint8_t> &En = tEn;
+    std::vector<uint64_t> &dfan = tdfan, &dlev = tdlev;
+    std::vector<Cut> &K = tK;
+    D.clear();
+    for (const std::vector<Cut> *L : {&Pa, &Pb})
+        for (const Cut &u : *L) D.insert(D.end(), u.leaf, u.leaf + u.n);
+    D.insert(D.end(), ta.leaf, ta.leaf + ta.n);
+    D.insert(D.end(), tb.leaf, tb.leaf + tb.n);
+    std::sort(D.begin(), D.end());
+    D.erase(std::unique(D.begin(), D.end()), D.end());
+    if (D.size() > 128) return false;
+    auto mask_of = [&](const Cut &u) {
+        u128 m = 0;
+        for (int t = 0; t < u.n; ++t) m |= (u128)1 << (std::lower_bound(D.begin(), D.end(), u.leaf[t]) - D.begin());
+        return m;
+    };
+    ma.clear();
+    mb.clear();
+    for (const Cut &u : Pa) ma.push_back(mask_of(u));
+    ma.push_back(mask_of(ta));
+    for (const Cut &v : Pb) mb.push_back(mask_of(v));
+    mb.push_back(mask_of(tb));
+    // Eq. (1) candidates in the list path's order; drop the empty cut and the trivial cut {n}
+    // (n itself is never in the dictionary: every leaf id is below id)
+    E.clear();
+    En.clear();
+    for (u128 u : ma)
+        for (u128 v : mb) {
+            const u128 m = u | v;
+            const int n = pop128(m);
+            if (n > (int)J.k_l || n == 0) continue;
+            E.push_back(m);
+            En.push_back((uint8_t)n);
+        }
+    ord.resize(E.size());
+    for (uint32_t i = 0; i < ord.size(); ++i) ord[i] = i;
+    std::sort(ord.begin(), ord.end(), [&](uint32_t xi, uint32_t yi) {
+        if (En[xi] != En[yi]) return En[xi] < En[yi];
+        return lex_less_masks(E[xi], E[yi]);
+    });
+    kept.clear();
+    u128 prev = 0;
+    bool have_prev = false;
+    for (uint32_t xi : ord) {  // keep a cut unless a kept (not larger) cut is a subset of it
+        const u128 x = E[xi];
+        // equal candidates are adjacent after the sort: a repeat is dominated by its first copy
+        // (kept, or itself dominated by a kept cut that is then a subset of the repeat too)
+        if (have_prev && x == prev) continue;
+        prev = x;
+        have_prev = true;
+        bool dom = false;
+        for (uint32_t ki : kept)
+            if ((E[ki] & ~x) == 0) {
+                dom = true;
+                break;
+            }
+        if (!dom) kept.push_back(xi);
+    }
+    // metrics per dictionary entry
+    dfan.resize(D.size());
+    dlev.resize(D.size());
+    for (size_t i = 0; i < D.size(); ++i) {
+        dfan[i] = (*J.fanout)[D[i]];
+        dlev[i] = c->level[D[i]];
+    }
+    K.resize(kept.size());
+    for (size_t t = 0; t < kept.size(); ++t) {
+        Cut &x = K[t];
+        u128 m = E[kept[t]];
+        x.n = 0;
+        x.sig = 0;
+        x.sum_fanout = x.sum_level = 0;
+        x.sim = 0;
+        while (m) {
+            const int i = ctz128(m);
+            m &= m - 1;
+            x.leaf[x.n++] = D[i];
+            x.sig |= bit_of(D[i]);
+            x.sum_fanout += dfan[i];
+            x.sum_level += dlev[i];
+        }
+    }
+    rk.resize(K.size());
+    for (uint32_t i = 0; i < rk.size(); ++i) rk[i] = i;
+    const uint32_t r = (*J.repr_of)[id];
+    if (r != 0xFFFFFFFFu && !P[r].empty()) {
+        static const unsigned __int128 L = lcm_upto(2 * KMAX);
+        for (Cut &x : K) {
+            unsigned __int128 sv = 0;
+            for (const Cut &y : P[r]) {
+                const int in = inter(x, y);
+                sv += (unsigned __int128)in * (L / (unsigned __int128)(x.n + y.n - in));
+            }
+            x.sim = sv;
+        }
+        std::sort(rk.begin(), rk.end(), [&](uint32_t xi, uint32_t yi) {
+            const Cut &x = K[xi], &y = K[yi];
+            if (x.sim != y.sim) return x.sim > y.sim;
+            return table1_less(x, y, J.pass);
+        });
+    } else {
+        std::sort(rk.begin(), rk.end(), [&](uint32_t xi, uint32_t yi) { return table1_less(K[xi], K[yi], J.pass); });
+    }
+    std::vector<Cut> out;
+    out.reserve(std::min<size_t>(rk.size(), J.C));
+    for (size_t t = 0; t < rk.size() && t < J.C; ++t) out.push_back(K[rk[t]]);
+    P[id].swap(out);
+    return true;
+}
+
 // P(id) from P(fanins) (and P(repr) for a member): Eq. (1), dominance, Table I / similarity order.
 void node_cuts(const CutJob &J, uint32_t id, std::vector<std::vector<Cut>> &P) {
+    static const bool lists_only = getenv("CEC_CUTS_LISTS") != nullptr;  // the list path (A/B, tests)
+    if (!lists_only && node_cuts_masks(J, id, P)) return;
     const cec_ctx *c = J.c;
     const uint32_t a = c->f0[id] >> 1, b = c->f1[id] >> 1;
     const std::vector<Cut> &Pa = P[a], &Pb = P[b];
     const Cut ta = trivial_cut(a), tb = trivial_cut(b);
     // candidates in the order P(n0) + {{n0}} x P(n1) + {{n1}}; ranked through index arrays (a Cut
     // is ~150 bytes: sorting the objects themselves dominated the enumeration)
-    thread_local std::vector<Cut> E;
-    thread_local std::vector<uint32_t> ord, kept;
+    thread_local std::vector<Cut> tE;
+    thread_local std::vector<uint32_t> tord, tkept;
+    std::vector<Cut> &E = tE;
+    std::vector<uint32_t> &ord = tord, &kept = tkept;
     E.clear();
     Cut m;
     for (size_t i = 0; i <= Pa.size(); ++i) {
@@ -176,7 +324,7 @@ void node_cuts(const CutJob &J, uint32_t id, std::vector<std::vector<Cut>> &P) {
     // dedupe + drop dominated: process by size, keep a cut unless a kept cut is its subset
     ord.resize(E.size());
     for (uint32_t i = 0; i < ord.size(); ++i) ord[i] = i;
-    std::sort(ord.begin(), ord.end(), [](uint32_t xi, uint32_t yi) {
+    std::sort(ord.begin(), ord.end(), [&](uint32_t xi, uint32_t yi) {
         const Cut &x = E[xi], &y = E[yi];
         if (x.n != y.n) return x.n < y.n;
         return std::lexicographical_compare(x.leaf, x.leaf + x.n, y.leaf, y.leaf + y.n);

@@ -1,6 +1,8 @@
 """Host logic of the CEC driver (no GPU): Eq. (1) cut enumeration on hand graphs, Table I orders,
 class formation from signatures, and miter reduction preserving PO functions (checked with the
 oracle's evaluator on random assignments)."""
+import os
+
 import numpy as np
 import pytest
 
@@ -153,3 +155,34 @@ def test_tried_pairs_follow_the_reduction():
              (3, 9, 0),   # 6 vs 9 -> (3, 4, 1)
              (8, 2, 1)}   # 14 vs 4 ^ 1 = 5 -> lower id first: (2, 7, 1)
     assert _remap_tried(tried, image) == {(4, 5, 0), (5, 6, 0), (3, 4, 1), (2, 7, 1)}
+
+
+def test_cut_masks_path_equals_lists_path():
+    """node_cuts' 128-bit dictionary path (csrc/cuts.cpp) and its list path (CEC_CUTS_LISTS=1) give
+    identical common cuts at C4's parameters (k_l = C = 16, 64-bit datapath, all three passes)."""
+    import subprocess
+    import sys
+    script = r"""
+import hashlib, sys
+sys.path.insert(0, %r)
+import numpy as np
+from paper_conf_dac_liuy25_b200 import capi
+from workloads import c4_dp
+m = c4_dp(64)
+ctx = capi.Context.from_aig(m.aig, device=-1)
+I = m.aig.num_pis
+pairs = sorted({(min(a >> 1, b >> 1), max(a >> 1, b >> 1)) for a, b in zip(m.lit_a.tolist(), m.lit_b.tolist())
+                if (a >> 1) != (b >> 1) and min(a >> 1, b >> 1) > I})
+h = hashlib.sha1()
+for pass_id in range(3):
+    for a in capi.cec_common_cuts(ctx.handle, [p[0] for p in pairs], [p[1] for p in pairs], 16, 16, pass_id, 16):
+        h.update(np.ascontiguousarray(a).tobytes())
+print(h.hexdigest())
+""" % os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ)
+    env.pop("CEC_CUTS_LISTS", None)
+    a = subprocess.run([sys.executable, "-c", script], capture_output=True, text=True, env=env, timeout=600)
+    env["CEC_CUTS_LISTS"] = "1"
+    b = subprocess.run([sys.executable, "-c", script], capture_output=True, text=True, env=env, timeout=600)
+    assert a.returncode == 0 and b.returncode == 0, a.stderr[-500:] + b.stderr[-500:]
+    assert a.stdout.strip() == b.stdout.strip() and len(a.stdout.strip()) == 40
