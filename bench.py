@@ -443,8 +443,9 @@ def main():
     peak = props.multi_processor_count * LOP3_PER_CLK_PER_SM * sm_clock * 1e6 / 1e12  # TLOP3/s
     # algorithmic LOP3s of the path: one 3-input LUT per mapped node group per u32 word (JIT), one
     # per AND (interpreter) — the AND-node count itself is the metric W — over the window kernels'
-    # own device time per launch (CUDA events around them on the launch stream, every timed step;
-    # the step adds the reset kernel and the graph launch); step_frac is the same over the step
+    # own device time per launch (CUDA events around them on the launch stream, mean over the
+    # second pass of K steps; the step adds the reset kernel and the graph launch); step_frac is
+    # the same rate over the timed step
     kern_ms = statistics.mean(sweep_ms) if sweep_ms else ms
     if world > 1:
         kern_ms = allreduce(kern_ms, dist.ReduceOp.MAX)
