@@ -25,9 +25,17 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--seeds", type=int, default=300)
     ap.add_argument("--start", type=int, default=0)
+    ap.add_argument("--engine", default="jit", choices=["jit", "auto", "interp"],
+                    help="engine under test (auto: per-window JIT / interpreter choice, as the product runs)")
+    ap.add_argument("--split", type=float, default=-1.0,
+                    help="CEC_PIPE_SPLIT for the public call (with CEC_PIPE_SPLIT_MINWIN=2): large windows first")
     ap.add_argument("--miters", action="store_true",
                     help="random-block miters A vs rewritten A (mostly EQ: full sweeps) instead of random pairs")
     a = ap.parse_args()
+    engine = {"jit": capi.CEC_ENGINE_JIT, "auto": capi.CEC_ENGINE_AUTO, "interp": capi.CEC_ENGINE_INTERP}[a.engine]
+    if a.split >= 0:
+        os.environ["CEC_PIPE_SPLIT"] = str(a.split)
+        os.environ["CEC_PIPE_SPLIT_MINWIN"] = "2"
     bad, pairs, neq, t0 = [], 0, 0, time.time()
     for seed in range(a.start, a.start + a.seeds):
         rng = np.random.default_rng(70000 + seed)
@@ -42,7 +50,7 @@ def main():
         else:
             m = tiny_random(I, int(rng.integers(30, 400)), 24, 80000 + seed)
         merge = int(rng.integers(0, 3))
-        ctx = capi.Context.from_aig(m.aig, k_max=16, merge=merge, engine=capi.CEC_ENGINE_JIT)
+        ctx = capi.Context.from_aig(m.aig, k_max=16, merge=merge, engine=engine)
         gv, gc, gk = ctx.sim_exhaustive(m.lit_a, m.lit_b)
         orc = oracle.Oracle.from_aig(m.aig)
         ov, oc, ok, _ = orc.check_pairs(m.lit_a, m.lit_b, k_max=16)
@@ -58,7 +66,8 @@ def main():
         pairs += m.num_pairs
         neq += int((ov == oracle.NOT_EQUIVALENT).sum())
         ctx.close()
-    print(json.dumps({"fuzz": "jit engine vs oracle" + (" (A vs rewritten A miters)" if a.miters else ""), "seeds": a.seeds, "start": a.start, "pairs": pairs,
+    print(json.dumps({"fuzz": f"{a.engine} engine vs oracle" + (" (A vs rewritten A miters)" if a.miters else "")
+                      + (f", split {a.split}" if a.split >= 0 else ""), "seeds": a.seeds, "start": a.start, "pairs": pairs,
                       "neq_pairs": neq, "mismatching_seeds": bad, "ok": not bad,
                       "seconds": round(time.time() - t0, 1)}), flush=True)
     return 1 if bad else 0
