@@ -615,3 +615,19 @@ def test_plan_sweep_timing_events():
     with pytest.raises(capi.CecError):
         capi.cec_plan_sweep_ms(plan)
     capi.cec_plan_free(plan)
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_shard_emulation_with_split_pipeline(world, monkeypatch):
+    """Pattern-space shards (rank g of G, shard-only mode) through the public call with the
+    large-windows-first split forced: the min over ranks is still the 1-GPU result."""
+    m = _c3_small()
+    ref = gpu_ctx(m.aig, merge=capi.CEC_MERGE_COST).sim_exhaustive(m.lit_a, m.lit_b)
+    monkeypatch.setenv("CEC_PIPE_SPLIT", str(float(1 << 12)))
+    monkeypatch.setenv("CEC_PIPE_SPLIT_MINWIN", "2")
+    parts = [gpu_ctx(m.aig, merge=capi.CEC_MERGE_COST, rank=g, world=world).sim_exhaustive(m.lit_a, m.lit_b)
+             for g in range(world)]
+    v, c, k = combine_shards(parts)
+    assert np.array_equal(v, ref[0]) and np.array_equal(k, ref[2])
+    neq = ref[0] == capi.CEC_NOT_EQUIVALENT
+    assert neq.any() and np.array_equal(np.asarray(c)[neq], ref[1][neq])
