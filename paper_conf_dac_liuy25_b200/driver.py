@@ -45,6 +45,7 @@ class CecParams:
     distance1: bool = True        # also simulate every distance-1 neighbour of each CEX
     device: int = 0
     engine: int = capi.CEC_ENGINE_AUTO
+    reuse_context: bool = True    # keep the device context(s) for the next check_miter call
 
 
 @dataclasses.dataclass
@@ -216,8 +217,12 @@ def check_miter(aig: Aig, lit_a, lit_b, params: Optional[CecParams] = None) -> C
 
     # One device context serves every phase: each new miter version is loaded into it
     # (cec_reload_aig), keeping streams, workers, device pools and JIT kernels.
-    # A second one (slot 1) holds the local-check limit when k_l > k_g.
-    dev: List[Optional[capi.Context]] = [None, None]
+    # A second one (slot 1) holds the local-check limit when k_l > k_g. With reuse_context the
+    # contexts also outlive the call (release_contexts() frees them): the next miter is loaded into
+    # them instead of creating contexts and freeing their device memory per call (context creation
+    # is excluded from end-to-end time; cudaFree of a pool can take 0.3 s).
+    dev: List[Optional[capi.Context]] = (_DEV_CACHE.setdefault((p.device, p.engine), [None, None])
+                                         if p.reuse_context else [None, None])
 
     def dctx(m: Miter, k_max: int, slot: int = 0) -> capi.Context:
         if dev[slot] is None:
@@ -231,14 +236,33 @@ def check_miter(aig: Aig, lit_a, lit_b, params: Optional[CecParams] = None) -> C
     # in random phases, so it is paused for the flow and restored afterwards.
     gc_was_on = gc.isenabled()
     gc.disable()
+    ok = False
     try:
-        return _flow(p, cur, log, checks, versions, P, po_v, po_status, dctx)
+        res = _flow(p, cur, log, checks, versions, P, po_v, po_status, dctx)
+        ok = True
+        return res
     finally:
-        for c in dev:
-            if c is not None:
-                c.close()
+        if not p.reuse_context or not ok:  # a failed flow does not leave its contexts for the next
+            for i, c in enumerate(dev):
+                if c is not None:
+                    c.close()
+                    dev[i] = None
         if gc_was_on:
             gc.enable()
+
+
+# device contexts kept between check_miter calls, per (device, engine); one caller thread at a time
+_DEV_CACHE: Dict[Tuple[int, int], List[Optional[capi.Context]]] = {}
+
+
+def release_contexts() -> None:
+    """Free the device contexts check_miter keeps between calls (reuse_context)."""
+    for slots in _DEV_CACHE.values():
+        for i, c in enumerate(slots):
+            if c is not None:
+                c.close()
+                slots[i] = None
+    _DEV_CACHE.clear()
 
 
 def _flow(p, cur, log, checks, versions, P, po_v, po_status, dctx) -> CecResult:
