@@ -16,6 +16,7 @@ then hands the reduced miter to ABC, which is out of scope).
 """
 from __future__ import annotations
 
+import atexit
 import dataclasses
 import gc
 import time
@@ -263,6 +264,9 @@ def release_contexts() -> None:
                 c.close()
                 slots[i] = None
     _DEV_CACHE.clear()
+
+
+atexit.register(release_contexts)  # before the CUDA runtime's own teardown (registered earlier)
 
 
 def _flow(p, cur, log, checks, versions, P, po_v, po_status, dctx) -> CecResult:
