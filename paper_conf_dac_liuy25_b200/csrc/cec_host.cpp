@@ -1570,11 +1570,13 @@ static cec_status plan_route(cec_ctx *c, uint32_t n, const uint32_t *la, const u
         cm.S = std::move(S);
         P->cmps.push_back(std::move(cm));
     }
+    tm.lap("routing: pairs -> windows");
     // a5: window merging: windows sorted lexicographically by input list.
     std::vector<uint32_t> order(wins0.size());
     for (uint32_t i = 0; i < order.size(); ++i) order[i] = i;
     std::stable_sort(order.begin(), order.end(),
                      [&](uint32_t a, uint32_t b) { return lex_less(wins0[a].inputs, wins0[b].inputs); });
+    tm.lap("routing: lexicographic sort");
     // a merged window is enumerated like a single pair's: never more than MAX_K_ENUM inputs
     // (its slice indices are u32), whatever k_s / k_max the caller passed
     const uint32_t ks = std::min({c->opts.k_s, kmax, (uint32_t)MAX_K_ENUM});
