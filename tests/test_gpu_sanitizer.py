@@ -34,6 +34,10 @@ print("SANITIZER-RUN-OK")
 def test_compute_sanitizer(tool):
     if not torch.cuda.is_available():
         pytest.skip("no CUDA device")
+    # opt-in: on the B200 pool, runs under compute-sanitizer have left GPUs needing a reset (the
+    # operators disabled the tool there); the round-2 runs with 0 errors are in profiles/
+    if os.environ.get("CEC_RUN_SANITIZER") != "1":
+        pytest.skip("compute-sanitizer runs are opt-in (CEC_RUN_SANITIZER=1)")
     cs = shutil.which("compute-sanitizer") or "/usr/local/cuda/bin/compute-sanitizer"
     if not os.path.exists(cs):
         pytest.skip("compute-sanitizer not found")
