@@ -99,7 +99,16 @@ typedef struct {
     uint32_t k_s;              /* window-merge threshold; 0 = k_max */
     int32_t merge;             /* cec_merge_policy; default CEC_MERGE_PAPER */
     int32_t engine;            /* cec_engine; default CEC_ENGINE_AUTO */
-    uint64_t reserved[6];      /* must be zero */
+    void *workspace;           /* caller-owned device memory for CEC_ENGINE_SIMT's simulation table:
+                                  Alg. 1's memory budget M. E = the largest
+                                  power of two with E x rows x 4 B <= workspace_bytes; the table
+                                  lives in the workspace (not freed by the library; the caller keeps
+                                  it alive and unused while plans of the context run). NULL = the
+                                  library allocates M itself (CEC_SIMT_MB, default 16 GiB). The
+                                  product engines (JIT, interpreter) keep truth tables on chip and
+                                  ignore it. */
+    uint64_t workspace_bytes;
+    uint64_t reserved[4];      /* must be zero */
 } cec_opts;
 
 typedef struct {

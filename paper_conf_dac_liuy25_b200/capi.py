@@ -37,7 +37,7 @@ class CecOpts(ctypes.Structure):
     _fields_ = [("device", ctypes.c_int32), ("rank", ctypes.c_int32), ("world", ctypes.c_int32),
                 ("nccl_unique_id", ctypes.c_void_p), ("stream", ctypes.c_void_p), ("k_max", ctypes.c_uint32),
                 ("k_s", ctypes.c_uint32), ("merge", ctypes.c_int32), ("engine", ctypes.c_int32),
-                ("reserved", ctypes.c_uint64 * 6)]
+                ("workspace", ctypes.c_void_p), ("workspace_bytes", ctypes.c_uint64), ("reserved", ctypes.c_uint64 * 4)]
 
 
 class CecAig(ctypes.Structure):

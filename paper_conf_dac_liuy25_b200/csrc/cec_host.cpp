@@ -1018,6 +1018,7 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         S.level_off.push_back((uint32_t)S.h_nodes.size());
         uint64_t M = 16384ull << 18;  // words (16 GiB)
         if (const char *e = getenv("CEC_SIMT_MB")) M = strtoull(e, nullptr, 10) << 18;
+        if (c->opts.workspace) M = c->opts.workspace_bytes / 4;  // the caller's budget (Alg. 1 input M)
         uint64_t E = 4;  // Alg. 1 l.2: the largest power of two with E x rows <= M
         while (E * 2 * rows <= M && E < max_ttw) E *= 2;
         if (E * rows > M) return fail(c, CEC_E_NOMEM, "simulation table: %llu rows do not fit M", (unsigned long long)rows);
@@ -1347,7 +1348,12 @@ cec_status upload(cec_ctx *c, cec_plan *P) {
     }
     if (P->simt.E) {
         SimtPlan &S = P->simt;
-        CUDA_TRY(c, dev_alloc((void **)&S.d_simt, sizeof(uint32_t) * (size_t)S.E * S.rows));
+        if (c->opts.workspace && sizeof(uint32_t) * (uint64_t)S.E * S.rows <= c->opts.workspace_bytes) {
+            S.d_simt = (uint4 *)c->opts.workspace;  // 16-byte aligned: cudaMalloc / torch allocations
+            S.simt_in_workspace = true;
+        } else {
+            CUDA_TRY(c, dev_alloc((void **)&S.d_simt, sizeof(uint32_t) * (size_t)S.E * S.rows));
+        }
         CUDA_TRY(c, dev_alloc((void **)&S.d_inputs, sizeof(uint4) * std::max<size_t>(1, S.h_inputs.size())));
         CUDA_TRY(c, dev_alloc((void **)&S.d_nodes, sizeof(uint4) * std::max<size_t>(1, S.h_nodes.size())));
         CUDA_TRY(c, dev_alloc((void **)&S.d_pairs, sizeof(uint4) * std::max<size_t>(1, S.h_pairs.size())));
@@ -1374,7 +1380,8 @@ void free_dev(cec_plan *P) {
     P->arena_cap = 0;
     P->pool.reset();
     P->d = DevPlan{};
-    dev_free(P->simt.d_simt);
+    if (!P->simt.simt_in_workspace) dev_free(P->simt.d_simt);
+    P->simt.simt_in_workspace = false;
     dev_free(P->simt.d_inputs);
     dev_free(P->simt.d_nodes);
     dev_free(P->simt.d_pairs);

@@ -156,6 +156,7 @@ struct SimtPlan {
     uint32_t E = 0;                 // words per row per round (0 = plan does not use this engine)
     uint64_t rounds = 0, rows = 0;
     uint4 *d_simt = nullptr;        // rows x E words
+    bool simt_in_workspace = false; // d_simt is the caller's workspace (cec_opts.workspace): not freed
     uint4 *d_inputs = nullptr;      // {row, window, j, 0}
     uint4 *d_nodes = nullptr;       // by level: {row, row_f0 | c0 << 31, row_f1 | c1 << 31, window}
     uint4 *d_pairs = nullptr;       // {row_a | ca << 31, row_b | cb << 31, window, cmp}

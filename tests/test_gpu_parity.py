@@ -631,3 +631,20 @@ def test_shard_emulation_with_split_pipeline(world, monkeypatch):
     assert np.array_equal(v, ref[0]) and np.array_equal(k, ref[2])
     neq = ref[0] == capi.CEC_NOT_EQUIVALENT
     assert neq.any() and np.array_equal(np.asarray(c)[neq], ref[1][neq])
+
+
+@pytest.mark.parametrize("kib", [64, 256, 4096])
+def test_simt_engine_caller_workspace(kib):
+    """cec_opts.workspace (include/cec.h): the paper's Alg. 1 engine sizes E from the caller's memory
+    budget M and keeps its simulation table in the caller's device buffer; a small M
+    means more rounds (E words per row per round), never different results."""
+    m = circuits.c2_mul12_bug(seed=1, n=8)
+    ws = torch.empty(kib * 1024, dtype=torch.uint8, device="cuda")
+    ctx = gpu_ctx(m.aig, engine=capi.CEC_ENGINE_SIMT, workspace=ws.data_ptr(), workspace_bytes=ws.numel())
+    got = ctx.sim_exhaustive(m.lit_a, m.lit_b)
+    orc = Oracle.from_aig(m.aig)
+    ov, oc, ok, _ = orc.check_pairs(m.lit_a, m.lit_b, k_max=32)
+    assert_same(*got, ov, oc, ok, f"simt workspace {kib} KiB")
+    ref = gpu_ctx(m.aig, engine=capi.CEC_ENGINE_SIMT).sim_exhaustive(m.lit_a, m.lit_b)
+    for a, b in zip(got, ref):
+        assert np.array_equal(a, b)
