@@ -648,3 +648,34 @@ def test_simt_engine_caller_workspace(kib):
     ref = gpu_ctx(m.aig, engine=capi.CEC_ENGINE_SIMT).sim_exhaustive(m.lit_a, m.lit_b)
     for a, b in zip(got, ref):
         assert np.array_equal(a, b)
+
+
+def test_cli_diffable_output_matches_oracle_byte_for_byte(tmp_path):
+    """SURVEY.md §8(c) "Diffable output": the GPU path's CLI and the oracle's CLI, given the same
+    AIGER, pair and check files, print byte-identical text (verdicts, k, CEX indices, CEX vectors;
+    local checks)."""
+    import subprocess
+    import sys as _sys
+
+    from workloads import write_aag, write_checks, write_pairs
+
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    m = circuits.c2_mul12_bug(seed=3, n=8)
+    write_aag(m.aig, str(tmp_path / "m.aag"))
+    write_pairs(str(tmp_path / "p.txt"), m.lit_a, m.lit_b)
+    orc = Oracle.from_aig(m.aig)
+    off, lv = [0], []
+    for a, b in zip(m.lit_a, m.lit_b):  # cut = the pair's support (local verdict = global, P:25)
+        s = orc.support(int(a), int(b))
+        lv += s
+        off.append(len(lv))
+    write_checks(str(tmp_path / "c.txt"), m.lit_a, m.lit_b, off, lv)
+    outs = {}
+    for cmd, f in (("check", "p.txt"), ("local", "c.txt")):
+        want = oracle.run_cli(cmd, str(tmp_path / "m.aag"), str(tmp_path / f))
+        got = subprocess.run([_sys.executable, "-m", "paper_conf_dac_liuy25_b200.cli", cmd, str(tmp_path / "m.aag"),
+                              str(tmp_path / f)], capture_output=True, text=True, cwd=root, timeout=300)
+        assert got.returncode == 0, got.stderr[-2000:]
+        assert got.stdout == want, cmd
+        outs[cmd] = want
+    assert " NEQ " in outs["check"] and "\ncex " in outs["check"]  # the bug is refuted, with a CEX line
