@@ -36,6 +36,7 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 METRIC = "AIG node-pattern evals/s"
+WORKLOAD_SEEDS = {"c5": 5, "c3": 3, "c2bug": 1, "c2": None, "c1": None}  # generator seeds (workloads/circuits.py)
 UNIT = "node-patterns/s"
 LOP3_PER_CLK_PER_SM = 64  # alu pipe: rt = 2 cycles per warp-instr per SMSP, 4 SMSPs (B300_MICROARCH.md)
 
@@ -493,6 +494,42 @@ def main():
             parity = {"vs": f"tests/golden/{gold_name}.json (oracle/, every pair)", "pairs": int(gv.size),
                       "diffs": diffs, "ok": diffs == 0}
 
+    # SURVEY.md §8(d) "Runs and reporting": the per-run record under the survey's own field names
+    h2d_ms = None
+    if st_e2e["h2d_bytes"]:  # one pinned host -> device copy of the call's H2D bytes, CUDA events
+        hb = torch.empty(int(st_e2e["h2d_bytes"]), dtype=torch.uint8, pin_memory=True)
+        db = torch.empty_like(hb, device="cuda")
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        db.copy_(hb, non_blocking=True)
+        e0.record(stream)
+        db.copy_(hb, non_blocking=True)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        h2d_ms = e0.elapsed_time(e1)
+    ncu = {}
+    if os.path.exists(prof):
+        try:
+            ncu = json.load(open(prof)).get(args.config, {})
+        except Exception:
+            ncu = {}
+    record = {
+        "config": args.config, "seed": WORKLOAD_SEEDS.get(args.config), "gpus": world, "W": W_all,
+        "t_kernel_ms": statistics.median(step_ms), "node_patterns_per_s": value, "t_e2e_ms": e2e,
+        "t_hostprep_ms": st_e2e["host_prep_ms"], "t_h2d_ms": h2d_ms,
+        "t_allreduce_us": 1e3 * max(0.0, ms - kern_ms) if world > 1 else 0.0,
+        "dram_GBps": (ncu["dram_bytes_per_launch"] / ncu["profiled_launch_ns"]
+                      if ncu.get("dram_bytes_per_launch") and ncu.get("profiled_launch_ns") else None),
+        "alu_pipe_pct": ncu.get("alu_pipe_pct"),
+        "lop3_count_per_W32": stats["lop3_words"] / max(1.0, W_rank / 32.0),
+        "sm_clock_MHz": sm_clock,
+        "oracle_wall_s": cpu["seconds"] if cpu else None, "oracle_cores": cpu["cores"] if cpu else None,
+        "oracle_cpu_s": cpu["seconds"] * cpu["cores"] if cpu else None,
+        "parity": parity,
+        "notes": ("t_kernel_ms: median step; t_h2d_ms: one pinned copy of the call's H2D bytes; "
+                  "t_allreduce_us: step minus window-kernel time (reset + reduction + launch), N > 1; "
+                  "dram_GBps / alu_pipe_pct: ncu --set full of the largest kernel (profiles/ncu_summary.json)"),
+    }
+
     if rank == 0:
         line = {
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
@@ -506,6 +543,7 @@ def main():
                        "verdicts": verdicts},
             "clocks": clocks,
             "parity": parity,
+            "record": record,
             "gpu_launches": int(launches_per_step * args.steps),
             "e2e": {"value": W_all / (e2e / 1e3), "unit": UNIT, "ms_per_miter": e2e,
                     "h2d_bytes_per_step": int(st_e2e["h2d_bytes"]), "d2h_bytes_per_step": int(st_e2e["d2h_bytes"]),

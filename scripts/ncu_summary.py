@@ -56,6 +56,7 @@ def main():
     if a.note:
         md += [a.note, ""]
     dram_per_launch = []
+    alu_pct, dur_ns = [], []
     for rep in a.rep:
         hdr, units, rows = raw_rows(rep)
         idx = {n: i for i, n in enumerate(hdr)}
@@ -83,6 +84,13 @@ def main():
                                 for v, n in sorted(stalls, reverse=True)))
             md.append("")
             scale = {"byte": 1.0, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}
+            for key, acc in (("sm__pipe_alu_cycles_active.avg.pct_of_peak_sustained_active", alu_pct),
+                             ("gpu__time_duration.sum", dur_ns)):
+                try:
+                    acc.append(float(r[idx[key]]) * ({"ms": 1e6, "us": 1e3, "usecond": 1e3, "msecond": 1e6}.get(units[idx[key]], 1.0)
+                                                     if key == "gpu__time_duration.sum" else 1.0))
+                except (KeyError, ValueError):
+                    pass
             try:
                 rd, wr = idx["dram__bytes_read.sum"], idx["dram__bytes_write.sum"]
                 dram_per_launch.append(float(r[rd]) * scale.get(units[rd], 1.0) + float(r[wr]) * scale.get(units[wr], 1.0))
@@ -117,6 +125,10 @@ def main():
     if dram_per_launch:
         summ.setdefault(a.config, {})["dram_bytes_per_launch"] = sum(dram_per_launch) / len(dram_per_launch)
         summ[a.config]["source"] = a.name
+    if alu_pct:
+        summ.setdefault(a.config, {})["alu_pipe_pct"] = sum(alu_pct) / len(alu_pct)
+    if dur_ns:
+        summ.setdefault(a.config, {})["profiled_launch_ns"] = sum(dur_ns) / len(dur_ns)
     with open(sp, "w") as fh:
         json.dump(summ, fh, indent=1)
 
