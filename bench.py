@@ -527,7 +527,8 @@ def main():
         "parity": parity,
         "notes": ("t_kernel_ms: median step; t_h2d_ms: one pinned copy of the call's H2D bytes; "
                   "t_allreduce_us: step minus window-kernel time (reset + reduction + launch), N > 1; "
-                  "dram_GBps / alu_pipe_pct: ncu --set full of the largest kernel (profiles/ncu_summary.json)"),
+                  "dram_GBps / alu_pipe_pct: ncu --set full of one window kernel of this config "
+                  f"(profiles/ncu_summary.json, {ncu.get('source', 'none')})"),
     }
 
     if rank == 0:
@@ -558,7 +559,7 @@ def main():
                          {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "TLOP3/s",
                          "frac": achieved / peak, "traffic": traffic,
                          "kernel_ms": kern_ms, "kernel_timing": "CUDA events around the window kernels "
-                         "(cec_plan_sweep_ms), mean over the timed steps",
+                         "(cec_plan_sweep_ms), mean over a second pass of the K steps",
                          "step_frac": stats["lop3_words"] / (ms / 1e3) / 1e12 / peak,
                          "peak_basis": f"{props.multi_processor_count} SMs x {LOP3_PER_CLK_PER_SM} LOP3/clk x {sm_clock:.0f} MHz (guide unit counts, SM clock; microbenchmark scripts/peaks.cu measured 64.00 LOP3/clk/SM = 18.53 TLOP3/s at 1957 MHz, profiles/round1_peaks.json)",
                          "lop3_per_word_per_and": stats["lop3_words"] / max(1.0, W_rank / 32.0),
