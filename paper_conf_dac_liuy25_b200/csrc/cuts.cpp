@@ -217,29 +217,38 @@ bool node_cuts_masks(const CutJob &J, uint32_t id, std::vector<std::vector<Cut>>
             E.push_back(m);
             En.push_back((uint8_t)n);
         }
+    // Dominance filter: the kept set is the set of minimal candidates (no kept cut is a subset of
+    // another), which does not depend on the order inside one size class, only on visiting smaller
+    // sizes first; the final Table I / similarity ranking below is a total order. So candidates are
+    // bucketed by size (counting sort) and, inside a bucket, sorted by mask value only to find
+    // repeats; a candidate is checked against kept cuts of strictly smaller size (two different
+    // cuts of one size are never subsets of each other).
+    uint32_t bstart[KMAX + 2] = {0};
+    for (uint8_t n : En) ++bstart[n + 1];
+    for (int b = 0; b <= KMAX; ++b) bstart[b + 1] += bstart[b];
     ord.resize(E.size());
-    for (uint32_t i = 0; i < ord.size(); ++i) ord[i] = i;
-    std::sort(ord.begin(), ord.end(), [&](uint32_t xi, uint32_t yi) {
-        if (En[xi] != En[yi]) return En[xi] < En[yi];
-        return lex_less_masks(E[xi], E[yi]);
-    });
+    {
+        uint32_t fillp[KMAX + 1];
+        for (int b = 0; b <= KMAX; ++b) fillp[b] = bstart[b];
+        for (uint32_t i = 0; i < E.size(); ++i) ord[fillp[En[i]]++] = i;
+    }
     kept.clear();
-    u128 prev = 0;
-    bool have_prev = false;
-    for (uint32_t xi : ord) {  // keep a cut unless a kept (not larger) cut is a subset of it
-        const u128 x = E[xi];
-        // equal candidates are adjacent after the sort: a repeat is dominated by its first copy
-        // (kept, or itself dominated by a kept cut that is then a subset of the repeat too)
-        if (have_prev && x == prev) continue;
-        prev = x;
-        have_prev = true;
-        bool dom = false;
-        for (uint32_t ki : kept)
-            if ((E[ki] & ~x) == 0) {
-                dom = true;
-                break;
-            }
-        if (!dom) kept.push_back(xi);
+    for (int b = 1; b <= (int)J.k_l && b <= KMAX; ++b) {
+        const uint32_t lo = bstart[b], hi = bstart[b + 1];
+        if (lo == hi) continue;
+        std::sort(ord.begin() + lo, ord.begin() + hi, [&](uint32_t xi, uint32_t yi) { return E[xi] < E[yi]; });
+        const size_t smaller = kept.size();  // kept cuts of size < b
+        for (uint32_t t = lo; t < hi; ++t) {
+            const u128 x = E[ord[t]];
+            if (t > lo && x == E[ord[t - 1]]) continue;  // a repeat of the previous candidate
+            bool dom = false;
+            for (size_t q = 0; q < smaller; ++q)
+                if ((E[kept[q]] & ~x) == 0) {
+                    dom = true;
+                    break;
+                }
+            if (!dom) kept.push_back(ord[t]);
+        }
     }
     // metrics per dictionary entry
     dfan.resize(D.size());
