@@ -387,8 +387,69 @@ void node_cuts(const CutJob &J, uint32_t id, std::vector<std::vector<Cut>> &P) {
 }
 
 // common cuts u|v of a pair (no trivial cuts, <= k_l leaves), smallest first, at most max_cuts
+// Mask path of common_cuts_of (the same dictionary trick as node_cuts_masks): unions by OR, size by
+// popcount, (size, lexicographic) order by lex_less_masks, repeats adjacent after the sort; only the
+// first max_cuts survivors are turned back into leaf lists. False when > 128 distinct leaves.
+bool common_cuts_masks(const std::vector<std::vector<Cut>> &P, uint32_t r, uint32_t mbr, uint32_t k_l,
+                       uint32_t max_cuts, std::vector<Cut> &common) {
+    thread_local std::vector<uint32_t> tD;
+    thread_local std::vector<u128> tmr, tmm, tE;
+    thread_local std::vector<uint8_t> tEn;
+    thread_local std::vector<uint32_t> tord;
+    std::vector<uint32_t> &D = tD, &ord = tord;
+    std::vector<u128> &mr = tmr, &mm = tmm, &E = tE;
+    std::vector<uint8_t> &En = tEn;
+    D.clear();
+    for (const std::vector<Cut> *L : {&P[r], &P[mbr]})
+        for (const Cut &u : *L) D.insert(D.end(), u.leaf, u.leaf + u.n);
+    std::sort(D.begin(), D.end());
+    D.erase(std::unique(D.begin(), D.end()), D.end());
+    if (D.size() > 128) return false;
+    auto mask_of = [&](const Cut &u) {
+        u128 m = 0;
+        for (int t = 0; t < u.n; ++t) m |= (u128)1 << (std::lower_bound(D.begin(), D.end(), u.leaf[t]) - D.begin());
+        return m;
+    };
+    mr.clear();
+    mm.clear();
+    for (const Cut &u : P[r]) mr.push_back(mask_of(u));
+    for (const Cut &v : P[mbr]) mm.push_back(mask_of(v));
+    E.clear();
+    En.clear();
+    for (u128 u : mr)
+        for (u128 v : mm) {
+            const u128 m = u | v;
+            const int n = pop128(m);
+            if (n == 0 || n > (int)k_l) continue;
+            E.push_back(m);
+            En.push_back((uint8_t)n);
+        }
+    ord.resize(E.size());
+    for (uint32_t i = 0; i < ord.size(); ++i) ord[i] = i;
+    std::sort(ord.begin(), ord.end(), [&](uint32_t xi, uint32_t yi) {
+        if (En[xi] != En[yi]) return En[xi] < En[yi];
+        return lex_less_masks(E[xi], E[yi]);
+    });
+    common.clear();
+    for (size_t t = 0; t < ord.size() && common.size() < max_cuts; ++t) {
+        if (t > 0 && E[ord[t]] == E[ord[t - 1]]) continue;
+        Cut x;
+        u128 m = E[ord[t]];
+        while (m) {
+            const int i = ctz128(m);
+            m &= m - 1;
+            x.leaf[x.n++] = D[i];
+            x.sig |= bit_of(D[i]);
+        }
+        common.push_back(x);
+    }
+    return true;
+}
+
 void common_cuts_of(const std::vector<std::vector<Cut>> &P, uint32_t r, uint32_t mbr, uint32_t k_l, uint32_t max_cuts,
                     std::vector<Cut> &common) {
+    static const bool lists_only = getenv("CEC_CUTS_LISTS") != nullptr;
+    if (!lists_only && common_cuts_masks(P, r, mbr, k_l, max_cuts, common)) return;
     common.clear();
     Cut m;
     for (const Cut &u : P[r])
