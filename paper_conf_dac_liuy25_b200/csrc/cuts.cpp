@@ -22,6 +22,8 @@
 #include <atomic>
 #include <functional>
 #include <memory>
+#include <mutex>
+#include <condition_variable>
 #include <thread>
 #include <cstdint>
 #include <cstdlib>
@@ -690,9 +692,104 @@ extern "C" cec_status cec_local_pass(cec_ctx *c, uint32_t npairs, const uint32_t
     };
     uint32_t n_par = 0, n_flush = 0, nodes_par = 0, nodes_ser = 0;
     double t_ser = 0;
+    // Small cones (<= 64k needed nodes, e.g. C4's 2k): the priority cuts are enumerated without
+    // level barriers first — a node starts as soon as its fanins and representative are done (the
+    // dependencies of Eq. 2) — and the common cuts of all pairs in parallel; the level loop below
+    // then only fills and flushes the buffer, in exactly the level order and at exactly the flush
+    // points of Alg. 2, so the checks and verdicts are the same. (Large cones keep the level-by-level
+    // loop, whose flushes overlap the enumeration of the next levels.) CEC_ALG2_LEVEL_SYNC=1 forces it.
+    size_t n_need = 0;
+    for (const auto &L : lists) n_need += L.size();
+    const bool dataflow = n_need <= 65536 && getenv("CEC_ALG2_LEVEL_SYNC") == nullptr;
+    std::vector<std::vector<Cut>> cmn_all;
+    if (dataflow && n_need) {
+        if (lt) tq = clk::now();
+        std::vector<uint32_t> indeg(N, 0), coff(N + 1, 0), child;
+        auto prereq = [&](uint32_t id, uint32_t *out) {  // AND prerequisites of a needed AND node
+            int n = 0;
+            for (uint32_t p : {c->f0[id] >> 1, c->f1[id] >> 1, repr_of[id]})
+                if (p != 0xFFFFFFFFu && p > c->I) out[n++] = p;
+            return n;
+        };
+        uint32_t pq[3];
+        for (const auto &L : lists)
+            for (uint32_t id : L) {
+                const int n = prereq(id, pq);
+                indeg[id] = (uint32_t)n;
+                for (int t = 0; t < n; ++t) ++coff[pq[t] + 1];
+            }
+        for (uint32_t i = 0; i < N; ++i) coff[i + 1] += coff[i];
+        child.resize(coff[N]);
+        {
+            std::vector<uint32_t> fillc(coff.begin(), coff.end() - 1);
+            for (const auto &L : lists)
+                for (uint32_t id : L) {
+                    const int n = prereq(id, pq);
+                    for (int t = 0; t < n; ++t) child[fillc[pq[t]]++] = id;
+                }
+        }
+        std::mutex mu;
+        std::condition_variable cv;
+        std::vector<uint32_t> ready;
+        size_t remaining = n_need;
+        for (const auto &L : lists)
+            for (uint32_t id : L)
+                if (!indeg[id]) ready.push_back(id);
+        pool.run(pool.size() + 1, [&](uint32_t, unsigned) {
+            for (;;) {
+                uint32_t id;
+                {
+                    std::unique_lock<std::mutex> l(mu);
+                    cv.wait(l, [&]() { return !ready.empty() || remaining == 0; });
+                    if (ready.empty()) return;
+                    id = ready.back();
+                    ready.pop_back();
+                }
+                node_cuts(J, id, P);
+                size_t woke = 0;
+                {
+                    std::lock_guard<std::mutex> l(mu);
+                    --remaining;
+                    for (uint32_t t = coff[id]; t < coff[id + 1]; ++t)
+                        if (--indeg[child[t]] == 0) ready.push_back(child[t]), ++woke;
+                }
+                if (woke > 1 || remaining == 0) cv.notify_all();
+                else if (woke == 1) cv.notify_one();
+            }
+        });
+        nodes_par = (uint32_t)n_need;
+        acc(t_enum);
+        cmn_all.resize(npairs);
+        pool.run(npairs, [&](uint32_t q, unsigned) { common_cuts_of(P, repr[q], member[q], k_l, max_cuts, cmn_all[q]); });
+        acc(t_common);
+    }
     for (size_t e = 1; e < lists.size(); ++e) {
         const std::vector<uint32_t> &L = lists[e];
         if (lt) tq = clk::now();
+        if (dataflow) {  // cuts and common cuts are ready: Alg. 2 l.11-16 in level order
+            for (uint32_t q : pairs_at[e]) {
+                const uint32_t la = 2u * repr[q], lb = 2u * member[q] ^ (phase[q] & 1u);
+                for (const Cut &x : cmn_all[q]) {
+                    buf.pair.push_back(q);
+                    buf.la.push_back(la);
+                    buf.lb.push_back(lb);
+                    buf.leaves.insert(buf.leaves.end(), x.leaf, x.leaf + x.n);
+                    buf.off.push_back((uint32_t)buf.leaves.size());
+                    log_pair.push_back(q);
+                    log_leaves.insert(log_leaves.end(), x.leaf, x.leaf + x.n);
+                    log_off.push_back((uint32_t)log_leaves.size());
+                    ++nchecks;
+                }
+            }
+            acc(t_common);
+            if (buf.pair.size() >= std::max<uint32_t>(1, buffer_checks)) {  // Alg. 2 l.13-14: flush
+                ++n_flush;
+                cec_status st = flush();
+                if (st != CEC_OK) return st;
+                acc(t_flush);
+            }
+            continue;
+        }
         // a node's enumeration (~10-25 us at k_l = C = 16) outweighs a pool hand-off, so even
         // levels of 2 nodes run in parallel (C4's carry chains: 109 of 133 levels have < 8 nodes)
         if (L.size() < par_min) {
