@@ -17,6 +17,8 @@ then hands the reduced miter to ABC, which is out of scope).
 from __future__ import annotations
 
 import atexit
+import bisect
+import collections.abc
 import dataclasses
 import gc
 import time
@@ -49,6 +51,51 @@ class CecParams:
     reuse_context: bool = True    # keep the device context(s) for the next check_miter call
 
 
+class CheckLog(collections.abc.Sequence):
+    """Replay log of every local check (SURVEY.md §5 "checkpoint / resume": the oracle re-checks
+    each (miter version, pair, cut) and its verdict). Kept as the per-pass arrays the native pass
+    returns; entries are dicts {version, phase, pass, lit_a, lit_b, leaves, verdict} made on access
+    (building 57k dicts inside the flow cost ~20% of C4's end-to-end time)."""
+
+    def __init__(self):
+        self._chunks = []  # (version, phase, pass, lit_a[], lit_b[], cut_off[], leaves[], verdict[])
+        self._starts = [0]
+
+    def add(self, version, phase, pass_id, lit_a, lit_b, cut_off, leaves, verdict) -> None:
+        n = len(lit_a)
+        if n:
+            self._chunks.append((version, phase, pass_id, np.array(lit_a), np.array(lit_b), np.array(cut_off),
+                                 np.array(leaves), np.array(verdict)))  # copies: the pass's buffers are larger
+            self._starts.append(self._starts[-1] + n)
+
+    def append(self, ch: dict) -> None:
+        self.add(ch["version"], ch["phase"], ch["pass"], [ch["lit_a"]], [ch["lit_b"]], [0, len(ch["leaves"])],
+                 list(ch["leaves"]), [ch["verdict"]])
+
+    def __len__(self) -> int:
+        return self._starts[-1]
+
+    def _entry(self, k: int, i: int) -> dict:
+        v, ph, pa, la, lb, off, lv, vd = self._chunks[k]
+        return {"version": v, "phase": ph, "pass": pa, "lit_a": int(la[i]), "lit_b": int(lb[i]),
+                "leaves": [int(x) for x in lv[off[i]:off[i + 1]]], "verdict": int(vd[i])}
+
+    def __getitem__(self, idx):
+        if isinstance(idx, slice):
+            return [self[i] for i in range(*idx.indices(len(self)))]
+        if idx < 0:
+            idx += len(self)
+        if not 0 <= idx < len(self):
+            raise IndexError(idx)
+        k = bisect.bisect_right(self._starts, idx) - 1
+        return self._entry(k, idx - self._starts[k])
+
+    def __iter__(self):
+        for k, ch in enumerate(self._chunks):
+            for i in range(len(ch[3])):
+                yield self._entry(k, i)
+
+
 @dataclasses.dataclass
 class CecResult:
     verdict: int                      # CEC_EQUIVALENT / CEC_NOT_EQUIVALENT / CEC_UNDECIDED
@@ -56,7 +103,7 @@ class CecResult:
     cex: Optional[np.ndarray] = None  # PI values (PI id i+1 = cex[i]) of the lowest NEQ PO pair
     cex_pair: int = -1
     log: List[dict] = dataclasses.field(default_factory=list)
-    checks: List[dict] = dataclasses.field(default_factory=list)  # replay log of every local check
+    checks: "CheckLog" = dataclasses.field(default_factory=lambda: CheckLog())  # replay log of every local check
     versions: List[Aig] = dataclasses.field(default_factory=list)  # miter versions the checks refer to
     final_ands: int = 0
 
@@ -207,7 +254,7 @@ def check_miter(aig: Aig, lit_a, lit_b, params: Optional[CecParams] = None) -> C
     p = params or CecParams()
     cur = Miter(aig, lit_a, lit_b)
     log: List[dict] = []
-    checks: List[dict] = []
+    checks = CheckLog()
     versions: List[Aig] = []
     P = cur.lit_a.size
     po_v = np.full(P, capi.CEC_UNDECIDED, dtype=np.int32)
@@ -373,11 +420,12 @@ def _flow(p, cur, log, checks, versions, P, po_v, po_status, dctx) -> CecResult:
                     pass_id, p.max_cuts_per_pair, p.buffer_checks)
                 tk["local"] += time.perf_counter() - t1
                 ver = len(versions) - 1
-                for i in range(cp.size):
-                    r, m_, f = todo[int(cp[i])]
-                    checks.append({"version": ver, "phase": phase_no, "pass": pass_id, "lit_a": 2 * r,
-                                   "lit_b": 2 * m_ ^ f, "leaves": cl[cof[i]:cof[i + 1]].tolist(),
-                                   "verdict": int(cv[i])})
+                if cp.size:
+                    ta = np.array([x[0] for x in todo], dtype=np.int64)
+                    tm_ = np.array([x[1] for x in todo], dtype=np.int64)
+                    tf = np.array([x[2] for x in todo], dtype=np.int64)
+                    idx = cp.astype(np.int64)
+                    checks.add(ver, phase_no, pass_id, 2 * ta[idx], (2 * tm_[idx]) ^ tf[idx], cof, cl, cv)
                 for i, (r, m_, f) in enumerate(todo):
                     if pv[i] == capi.CEC_EQUIVALENT and m_ not in subst:
                         subst[m_] = 2 * r ^ f

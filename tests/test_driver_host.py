@@ -186,3 +186,15 @@ print(h.hexdigest())
     b = subprocess.run([sys.executable, "-c", script], capture_output=True, text=True, env=env, timeout=600)
     assert a.returncode == 0 and b.returncode == 0, a.stderr[-500:] + b.stderr[-500:]
     assert a.stdout.strip() == b.stdout.strip() and len(a.stdout.strip()) == 40
+
+
+def test_check_log_entries():
+    """driver.CheckLog: per-pass arrays in, the replay entries (dicts) out, in issue order."""
+    L = driver.CheckLog()
+    assert len(L) == 0 and not L
+    L.add(0, 1, 2, np.array([2, 4]), np.array([6, 9]), np.array([0, 2, 3]), np.array([1, 2, 3]), np.array([1, 0]))
+    L.append({"version": 1, "phase": 2, "pass": 0, "lit_a": 10, "lit_b": 12, "leaves": [5, 6], "verdict": 1})
+    assert len(L) == 3 and L
+    assert L[0] == {"version": 0, "phase": 1, "pass": 2, "lit_a": 2, "lit_b": 6, "leaves": [1, 2], "verdict": 1}
+    assert L[1]["leaves"] == [3] and L[1]["verdict"] == 0 and L[-1]["lit_a"] == 10
+    assert [c["lit_b"] for c in L] == [6, 9, 12] and [c["lit_a"] for c in L[1:]] == [4, 10]
