@@ -269,7 +269,7 @@ struct cec_plan {
 // a12 in two steps (cec_host.cpp): validate + plan + upload + launch asynchronously, then collect
 cec_status local_checks_launch(cec_ctx *c, uint32_t n, const uint32_t *la, const uint32_t *lb, const uint32_t *cut_off,
                                const uint32_t *leaves, std::unique_ptr<cec_plan> &out, uint32_t *bad_out,
-                               uint32_t *first_bad_out);
+                               uint32_t *first_bad_out, bool trusted_cuts = false);
 cec_status local_checks_collect(cec_ctx *c, cec_plan *P, int32_t *verdict);
 
 // device copy of the AIG (fanin literals + level CSR), uploaded on first use (cec_host.cpp)

@@ -2157,7 +2157,7 @@ cec_status cec_check_local_cuts(cec_ctx *c, uint32_t n, const uint32_t *la, cons
 // (asynchronous on the context stream), then collect (wait, read back, free the device block).
 cec_status local_checks_launch(cec_ctx *c, uint32_t n, const uint32_t *la, const uint32_t *lb, const uint32_t *cut_off,
                                const uint32_t *leaves, std::unique_ptr<cec_plan> &out, uint32_t *bad_out,
-                               uint32_t *first_bad_out) {
+                               uint32_t *first_bad_out, bool trusted_cuts) {
     auto t0 = std::chrono::steady_clock::now();
     std::unique_ptr<cec_plan> P(new (std::nothrow) cec_plan());
     if (!P) return CEC_E_NOMEM;
@@ -2182,14 +2182,19 @@ cec_status local_checks_launch(cec_ctx *c, uint32_t n, const uint32_t *la, const
         L.erase(std::unique(L.begin(), L.end()), L.end());
         if (L.size() > kcap) return fail(c, CEC_E_ARG, "check %u: %zu leaves > %u", q, L.size(), kcap);
         P->k[q] = (uint32_t)L.size();
-        // cut validation: no PI outside L reachable from a root without crossing L
-        ++sep;
-        for (uint32_t x : L) stop[x] = sep;
+        // cut validation: no PI outside L reachable from a root without crossing L.
+        // Skipped for the Alg. 2 pass's own common cuts (trusted_cuts): u | v with u a cut of one root
+        // and v of the other is a cut of both by construction (CEC_VALIDATE_CUTS=1 checks them anyway)
         bool ok = true;
-        uint32_t roots[2] = {la[q] >> 1, lb[q] >> 1};
-        walk_tfi(c, c->scratch, roots, 2, &stop, sep, [&](uint32_t v) {
-            if (v >= 1 && v <= c->I && stop[v] != sep) ok = false;
-        });
+        static const bool force_validate = getenv("CEC_VALIDATE_CUTS") != nullptr;
+        if (!trusted_cuts || force_validate) {
+            ++sep;
+            for (uint32_t x : L) stop[x] = sep;
+            uint32_t roots[2] = {la[q] >> 1, lb[q] >> 1};
+            walk_tfi(c, c->scratch, roots, 2, &stop, sep, [&](uint32_t v) {
+                if (v >= 1 && v <= c->I && stop[v] != sep) ok = false;
+            });
+        }
         if (!ok) {
             P->pre_verdict[q] = CEC_BAD_CUT;
             if (!bad++) first_bad = q;

@@ -653,7 +653,7 @@ extern "C" cec_status cec_local_pass(cec_ctx *c, uint32_t npairs, const uint32_t
         if (F.pair.empty()) return CEC_OK;
         uint32_t bad = 0, first_bad = 0;
         cec_status st = local_checks_launch(c, (uint32_t)F.pair.size(), F.la.data(), F.lb.data(), F.off.data(),
-                                            F.leaves.data(), F.plan, &bad, &first_bad);
+                                            F.leaves.data(), F.plan, &bad, &first_bad, true);
         if (st != CEC_OK) return st;
         if (bad) {
             c->err = "common cut is not a cut (internal error)";
