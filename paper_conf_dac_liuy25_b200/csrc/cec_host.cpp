@@ -1453,8 +1453,13 @@ static cec_status plan_route(cec_ctx *c, uint32_t n, const uint32_t *la, const u
     // the whole AIG, lists saturating at k_max + 1); only pairs above k_max (exact k) and the
     // cost-aware merge (which needs cone sizes) walk cones on the host.
     std::vector<uint8_t> need_walk(n, 1);
-    bool gpu_supp = !c->host_only && c->opts.merge != CEC_MERGE_COST && n >= 64 && c->N() >= (1u << 16);
-    if (const char *e = getenv("CEC_SUPP_GPU")) gpu_supp = !c->host_only && c->opts.merge != CEC_MERGE_COST && atoi(e) != 0;
+    // The cost-aware merge also needs each pair's cone size: the GPU walks those too (cone_sizes,
+    // supp_gpu.cu; CEC_CONES_GPU=0 walks them on the host), cones too large for its shared memory
+    // fall back to the host walk.
+    const bool cost = c->opts.merge == CEC_MERGE_COST;
+    bool cones_gpu = !getenv("CEC_CONES_GPU") || atoi(getenv("CEC_CONES_GPU")) != 0;
+    bool gpu_supp = !c->host_only && (!cost || cones_gpu) && n >= 64 && c->N() >= (1u << 16);
+    if (const char *e = getenv("CEC_SUPP_GPU")) gpu_supp = !c->host_only && (!cost || cones_gpu) && atoi(e) != 0;
     if (gpu_supp) {
         cec_status st = cec_ensure_device_aig(c);
         if (st != CEC_OK) return st;
@@ -1466,12 +1471,15 @@ static cec_status plan_route(cec_ctx *c, uint32_t n, const uint32_t *la, const u
         uint32_t nl = 0;
         CUDA_TRY(c, gpu_supports(*c->devpool, c->d_f0, c->d_f1, c->d_level_ids, c->level_off, c->I, c->N(), cap, roots,
                                  lists, cnt, c->stream, &nl, &c->supp_table));
+        std::vector<uint32_t> gcone;
+        if (cost) CUDA_TRY(c, gpu_cones(*c->devpool, c->d_f0, c->d_f1, c->I, roots, gcone, c->stream));
         for (uint32_t p = 0; p < n; ++p)
-            if (cnt[p] < cap) {
+            if (cnt[p] < cap && (!cost || gcone[p] != 0xFFFFFFFFu)) {
                 supp[p].assign(lists.begin() + (size_t)p * cap, lists.begin() + (size_t)p * cap + cnt[p]);
+                if (cost) cones[p] = gcone[p];
                 need_walk[p] = 0;
             }
-        tm.lap("supports (gpu)");
+        tm.lap(cost ? "supports + cones (gpu)" : "supports (gpu)");
     }
     if (std::find(need_walk.begin(), need_walk.end(), (uint8_t)1) != need_walk.end()) {
         WorkPool &wp = c->workers();

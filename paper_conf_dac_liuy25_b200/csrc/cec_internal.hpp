@@ -119,6 +119,10 @@ const char *gpu_supports(DevPool &pool, const uint32_t *d_f0, const uint32_t *d_
                          const std::vector<uint32_t> &level_off, uint32_t I, uint32_t N, uint32_t cap,
                          const std::vector<uint2> &roots, std::vector<uint32_t> &lists_out,
                          std::vector<uint32_t> &cnt_out, void *stream, uint32_t *launches, NodeSupports *table);
+// supp_gpu.cu: AND-cone sizes |TFI(a) u TFI(b)| of pairs (the cost-aware merge's estimates);
+// UINT32_MAX where the cone does not fit the block's shared-memory walk (the host walks those).
+const char *gpu_cones(DevPool &pool, const uint32_t *d_f0, const uint32_t *d_f1, uint32_t I,
+                      const std::vector<uint2> &roots, std::vector<uint32_t> &cone_out, void *stream);
 
 // jit.cpp
 std::string jit_key(const JitProgram &p);

@@ -115,7 +115,103 @@ __global__ void supp_pairs(const uint2 *__restrict__ roots, uint32_t n, const ui
 
 inline const char *ck(cudaError_t e) { return e == cudaSuccess ? nullptr : cudaGetErrorString(e); }
 
+// Cone sizes for the cost-aware merge: |TFI(a) u TFI(b)| in AND nodes (roots included, PIs and the
+// constant excluded), one block per pair: a breadth-first walk whose visited set is an
+// open-addressing hash table in shared memory and whose frontiers are two shared arrays. A cone that
+// does not fit (hash over half full, frontier overflow) reports UINT32_MAX and is walked on the host.
+constexpr uint32_t CONE_HS = 8192, CONE_FC = 4096, CONE_EMPTY = 0xFFFFFFFFu;
+constexpr size_t CONE_SMEM = sizeof(uint32_t) * (CONE_HS + 2 * CONE_FC);
+
+__device__ __forceinline__ int cone_insert(uint32_t *keys, uint32_t key) {  // 1 new, 0 present, -1 full
+    uint32_t h = (key * 0x9E3779B1u) >> (32 - 13);  // 13 = log2(CONE_HS)
+    for (uint32_t probe = 0; probe < 64; ++probe) {
+        const uint32_t old = atomicCAS(&keys[h], CONE_EMPTY, key);
+        if (old == CONE_EMPTY) return 1;
+        if (old == key) return 0;
+        h = (h + 1) & (CONE_HS - 1);
+    }
+    return -1;
+}
+
+__global__ void __launch_bounds__(256) cone_sizes(const uint2 *__restrict__ roots, uint32_t n,
+                                                  const uint32_t *__restrict__ f0, const uint32_t *__restrict__ f1,
+                                                  uint32_t I, uint32_t *out) {
+    extern __shared__ uint32_t sm[];
+    uint32_t *keys = sm, *fr[2] = {sm + CONE_HS, sm + CONE_HS + CONE_FC};
+    __shared__ uint32_t s_cnt, s_nf[2], s_over;
+    for (uint32_t p = blockIdx.x; p < n; p += gridDim.x) {
+        for (uint32_t i = threadIdx.x; i < CONE_HS; i += blockDim.x) keys[i] = CONE_EMPTY;
+        if (threadIdx.x == 0) s_cnt = 0, s_nf[0] = 0, s_nf[1] = 0, s_over = 0;
+        __syncthreads();
+        if (threadIdx.x < 2) {
+            const uint32_t r = threadIdx.x ? roots[p].y : roots[p].x;
+            if (r > I) {
+                const int ins = cone_insert(keys, r);
+                if (ins < 0) s_over = 1;
+                if (ins > 0) {
+                    atomicAdd(&s_cnt, 1u);
+                    fr[0][atomicAdd(&s_nf[0], 1u)] = r;
+                }
+            }
+        }
+        __syncthreads();
+        for (uint32_t cur = 0;; cur ^= 1u) {
+            const uint32_t nf = s_nf[cur];
+            if (nf == 0 || s_over) break;
+            if (threadIdx.x == 0) s_nf[cur ^ 1u] = 0;
+            __syncthreads();
+            for (uint32_t i = threadIdx.x; i < nf; i += blockDim.x) {
+                const uint32_t v = fr[cur][i];
+                const uint32_t fa[2] = {f0[v] >> 1, f1[v] >> 1};
+                for (int t = 0; t < 2; ++t) {
+                    if (fa[t] <= I) continue;  // PI or constant: not part of the AND cone
+                    const int ins = cone_insert(keys, fa[t]);
+                    if (ins < 0) s_over = 1;
+                    if (ins <= 0) continue;
+                    atomicAdd(&s_cnt, 1u);
+                    const uint32_t slot = atomicAdd(&s_nf[cur ^ 1u], 1u);
+                    if (slot < CONE_FC) fr[cur ^ 1u][slot] = fa[t];
+                    else s_over = 1;
+                }
+            }
+            __syncthreads();
+        }
+        if (threadIdx.x == 0) out[p] = (s_over || s_cnt > CONE_HS / 2) ? 0xFFFFFFFFu : s_cnt;
+        __syncthreads();
+    }
+}
+
 }  // namespace
+
+const char *gpu_cones(DevPool &pool, const uint32_t *d_f0, const uint32_t *d_f1, uint32_t I,
+                      const std::vector<uint2> &roots, std::vector<uint32_t> &cone_out, void *stream) {
+    cudaStream_t st = (cudaStream_t)stream;
+    const uint32_t n = (uint32_t)roots.size();
+    cone_out.assign(n, 0xFFFFFFFFu);
+    if (!n) return nullptr;
+    auto al = [](size_t x) { return (x + 255) / 256 * 256; };
+    const size_t b_roots = al(sizeof(uint2) * n), b_out = al(sizeof(uint32_t) * n);
+    void *blk = nullptr;
+    size_t blk_cap = 0;
+    const char *e;
+    if ((e = pool.get(b_roots + b_out, &blk, &blk_cap))) return e;
+    uint2 *d_roots = (uint2 *)blk;
+    uint32_t *d_out = (uint32_t *)((char *)blk + b_roots);
+    if ((e = ck(cudaFuncSetAttribute(cone_sizes, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)CONE_SMEM)))) {
+        pool.put(blk, blk_cap);
+        return e;
+    }
+    e = ck(cudaMemcpyAsync(d_roots, roots.data(), sizeof(uint2) * n, cudaMemcpyHostToDevice, st));
+    if (!e) {
+        cone_sizes<<<(unsigned)std::min<uint32_t>(n, 148u * 3u), 256, CONE_SMEM, st>>>(d_roots, n, d_f0, d_f1, I, d_out);
+        e = ck(cudaGetLastError());
+    }
+    if (!e) e = ck(cudaMemcpyAsync(cone_out.data(), d_out, sizeof(uint32_t) * n, cudaMemcpyDeviceToHost, st));
+    if (!e) e = ck(cudaStreamSynchronize(st));
+    if (e) cudaStreamSynchronize(st);
+    pool.put(blk, blk_cap);
+    return e;
+}
 
 const char *gpu_supports(DevPool &pool, const uint32_t *d_f0, const uint32_t *d_f1, const uint32_t *d_level_ids,
                          const std::vector<uint32_t> &level_off, uint32_t I, uint32_t N, uint32_t cap,

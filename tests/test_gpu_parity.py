@@ -679,3 +679,30 @@ def test_cli_diffable_output_matches_oracle_byte_for_byte(tmp_path):
         assert got.stdout == want, cmd
         outs[cmd] = want
     assert " NEQ " in outs["check"] and "\ncex " in outs["check"]  # the bug is refuted, with a CEX line
+
+
+@pytest.mark.parametrize("which", ["small", "full"])
+def test_gpu_cone_sizes_give_the_host_merge(which, monkeypatch):
+    """The cost-aware merge's cone sizes from the GPU walk (supp_gpu.cu cone_sizes) equal the host
+    walk's: the merged windows (inputs, node counts, pairs) and W are identical to the host-walk
+    plan (CEC_CONES_GPU=0), and so are the results."""
+    from workloads import c3_rand
+
+    m = _c3_small() if which == "small" else c3_rand()
+
+    def plan_of():
+        ctx = gpu_ctx(m.aig, merge=capi.CEC_MERGE_COST, engine=capi.CEC_ENGINE_INTERP)
+        pl = capi.cec_plan_exhaustive(ctx.handle, m.lit_a, m.lit_b)
+        info = capi.cec_plan_info(pl)
+        wins = [capi.cec_plan_window(pl, w) for w in range(info["num_windows"])]
+        capi.cec_plan_run(ctx.handle, pl)
+        res = capi.cec_plan_results(ctx.handle, pl, m.num_pairs)
+        capi.cec_plan_free(pl)
+        return info, wins, res
+
+    gi, gw, gr = plan_of()
+    monkeypatch.setenv("CEC_CONES_GPU", "0")
+    hi, hw, hr = plan_of()
+    assert gi == hi and gw == hw
+    for a, b in zip(gr, hr):
+        assert np.array_equal(a, b)
