@@ -944,7 +944,7 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
             if (!res[w].jit && !res[w].sc.ops.empty())
                 std::copy(res[w].sc.ops.begin(), res[w].sc.ops.end(), P->prog.begin() + P->dwin[w].prog_off);
         };
-        if (wins.size() < 2) {
+        if (wins.size() < 2 || prog_total < (1u << 16)) {  // small: a pool hand-off costs more than the copy
             for (uint32_t w = 0; w < wins.size(); ++w) copy(w, 0);
         } else {
             c->workers().run((uint32_t)wins.size(), copy);
@@ -958,7 +958,9 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
             const int32_t pi = win_jit[w];
             if (pi >= 0 && jit_rep[pi] != w && res[w].key != res[jit_rep[pi]].key) bad[w] = 1;
         };
-        if (wins.size() < 2) {
+        size_t njit = 0;  // only JIT windows have keys to compare
+        for (uint32_t w = 0; w < wins.size(); ++w) njit += win_jit[w] >= 0;
+        if (njit < 64) {
             for (uint32_t w = 0; w < wins.size(); ++w) verify(w, 0);
         } else {
             c->workers().run((uint32_t)wins.size(), verify);
