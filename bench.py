@@ -245,7 +245,7 @@ def main():
     ap.add_argument("--config", default="c5")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--engine", type=int, default=0, help="0 auto, 1 interpreter, 2 JIT, 3 paper Alg. 1 (simt in HBM)")
-    ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--merge", type=int, default=-1, help="0 off, 1 paper (default), 2 cost-aware (default for c3)")
     ap.add_argument("--cpu-log2-patterns", type=int, default=19)
     ap.add_argument("--ref-log2-patterns", type=int, default=17)
