@@ -1423,6 +1423,39 @@ extern "C" {
 }  // extern "C"
 
 // a2-a5 of a global check: supports, trivial pairs, routing by k, compares, windows and merging.
+// Open-addressing map uint64 -> uint32 for the routing of all pairs (one probe sequence per lookup,
+// no node allocations: the routing loop was bound by std::unordered_map). Key ~0 is the empty mark.
+struct FlatMap64 {
+    std::vector<uint64_t> key;
+    std::vector<uint32_t> val;
+    size_t mask = 0;
+    explicit FlatMap64(size_t n) {
+        size_t cap = 16;
+        while (cap < 2 * n) cap <<= 1;
+        key.assign(cap, ~0ull);
+        val.assign(cap, 0);
+        mask = cap - 1;
+    }
+    // the value slot of `k` (inserted with value `dflt` if absent; *inserted says which)
+    uint32_t *slot(uint64_t k, uint32_t dflt, bool *inserted) {
+        uint64_t h = k + 0x9E3779B97F4A7C15ull;
+        h = (h ^ (h >> 30)) * 0xBF58476D1CE4E5B9ull;
+        h = (h ^ (h >> 27)) * 0x94D049BB133111EBull;
+        for (size_t i = (h ^ (h >> 31)) & mask;; i = (i + 1) & mask) {
+            if (key[i] == k) {
+                *inserted = false;
+                return &val[i];
+            }
+            if (key[i] == ~0ull) {
+                key[i] = k;
+                val[i] = dflt;
+                *inserted = true;
+                return &val[i];
+            }
+        }
+    }
+};
+
 static cec_status plan_route(cec_ctx *c, uint32_t n, const uint32_t *la, const uint32_t *lb, cec_plan *P,
                              std::vector<WinHost> &wins, PhaseTimer &tm) {
     P->num_pairs = n;
@@ -1434,10 +1467,10 @@ static cec_status plan_route(cec_ctx *c, uint32_t n, const uint32_t *la, const u
     P->pair_cmp.assign(n, -1);
     const uint32_t kmax = c->opts.k_max;
     // a2/a3: supports, trivial pairs, routing by k; identical (unordered) pairs share one compare
-    std::unordered_map<uint64_t, uint32_t> seen;  // unordered literal pair -> compare
+    FlatMap64 seen(n);  // unordered literal pair -> compare (key < ~0: literals < 2^32 - 1)
     // identical supports share a window: hash of S -> first window with that hash, then a chain
     // through win_next (exact compare below); no per-window allocation
-    std::unordered_map<uint64_t, uint32_t> by_support;
+    FlatMap64 by_support(n);
     std::vector<uint32_t> win_next;
     auto supp_hash = [](const std::vector<uint32_t> &S) {
         uint64_t h = 0x9E3779B97F4A7C15ull ^ S.size();
@@ -1532,8 +1565,6 @@ static cec_status plan_route(cec_ctx *c, uint32_t n, const uint32_t *la, const u
         }
     }
     tm.lap("supports");
-    seen.reserve(2 * (size_t)n);
-    by_support.reserve(2 * (size_t)n);
     P->cmps.reserve(n);
     wins0.reserve(n);
     win_next.reserve(n);
@@ -1556,21 +1587,23 @@ static cec_status plan_route(cec_ctx *c, uint32_t n, const uint32_t *la, const u
         }
         P->pre_verdict[p] = DECIDED_BY_SIM;
         const uint64_t key = (uint64_t)std::min(la[p], lb[p]) << 32 | std::max(la[p], lb[p]);
-        auto it = seen.find(key);
-        if (it != seen.end()) {
-            P->pair_cmp[p] = (int32_t)it->second;
+        bool fresh = false;
+        uint32_t *cslot = seen.slot(key, (uint32_t)P->cmps.size(), &fresh);
+        if (!fresh) {
+            P->pair_cmp[p] = (int32_t)*cslot;
             continue;
         }
-        const uint32_t ci = (uint32_t)P->cmps.size();
-        seen.emplace(key, ci);
+        const uint32_t ci = *cslot;
         P->pair_cmp[p] = (int32_t)ci;
-        auto hit = by_support.emplace(supp_hash(S), UINT32_MAX).first;
+        uint64_t sh = supp_hash(S);
+        if (sh == ~0ull) sh = 0;  // the empty mark (a hash collision is resolved by the exact compare)
+        uint32_t *head = by_support.slot(sh, UINT32_MAX, &fresh);
         uint32_t wi = UINT32_MAX;
-        for (uint32_t x = hit->second; x != UINT32_MAX && wi == UINT32_MAX; x = win_next[x])
+        for (uint32_t x = *head; x != UINT32_MAX && wi == UINT32_MAX; x = win_next[x])
             if (wins0[x].inputs == S) wi = x;
         if (wi == UINT32_MAX) {
-            win_next.push_back(hit->second);
-            hit->second = (uint32_t)wins0.size();
+            win_next.push_back(*head);
+            *head = (uint32_t)wins0.size();
             WinHost w;
             w.inputs = S;
             w.cmps.push_back(ci);
