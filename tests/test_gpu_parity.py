@@ -681,14 +681,17 @@ def test_cli_diffable_output_matches_oracle_byte_for_byte(tmp_path):
     assert " NEQ " in outs["check"] and "\ncex " in outs["check"]  # the bug is refuted, with a CEX line
 
 
-@pytest.mark.parametrize("which", ["small", "full"])
+@pytest.mark.parametrize("which", ["small", "full", "bigcones"])
 def test_gpu_cone_sizes_give_the_host_merge(which, monkeypatch):
     """The cost-aware merge's cone sizes from the GPU walk (supp_gpu.cu cone_sizes) equal the host
     walk's: the merged windows (inputs, node counts, pairs) and W are identical to the host-walk
     plan (CEC_CONES_GPU=0), and so are the results."""
     from workloads import c3_rand
 
-    m = _c3_small() if which == "small" else c3_rand()
+    if which == "bigcones":  # 10k-AND copies: cones beyond the kernel's shared memory -> host fallback
+        m = c5_big(copies=8, n_random=6, n_bugs=2)
+    else:
+        m = _c3_small() if which == "small" else c3_rand()
 
     def plan_of():
         ctx = gpu_ctx(m.aig, merge=capi.CEC_MERGE_COST, engine=capi.CEC_ENGINE_INTERP)
