@@ -903,9 +903,14 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
         dw.tt_words_lo = (uint32_t)ttw;
         dw.tt_words_hi = (uint32_t)(ttw >> 32);
         P->dwin.push_back(dw);
-        P->win_inputs.push_back(W.inputs);
         P->win_nodes.push_back((uint32_t)nodes.size());
-        P->win_cmps.push_back(wc);
+        if (c->opts.engine == CEC_ENGINE_SIMT && !local) {  // the Alg. 1 layout below reads them again
+            P->win_inputs.push_back(W.inputs);
+            P->win_cmps.push_back(wc);
+        } else {  // the caller's windows are discarded after planning: no copies
+            P->win_inputs.push_back(std::move(W.inputs));
+            P->win_cmps.push_back(std::move(wcs[w]));
+        }
         nslots_of.push_back(sc.nslots);
         const bool jit = R.jit;
         if (jit) {  // windows of identical structure share one program (by hash; verified below)
