@@ -917,6 +917,7 @@ cec_status finish_plan(cec_ctx *c, cec_plan *P, std::vector<WinHost> &wins, cons
             auto it = jit_hindex.find(R.hkey);
             if (it == jit_hindex.end()) {
                 it = jit_hindex.emplace(R.hkey, (uint32_t)jit_progs.size()).first;
+                R.jp.key = R.key;  // the cache lookup's key part (R.key stays for the exact verify)
                 jit_progs.push_back(std::move(R.jp));
                 jit_rep.push_back((uint32_t)w);
             }

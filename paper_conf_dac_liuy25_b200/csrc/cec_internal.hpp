@@ -49,6 +49,7 @@ struct JitProgram {
     uint32_t k = 0;
     std::vector<uint32_t> nodes;
     std::vector<uint32_t> cmps;
+    std::string key;  // jit_key(*this) when the planner already built it (cache lookups reuse it)
 };
 struct JItem {             // a slice range of one JIT window instance
     uint32_t win;          // window index (bound / neq_cnt)

@@ -1228,7 +1228,7 @@ const char *jit_get_unit(const std::vector<const JitProgram *> &ps, const JitCon
     snprintf(ck, sizeof ck, "|%d,%d,%d,%d,%d,%d,%d", cfg.threads, cfg.min_blocks, cfg.sync_every, (int)cfg.fuse,
              (int)cfg.splice, (int)cfg.free_warps, cfg.ilp);
     std::string key;
-    for (const JitProgram *p : ps) key += jit_key(*p) + "#";
+    for (const JitProgram *p : ps) (key += p->key.empty() ? jit_key(*p) : p->key) += "#";
     key += ck;
     {
         std::lock_guard<std::mutex> g(g_mu);
